@@ -1,0 +1,365 @@
+#!/usr/bin/env python
+"""Benchmark of the single-parity HISQ Dslash (BASELINE.json metric: Dslash GFLOP/s and
+achieved HBM GB/s, % of B200 peak, at 1/2/4/8 GPUs).
+
+One step = one Dslash apply (every row of SURVEY.md §8(a): site decode, neighbour addressing,
+link stream, neighbour gather, 16 matvecs, store; plus the depth-3 halo exchange when N > 1)
+on one batch of synthetic fp64 input.
+
+  N = 1 : 32^4 lattice (BASELINE.json configs[2], the paper's workload).
+  N > 1 : weak scaling, 32^3 x 32N global lattice t-partitioned over N GPUs (configs[4] shape:
+          32^3 x 32 per GPU), halo overlapped with the interior kernel.
+
+GFLOP/s = 1146 flop x target sites / time (PAPER.md L278 convention, 600.8 MFLOP per 32^4
+apply).  Algorithmic bytes = 2400 per target site.  Inputs are larger
+than L2: the 1.2 GB of links stream through every apply and the source/output vectors rotate
+over R pairs whose footprint exceeds the 126 MB L2.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--kernel site|dir4] [--block B]
+  python bench.py --impl reference ...   # the CPU oracle on the host cores (reference arm)
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+FLOP_PER_SITE = 1146
+ALGO_BYTES_PER_SITE = 2400
+METRIC = "Dslash GFLOP/s and achieved HBM GB/s (% of B200 peak) at 1/2/4/8 GPUs"
+NOMINAL_HBM_GBS = 8000.0
+FALLBACK_HBM_GBS = 6650.0  # /opt/skills/guides/B200_PROFILING.md fallback
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=2000)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--kernel", default="site", choices=["site", "dir4"])
+    ap.add_argument("--block", type=int, default=0)
+    ap.add_argument("--local", default="32,32,32,32", help="per-GPU local extents x,y,z,t")
+    ap.add_argument("--parity", type=int, default=0)
+    ap.add_argument("--no-overlap", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0, help="oracle CPU-baseline budget")
+    return ap.parse_args()
+
+
+def workload(args, world):
+    loc = tuple(int(v) for v in args.local.split(","))
+    gdims = (loc[0], loc[1], loc[2], loc[3] * world)
+    grid = (1, 1, 1, world)
+    if world == 1 and loc == (32, 32, 32, 32):
+        name = "32^4 fp64 single-parity HISQ Dslash, 1 GPU (BASELINE.json configs[2])"
+    else:
+        name = (f"{gdims[0]}^3x{gdims[3]} fp64 single-parity HISQ Dslash, weak scaling "
+                f"{loc[0]}x{loc[1]}x{loc[2]}x{loc[3]} per GPU, t-partitioned over {world} (configs[4] shape)")
+    return gdims, grid, loc, name
+
+
+def measured_peak():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            v = float(json.load(f)["hbm_gbs"])
+            return v, "measured (MEASURED_PEAKS.json hbm_gbs, copy burst)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic(kernel_name, local_dims):
+    """dram read+write bytes per launch from the committed ncu --set full summary, if it matches."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_summary.json")) as f:
+            s = json.load(f)
+        for e in s.get("kernels", []):
+            if e.get("variant") == kernel_name and tuple(e.get("local_dims", ())) == tuple(local_dims):
+                return int(e["dram_bytes_per_launch"])
+    except Exception:
+        pass
+    return None
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons with NVML while the timed region runs."""
+
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, device_index):
+        self.samples, self.reasons, self.max_mhz = [], 0, None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.hdl = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.hdl, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.hdl, self.nv.NVML_CLOCK_SM))
+                self.reasons |= int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.hdl))
+            except Exception:
+                pass
+            time.sleep(0.01)
+
+    def __enter__(self):
+        if self.nv:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv:
+            self.t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["unavailable"]}
+        s = sorted(self.samples)
+        names = [n for b, n in self.REASONS.items() if self.reasons & b and n != "gpu_idle"]
+        return {"sm_mhz": s[len(s) // 2], "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(s)}
+
+
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count()
+
+
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def run_oracle_baseline(gdims, parity, budget_s, steps=None, warmup=0):
+    """Time the CPU oracle (as it stands) on the host cores.  Returns a dict for cpu_baseline.
+
+    steps=None: full-lattice applies until `budget_s` is spent (>= 1).  steps=K: the reference
+    arm, K timed steps after `warmup`, each a bounded sample of target sites sized so the whole
+    run takes about `budget_s`.
+    """
+    import numpy as np
+
+    import fieldgen
+    import oracle
+
+    fat, lng = fieldgen.workload_links(gdims)
+    psi = fieldgen.vector(gdims, fieldgen.SEED_PSI)
+    vh = int(np.prod(gdims)) // 2
+    cores = host_cores()
+    t0 = time.perf_counter()
+    oracle.dslash(fat, lng, psi, parity, cores)                 # warm-up full apply
+    t_full = time.perf_counter() - t0
+    if steps is None:
+        n, t0 = 0, time.perf_counter()
+        while True:
+            oracle.dslash(fat, lng, psi, parity, cores)
+            n += 1
+            el = time.perf_counter() - t0
+            if el >= budget_s:
+                break
+        return {"value": FLOP_PER_SITE * vh * n / el / 1e9, "unit": "GFLOP/s", "cores": cores,
+                "kind": "oracle", "cpu": cpu_model(),
+                "sample": f"{n} full {gdims[0]}x{gdims[1]}x{gdims[2]}x{gdims[3]} applies (parity {parity}), "
+                          f"{el:.1f} s, OpenMP over target sites"}, el / n
+    sites_all = oracle.lex_sites_of_parity(gdims, parity)
+    frac = min(1.0, budget_s / max(1, steps + warmup) / t_full)
+    stride = max(1, int(round(1.0 / frac)))
+    sites = np.ascontiguousarray(sites_all[::stride])
+    for _ in range(warmup):
+        oracle.dslash_sites(fat, lng, psi, sites, cores)
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        oracle.dslash_sites(fat, lng, psi, sites, cores)
+    el = time.perf_counter() - t0
+    return {"value": FLOP_PER_SITE * sites.size * steps / el / 1e9, "unit": "GFLOP/s", "cores": cores,
+            "kind": "oracle", "cpu": cpu_model(),
+            "sample": f"each step: every {stride}-th target site of the {gdims[0]}x{gdims[1]}x{gdims[2]}x{gdims[3]} "
+                      f"lattice ({sites.size} of {vh} sites), parity {parity}"}, el / steps
+
+
+def reference_arm(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    world = args.gpus
+    gdims, grid, loc, name = workload(args, 1)   # the oracle runs the N=1 workload of one rank
+    budget = max(20.0, min(150.0, 0.05 * (args.steps + args.warmup)))
+    cb, per_step = run_oracle_baseline(gdims, args.parity, budget, args.steps, args.warmup)
+    line = {"metric": METRIC, "value": cb["value"], "unit": "GFLOP/s", "impl": "reference", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": per_step * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": name, "global_dims": list(gdims), "parity": args.parity,
+                       "oracle": "oracle/hisq_oracle.c (plain C99 complex, -O2 -ffp-contract=off, OpenMP)"},
+            "cpu_baseline": cb,
+            "e2e": {"value": cb["value"], "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return reference_arm(args)
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import fieldgen
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.gpus != world:
+        if world == 1 and args.gpus > 1:
+            print(json.dumps({"error": f"--gpus {args.gpus} needs torchrun with {args.gpus} ranks"}))
+            return 2
+    torch.cuda.set_device(local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    gdims, grid, loc, name = workload(args, world)
+    parity = args.parity
+
+    D = Dslash(gdims, grid, parity_mask=parity, kernel=args.kernel, block=args.block,
+               overlap=not args.no_overlap, timing=True, rank=rank, world_size=world)
+    origin, extent = D.origin, D.local_dims
+    fat, lng = fieldgen.workload_links(gdims, origin=origin, extent=extent)
+    D.load_links(fat, lng)
+    del fat, lng
+    vh = D.vh
+    vec_bytes = 3 * vh * 16
+    l2_bytes = torch.cuda.get_device_properties(local_rank).L2_cache_size
+    R = max(2, int(np.ceil(2 * l2_bytes / (2 * vec_bytes))) + 1)
+    srcs = [torch.from_numpy(fieldgen.vector_cb(gdims, fieldgen.SEED_PSI + r, 1 - parity, origin=origin,
+                                                extent=extent)).cuda() for r in range(R)]
+    outs = [D.empty_vector() for _ in range(R)]
+    stream = torch.cuda.current_stream()
+
+    def step(i):
+        D.apply(outs[i % R], srcs[i % R], parity, stream)
+
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    D.kernel_timing_reset()   # discard warm-up records
+
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(torch.cuda.current_device()) as clk:
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        for i in range(args.steps):
+            step(i)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+    ms = ev0.elapsed_time(ev1)
+    t_int, n_int = D.kernel_timing(0)
+    t_bnd, n_bnd = D.kernel_timing(1)
+    D.kernel_timing_reset()
+    t_max = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
+    ms_max = float(t_max.item())
+    total_sites = vh * world
+    gflops = FLOP_PER_SITE * total_sites * args.steps / (ms_max * 1e-3) / 1e9
+    algo_gbs = ALGO_BYTES_PER_SITE * total_sites * args.steps / (ms_max * 1e-3) / 1e9
+
+    # dominant kernel: the full-lattice kernel at N = 1, the interior kernel at N > 1
+    plan = D.plan
+    dom_sites = int(plan.interior_sites) if plan.n_interior else int(plan.boundary_sites)
+    peak, peak_src = measured_peak()
+    kern_ms = t_int / max(1, n_int) if n_int else None
+    roof = None
+    if kern_ms:
+        achieved = ALGO_BYTES_PER_SITE * dom_sites / (kern_ms * 1e-3) / 1e9
+        roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": ncu_traffic(args.kernel, extent),
+                "kernel": f"dslash_{args.kernel}_kernel" + ("<ghost=false> interior" if world > 1 else "<ghost=false>"),
+                "bytes_per_launch": ALGO_BYTES_PER_SITE * dom_sites, "avg_launch_us": round(kern_ms * 1e3, 2),
+                "launches": n_int, "peak_source": peak_src,
+                "frac_of_nominal_8TBs": round(achieved / NOMINAL_HBM_GBS, 4)}
+
+    # end to end through the C ABI from pinned host buffers (H2D of psi, apply, D2H of chi)
+    e2e = None
+    if not args.no_e2e:
+        hin = torch.from_numpy(fieldgen.vector_cb(gdims, fieldgen.SEED_PSI, 1 - parity, origin=origin,
+                                                  extent=extent)).pin_memory()
+        hout = torch.empty_like(hin).pin_memory()
+        ke = max(10, min(args.steps, 300))
+        for _ in range(3):
+            D.apply_host(hout, hin, parity, stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ev0.record(stream)
+        for _ in range(ke):
+            D.apply_host(hout, hin, parity, stream)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        D.kernel_timing_reset()
+        te = torch.tensor([ev0.elapsed_time(ev1)], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e = {"value": FLOP_PER_SITE * total_sites * ke / (float(te.item()) * 1e-3) / 1e9, "unit": "GFLOP/s",
+               "h2d_bytes_per_step": vec_bytes * world, "d2h_bytes_per_step": vec_bytes * world, "steps": ke,
+               "path": "dslash_apply_host (C ABI): pinned host psi -> device, apply, device -> pinned host chi"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu, _ = run_oracle_baseline(gdims, parity, args.cpu_seconds)
+
+    launches_per_step = (1 if not any(plan.halo) else (int(plan.n_interior > 0) + 1))
+    if rank == 0:
+        line = {"metric": METRIC, "value": round(gflops, 2), "unit": "GFLOP/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic",
+                "config": {"workload": name, "global_dims": list(gdims), "local_dims": list(extent),
+                           "proc_grid": list(grid), "parallelism": f"t{world}", "parity": parity,
+                           "kernel": args.kernel, "block": args.block or None,
+                           "overlap": not args.no_overlap,
+                           "l2": f"inputs > L2: 1.21 GB links/apply streamed; {R} rotating (psi, chi) pairs = "
+                                 f"{R * 2 * vec_bytes / 1e6:.0f} MB > {l2_bytes / 1e6:.0f} MB L2",
+                           "links": "random SU(3) fat (seed 1), -1/24 random SU(3) long (seed 2)"},
+                "algorithmic_gbs": round(algo_gbs, 1),
+                "pct_hbm_measured": round(100 * algo_gbs / peak, 2),
+                "pct_hbm_nominal_8TBs": round(100 * algo_gbs / NOMINAL_HBM_GBS, 2),
+                "roofline": roof, "clocks": clk.summary(), "e2e": e2e,
+                "gpu_launches": launches_per_step * args.steps,
+                "cpu_baseline": cpu}
+        print(json.dumps(line), flush=True)
+    D.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -158,15 +158,16 @@ FG_API int64_t fg_vector(const int32_t G[4], const int32_t O[4], const int32_t E
 }
 
 /*
- * The same vector values, but only the sites of global parity `parity`, in the
+ * The same vector values, but only the sites of GLOBAL parity `parity`, in the
  * library's checkerboard vector layout: out[c][cb] complex, c < 3, where
- * cb = (local lex) / 2 over the sites of that parity (requires E[0] even and an
- * even origin sum, which the library's partition rules guarantee).  Vh = nloc/2.
+ * cb = (local lex) / 2 over the sites of that parity.  Requires E[0] even (then every
+ * x-row holds E[0]/2 sites of each parity and cb is a bijection onto [0, Vh)), any
+ * origin (odd origins describe ghost slabs).  Vh = nloc/2.
  */
 FG_API int64_t fg_vector_cb(const int32_t G[4], const int32_t O[4], const int32_t E[4], uint64_t seed,
                             int32_t parity, double* out) {
-    if (fg_check_box(G, O, E) || !out || (parity & ~1) || (E[0] & 1) || ((O[0] + O[1] + O[2] + O[3]) & 1))
-        return -1;
+    if (fg_check_box(G, O, E) || !out || (parity & ~1) || (E[0] & 1)) return -1;
+    const int64_t osum = (int64_t)O[0] + O[1] + O[2] + O[3];
     const int64_t nloc = (int64_t)E[0] * E[1] * E[2] * E[3];
     const int64_t vh = nloc / 2;
 #pragma omp parallel for schedule(static)
@@ -176,7 +177,7 @@ FG_API int64_t fg_vector_cb(const int32_t G[4], const int32_t O[4], const int32_
         const int64_t y = r % E[1]; r /= E[1];
         const int64_t z = r % E[2]; r /= E[2];
         const int64_t t = r;
-        if (((x + y + z + t) & 1) != parity) continue;
+        if (((x + y + z + t + osum) & 1) != parity) continue;
         const uint64_t g = fg_glex(G, O[0] + x, O[1] + y, O[2] + z, O[3] + t);
         const int64_t cb = l >> 1;
         for (int c = 0; c < 3; ++c)

@@ -1,0 +1,196 @@
+/*
+ * hisq_dslash.h -- C ABI of the B200-native single-parity HISQ (improved-staggered)
+ * Dslash library (libhisq_dslash.so, sm_100a).
+ *
+ * The operation (§II, Eq. (1) "C = Dslash x B", with the third-
+ * neighbour Naik terms of L27/L51; readings Z1-Z10): for every local
+ * site x of the target parity p,
+ *
+ *   chi(x) = sum_{mu=0..3} [  F(x,mu) psi(x+mu)   - F(x-mu,mu)^dag  psi(x-mu)
+ *                           + N(x,mu) psi(x+3mu)  - N(x-3mu,mu)^dag psi(x-3mu) ]
+ *
+ * on a periodic 4-D lattice, fp64 complex.  F = fat links, N = long (Naik) links,
+ * psi lives on parity 1-p (target sites s* in [0, L^4/2)).
+ *
+ * Conventions (all functions):
+ *   - dims are {Lx, Ly, Lz, Lt}, x fastest; lex(x,y,z,t) = x + Lx*(y + Ly*(z + Lz*t));
+ *     parity p(x) = (x+y+z+t) mod 2 in GLOBAL coordinates.
+ *   - Complex numbers are two interleaved doubles (re, im), 16 B.
+ *   - Vector layout (in, out): [3][Vh_local] complex, colour-major ("SoA"), where the
+ *     checkerboard index cb = (local lex) / 2 enumerates the local sites of one parity
+ *     in lexicographic order (Z8).  Vh_local = local volume / 2.
+ *   - Canonical link layout (load_links input): [t][z][y][x][mu][3][3] complex over the
+ *     LOCAL volume, forward links only, row-major 3x3 (|i| x |j| complex
+ *     matrices, an array of L^4 x |k| per link kind).
+ *   - Every function returns a dslash_status; no C++ exception crosses the ABI.  Errors
+ *     are sticky per handle: once a call fails, dslash_error_string(h) describes the
+ *     first failure; later calls still run their own argument checks.
+ *   - Streams are cudaStream_t passed as void* (NULL = the legacy default stream).
+ *
+ * Multi-GPU: one process per GPU; the lattice may be split along
+ * z and t only (proc_grid = {1, 1, Pz, Pt}); rank = cz + Pz * ct.  Each apply exchanges
+ * a depth-3 halo of the source parity (the Naik hop reaches 3 sites) with NCCL
+ * send/recv on an internal communication stream, overlapped with the interior kernel.
+ */
+#ifndef HISQ_DSLASH_H
+#define HISQ_DSLASH_H
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define DSLASH_API __attribute__((visibility("default")))
+#else
+#define DSLASH_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct dslash_s* dslash_t;
+typedef void* dslash_stream_t; /* cudaStream_t */
+
+typedef enum {
+    DSLASH_OK = 0,
+    DSLASH_ERR_ARG = 1,         /* invalid argument (odd/small extents, bad parity, NULL/aliased pointers) */
+    DSLASH_ERR_STATE = 2,       /* call out of order (apply before load_links, option after load_links) */
+    DSLASH_ERR_CUDA = 3,        /* a CUDA runtime call failed (message carries cudaGetErrorString) */
+    DSLASH_ERR_NCCL = 4,        /* an NCCL call failed */
+    DSLASH_ERR_OOM = 5,         /* device allocation failed */
+    DSLASH_ERR_UNSUPPORTED = 6  /* valid but not implemented (x/y partitioning, fp32 before it exists) */
+} dslash_status;
+
+enum { DSLASH_EVEN = 0, DSLASH_ODD = 1, DSLASH_BOTH = 2 }; /* parity_mask */
+enum { DSLASH_F64 = 0, DSLASH_F32 = 1 };                   /* precision */
+
+/* Kernel variants (DSLASH_OPT_KERNEL); DESIGN.md §Kernels. */
+enum {
+    DSLASH_KERNEL_SITE = 0, /* one thread per target site, 16 link matrices streamed per thread   */
+    DSLASH_KERNEL_DIR4 = 1  /* four lanes per site (one per mu), 2-step shuffle reduction ("3LP") */
+};
+
+/* Options (dslash_set_option). */
+enum {
+    DSLASH_OPT_KERNEL = 0,      /* kernel variant; before load_links (it fixes the link layout)        */
+    DSLASH_OPT_BLOCK = 1,       /* threads per block, 0 = variant default; any time                    */
+    DSLASH_OPT_FORCE_HALO = 2,  /* bitmask of directions (bit mu) exchanged through the halo path even
+                                   when Pmu == 1 (self-halo: neighbour = self); before load_links      */
+    DSLASH_OPT_OVERLAP = 3,     /* 1 (default): interior kernel overlaps the halo exchange; 0: one
+                                   kernel over all sites after the exchange                            */
+    DSLASH_OPT_TIMING = 4       /* 1: record CUDA events around every kernel (dslash_kernel_timing)   */
+};
+
+/* Kernel classes for dslash_kernel_timing. */
+enum { DSLASH_TIMING_INTERIOR = 0, DSLASH_TIMING_BOUNDARY = 1, DSLASH_TIMING_ALL = 2 };
+
+/* Host-only decomposition of the local lattice (no CUDA calls).  A "box" is
+ * [lo[d], hi[d]) per dimension in local coordinates; the target-parity sites of a
+ * box number (hi0-lo0)/2 * (hi1-lo1) * (hi2-lo2) * (hi3-lo3). */
+typedef struct {
+    int32_t lo[4];
+    int32_t hi[4];
+} dslash_box_t;
+
+typedef struct {
+    int32_t global_dims[4];
+    int32_t proc_grid[4];
+    int32_t proc_coords[4];
+    int32_t local_dims[4];
+    int32_t origin[4];         /* global coordinate of local (0,0,0,0); always even */
+    int32_t halo[4];           /* 1 if direction mu exchanges a depth-3 halo        */
+    int32_t nbr_rank[4][2];    /* [mu][0 = minus, 1 = plus] neighbour rank (self if Pmu == 1) */
+    int32_t rank, nranks;
+    int64_t vh_local;          /* local target (= source) sites per parity           */
+    int64_t face_vh[4];        /* source sites in one depth-3 face slab (0 if no halo) */
+    int32_t n_interior, n_boundary;
+    dslash_box_t interior[1];  /* sites whose 16 sources are all local               */
+    dslash_box_t boundary[4];  /* the remaining sites (disjoint boxes)               */
+    int64_t interior_sites, boundary_sites;
+} dslash_plan_t;
+
+/* Compute the decomposition for `rank` of `nranks` (no CUDA, no allocation).
+ * force_halo_mask: as DSLASH_OPT_FORCE_HALO.  Errors: DSLASH_ERR_ARG for odd or < 2
+ * extents, a halo direction with an odd local extent or one < 4 (depth-3 halo plus
+ * parity), extents not divisible by proc_grid, prod(proc_grid) != nranks, rank out of
+ * range; DSLASH_ERR_UNSUPPORTED for proc_grid[0] or proc_grid[1] != 1. */
+DSLASH_API dslash_status dslash_plan(const int32_t global_dims[4], const int32_t proc_grid[4], int32_t rank,
+                          int32_t nranks, int32_t force_halo_mask, dslash_plan_t* plan);
+
+/* Create a handle on the current CUDA device.  parity_mask selects for which target
+ * parities links are prepared (DSLASH_BOTH doubles link memory).  precision must be
+ * DSLASH_F64 (DSLASH_F32 returns DSLASH_ERR_UNSUPPORTED in this version).
+ * nccl_unique_id: the 128-byte ncclUniqueId from dslash_get_unique_id() on rank 0,
+ * broadcast to all ranks by the caller; NULL when nranks == 1.  On success *out owns
+ * a CUDA communication stream, events, ghost buffers and (nranks > 1) an NCCL
+ * communicator; release it with dslash_destroy.  On failure *out is NULL. */
+DSLASH_API dslash_status dslash_create(const int32_t global_dims[4], const int32_t proc_grid[4], int32_t parity_mask,
+                            int32_t precision, const void* nccl_unique_id, int32_t nranks, int32_t rank,
+                            dslash_t* out);
+
+/* Write a fresh ncclUniqueId (128 bytes) to id_out.  Call on rank 0 only. */
+DSLASH_API dslash_status dslash_get_unique_id(void* id_out);
+
+/* Set an option (see DSLASH_OPT_*).  DSLASH_ERR_STATE if the option must precede
+ * load_links and links are loaded; DSLASH_ERR_ARG for unknown keys or bad values. */
+DSLASH_API dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t value);
+
+/* Copy the caller's forward links into the library's internal parity-split layout,
+ * building the back-links F(x-mu,mu)^dag and N(x-3mu,mu)^dag (|l| = 4
+ * link arrays; Z2).  fat, lng: canonical layout over the local volume,
+ * fp64 complex; on_device = 1 if they are device pointers, 0 for host memory.  When
+ * partitioned, one NCCL exchange fetches the 3 link slices below each halo face.
+ * Synchronous: on return the caller may free fat and lng.  Callable again to replace
+ * the links. */
+DSLASH_API dslash_status dslash_load_links(dslash_t h, const void* fat, const void* lng, int32_t on_device,
+                                dslash_stream_t stream);
+
+/* chi = D psi on target parity `parity`.  out: device [3][Vh_local] complex on parity
+ * `parity`; in: device [3][Vh_local] complex on parity 1-parity.  Both caller-owned,
+ * 16-byte aligned, non-overlapping.  Stream-ordered and asynchronous: it runs
+ * halo_start / interior kernel / halo_wait / boundary kernel internally.  Errors:
+ * DSLASH_ERR_STATE before load_links, DSLASH_ERR_ARG for parity not in parity_mask,
+ * NULL, misaligned or overlapping buffers. */
+DSLASH_API dslash_status dslash_apply(dslash_t h, void* out, const void* in, int32_t parity, dslash_stream_t stream);
+
+/* The same operation from HOST buffers (end-to-end path): copies in (host) to an
+ * internal device buffer, applies, copies the result to out (host), all ordered on
+ * `stream`; returns after enqueueing (synchronise the stream before reading out).
+ * Pinned host memory gives asynchronous copies. */
+DSLASH_API dslash_status dslash_apply_host(dslash_t h, void* out_host, const void* in_host, int32_t parity,
+                                dslash_stream_t stream);
+
+/* Halo exchange only: start sending the depth-3 faces of `in` (source parity
+ * src_parity) after the work already queued on `stream`; dslash_halo_wait makes
+ * `stream` wait for the ghost zones.  No-op when no direction has a halo.  Exposed
+ * so callers can overlap their own work; dslash_apply calls both itself. */
+DSLASH_API dslash_status dslash_halo_start(dslash_t h, const void* in, int32_t src_parity, dslash_stream_t stream);
+DSLASH_API dslash_status dslash_halo_wait(dslash_t h, dslash_stream_t stream);
+
+/* Synchronise the handle's streams and surface asynchronous CUDA/NCCL errors. */
+DSLASH_API dslash_status dslash_sync(dslash_t h);
+
+/* Sum of the durations of the kernels of class `which` (DSLASH_TIMING_INTERIOR / _BOUNDARY,
+ * or DSLASH_TIMING_ALL for every class) recorded since the last dslash_kernel_timing_reset
+ * (DSLASH_OPT_TIMING = 1); synchronises on the recorded events.  Every timed launch keeps
+ * one event pair until the next reset. */
+DSLASH_API dslash_status dslash_kernel_timing(dslash_t h, int32_t which, double* total_ms, int64_t* launches);
+DSLASH_API dslash_status dslash_kernel_timing_reset(dslash_t h);
+
+/* Copy the plan the handle uses. */
+DSLASH_API dslash_status dslash_get_plan(dslash_t h, dslash_plan_t* plan);
+
+/* Number of local target sites per parity (Vh_local), or -1 for a NULL handle. */
+DSLASH_API int64_t dslash_local_half_volume(dslash_t h);
+
+/* Release everything the handle owns (synchronises first).  NULL is a no-op. */
+DSLASH_API dslash_status dslash_destroy(dslash_t h);
+
+/* Human-readable description of the handle's first error ("" if none); with h = NULL,
+ * the last error of a failed dslash_create / dslash_plan in this thread. */
+DSLASH_API const char* dslash_error_string(dslash_t h);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* HISQ_DSLASH_H */

@@ -1,0 +1,148 @@
+"""B200-native single-parity HISQ Dslash (MILC-Dslash hot path, Dufek et al. SC'24 workshops).
+
+The product is the C-ABI library ``libhisq_dslash.so`` (include/hisq_dslash.h):
+hand-written sm_100a CUDA kernels plus a C++ host runtime with an NCCL depth-3 halo
+exchange.  This package is a thin Python binding: ``_abi`` exposes the C functions
+under their own names (argument marshalling only) and :class:`Dslash` wraps a handle,
+taking device memory and streams from PyTorch.  There is no CPU fallback: importing
+without the built library raises.
+"""
+from __future__ import annotations
+
+from . import _abi
+from ._abi import (DSLASH_BOTH, DSLASH_EVEN, DSLASH_F64, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_SITE,  # noqa: F401
+                   DSLASH_ODD, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_KERNEL, DSLASH_OPT_OVERLAP,
+                   DSLASH_OPT_TIMING, DSLASH_TIMING_ALL, DSLASH_TIMING_BOUNDARY, DSLASH_TIMING_INTERIOR,
+                   KERNELS, DslashError, dslash_plan)
+
+FLOP_PER_SITE = 1146          # 600.8 MFLOP per 32^4 apply = 1146 per target site
+LINK_BYTES_PER_SITE = 2304    # 16 matrices x 9 complex x 16 B (fp64), streamed once
+ALGO_BYTES_PER_SITE = 2400    # + 48 B source (ideal reuse) + 48 B output
+
+__all__ = ["Dslash", "DslashError", "dslash_plan", "FLOP_PER_SITE", "ALGO_BYTES_PER_SITE"]
+
+
+def _stream_handle(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+
+
+class Dslash:
+    """One handle of the library on the current CUDA device.
+
+    Vectors are torch complex128 CUDA tensors of shape (3, Vh_local) (colour-major,
+    checkerboard site order cb = local lex // 2); links are canonical forward links
+    (Lt, Lz, Ly, Lx, 4, 3, 3) complex128 over the local volume, numpy (host) or torch
+    (device).  With ``world_size > 1`` the NCCL unique id is broadcast through the
+    default torch.distributed process group.
+    """
+
+    def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="site", block=0,
+                 force_halo=0, overlap=True, timing=False, rank=0, world_size=1):
+        self.global_dims = tuple(int(d) for d in global_dims)
+        self.proc_grid = tuple(int(p) for p in proc_grid)
+        uid = None
+        if world_size > 1:
+            import torch
+            import torch.distributed as dist
+            t = torch.zeros(128, dtype=torch.uint8, device="cuda" if dist.get_backend() == "nccl" else "cpu")
+            if rank == 0:
+                t.copy_(torch.frombuffer(bytearray(_abi.dslash_get_unique_id()), dtype=torch.uint8))
+            dist.broadcast(t, 0)
+            uid = bytes(t.cpu().numpy().tobytes())
+        self.h = _abi.dslash_create(self.global_dims, self.proc_grid, parity_mask, DSLASH_F64, uid, world_size, rank)
+        try:
+            _abi.dslash_set_option(self.h, DSLASH_OPT_KERNEL, KERNELS[kernel] if isinstance(kernel, str) else kernel)
+            if block:
+                _abi.dslash_set_option(self.h, DSLASH_OPT_BLOCK, block)
+            if force_halo:
+                _abi.dslash_set_option(self.h, DSLASH_OPT_FORCE_HALO, force_halo)
+            _abi.dslash_set_option(self.h, DSLASH_OPT_OVERLAP, int(bool(overlap)))
+            if timing:
+                _abi.dslash_set_option(self.h, DSLASH_OPT_TIMING, 1)
+        except Exception:
+            self.close()
+            raise
+        self.plan = _abi.dslash_get_plan(self.h)
+        self.vh = int(self.plan.vh_local)
+        self.local_dims = tuple(self.plan.local_dims)
+        self.origin = tuple(self.plan.origin)
+
+    # -- links
+    def load_links(self, fat, lng, stream=None):
+        import numpy as np
+        if isinstance(fat, np.ndarray):
+            fat = np.ascontiguousarray(fat, dtype=np.complex128)
+            lng = np.ascontiguousarray(lng, dtype=np.complex128)
+            self._check_links(fat.shape, lng.shape)
+            _abi.dslash_load_links(self.h, fat.ctypes.data, lng.ctypes.data, 0, _stream_handle(stream))
+        else:
+            import torch
+            assert fat.is_cuda and fat.dtype == torch.complex128 and fat.is_contiguous()
+            assert lng.is_cuda and lng.dtype == torch.complex128 and lng.is_contiguous()
+            self._check_links(tuple(fat.shape), tuple(lng.shape))
+            _abi.dslash_load_links(self.h, fat.data_ptr(), lng.data_ptr(), 1, _stream_handle(stream))
+
+    def _check_links(self, a, b):
+        lx, ly, lz, lt = self.local_dims
+        want = (lt, lz, ly, lx, 4, 3, 3)
+        if tuple(a) != want or tuple(b) != want:
+            raise ValueError(f"links must have shape {want}, got {a} and {b}")
+
+    # -- vectors
+    def empty_vector(self):
+        import torch
+        return torch.empty((3, self.vh), dtype=torch.complex128, device="cuda")
+
+    def _check_vec(self, v):
+        import torch
+        if not (v.is_cuda and v.dtype == torch.complex128 and v.is_contiguous() and tuple(v.shape) == (3, self.vh)):
+            raise ValueError(f"vector must be a contiguous complex128 CUDA tensor of shape (3, {self.vh})")
+
+    def apply(self, out, inp, parity, stream=None):
+        """out = D inp on target parity `parity` (stream-ordered, asynchronous)."""
+        self._check_vec(out)
+        self._check_vec(inp)
+        _abi.dslash_apply(self.h, out.data_ptr(), inp.data_ptr(), int(parity), _stream_handle(stream))
+        return out
+
+    def __call__(self, inp, parity, stream=None):
+        return self.apply(self.empty_vector(), inp, parity, stream)
+
+    def apply_host(self, out, inp, parity, stream=None):
+        """Host-buffer path (end-to-end): torch CPU complex128 tensors (pin them for async copies)."""
+        import torch
+        for v in (out, inp):
+            if v.is_cuda or v.dtype != torch.complex128 or not v.is_contiguous() or tuple(v.shape) != (3, self.vh):
+                raise ValueError(f"host vectors must be contiguous complex128 CPU tensors of shape (3, {self.vh})")
+        _abi.dslash_apply_host(self.h, out.data_ptr(), inp.data_ptr(), int(parity), _stream_handle(stream))
+        return out
+
+    def kernel_timing(self, which=DSLASH_TIMING_ALL):
+        """(total ms, launches) of the kernels of class `which` recorded since the last reset."""
+        return _abi.dslash_kernel_timing(self.h, which)
+
+    def kernel_timing_reset(self):
+        _abi.dslash_kernel_timing_reset(self.h)
+
+    def sync(self):
+        _abi.dslash_sync(self.h)
+
+    def close(self):
+        if getattr(self, "h", None):
+            _abi.dslash_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

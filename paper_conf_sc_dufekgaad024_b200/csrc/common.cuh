@@ -1,0 +1,97 @@
+// common.cuh -- shared device-side types and PTX helpers for the HISQ Dslash kernels (sm_100a).
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace hisq {
+
+// ---------------------------------------------------------------- fast unsigned division
+// q = n / d for 0 <= n < 2^31 and d >= 1 via one mul.hi (round-up multiplier method).
+struct FastDiv {
+    uint32_t d, m, s;
+    __host__ void init(uint32_t div) {
+        d = div;
+        s = 0;
+        while ((1ull << s) < div) ++s;
+        m = (uint32_t)((((1ull << 32) * ((1ull << s) - div)) / div) + 1);
+    }
+    __device__ __forceinline__ uint32_t div(uint32_t n) const {
+        return (uint32_t)(((uint64_t)__umulhi(n, m) + n) >> s);
+    }
+};
+
+// ---------------------------------------------------------------- cache-policy loads/stores
+// Links are streamed exactly once: keep them out of L1 and mark their L2 lines evict-first so
+// the reused source vectors (16 consumers each) stay L2-resident.
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+__device__ __forceinline__ double2 ld_stream(const double2* p, uint64_t pol) {
+    double2 r;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;"
+        : "=d"(r.x), "=d"(r.y)
+        : "l"(p), "l"(pol));
+    return r;
+}
+
+__device__ __forceinline__ double2 ld_reuse(const double2* p, uint64_t pol) {
+    double2 r;
+    asm("ld.global.nc.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(r.x), "=d"(r.y) : "l"(p), "l"(pol));
+    return r;
+}
+
+__device__ __forceinline__ void st_stream(double2* p, double2 v) {
+    asm volatile("st.global.cs.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
+}
+
+// ---------------------------------------------------------------- complex fp64 arithmetic
+// acc += a * b
+__device__ __forceinline__ void cmadd(double2& acc, double2 a, double2 b) {
+    acc.x = fma(a.x, b.x, acc.x);
+    acc.x = fma(-a.y, b.y, acc.x);
+    acc.y = fma(a.x, b.y, acc.y);
+    acc.y = fma(a.y, b.x, acc.y);
+}
+// acc -= a * b
+__device__ __forceinline__ void cmsub(double2& acc, double2 a, double2 b) {
+    acc.x = fma(-a.x, b.x, acc.x);
+    acc.x = fma(a.y, b.y, acc.x);
+    acc.y = fma(-a.x, b.y, acc.y);
+    acc.y = fma(-a.y, b.x, acc.y);
+}
+
+// ---------------------------------------------------------------- kernel parameters
+constexpr int kMaxBoxes = 4;
+
+struct Box {
+    int lo[4];
+    int n[4];  // extent per dim; n[0] counts full x extent (sites per row = n[0] / 2)
+};
+
+struct StencilParams {
+    const double2* links;      // internal link layout for the target parity (variant-specific)
+    const double2* in;         // [3][vh] source parity, local
+    double2* out;              // [3][vh] target parity, local
+    const double2* ghost[4][2];  // [mu][side] -> [3][face_vh[mu]] (only where halo[mu])
+    int64_t vh;
+    int64_t face_vh[4];
+    int L[4];                  // local extents
+    int lxh;                   // L[0] / 2
+    int parity;                // (target parity + origin sum) & 1, origin sum is even -> target parity
+    int halo_mask;             // bit mu set: direction mu reads ghosts outside [0, L[mu])
+    int nbox;
+    Box box[kMaxBoxes];
+    int64_t box_start[kMaxBoxes + 1];  // prefix sum of target sites per box
+    FastDiv div_xh[kMaxBoxes], div_y[kMaxBoxes], div_z[kMaxBoxes];
+};
+
+}  // namespace hisq

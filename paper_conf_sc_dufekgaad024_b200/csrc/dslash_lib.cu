@@ -1,0 +1,723 @@
+// dslash_lib.cu -- C ABI of the B200-native HISQ Dslash (include/hisq_dslash.h).
+//
+// Host runtime: lattice decomposition (dslash_plan), device memory ownership, the depth-3
+// halo exchange (NCCL send/recv over NVLink on an internal stream, or device copies when the
+// neighbour is this rank), kernel launches and error reporting.  Every step of the Dslash
+// itself runs in the kernels of stencil.cuh / links.cuh.
+#include <nccl.h>
+
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "hisq_dslash.h"
+#include "common.cuh"
+#include "links.cuh"
+#include "stencil.cuh"
+
+using namespace hisq;
+
+// ============================================================================ errors
+static thread_local std::string g_last_error;
+
+struct dslash_s {
+    dslash_plan_t plan{};
+    int32_t global_dims[4]{}, proc_grid[4]{};
+    int parity_mask = 0, precision = 0, device = 0;
+    int kernel = DSLASH_KERNEL_SITE, block = 0, force_halo = 0, overlap = 1, timing = 0;
+    bool loaded = false;
+    double2* links[2] = {nullptr, nullptr};
+    double2* ghost[4][2] = {};     // source-vector ghost faces [3][face_vh]
+    double2* zsend[2] = {};        // packed z faces to send (NCCL path)
+    double2* stage_in = nullptr;   // apply_host staging
+    double2* stage_out = nullptr;
+    cudaStream_t comm = nullptr;
+    cudaEvent_t ev_start = nullptr, ev_halo = nullptr;
+    bool halo_pending = false;
+    ncclComm_t nccl = nullptr;
+    struct TimedLaunch {
+        cudaEvent_t a, b;
+        int kind;
+    };
+    std::vector<TimedLaunch> tpool;
+    size_t tused = 0;
+    dslash_status err = DSLASH_OK;
+    std::string msg;
+};
+
+static dslash_status fail(dslash_t h, dslash_status st, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (h) {
+        if (h->err == DSLASH_OK) {
+            h->err = st;
+            h->msg = buf;
+        }
+    } else {
+        g_last_error = buf;
+    }
+    return st;
+}
+
+#define CU(h, call)                                                                                   \
+    do {                                                                                              \
+        cudaError_t e_ = (call);                                                                      \
+        if (e_ != cudaSuccess)                                                                        \
+            return fail((h), e_ == cudaErrorMemoryAllocation ? DSLASH_ERR_OOM : DSLASH_ERR_CUDA,      \
+                        "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e_));           \
+    } while (0)
+
+#define NC(h, call)                                                                                   \
+    do {                                                                                              \
+        ncclResult_t r_ = (call);                                                                     \
+        if (r_ != ncclSuccess)                                                                        \
+            return fail((h), DSLASH_ERR_NCCL, "%s:%d %s: %s", __FILE__, __LINE__, #call,              \
+                        ncclGetErrorString(r_));                                                      \
+    } while (0)
+
+// ============================================================================ plan (host only)
+extern "C" dslash_status dslash_plan(const int32_t G[4], const int32_t P[4], int32_t rank, int32_t nranks,
+                                     int32_t force_halo_mask, dslash_plan_t* out) {
+    if (!G || !P || !out) return fail(nullptr, DSLASH_ERR_ARG, "dslash_plan: NULL argument");
+    dslash_plan_t p;
+    memset(&p, 0, sizeof p);
+    int64_t prod = 1;
+    for (int d = 0; d < 4; ++d) {
+        if (G[d] < 2 || (G[d] & 1))
+            return fail(nullptr, DSLASH_ERR_ARG, "global extent %d of dim %d must be even and >= 2", G[d], d);
+        if (P[d] < 1) return fail(nullptr, DSLASH_ERR_ARG, "proc_grid[%d] = %d must be >= 1", d, P[d]);
+        if (G[d] % P[d])
+            return fail(nullptr, DSLASH_ERR_ARG, "global extent %d of dim %d not divisible by proc_grid %d", G[d], d,
+                        P[d]);
+        prod *= P[d];
+    }
+    if (P[0] != 1 || P[1] != 1)
+        return fail(nullptr, DSLASH_ERR_UNSUPPORTED, "only z and t may be partitioned (proc_grid = {1,1,Pz,Pt})");
+    if (prod != nranks) return fail(nullptr, DSLASH_ERR_ARG, "prod(proc_grid) = %lld != nranks = %d", (long long)prod, nranks);
+    if (rank < 0 || rank >= nranks) return fail(nullptr, DSLASH_ERR_ARG, "rank %d out of range [0,%d)", rank, nranks);
+    if (force_halo_mask & ~0xC)
+        return fail(nullptr, DSLASH_ERR_UNSUPPORTED, "halo directions other than z (bit 2) and t (bit 3)");
+    p.rank = rank;
+    p.nranks = nranks;
+    // rank = cx + Px*(cy + Py*(cz + Pz*ct)) with Px = Py = 1
+    int r = rank;
+    for (int d = 0; d < 4; ++d) {
+        p.global_dims[d] = G[d];
+        p.proc_grid[d] = P[d];
+        p.proc_coords[d] = r % P[d];
+        r /= P[d];
+        p.local_dims[d] = G[d] / P[d];
+        p.origin[d] = p.proc_coords[d] * p.local_dims[d];
+    }
+    for (int d = 0; d < 4; ++d) {
+        p.halo[d] = (P[d] > 1) || ((force_halo_mask >> d) & 1);
+        for (int side = 0; side < 2; ++side) {
+            int c[4] = {p.proc_coords[0], p.proc_coords[1], p.proc_coords[2], p.proc_coords[3]};
+            c[d] = (c[d] + (side ? 1 : P[d] - 1)) % P[d];
+            p.nbr_rank[d][side] = c[0] + P[0] * (c[1] + P[1] * (c[2] + P[2] * c[3]));
+        }
+        if (p.halo[d] && (p.local_dims[d] < 4 || (p.local_dims[d] & 1)))
+            return fail(nullptr, DSLASH_ERR_ARG,
+                        "local extent %d of halo dim %d must be even and >= 4 (depth-3 halo, parity)",
+                        p.local_dims[d], d);
+    }
+    const int64_t V = (int64_t)p.local_dims[0] * p.local_dims[1] * p.local_dims[2] * p.local_dims[3];
+    p.vh_local = V / 2;
+    for (int d = 0; d < 4; ++d) p.face_vh[d] = p.halo[d] ? 3 * (V / p.local_dims[d]) / 2 : 0;
+
+    // interior box: [3, L-3) along halo dims, full otherwise
+    dslash_box_t full;
+    for (int d = 0; d < 4; ++d) {
+        full.lo[d] = 0;
+        full.hi[d] = p.local_dims[d];
+    }
+    dslash_box_t in = full;
+    bool empty = false;
+    for (int d = 0; d < 4; ++d)
+        if (p.halo[d]) {
+            in.lo[d] = 3;
+            in.hi[d] = p.local_dims[d] - 3;
+            if (in.lo[d] >= in.hi[d]) empty = true;
+        }
+    auto count = [](const dslash_box_t& b) {
+        int64_t n = (b.hi[0] - b.lo[0]) / 2;
+        for (int d = 1; d < 4; ++d) n *= (b.hi[d] - b.lo[d]);
+        return n;
+    };
+    if (empty) {
+        p.n_interior = 0;
+        p.n_boundary = 1;
+        p.boundary[0] = full;
+    } else {
+        p.n_interior = 1;
+        p.interior[0] = in;
+        int nb = 0;
+        dslash_box_t rest = full;  // region still to be covered: shrinks as slabs are cut off
+        for (int d = 3; d >= 2; --d) {
+            if (!p.halo[d]) continue;
+            dslash_box_t lo = rest, hi = rest;
+            lo.hi[d] = 3;
+            hi.lo[d] = p.local_dims[d] - 3;
+            p.boundary[nb++] = lo;
+            p.boundary[nb++] = hi;
+            rest.lo[d] = 3;
+            rest.hi[d] = p.local_dims[d] - 3;
+        }
+        p.n_boundary = nb;
+    }
+    for (int i = 0; i < p.n_interior; ++i) p.interior_sites += count(p.interior[i]);
+    for (int i = 0; i < p.n_boundary; ++i) p.boundary_sites += count(p.boundary[i]);
+    *out = p;
+    return DSLASH_OK;
+}
+
+// ============================================================================ handle
+extern "C" dslash_status dslash_get_unique_id(void* id_out) {
+    if (!id_out) return fail(nullptr, DSLASH_ERR_ARG, "NULL id_out");
+    ncclUniqueId id;
+    ncclResult_t r = ncclGetUniqueId(&id);
+    if (r != ncclSuccess) return fail(nullptr, DSLASH_ERR_NCCL, "ncclGetUniqueId: %s", ncclGetErrorString(r));
+    memcpy(id_out, &id, sizeof id);
+    return DSLASH_OK;
+}
+
+static void free_links(dslash_t h) {
+    for (int p = 0; p < 2; ++p)
+        if (h->links[p]) {
+            cudaFree(h->links[p]);
+            h->links[p] = nullptr;
+        }
+    h->loaded = false;
+}
+
+static void free_halo(dslash_t h) {
+    for (int d = 0; d < 4; ++d)
+        for (int s = 0; s < 2; ++s)
+            if (h->ghost[d][s]) {
+                cudaFree(h->ghost[d][s]);
+                h->ghost[d][s] = nullptr;
+            }
+    for (int s = 0; s < 2; ++s)
+        if (h->zsend[s]) {
+            cudaFree(h->zsend[s]);
+            h->zsend[s] = nullptr;
+        }
+}
+
+static dslash_status alloc_halo(dslash_t h) {
+    free_halo(h);
+    const dslash_plan_t& p = h->plan;
+    for (int d = 2; d < 4; ++d) {
+        if (!p.halo[d]) continue;
+        for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->ghost[d][s], 3 * p.face_vh[d] * sizeof(double2)));
+    }
+    if (p.halo[2] && p.nbr_rank[2][0] != p.rank)
+        for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->zsend[s], 3 * p.face_vh[2] * sizeof(double2)));
+    return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_create(const int32_t G[4], const int32_t P[4], int32_t parity_mask, int32_t precision,
+                                       const void* nccl_unique_id, int32_t nranks, int32_t rank, dslash_t* out) {
+    if (!out) return fail(nullptr, DSLASH_ERR_ARG, "NULL out");
+    *out = nullptr;
+    if (parity_mask < DSLASH_EVEN || parity_mask > DSLASH_BOTH)
+        return fail(nullptr, DSLASH_ERR_ARG, "parity_mask %d not in {0,1,2}", parity_mask);
+    if (precision == DSLASH_F32) return fail(nullptr, DSLASH_ERR_UNSUPPORTED, "fp32 path not built in this version");
+    if (precision != DSLASH_F64) return fail(nullptr, DSLASH_ERR_ARG, "precision %d unknown", precision);
+    if (nranks > 1 && !nccl_unique_id) return fail(nullptr, DSLASH_ERR_ARG, "nranks > 1 needs an NCCL unique id");
+    dslash_plan_t plan;
+    dslash_status st = dslash_plan(G, P, rank, nranks, 0, &plan);
+    if (st != DSLASH_OK) return st;
+    dslash_t h = new dslash_s();
+    h->plan = plan;
+    memcpy(h->global_dims, G, sizeof h->global_dims);
+    memcpy(h->proc_grid, P, sizeof h->proc_grid);
+    h->parity_mask = parity_mask;
+    h->precision = precision;
+    auto bail = [&](dslash_status s) {
+        g_last_error = h->msg;
+        dslash_destroy(h);
+        return s;
+    };
+    cudaError_t e = cudaGetDevice(&h->device);
+    if (e != cudaSuccess) {
+        fail(h, DSLASH_ERR_CUDA, "cudaGetDevice: %s", cudaGetErrorString(e));
+        return bail(DSLASH_ERR_CUDA);
+    }
+    if ((e = cudaStreamCreateWithFlags(&h->comm, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&h->ev_start, cudaEventDisableTiming)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&h->ev_halo, cudaEventDisableTiming)) != cudaSuccess) {
+        fail(h, DSLASH_ERR_CUDA, "stream/event creation: %s", cudaGetErrorString(e));
+        return bail(DSLASH_ERR_CUDA);
+    }
+    if (nranks > 1) {
+        ncclUniqueId id;
+        memcpy(&id, nccl_unique_id, sizeof id);
+        ncclResult_t r = ncclCommInitRank(&h->nccl, nranks, id, rank);
+        if (r != ncclSuccess) {
+            h->nccl = nullptr;
+            fail(h, DSLASH_ERR_NCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+            return bail(DSLASH_ERR_NCCL);
+        }
+    }
+    if ((st = alloc_halo(h)) != DSLASH_OK) return bail(st);
+    *out = h;
+    return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t value) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    switch (key) {
+        case DSLASH_OPT_KERNEL:
+            if (value != DSLASH_KERNEL_SITE && value != DSLASH_KERNEL_DIR4)
+                return fail(h, DSLASH_ERR_ARG, "unknown kernel variant %lld", (long long)value);
+            if (h->loaded && value != h->kernel)
+                return fail(h, DSLASH_ERR_STATE, "kernel variant fixes the link layout: set it before load_links");
+            h->kernel = (int)value;
+            return DSLASH_OK;
+        case DSLASH_OPT_BLOCK:
+            if (value != 0 && (value < 32 || value > 1024 || (value & 31)))
+                return fail(h, DSLASH_ERR_ARG, "block size %lld must be 0 or a multiple of 32 in [32,1024]",
+                            (long long)value);
+            h->block = (int)value;
+            return DSLASH_OK;
+        case DSLASH_OPT_FORCE_HALO: {
+            if (h->loaded) return fail(h, DSLASH_ERR_STATE, "FORCE_HALO must be set before load_links");
+            dslash_plan_t p;
+            dslash_status st = dslash_plan(h->global_dims, h->proc_grid, h->plan.rank, h->plan.nranks, (int)value, &p);
+            if (st != DSLASH_OK) return fail(h, st, "%s", g_last_error.c_str());
+            h->plan = p;
+            h->force_halo = (int)value;
+            return alloc_halo(h);
+        }
+        case DSLASH_OPT_OVERLAP:
+            h->overlap = value != 0;
+            return DSLASH_OK;
+        case DSLASH_OPT_TIMING:
+            h->timing = value != 0;
+            return DSLASH_OK;
+        default:
+            return fail(h, DSLASH_ERR_ARG, "unknown option %d", key);
+    }
+}
+
+// ============================================================================ link loading
+extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const void* lng, int32_t on_device,
+                                           dslash_stream_t stream) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (!fat || !lng) return fail(h, DSLASH_ERR_ARG, "NULL link pointer");
+    cudaStream_t s = (cudaStream_t)stream;
+    const dslash_plan_t& p = h->plan;
+    const int64_t V = 2 * p.vh_local;
+    const size_t canon_bytes = (size_t)V * 36 * sizeof(double2);
+    std::vector<void*> tmp;
+    auto cleanup = [&]() {
+        for (void* q : tmp) cudaFree(q);
+    };
+#define CUL(call)                                                                                     \
+    do {                                                                                              \
+        cudaError_t e_ = (call);                                                                      \
+        if (e_ != cudaSuccess) {                                                                      \
+            cudaStreamSynchronize(s);                                                                 \
+            cleanup();                                                                                \
+            return fail(h, e_ == cudaErrorMemoryAllocation ? DSLASH_ERR_OOM : DSLASH_ERR_CUDA,        \
+                        "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e_));           \
+        }                                                                                             \
+    } while (0)
+    const double2* dfat = (const double2*)fat;
+    const double2* dlng = (const double2*)lng;
+    if (!on_device) {
+        void *a, *b;
+        CUL(cudaMalloc(&a, canon_bytes));
+        tmp.push_back(a);
+        CUL(cudaMalloc(&b, canon_bytes));
+        tmp.push_back(b);
+        CUL(cudaMemcpyAsync(a, fat, canon_bytes, cudaMemcpyHostToDevice, s));
+        CUL(cudaMemcpyAsync(b, lng, canon_bytes, cudaMemcpyHostToDevice, s));
+        dfat = (const double2*)a;
+        dlng = (const double2*)b;
+    }
+    // lower link slabs: the 3 slices just below the local origin in each halo direction
+    LinkConvParams C{};
+    C.fat = dfat;
+    C.lng = dlng;
+    for (int d = 0; d < 4; ++d) C.L[d] = p.local_dims[d];
+    C.lxh = p.local_dims[0] / 2;
+    C.vh = p.vh_local;
+    C.layout = h->kernel == DSLASH_KERNEL_DIR4 ? 1 : 0;
+    int halo_mask = 0;
+    for (int d = 2; d < 4; ++d)
+        if (p.halo[d]) halo_mask |= 1 << d;
+    C.halo_mask = halo_mask;
+    double2* slab[4][2] = {};   // [mu][fat/long] received
+    double2* send[4][2] = {};   // packed top slabs (z, NCCL only)
+    for (int d = 2; d < 4; ++d) {
+        if (!p.halo[d]) continue;
+        const int64_t slab_elems = 3 * (V / p.local_dims[d]) * 36;
+        for (int k = 0; k < 2; ++k) {
+            CUL(cudaMalloc(&slab[d][k], slab_elems * sizeof(double2)));
+            tmp.push_back(slab[d][k]);
+        }
+    }
+    // Exchange: rank sends its top 3 slices to its plus neighbour, receives into its lower
+    // slab from its minus neighbour.  All ranks issue t then z, fat then long (same order).
+    bool need_nccl = false;
+    for (int d = 3; d >= 2; --d)
+        if (p.halo[d] && p.nbr_rank[d][1] != p.rank) need_nccl = true;
+    const int L0 = p.local_dims[0], L1 = p.local_dims[1], L2 = p.local_dims[2], L3 = p.local_dims[3];
+    const size_t row = (size_t)L0 * L1 * 36 * sizeof(double2);  // one z-slice of one t
+    for (int d = 3; d >= 2; --d) {
+        if (!p.halo[d]) continue;
+        for (int k = 0; k < 2; ++k) {
+            const double2* src = k ? dlng : dfat;
+            if (d == 3) {
+                const double2* top = src + (size_t)(L3 - 3) * L2 * L1 * L0 * 36;
+                if (p.nbr_rank[3][1] == p.rank)
+                    CUL(cudaMemcpyAsync(slab[3][k], top, 3 * (size_t)L2 * row, cudaMemcpyDeviceToDevice, s));
+                else
+                    send[3][k] = (double2*)top;  // contiguous: zero copy
+            } else {
+                double2* dst = slab[2][k];
+                if (p.nbr_rank[2][1] != p.rank) {
+                    CUL(cudaMalloc(&send[2][k], 3 * (size_t)L3 * row));
+                    tmp.push_back(send[2][k]);
+                    dst = send[2][k];
+                }
+                // [t][z in L2-3..L2-1][y][x] -> [t][d][y][x]
+                CUL(cudaMemcpy2DAsync(dst, 3 * row, src + (size_t)(L2 - 3) * L1 * L0 * 36, (size_t)L2 * row, 3 * row,
+                                      L3, cudaMemcpyDeviceToDevice, s));
+            }
+        }
+    }
+    if (need_nccl) {
+        CUL(cudaStreamSynchronize(s));
+        ncclResult_t r = ncclGroupStart();
+        for (int d = 3; d >= 2 && r == ncclSuccess; --d) {
+            if (!p.halo[d] || p.nbr_rank[d][1] == p.rank) continue;
+            const size_t n = (size_t)3 * (V / p.local_dims[d]) * 36 * 2;  // doubles
+            for (int k = 0; k < 2 && r == ncclSuccess; ++k) {
+                r = ncclSend(send[d][k], n, ncclDouble, p.nbr_rank[d][1], h->nccl, s);
+                if (r == ncclSuccess) r = ncclRecv(slab[d][k], n, ncclDouble, p.nbr_rank[d][0], h->nccl, s);
+            }
+        }
+        ncclResult_t r2 = ncclGroupEnd();
+        if (r == ncclSuccess) r = r2;
+        if (r != ncclSuccess) {
+            cleanup();
+            return fail(h, DSLASH_ERR_NCCL, "link halo exchange: %s", ncclGetErrorString(r));
+        }
+    }
+    for (int d = 0; d < 4; ++d) {
+        C.slab_fat[d] = slab[d][0];
+        C.slab_lng[d] = slab[d][1];
+    }
+    const size_t link_bytes = (size_t)p.vh_local * 144 * sizeof(double2);
+    for (int par = 0; par < 2; ++par) {
+        const bool want = h->parity_mask == DSLASH_BOTH || h->parity_mask == par;
+        if (!want) continue;
+        if (!h->links[par]) CUL(cudaMalloc(&h->links[par], link_bytes));
+        C.links = h->links[par];
+        C.parity = par;  // origin sum is even, so local and global parity agree
+        const int64_t n = p.vh_local * 16;
+        const int bs = 256;
+        convert_links_kernel<<<(unsigned)((n + bs - 1) / bs), bs, 0, s>>>(C);
+        CUL(cudaGetLastError());
+    }
+    CUL(cudaStreamSynchronize(s));
+    cleanup();
+#undef CUL
+    h->loaded = true;
+    return DSLASH_OK;
+}
+
+// ============================================================================ halo exchange
+static bool any_halo(const dslash_plan_t& p) { return p.halo[2] || p.halo[3]; }
+
+extern "C" dslash_status dslash_halo_start(dslash_t h, const void* in, int32_t src_parity, dslash_stream_t stream) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (!in || ((uintptr_t)in & 15)) return fail(h, DSLASH_ERR_ARG, "in is NULL or not 16-byte aligned");
+    if (src_parity & ~1) return fail(h, DSLASH_ERR_ARG, "src_parity %d not in {0,1}", src_parity);
+    const dslash_plan_t& p = h->plan;
+    if (!any_halo(p)) return DSLASH_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    const double2* src = (const double2*)in;
+    const int64_t vh = p.vh_local;
+    const int L0 = p.local_dims[0], L1 = p.local_dims[1], L2 = p.local_dims[2], L3 = p.local_dims[3];
+    const int lxh = L0 / 2;
+    CU(h, cudaEventRecord(h->ev_start, s));
+    CU(h, cudaStreamWaitEvent(h->comm, h->ev_start, 0));
+    bool nccl_work = false;
+    // --- local copies (neighbour == self) and z packing
+    if (p.halo[3]) {
+        const size_t slab = (size_t)3 * lxh * L1 * L2;  // sites in 3 t-slices of one parity
+        if (p.nbr_rank[3][0] == p.rank) {
+            // minus ghost <- my top slices, plus ghost <- my bottom slices (periodic self-halo)
+            CU(h, cudaMemcpy2DAsync(h->ghost[3][0], slab * sizeof(double2), src + (size_t)(L3 - 3) * lxh * L1 * L2,
+                                    vh * sizeof(double2), slab * sizeof(double2), 3, cudaMemcpyDeviceToDevice, h->comm));
+            CU(h, cudaMemcpy2DAsync(h->ghost[3][1], slab * sizeof(double2), src, vh * sizeof(double2),
+                                    slab * sizeof(double2), 3, cudaMemcpyDeviceToDevice, h->comm));
+        } else {
+            nccl_work = true;
+        }
+    }
+    if (p.halo[2]) {
+        // [c][t][z0..z0+2][y][xh] -> [c][t][d][y][xh]: rows of 3 z-slices, one row per (c, t)
+        const size_t row = (size_t)lxh * L1;  // sites of one z-slice of one t
+        const bool self = p.nbr_rank[2][0] == p.rank;
+        double2* to_minus = self ? h->ghost[2][1] : h->zsend[0];  // my bottom slices
+        double2* to_plus = self ? h->ghost[2][0] : h->zsend[1];   // my top slices
+        CU(h, cudaMemcpy2DAsync(to_minus, 3 * row * sizeof(double2), src, (size_t)L2 * row * sizeof(double2),
+                                3 * row * sizeof(double2), (size_t)3 * L3, cudaMemcpyDeviceToDevice, h->comm));
+        CU(h, cudaMemcpy2DAsync(to_plus, 3 * row * sizeof(double2), src + (size_t)(L2 - 3) * row,
+                                (size_t)L2 * row * sizeof(double2), 3 * row * sizeof(double2), (size_t)3 * L3,
+                                cudaMemcpyDeviceToDevice, h->comm));
+        if (!self) nccl_work = true;
+    }
+    if (nccl_work) {
+        if (!h->nccl) return fail(h, DSLASH_ERR_STATE, "halo to another rank without an NCCL communicator");
+        // Per direction: sends (bottom -> minus, top -> plus) then receives (plus ghost <- plus,
+        // minus ghost <- minus).  With P = 2 both neighbours are one rank and NCCL matches a pair's
+        // messages in issue order: my first message (bottom) is the peer's first receive (its plus
+        // ghost, since I am its plus neighbour).
+        NC(h, ncclGroupStart());
+        if (p.halo[3] && p.nbr_rank[3][0] != p.rank) {
+            const size_t slab = (size_t)3 * lxh * L1 * L2;
+            const size_t n = slab * 2;
+            for (int c = 0; c < 3; ++c)
+                NC(h, ncclSend(src + c * vh, n, ncclDouble, p.nbr_rank[3][0], h->nccl, h->comm));
+            for (int c = 0; c < 3; ++c)
+                NC(h, ncclSend(src + c * vh + (size_t)(L3 - 3) * lxh * L1 * L2, n, ncclDouble, p.nbr_rank[3][1], h->nccl,
+                               h->comm));
+            for (int c = 0; c < 3; ++c)
+                NC(h, ncclRecv(h->ghost[3][1] + c * slab, n, ncclDouble, p.nbr_rank[3][1], h->nccl, h->comm));
+            for (int c = 0; c < 3; ++c)
+                NC(h, ncclRecv(h->ghost[3][0] + c * slab, n, ncclDouble, p.nbr_rank[3][0], h->nccl, h->comm));
+        }
+        if (p.halo[2] && p.nbr_rank[2][0] != p.rank) {
+            const size_t n = (size_t)3 * p.face_vh[2] * 2;
+            NC(h, ncclSend(h->zsend[0], n, ncclDouble, p.nbr_rank[2][0], h->nccl, h->comm));
+            NC(h, ncclSend(h->zsend[1], n, ncclDouble, p.nbr_rank[2][1], h->nccl, h->comm));
+            NC(h, ncclRecv(h->ghost[2][1], n, ncclDouble, p.nbr_rank[2][1], h->nccl, h->comm));
+            NC(h, ncclRecv(h->ghost[2][0], n, ncclDouble, p.nbr_rank[2][0], h->nccl, h->comm));
+        }
+        NC(h, ncclGroupEnd());
+    }
+    (void)src_parity;  // faces are copied in the caller's cb order; parity only names the field
+    CU(h, cudaEventRecord(h->ev_halo, h->comm));
+    h->halo_pending = true;
+    return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_halo_wait(dslash_t h, dslash_stream_t stream) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (!h->halo_pending) return DSLASH_OK;
+    CU(h, cudaStreamWaitEvent((cudaStream_t)stream, h->ev_halo, 0));
+    h->halo_pending = false;
+    return DSLASH_OK;
+}
+
+// ============================================================================ launches
+static void fill_boxes(StencilParams& K, const dslash_box_t* boxes, int n) {
+    K.nbox = n;
+    K.box_start[0] = 0;
+    for (int b = 0; b < n; ++b) {
+        for (int d = 0; d < 4; ++d) {
+            K.box[b].lo[d] = boxes[b].lo[d];
+            K.box[b].n[d] = boxes[b].hi[d] - boxes[b].lo[d];
+        }
+        K.div_xh[b].init((uint32_t)(K.box[b].n[0] / 2));
+        K.div_y[b].init((uint32_t)K.box[b].n[1]);
+        K.div_z[b].init((uint32_t)K.box[b].n[2]);
+        K.box_start[b + 1] = K.box_start[b] + (int64_t)(K.box[b].n[0] / 2) * K.box[b].n[1] * K.box[b].n[2] * K.box[b].n[3];
+    }
+    for (int b = n; b < kMaxBoxes; ++b) K.box_start[b + 1] = K.box_start[n];
+}
+
+static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int kind, cudaStream_t s) {
+    const int64_t sites = K.box_start[K.nbox];
+    if (sites == 0) return DSLASH_OK;
+    const bool dir4 = h->kernel == DSLASH_KERNEL_DIR4;
+    const int bs = h->block ? h->block : (dir4 ? 256 : 128);
+    const int64_t threads = dir4 ? sites * 4 : sites;
+    const unsigned grid = (unsigned)((threads + bs - 1) / bs);
+    dslash_s::TimedLaunch* tl = nullptr;
+    if (h->timing) {
+        if (h->tused == h->tpool.size()) {
+            dslash_s::TimedLaunch t{};
+            CU(h, cudaEventCreate(&t.a));
+            CU(h, cudaEventCreate(&t.b));
+            h->tpool.push_back(t);
+        }
+        tl = &h->tpool[h->tused++];
+        tl->kind = kind;
+        CU(h, cudaEventRecord(tl->a, s));
+    }
+    if (dir4) {
+        if (ghost)
+            dslash_dir4_kernel<true><<<grid, bs, 0, s>>>(K);
+        else
+            dslash_dir4_kernel<false><<<grid, bs, 0, s>>>(K);
+    } else {
+        if (ghost)
+            dslash_site_kernel<true><<<grid, bs, 0, s>>>(K);
+        else
+            dslash_site_kernel<false><<<grid, bs, 0, s>>>(K);
+    }
+    CU(h, cudaGetLastError());
+    if (tl) CU(h, cudaEventRecord(tl->b, s));
+    return DSLASH_OK;
+}
+
+static dslash_status check_vectors(dslash_t h, const void* out, const void* in) {
+    if (!out || !in) return fail(h, DSLASH_ERR_ARG, "NULL vector pointer");
+    if (((uintptr_t)out & 15) || ((uintptr_t)in & 15)) return fail(h, DSLASH_ERR_ARG, "vectors must be 16-byte aligned");
+    const uintptr_t n = (uintptr_t)(3 * h->plan.vh_local * sizeof(double2));
+    const uintptr_t a = (uintptr_t)out, b = (uintptr_t)in;
+    if (a < b + n && b < a + n) return fail(h, DSLASH_ERR_ARG, "in and out overlap");
+    return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_apply(dslash_t h, void* out, const void* in, int32_t parity, dslash_stream_t stream) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (parity & ~1) return fail(h, DSLASH_ERR_ARG, "parity %d not in {0,1}", parity);
+    if (h->parity_mask != DSLASH_BOTH && h->parity_mask != parity)
+        return fail(h, DSLASH_ERR_ARG, "parity %d not prepared (parity_mask %d)", parity, h->parity_mask);
+    if (!h->loaded) return fail(h, DSLASH_ERR_STATE, "apply before load_links");
+    dslash_status st = check_vectors(h, out, in);
+    if (st != DSLASH_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    const dslash_plan_t& p = h->plan;
+    StencilParams K{};
+    K.links = h->links[parity];
+    K.in = (const double2*)in;
+    K.out = (double2*)out;
+    K.vh = p.vh_local;
+    for (int d = 0; d < 4; ++d) {
+        K.L[d] = p.local_dims[d];
+        K.face_vh[d] = p.face_vh[d];
+        K.ghost[d][0] = h->ghost[d][0];
+        K.ghost[d][1] = h->ghost[d][1];
+        if (p.halo[d]) K.halo_mask |= 1 << d;
+    }
+    K.lxh = p.local_dims[0] / 2;
+    K.parity = parity;
+    if (!any_halo(p)) {
+        fill_boxes(K, p.interior, p.n_interior);
+        return launch(h, K, false, DSLASH_TIMING_INTERIOR, s);
+    }
+    if ((st = dslash_halo_start(h, in, 1 - parity, stream)) != DSLASH_OK) return st;
+    if (h->overlap) {
+        fill_boxes(K, p.interior, p.n_interior);
+        if ((st = launch(h, K, false, DSLASH_TIMING_INTERIOR, s)) != DSLASH_OK) return st;
+        if ((st = dslash_halo_wait(h, stream)) != DSLASH_OK) return st;
+        fill_boxes(K, p.boundary, p.n_boundary);
+        return launch(h, K, true, DSLASH_TIMING_BOUNDARY, s);
+    }
+    if ((st = dslash_halo_wait(h, stream)) != DSLASH_OK) return st;
+    dslash_box_t all[kMaxBoxes];
+    int n = 0;
+    for (int i = 0; i < p.n_interior; ++i) all[n++] = p.interior[i];
+    for (int i = 0; i < p.n_boundary && n < kMaxBoxes; ++i) all[n++] = p.boundary[i];
+    if (p.n_interior + p.n_boundary > kMaxBoxes) {
+        // 5 boxes (t and z halo): launch the interior part first, then the boundary boxes
+        fill_boxes(K, p.interior, p.n_interior);
+        if ((st = launch(h, K, true, DSLASH_TIMING_INTERIOR, s)) != DSLASH_OK) return st;
+        fill_boxes(K, p.boundary, p.n_boundary);
+        return launch(h, K, true, DSLASH_TIMING_BOUNDARY, s);
+    }
+    fill_boxes(K, all, n);
+    return launch(h, K, true, DSLASH_TIMING_ALL, s);
+}
+
+extern "C" dslash_status dslash_apply_host(dslash_t h, void* out_host, const void* in_host, int32_t parity,
+                                           dslash_stream_t stream) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (!out_host || !in_host) return fail(h, DSLASH_ERR_ARG, "NULL host buffer");
+    const size_t bytes = 3 * (size_t)h->plan.vh_local * sizeof(double2);
+    if (!h->stage_in) CU(h, cudaMalloc(&h->stage_in, bytes));
+    if (!h->stage_out) CU(h, cudaMalloc(&h->stage_out, bytes));
+    cudaStream_t s = (cudaStream_t)stream;
+    CU(h, cudaMemcpyAsync(h->stage_in, in_host, bytes, cudaMemcpyHostToDevice, s));
+    dslash_status st = dslash_apply(h, h->stage_out, h->stage_in, parity, stream);
+    if (st != DSLASH_OK) return st;
+    CU(h, cudaMemcpyAsync(out_host, h->stage_out, bytes, cudaMemcpyDeviceToHost, s));
+    return DSLASH_OK;
+}
+
+// ============================================================================ misc
+extern "C" dslash_status dslash_sync(dslash_t h) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    CU(h, cudaStreamSynchronize(h->comm));
+    CU(h, cudaDeviceSynchronize());
+    if (h->nccl) {
+        ncclResult_t async_err;
+        NC(h, ncclCommGetAsyncError(h->nccl, &async_err));
+        if (async_err != ncclSuccess)
+            return fail(h, DSLASH_ERR_NCCL, "NCCL async error: %s", ncclGetErrorString(async_err));
+    }
+    return h->err;
+}
+
+extern "C" dslash_status dslash_kernel_timing(dslash_t h, int32_t which, double* total_ms, int64_t* launches) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (!total_ms || !launches) return fail(h, DSLASH_ERR_ARG, "NULL output");
+    double tot = 0.0;
+    int64_t n = 0;
+    for (size_t i = 0; i < h->tused; ++i) {
+        const auto& t = h->tpool[i];
+        if (which != DSLASH_TIMING_ALL && t.kind != which) continue;
+        CU(h, cudaEventSynchronize(t.b));
+        float ms = 0.f;
+        CU(h, cudaEventElapsedTime(&ms, t.a, t.b));
+        tot += ms;
+        ++n;
+    }
+    *total_ms = tot;
+    *launches = n;
+    return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_kernel_timing_reset(dslash_t h) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (h->tused) CU(h, cudaEventSynchronize(h->tpool[h->tused - 1].b));
+    h->tused = 0;
+    return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_get_plan(dslash_t h, dslash_plan_t* plan) {
+    if (!h || !plan) return fail(h, DSLASH_ERR_ARG, "NULL argument");
+    *plan = h->plan;
+    return DSLASH_OK;
+}
+
+extern "C" int64_t dslash_local_half_volume(dslash_t h) { return h ? h->plan.vh_local : -1; }
+
+extern "C" dslash_status dslash_destroy(dslash_t h) {
+    if (!h) return DSLASH_OK;
+    if (h->comm) cudaStreamSynchronize(h->comm);
+    cudaDeviceSynchronize();
+    free_links(h);
+    free_halo(h);
+    if (h->stage_in) cudaFree(h->stage_in);
+    if (h->stage_out) cudaFree(h->stage_out);
+    for (auto& t : h->tpool) {
+        cudaEventDestroy(t.a);
+        cudaEventDestroy(t.b);
+    }
+    if (h->nccl) ncclCommDestroy(h->nccl);
+    if (h->ev_start) cudaEventDestroy(h->ev_start);
+    if (h->ev_halo) cudaEventDestroy(h->ev_halo);
+    if (h->comm) cudaStreamDestroy(h->comm);
+    delete h;
+    return DSLASH_OK;
+}
+
+extern "C" const char* dslash_error_string(dslash_t h) {
+    if (!h) return g_last_error.c_str();
+    return h->msg.c_str();
+}

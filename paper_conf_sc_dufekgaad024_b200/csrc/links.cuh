@@ -1,0 +1,86 @@
+// links.cuh -- one-time link preprocessing for dslash_load_links (not on the timed path).
+//
+// Canonical input: forward links [t][z][y][x][mu][3][3] complex over the local
+// volume.  Output: for target parity p the |l| = 4 link arrays of PAPER.md L51 indexed by the
+// target site (Fig. 1 caption L67: "each target site s* has |l| x |k| SU(3) matrices"):
+//   Ff(x,mu) = F(x,mu),  Fb(x,mu) = F(x-mu,mu)^dag,  Nf(x,mu) = N(x,mu),  Nb(x,mu) = N(x-3mu,mu)^dag
+// (reading Z2: back-links are adjoints of the neighbours' forward links).
+// In a halo direction the sites x-mu / x-3mu below the local volume come from `slab[mu]`, the
+// 3 coordinate slices just below the local origin received from the minus neighbour, stored
+// like the canonical array with that coordinate restricted to d = 0..2 (global coordinate
+// origin - 3 + d):  t: [d][z][y][x][mu][9],  z: [t][d][y][x][mu][9].
+#pragma once
+
+#include "common.cuh"
+#include "stencil.cuh"
+
+namespace hisq {
+
+struct LinkConvParams {
+    const double2* fat;           // canonical local [lex][4][9]
+    const double2* lng;
+    const double2* slab_fat[4];   // lower link slabs (halo directions only), see above
+    const double2* slab_lng[4];
+    double2* links;               // internal layout (SITE or DIR4)
+    int64_t vh;
+    int L[4];
+    int lxh;
+    int parity;
+    int halo_mask;
+    int layout;                   // 0 = SITE, 1 = DIR4
+};
+
+__device__ __forceinline__ const double2* canon_link(const LinkConvParams& P, bool is_long, int mu, int x, int y,
+                                                     int z, int t, int back) {
+    // the link of kind (fat/long) and direction mu at site (x,y,z,t) - back * mu^
+    int c[4] = {x, y, z, t};
+    int cn = c[mu] - back;
+    if (((P.halo_mask >> mu) & 1) && cn < 0) {
+        const int d = cn + 3;
+        int64_t off;
+        if (mu == 3)
+            off = x + (int64_t)P.L[0] * (y + (int64_t)P.L[1] * (z + (int64_t)P.L[2] * d));
+        else  // mu == 2
+            off = x + (int64_t)P.L[0] * (y + (int64_t)P.L[1] * (d + 3 * (int64_t)t));
+        return (is_long ? P.slab_lng[mu] : P.slab_fat[mu]) + (off * 4 + mu) * 9;
+    }
+    while (cn < 0) cn += P.L[mu];
+    c[mu] = cn;
+    const int64_t lex = c[0] + (int64_t)P.L[0] * (c[1] + (int64_t)P.L[1] * (c[2] + (int64_t)P.L[2] * c[3]));
+    return (is_long ? P.lng : P.fat) + (lex * 4 + mu) * 9;
+}
+
+// one thread per (target site, mu, l)
+__global__ void convert_links_kernel(const LinkConvParams P) {
+    const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (gid >= P.vh * 16) return;
+    const int64_t cb = gid >> 4;
+    const int mu = (int)(gid >> 2) & 3;
+    const int l = (int)gid & 3;
+    int64_t r = cb;
+    const int xh = (int)(r % P.lxh);
+    r /= P.lxh;
+    const int y = (int)(r % P.L[1]);
+    r /= P.L[1];
+    const int z = (int)(r % P.L[2]);
+    const int t = (int)(r / P.L[2]);
+    const int x = 2 * xh + ((P.parity + y + z + t) & 1);
+    const bool is_long = l >= 2;
+    const int back = (l == 1) ? 1 : (l == 3) ? 3 : 0;
+    const double2* A = canon_link(P, is_long, mu, x, y, z, t, back);
+    for (int i = 0; i < 3; ++i)
+        for (int j = 0; j < 3; ++j) {
+            double2 v;
+            if (back) {  // (A^dag)_{ij} = conj(A_{ji})
+                v = A[3 * j + i];
+                v.y = -v.y;
+            } else {
+                v = A[3 * i + j];
+            }
+            const int e = 3 * i + j;
+            const int64_t o = P.layout == 0 ? link_index_site(mu, l, e, P.vh, cb) : link_index_dir4(mu, l, e, P.vh, cb);
+            P.links[o] = v;
+        }
+}
+
+}  // namespace hisq

@@ -1,0 +1,236 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Tolerance (reading Z11): normwise  max|chi - chi_ref| / max|chi_ref|
+<= 1e-12 in fp64; summation order and FMA differ from the oracle, so bit equality with the
+oracle is not expected.  Bitwise equality IS required between the unpartitioned apply and
+the self-halo (interior + boundary) apply, and between repeated applies.
+"""
+import numpy as np
+import pytest
+
+import fieldgen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-12
+KERNELS = ["site", "dir4"]
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    torch.cuda.set_device(0)
+    return torch
+
+
+def _gpu_apply(torch, dims, fat, lng, src_cb, parity, **kw):
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    with Dslash(dims, **kw) as D:
+        D.load_links(fat, lng)
+        out = D(torch.from_numpy(src_cb).cuda(), parity)
+        torch.cuda.synchronize()
+        return out.cpu().numpy()
+
+
+# ragged: 6x8x10x12 has Vh = 2880 (not a multiple of the block); 4^4 aliases +3 with -1
+SMALL = [(4, 4, 4, 4), (8, 8, 8, 8), (8, 10, 12, 14), (6, 8, 10, 12), (2, 4, 6, 8), (16, 16, 16, 16)]
+
+
+@pytest.mark.parametrize("kernel", KERNELS)
+@pytest.mark.parametrize("dims", SMALL)
+@pytest.mark.parametrize("parity", [0, 1])
+def test_parity_vs_oracle(torch_cuda, kernel, dims, parity):
+    fat, lng = fieldgen.workload_links(dims)
+    psi = fieldgen.vector(dims, fieldgen.SEED_PSI)
+    ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, parity), parity)
+    got = _gpu_apply(torch_cuda, dims, fat, lng, fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 1 - parity), parity,
+                     kernel=kernel)
+    assert oracle.normwise_error(got, ref) <= TOL
+
+
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_parity_gaussian_links(torch_cuda, kernel):
+    """Non-unitary links: nothing in the kernel may assume SU(3) (reading Z14)."""
+    dims = (8, 10, 12, 14)
+    fat = fieldgen.links(dims, 101, "gauss")
+    lng = fieldgen.links(dims, 102, "gauss", scale=0.3)
+    psi = fieldgen.vector(dims, 103)
+    for parity in (0, 1):
+        ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, parity), parity)
+        got = _gpu_apply(torch_cuda, dims, fat, lng, fieldgen.vector_cb(dims, 103, 1 - parity), parity, kernel=kernel)
+        assert oracle.normwise_error(got, ref) <= TOL
+
+
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_point_source_exact(torch_cuda, kernel):
+    """P6 on the GPU: identity-scaled links and a point source give exact integers (bitwise)."""
+    dims = (8, 10, 12, 14)
+    lx, ly, lz, lt = dims
+    fat = np.zeros((lt, lz, ly, lx, 4, 3, 3), np.complex128)
+    lng = np.zeros_like(fat)
+    fat[...] = np.eye(3)
+    lng[...] = 2 * np.eye(3)
+    x0 = (3, 7, 5, 11)
+    psi = np.zeros((lt, lz, ly, lx, 3), np.complex128)
+    psi[x0[3], x0[2], x0[1], x0[0]] = [1 + 2j, -3, 4 - 5j]
+    parity = 1 - (sum(x0) & 1)
+    ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, parity), parity)
+    got = _gpu_apply(torch_cuda, dims, fat, lng, oracle.full_to_cb(psi, 1 - parity), parity, kernel=kernel)
+    assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("kernel", KERNELS)
+@pytest.mark.parametrize("dims,mask", [((8, 8, 8, 8), 0x8), ((8, 8, 8, 8), 0x4), ((8, 8, 8, 8), 0xC),
+                                       ((8, 10, 12, 14), 0xC), ((4, 4, 4, 4), 0xC), ((6, 8, 10, 12), 0x8)])
+@pytest.mark.parametrize("overlap", [True, False])
+def test_self_halo_bitwise(torch_cuda, kernel, dims, mask, overlap):
+    """The halo path with neighbour = self (ghost faces, interior/boundary split) must give the
+    unpartitioned result bit for bit (same per-site device function), and match the oracle."""
+    fat, lng = fieldgen.workload_links(dims)
+    psi = fieldgen.vector(dims, fieldgen.SEED_PSI)
+    for parity in (0, 1):
+        src = fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 1 - parity)
+        plain = _gpu_apply(torch_cuda, dims, fat, lng, src, parity, kernel=kernel)
+        halo = _gpu_apply(torch_cuda, dims, fat, lng, src, parity, kernel=kernel, force_halo=mask, overlap=overlap)
+        assert np.array_equal(plain, halo)
+        ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, parity), parity)
+        assert oracle.normwise_error(halo, ref) <= TOL
+
+
+def test_kernels_agree(torch_cuda):
+    dims = (16, 16, 16, 16)
+    fat, lng = fieldgen.workload_links(dims)
+    src = fieldgen.vector_cb(dims, 7, 1)
+    a = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel="site")
+    b = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel="dir4")
+    assert oracle.normwise_error(a, b) < 1e-14
+
+
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_full_size_32(torch_cuda, kernel):
+    """The benchmark size (32^4) in the bench's launch configuration, whole output vs the oracle."""
+    dims = (32, 32, 32, 32)
+    fat, lng = fieldgen.workload_links(dims)
+    psi = fieldgen.vector(dims, fieldgen.SEED_PSI)
+    parity = 0
+    ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, parity), parity)
+    got = _gpu_apply(torch_cuda, dims, fat, lng, fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 1), parity,
+                     kernel=kernel)
+    assert oracle.normwise_error(got, ref) <= TOL
+
+
+def test_sampled_48(torch_cuda):
+    """48^4 (strong-scaling global lattice) on one GPU: 4096 sampled sites vs the oracle, one by one."""
+    dims = (48, 48, 48, 48)
+    fat, lng = fieldgen.workload_links(dims)
+    psi = fieldgen.vector(dims, fieldgen.SEED_PSI)
+    parity = 1
+    got = _gpu_apply(torch_cuda, dims, fat, lng, fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 0), parity)
+    lex = oracle.lex_sites_of_parity(dims, parity)
+    rng = np.random.default_rng(48)
+    pick = np.sort(rng.choice(lex.size, 4096, replace=False))
+    pick = np.concatenate([[0, 1, lex.size - 1], pick])          # first/last sites (wrap in every dim)
+    ref = oracle.dslash_sites(fat, lng, psi, lex[pick])           # (n, 3)
+    assert oracle.normwise_error(got[:, pick].T, ref) <= TOL
+
+
+def test_antihermitian_gpu(torch_cuda):
+    """P3 through the library: <chi_e, D_eo psi_o> = -<D_oe chi_e, psi_o>."""
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    torch = torch_cuda
+    dims = (8, 10, 12, 14)
+    fat, lng = fieldgen.workload_links(dims)
+    with Dslash(dims) as D:
+        D.load_links(fat, lng)
+        psi_o = torch.from_numpy(fieldgen.vector_cb(dims, 5, 1)).cuda()
+        chi_e = torch.from_numpy(fieldgen.vector_cb(dims, 6, 0)).cuda()
+        d_psi = D(psi_o, 0)
+        d_chi = D(chi_e, 1)
+        lhs = torch.vdot(chi_e.reshape(-1), d_psi.reshape(-1)).item()
+        rhs = -torch.vdot(d_chi.reshape(-1), psi_o.reshape(-1)).item()
+        scale = (chi_e.norm() * d_psi.norm()).item()
+        assert abs(lhs - rhs) < 1e-13 * scale
+
+
+def test_apply_host_and_determinism(torch_cuda):
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    torch = torch_cuda
+    dims = (8, 8, 8, 16)
+    fat, lng = fieldgen.workload_links(dims)
+    with Dslash(dims) as D:
+        D.load_links(fat, lng)
+        src = torch.from_numpy(fieldgen.vector_cb(dims, 3, 1))
+        a = D(src.cuda(), 0)
+        b = D(src.cuda(), 0)
+        hout = torch.empty_like(src).pin_memory()
+        D.apply_host(hout, src.pin_memory(), 0)
+        torch.cuda.synchronize()
+        assert torch.equal(a, b)
+        assert torch.equal(a.cpu(), hout)
+
+
+def test_device_links_equal_host_links(torch_cuda):
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    torch = torch_cuda
+    dims = (8, 8, 8, 8)
+    fat, lng = fieldgen.workload_links(dims)
+    src = torch.from_numpy(fieldgen.vector_cb(dims, 3, 0)).cuda()
+    with Dslash(dims) as D:
+        D.load_links(fat, lng)
+        a = D(src, 1)
+        D.load_links(torch.from_numpy(fat).cuda(), torch.from_numpy(lng).cuda())
+        b = D(src, 1)
+        torch.cuda.synchronize()
+        assert torch.equal(a, b)
+
+
+def test_error_paths(torch_cuda):
+    from paper_conf_sc_dufekgaad024_b200 import Dslash, _abi
+    torch = torch_cuda
+    dims = (8, 8, 8, 8)
+    D = Dslash(dims, parity_mask=_abi.DSLASH_EVEN)
+    v = D.empty_vector()
+    w = D.empty_vector()
+    with pytest.raises(_abi.DslashError) as e:
+        D.apply(v, w, 0)
+    assert e.value.status == _abi.DSLASH_ERR_STATE
+    fat, lng = fieldgen.workload_links(dims)
+    D.load_links(fat, lng)
+    with pytest.raises(_abi.DslashError) as e:
+        _abi.dslash_apply(D.h, v.data_ptr(), v.data_ptr(), 0, 0)         # in == out
+    assert e.value.status == _abi.DSLASH_ERR_ARG
+    with pytest.raises(_abi.DslashError) as e:
+        D.apply(v, w, 1)                                                  # parity not prepared
+    assert e.value.status == _abi.DSLASH_ERR_ARG
+    with pytest.raises(_abi.DslashError) as e:
+        _abi.dslash_apply(D.h, v.data_ptr(), w.data_ptr(), 2, 0)         # bad parity
+    assert e.value.status == _abi.DSLASH_ERR_ARG
+    with pytest.raises(_abi.DslashError) as e:
+        _abi.dslash_apply(D.h, v.data_ptr() + 8, w.data_ptr(), 0, 0)     # misaligned
+    assert e.value.status == _abi.DSLASH_ERR_ARG
+    with pytest.raises(_abi.DslashError) as e:
+        _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_KERNEL, _abi.DSLASH_KERNEL_DIR4)  # after load_links
+    assert e.value.status == _abi.DSLASH_ERR_STATE
+    D.close()
+    with pytest.raises(_abi.DslashError) as e:
+        Dslash((8, 8, 8, 8), proc_grid=(1, 1, 1, 2))                       # nranks mismatch
+    assert e.value.status == _abi.DSLASH_ERR_ARG
+
+
+def test_kernel_timing_records(torch_cuda):
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    torch = torch_cuda
+    dims = (8, 8, 8, 16)
+    fat, lng = fieldgen.workload_links(dims)
+    with Dslash(dims, timing=True, force_halo=0x8) as D:
+        D.load_links(fat, lng)
+        src = torch.from_numpy(fieldgen.vector_cb(dims, 3, 1)).cuda()
+        out = D.empty_vector()
+        for _ in range(3):
+            D.apply(out, src, 0)
+        ms, n = D.kernel_timing()
+        assert n == 6 and ms > 0   # interior + boundary per apply
+        assert D.kernel_timing(0)[1] == 3 and D.kernel_timing(1)[1] == 3
+        D.kernel_timing_reset()
+        assert D.kernel_timing()[1] == 0
