@@ -15,7 +15,8 @@
  * Conventions (all functions):
  *   - dims are {Lx, Ly, Lz, Lt}, x fastest; lex(x,y,z,t) = x + Lx*(y + Ly*(z + Lz*t));
  *     parity p(x) = (x+y+z+t) mod 2 in GLOBAL coordinates.
- *   - Complex numbers are two interleaved doubles (re, im), 16 B.
+ *   - Complex numbers are two interleaved reals (re, im): 16 B (fp64), or 8 B for the
+ *     vectors of a DSLASH_F32 handle.
  *   - Vector layout (in, out): [3][Vh_local] complex, colour-major ("SoA"), where the
  *     checkerboard index cb = (local lex) / 2 enumerates the local sites of one parity
  *     in lexicographic order (Z8).  Vh_local = local volume / 2.
@@ -61,23 +62,31 @@ typedef enum {
 } dslash_status;
 
 enum { DSLASH_EVEN = 0, DSLASH_ODD = 1, DSLASH_BOTH = 2 }; /* parity_mask */
-enum { DSLASH_F64 = 0, DSLASH_F32 = 1 };                   /* precision */
+/* precision: F64 = fp64 links, vectors and arithmetic (the paper's, L278); F32 = fp32 links
+ * and vectors (complex64), fp32 accumulation; MIXED = fp32 links, fp64 vectors and fp64
+ * accumulation (links are widened before the FMAs).  load_links always takes fp64 input. */
+enum { DSLASH_F64 = 0, DSLASH_F32 = 1, DSLASH_MIXED = 2 };
 
 /* Kernel variants (DSLASH_OPT_KERNEL); DESIGN.md §Kernels. */
 enum {
     DSLASH_KERNEL_SITE = 0, /* one thread per target site, 16 link matrices streamed per thread   */
-    DSLASH_KERNEL_DIR4 = 1  /* four lanes per site (one per mu), 2-step shuffle reduction ("3LP") */
+    DSLASH_KERNEL_DIR4 = 1, /* four lanes per site (one per mu), 2-step shuffle reduction ("3LP") */
+    DSLASH_KERNEL_DIR2 = 2  /* two lanes per site (two directions each), 1-step shuffle reduction  */
 };
 
 /* Options (dslash_set_option). */
 enum {
-    DSLASH_OPT_KERNEL = 0,      /* kernel variant; before load_links (it fixes the link layout)        */
-    DSLASH_OPT_BLOCK = 1,       /* threads per block, 0 = variant default; any time                    */
+    DSLASH_OPT_KERNEL = 0,      /* kernel variant (default DSLASH_KERNEL_DIR2); before load_links, as
+                                   it fixes the link layout                                            */
+    DSLASH_OPT_BLOCK = 1,       /* threads per block (multiple of 32, <= 256), 0 = default; any time   */
     DSLASH_OPT_FORCE_HALO = 2,  /* bitmask of directions (bit mu) exchanged through the halo path even
                                    when Pmu == 1 (self-halo: neighbour = self); before load_links      */
     DSLASH_OPT_OVERLAP = 3,     /* 1 (default): interior kernel overlaps the halo exchange; 0: one
                                    kernel over all sites after the exchange                            */
-    DSLASH_OPT_TIMING = 4       /* 1: record CUDA events around every kernel (dslash_kernel_timing)   */
+    DSLASH_OPT_TIMING = 4,      /* 1: record CUDA events around every kernel (dslash_kernel_timing)   */
+    DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
+                                   resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
+                                   4 (<= 64); 0 = default; any time                                    */
 };
 
 /* Kernel classes for dslash_kernel_timing. */
@@ -117,8 +126,8 @@ DSLASH_API dslash_status dslash_plan(const int32_t global_dims[4], const int32_t
                           int32_t nranks, int32_t force_halo_mask, dslash_plan_t* plan);
 
 /* Create a handle on the current CUDA device.  parity_mask selects for which target
- * parities links are prepared (DSLASH_BOTH doubles link memory).  precision must be
- * DSLASH_F64 (DSLASH_F32 returns DSLASH_ERR_UNSUPPORTED in this version).
+ * parities links are prepared (DSLASH_BOTH doubles link memory).  precision: DSLASH_F64,
+ * DSLASH_F32 or DSLASH_MIXED (it fixes the stored link type and the vector type).
  * nccl_unique_id: the 128-byte ncclUniqueId from dslash_get_unique_id() on rank 0,
  * broadcast to all ranks by the caller; NULL when nranks == 1.  On success *out owns
  * a CUDA communication stream, events, ghost buffers and (nranks > 1) an NCCL
@@ -158,6 +167,16 @@ DSLASH_API dslash_status dslash_apply(dslash_t h, void* out, const void* in, int
  * Pinned host memory gives asynchronous copies. */
 DSLASH_API dslash_status dslash_apply_host(dslash_t h, void* out_host, const void* in_host, int32_t parity,
                                 dslash_stream_t stream);
+
+/* n applies from HOST buffers, pipelined: apply i reads in_host[i] and writes out_host[i]
+ * (all [3][Vh_local] complex, pinned for overlap; inputs must not alias outputs).  The
+ * host->device copy of apply i+1 and the device->host copy of apply i-1 run on internal
+ * copy streams while apply i computes on `stream`, through 3 rotating device slots.  The
+ * first copy waits for the work already queued on `stream`; `stream` waits for the last
+ * copy, so synchronising `stream` makes every out_host[i] valid. */
+DSLASH_API dslash_status dslash_apply_host_batch(dslash_t h, int32_t n, void* const* out_host,
+                                                 const void* const* in_host, int32_t parity,
+                                                 dslash_stream_t stream);
 
 /* Halo exchange only: start sending the depth-3 faces of `in` (source parity
  * src_parity) after the work already queued on `stream`; dslash_halo_wait makes

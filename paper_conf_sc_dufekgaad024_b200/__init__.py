@@ -17,7 +17,9 @@ from ._abi import (DSLASH_BOTH, DSLASH_EVEN, DSLASH_F64, DSLASH_KERNEL_DIR4, DSL
 
 FLOP_PER_SITE = 1146          # 600.8 MFLOP per 32^4 apply = 1146 per target site
 LINK_BYTES_PER_SITE = 2304    # 16 matrices x 9 complex x 16 B (fp64), streamed once
-ALGO_BYTES_PER_SITE = 2400    # + 48 B source (ideal reuse) + 48 B output (DESIGN.md §Roofline)
+ALGO_BYTES_PER_SITE = 2400    # + 48 B source (ideal reuse) + 48 B output (DESIGN.md §6)
+# algorithmic bytes per target site by precision: links + source + output
+ALGO_BYTES = {"f64": 2304 + 48 + 48, "f32": 1152 + 24 + 24, "mixed": 1152 + 48 + 48}
 
 __all__ = ["Dslash", "DslashError", "dslash_plan", "FLOP_PER_SITE", "ALGO_BYTES_PER_SITE"]
 
@@ -32,16 +34,21 @@ def _stream_handle(stream):
 class Dslash:
     """One handle of the library on the current CUDA device.
 
-    Vectors are torch complex128 CUDA tensors of shape (3, Vh_local) (colour-major,
+    precision: "f64" (default), "f32" (complex64 vectors and fp32 links) or "mixed"
+    (fp32 links, complex128 vectors, fp64 accumulation).
+    Vectors are torch complex128 (complex64 for "f32") CUDA tensors of shape (3, Vh_local) (colour-major,
     checkerboard site order cb = local lex // 2); links are canonical forward links
     (Lt, Lz, Ly, Lx, 4, 3, 3) complex128 over the local volume, numpy (host) or torch
     (device).  With ``world_size > 1`` the NCCL unique id is broadcast through the
     default torch.distributed process group.
     """
 
-    def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="site", block=0,
-                 force_halo=0, overlap=True, timing=False, rank=0, world_size=1):
+    def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="dir2", block=0,
+                 force_halo=0, overlap=True, timing=False, rank=0, world_size=1, min_blocks=0, precision="f64"):
+        import torch
         self.global_dims = tuple(int(d) for d in global_dims)
+        self.precision = precision
+        self.dtype = torch.complex64 if precision == "f32" else torch.complex128
         self.proc_grid = tuple(int(p) for p in proc_grid)
         uid = None
         if world_size > 1:
@@ -52,11 +59,14 @@ class Dslash:
                 t.copy_(torch.frombuffer(bytearray(_abi.dslash_get_unique_id()), dtype=torch.uint8))
             dist.broadcast(t, 0)
             uid = bytes(t.cpu().numpy().tobytes())
-        self.h = _abi.dslash_create(self.global_dims, self.proc_grid, parity_mask, DSLASH_F64, uid, world_size, rank)
+        self.h = _abi.dslash_create(self.global_dims, self.proc_grid, parity_mask, _abi.PRECISIONS[precision], uid,
+                                    world_size, rank)
         try:
             _abi.dslash_set_option(self.h, DSLASH_OPT_KERNEL, KERNELS[kernel] if isinstance(kernel, str) else kernel)
             if block:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_BLOCK, block)
+            if min_blocks:
+                _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_MIN_BLOCKS, min_blocks)
             if force_halo:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_FORCE_HALO, force_halo)
             _abi.dslash_set_option(self.h, DSLASH_OPT_OVERLAP, int(bool(overlap)))
@@ -94,12 +104,12 @@ class Dslash:
     # -- vectors
     def empty_vector(self):
         import torch
-        return torch.empty((3, self.vh), dtype=torch.complex128, device="cuda")
+        return torch.empty((3, self.vh), dtype=self.dtype, device="cuda")
 
-    def _check_vec(self, v):
-        import torch
-        if not (v.is_cuda and v.dtype == torch.complex128 and v.is_contiguous() and tuple(v.shape) == (3, self.vh)):
-            raise ValueError(f"vector must be a contiguous complex128 CUDA tensor of shape (3, {self.vh})")
+    def _check_vec(self, v, cuda=True):
+        if not (v.is_cuda == cuda and v.dtype == self.dtype and v.is_contiguous() and tuple(v.shape) == (3, self.vh)):
+            where = "CUDA" if cuda else "CPU"
+            raise ValueError(f"vector must be a contiguous {self.dtype} {where} tensor of shape (3, {self.vh})")
 
     def apply(self, out, inp, parity, stream=None):
         """out = D inp on target parity `parity` (stream-ordered, asynchronous)."""
@@ -113,12 +123,18 @@ class Dslash:
 
     def apply_host(self, out, inp, parity, stream=None):
         """Host-buffer path (end-to-end): torch CPU complex128 tensors (pin them for async copies)."""
-        import torch
         for v in (out, inp):
-            if v.is_cuda or v.dtype != torch.complex128 or not v.is_contiguous() or tuple(v.shape) != (3, self.vh):
-                raise ValueError(f"host vectors must be contiguous complex128 CPU tensors of shape (3, {self.vh})")
+            self._check_vec(v, cuda=False)
         _abi.dslash_apply_host(self.h, out.data_ptr(), inp.data_ptr(), int(parity), _stream_handle(stream))
         return out
+
+    def apply_host_batch(self, outs, inps, parity, stream=None):
+        """Pipelined host-buffer applies: outs[i] = D inps[i] (torch CPU complex128, pinned)."""
+        for v in list(outs) + list(inps):
+            self._check_vec(v, cuda=False)
+        _abi.dslash_apply_host_batch(self.h, [o.data_ptr() for o in outs], [v.data_ptr() for v in inps],
+                                     int(parity), _stream_handle(stream))
+        return outs
 
     def kernel_timing(self, which=DSLASH_TIMING_ALL):
         """(total ms, launches) of the kernels of class `which` recorded since the last reset."""

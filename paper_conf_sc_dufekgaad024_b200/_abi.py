@@ -18,11 +18,13 @@ DSLASH_OK, DSLASH_ERR_ARG, DSLASH_ERR_STATE, DSLASH_ERR_CUDA, DSLASH_ERR_NCCL, D
 STATUS_NAMES = {0: "DSLASH_OK", 1: "DSLASH_ERR_ARG", 2: "DSLASH_ERR_STATE", 3: "DSLASH_ERR_CUDA",
                 4: "DSLASH_ERR_NCCL", 5: "DSLASH_ERR_OOM", 6: "DSLASH_ERR_UNSUPPORTED"}
 DSLASH_EVEN, DSLASH_ODD, DSLASH_BOTH = 0, 1, 2
-DSLASH_F64, DSLASH_F32 = 0, 1
-DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4 = 0, 1
-DSLASH_OPT_KERNEL, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_OVERLAP, DSLASH_OPT_TIMING = range(5)
+DSLASH_F64, DSLASH_F32, DSLASH_MIXED = 0, 1, 2
+PRECISIONS = {"f64": DSLASH_F64, "f32": DSLASH_F32, "mixed": DSLASH_MIXED}
+DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_DIR2 = 0, 1, 2
+DSLASH_OPT_KERNEL, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_OVERLAP, DSLASH_OPT_TIMING, \
+    DSLASH_OPT_MIN_BLOCKS = range(6)
 DSLASH_TIMING_INTERIOR, DSLASH_TIMING_BOUNDARY, DSLASH_TIMING_ALL = range(3)
-KERNELS = {"site": DSLASH_KERNEL_SITE, "dir4": DSLASH_KERNEL_DIR4}
+KERNELS = {"site": DSLASH_KERNEL_SITE, "dir4": DSLASH_KERNEL_DIR4, "dir2": DSLASH_KERNEL_DIR2}
 
 
 class dslash_box_t(ctypes.Structure):
@@ -77,6 +79,8 @@ _SIGS = {
     "dslash_load_links": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply_host": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
+    "dslash_apply_host_batch": ([_h, ctypes.c_int32, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.c_int32,
+                                 _vp], ctypes.c_int),
     "dslash_halo_start": ([_h, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_halo_wait": ([_h, _vp], ctypes.c_int),
     "dslash_sync": ([_h], ctypes.c_int),
@@ -148,6 +152,15 @@ def dslash_apply(h, out_ptr, in_ptr, parity, stream=0):
 
 def dslash_apply_host(h, out_ptr, in_ptr, parity, stream=0):
     return check(lib.dslash_apply_host(h, out_ptr, in_ptr, parity, stream), h)
+
+
+def dslash_apply_host_batch(h, out_ptrs, in_ptrs, parity, stream=0):
+    n = len(out_ptrs)
+    if len(in_ptrs) != n:
+        raise ValueError("out_ptrs and in_ptrs differ in length")
+    outs = (ctypes.c_void_p * max(n, 1))(*out_ptrs)
+    ins = (ctypes.c_void_p * max(n, 1))(*in_ptrs)
+    return check(lib.dslash_apply_host_batch(h, n, outs, ins, parity, stream), h)
 
 
 def dslash_halo_start(h, in_ptr, src_parity, stream=0):

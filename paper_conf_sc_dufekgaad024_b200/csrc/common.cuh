@@ -53,6 +53,39 @@ __device__ __forceinline__ void st_stream(double2* p, double2 v) {
     asm volatile("st.global.cs.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
 }
 
+__device__ __forceinline__ float2 ld_stream(const float2* p, uint64_t pol) {
+    float2 r;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f32 {%0, %1}, [%2], %3;"
+        : "=f"(r.x), "=f"(r.y)
+        : "l"(p), "l"(pol));
+    return r;
+}
+
+__device__ __forceinline__ float2 ld_reuse(const float2* p, uint64_t pol) {
+    float2 r;
+    asm("ld.global.nc.L2::cache_hint.v2.f32 {%0, %1}, [%2], %3;" : "=f"(r.x), "=f"(r.y) : "l"(p), "l"(pol));
+    return r;
+}
+
+__device__ __forceinline__ void st_stream(float2* p, float2 v) {
+    asm volatile("st.global.cs.v2.f32 [%0], {%1, %2};" ::"l"(p), "f"(v.x), "f"(v.y) : "memory");
+}
+
+// ---------------------------------------------------------------- precision
+// complex type of a real type: cplx_t<double> = double2, cplx_t<float> = float2
+template <typename R> struct CplxOf;
+template <> struct CplxOf<double> { using type = double2; };
+template <> struct CplxOf<float> { using type = float2; };
+template <typename R> using cplx_t = typename CplxOf<R>::type;
+
+template <typename T> __device__ __forceinline__ T to_cplx(double2 v);
+template <> __device__ __forceinline__ double2 to_cplx<double2>(double2 v) { return v; }
+template <> __device__ __forceinline__ float2 to_cplx<float2>(double2 v) {
+    return make_float2((float)v.x, (float)v.y);
+}
+__device__ __forceinline__ double2 widen(double2 v) { return v; }
+__device__ __forceinline__ double2 widen(float2 v) { return make_double2(v.x, v.y); }
+
 // ---------------------------------------------------------------- complex fp64 arithmetic
 // acc += a * b
 __device__ __forceinline__ void cmadd(double2& acc, double2 a, double2 b) {
@@ -68,6 +101,18 @@ __device__ __forceinline__ void cmsub(double2& acc, double2 a, double2 b) {
     acc.y = fma(-a.x, b.y, acc.y);
     acc.y = fma(-a.y, b.x, acc.y);
 }
+__device__ __forceinline__ void cmadd(float2& acc, float2 a, float2 b) {
+    acc.x = fmaf(a.x, b.x, acc.x);
+    acc.x = fmaf(-a.y, b.y, acc.x);
+    acc.y = fmaf(a.x, b.y, acc.y);
+    acc.y = fmaf(a.y, b.x, acc.y);
+}
+__device__ __forceinline__ void cmsub(float2& acc, float2 a, float2 b) {
+    acc.x = fmaf(-a.x, b.x, acc.x);
+    acc.x = fmaf(a.y, b.y, acc.x);
+    acc.y = fmaf(-a.x, b.y, acc.y);
+    acc.y = fmaf(-a.y, b.x, acc.y);
+}
 
 // ---------------------------------------------------------------- kernel parameters
 constexpr int kMaxBoxes = 4;
@@ -77,11 +122,13 @@ struct Box {
     int n[4];  // extent per dim; n[0] counts full x extent (sites per row = n[0] / 2)
 };
 
+// Pointers are untyped: the kernel instantiation fixes the link type (double2 or float2) and
+// the vector type (double2 or float2).
 struct StencilParams {
-    const double2* links;      // internal link layout for the target parity (variant-specific)
-    const double2* in;         // [3][vh] source parity, local
-    double2* out;              // [3][vh] target parity, local
-    const double2* ghost[4][2];  // [mu][side] -> [3][face_vh[mu]] (only where halo[mu])
+    const void* links;         // internal link layout for the target parity (variant-specific)
+    const void* in;            // [3][vh] source parity, local
+    void* out;                 // [3][vh] target parity, local
+    const void* ghost[4][2];   // [mu][side] -> [3][face_vh[mu]] (only where halo[mu])
     int64_t vh;
     int64_t face_vh[4];
     int L[4];                  // local extents

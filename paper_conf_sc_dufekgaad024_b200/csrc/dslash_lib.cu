@@ -26,13 +26,20 @@ struct dslash_s {
     dslash_plan_t plan{};
     int32_t global_dims[4]{}, proc_grid[4]{};
     int parity_mask = 0, precision = 0, device = 0;
-    int kernel = DSLASH_KERNEL_SITE, block = 0, force_halo = 0, overlap = 1, timing = 0;
+    int kernel = DSLASH_KERNEL_DIR2, block = 0, force_halo = 0, overlap = 1, timing = 0, min_blocks = 0;
     bool loaded = false;
-    double2* links[2] = {nullptr, nullptr};
-    double2* ghost[4][2] = {};     // source-vector ghost faces [3][face_vh]
-    double2* zsend[2] = {};        // packed z faces to send (NCCL path)
-    double2* stage_in = nullptr;   // apply_host staging
-    double2* stage_out = nullptr;
+    void* links[2] = {nullptr, nullptr};
+    char* ghost[4][2] = {};        // source-vector ghost faces [nrhs][3][face_vh]
+    char* zsend[2] = {};           // packed z faces to send (NCCL path)
+    int ghost_rhs = 0;             // number of right-hand sides the ghost buffers hold
+    void* stage_in = nullptr;      // apply_host staging
+    void* stage_out = nullptr;
+    static constexpr int kSlots = 3;  // apply_host_batch pipeline depth
+    void* slot_in[kSlots] = {};
+    void* slot_out[kSlots] = {};
+    cudaStream_t h2d = nullptr, d2h = nullptr;
+    cudaEvent_t ev_in_ready[kSlots] = {}, ev_in_free[kSlots] = {}, ev_out_ready[kSlots] = {},
+                ev_out_free[kSlots] = {}, ev_batch = nullptr;
     cudaStream_t comm = nullptr;
     cudaEvent_t ev_start = nullptr, ev_halo = nullptr;
     bool halo_pending = false;
@@ -209,15 +216,17 @@ static void free_halo(dslash_t h) {
         }
 }
 
-static dslash_status alloc_halo(dslash_t h) {
+static dslash_status alloc_halo(dslash_t h, int nrhs) {
     free_halo(h);
     const dslash_plan_t& p = h->plan;
+    const size_t es = h->precision == DSLASH_F32 ? 8 : 16;
     for (int d = 2; d < 4; ++d) {
         if (!p.halo[d]) continue;
-        for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->ghost[d][s], 3 * p.face_vh[d] * sizeof(double2)));
+        for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->ghost[d][s], (size_t)nrhs * 3 * p.face_vh[d] * es));
     }
     if (p.halo[2] && p.nbr_rank[2][0] != p.rank)
-        for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->zsend[s], 3 * p.face_vh[2] * sizeof(double2)));
+        for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->zsend[s], (size_t)nrhs * 3 * p.face_vh[2] * es));
+    h->ghost_rhs = nrhs;
     return DSLASH_OK;
 }
 
@@ -227,8 +236,8 @@ extern "C" dslash_status dslash_create(const int32_t G[4], const int32_t P[4], i
     *out = nullptr;
     if (parity_mask < DSLASH_EVEN || parity_mask > DSLASH_BOTH)
         return fail(nullptr, DSLASH_ERR_ARG, "parity_mask %d not in {0,1,2}", parity_mask);
-    if (precision == DSLASH_F32) return fail(nullptr, DSLASH_ERR_UNSUPPORTED, "fp32 path not built in this version");
-    if (precision != DSLASH_F64) return fail(nullptr, DSLASH_ERR_ARG, "precision %d unknown", precision);
+    if (precision != DSLASH_F64 && precision != DSLASH_F32 && precision != DSLASH_MIXED)
+        return fail(nullptr, DSLASH_ERR_ARG, "precision %d unknown", precision);
     if (nranks > 1 && !nccl_unique_id) return fail(nullptr, DSLASH_ERR_ARG, "nranks > 1 needs an NCCL unique id");
     dslash_plan_t plan;
     dslash_status st = dslash_plan(G, P, rank, nranks, 0, &plan);
@@ -265,7 +274,7 @@ extern "C" dslash_status dslash_create(const int32_t G[4], const int32_t P[4], i
             return bail(DSLASH_ERR_NCCL);
         }
     }
-    if ((st = alloc_halo(h)) != DSLASH_OK) return bail(st);
+    if ((st = alloc_halo(h, 1)) != DSLASH_OK) return bail(st);
     *out = h;
     return DSLASH_OK;
 }
@@ -274,15 +283,15 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     switch (key) {
         case DSLASH_OPT_KERNEL:
-            if (value != DSLASH_KERNEL_SITE && value != DSLASH_KERNEL_DIR4)
+            if (value != DSLASH_KERNEL_SITE && value != DSLASH_KERNEL_DIR4 && value != DSLASH_KERNEL_DIR2)
                 return fail(h, DSLASH_ERR_ARG, "unknown kernel variant %lld", (long long)value);
             if (h->loaded && value != h->kernel)
                 return fail(h, DSLASH_ERR_STATE, "kernel variant fixes the link layout: set it before load_links");
             h->kernel = (int)value;
             return DSLASH_OK;
         case DSLASH_OPT_BLOCK:
-            if (value != 0 && (value < 32 || value > 1024 || (value & 31)))
-                return fail(h, DSLASH_ERR_ARG, "block size %lld must be 0 or a multiple of 32 in [32,1024]",
+            if (value != 0 && (value < 32 || value > 256 || (value & 31)))
+                return fail(h, DSLASH_ERR_ARG, "block size %lld must be 0 or a multiple of 32 in [32,256]",
                             (long long)value);
             h->block = (int)value;
             return DSLASH_OK;
@@ -293,7 +302,7 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             if (st != DSLASH_OK) return fail(h, st, "%s", g_last_error.c_str());
             h->plan = p;
             h->force_halo = (int)value;
-            return alloc_halo(h);
+            return alloc_halo(h, 1);
         }
         case DSLASH_OPT_OVERLAP:
             h->overlap = value != 0;
@@ -301,9 +310,22 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
         case DSLASH_OPT_TIMING:
             h->timing = value != 0;
             return DSLASH_OK;
+        case DSLASH_OPT_MIN_BLOCKS:
+            if (value != 0 && (value < 2 || value > 4))
+                return fail(h, DSLASH_ERR_ARG, "min_blocks %lld must be 0, 2, 3 or 4", (long long)value);
+            h->min_blocks = (int)value;
+            return DSLASH_OK;
         default:
             return fail(h, DSLASH_ERR_ARG, "unknown option %d", key);
     }
+}
+
+// bytes of one complex element of the vectors / of the stored links
+static size_t vec_elem(const dslash_s* h) { return h->precision == DSLASH_F32 ? 8 : 16; }
+static size_t link_elem(const dslash_s* h) { return h->precision == DSLASH_F64 ? 16 : 8; }
+
+static int lanes_of(int kernel) {
+    return kernel == DSLASH_KERNEL_DIR4 ? 4 : kernel == DSLASH_KERNEL_DIR2 ? 2 : 1;
 }
 
 // ============================================================================ link loading
@@ -349,7 +371,7 @@ extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
     for (int d = 0; d < 4; ++d) C.L[d] = p.local_dims[d];
     C.lxh = p.local_dims[0] / 2;
     C.vh = p.vh_local;
-    C.layout = h->kernel == DSLASH_KERNEL_DIR4 ? 1 : 0;
+    C.lanes = lanes_of(h->kernel);
     int halo_mask = 0;
     for (int d = 2; d < 4; ++d)
         if (p.halo[d]) halo_mask |= 1 << d;
@@ -416,7 +438,7 @@ extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
         C.slab_fat[d] = slab[d][0];
         C.slab_lng[d] = slab[d][1];
     }
-    const size_t link_bytes = (size_t)p.vh_local * 144 * sizeof(double2);
+    const size_t link_bytes = (size_t)p.vh_local * 144 * link_elem(h);
     for (int par = 0; par < 2; ++par) {
         const bool want = h->parity_mask == DSLASH_BOTH || h->parity_mask == par;
         if (!want) continue;
@@ -425,7 +447,10 @@ extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
         C.parity = par;  // origin sum is even, so local and global parity agree
         const int64_t n = p.vh_local * 16;
         const int bs = 256;
-        convert_links_kernel<<<(unsigned)((n + bs - 1) / bs), bs, 0, s>>>(C);
+        if (h->precision == DSLASH_F64)
+            convert_links_kernel<double><<<(unsigned)((n + bs - 1) / bs), bs, 0, s>>>(C);
+        else
+            convert_links_kernel<float><<<(unsigned)((n + bs - 1) / bs), bs, 0, s>>>(C);
         CUL(cudaGetLastError());
     }
     CUL(cudaStreamSynchronize(s));
@@ -438,44 +463,47 @@ extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
 // ============================================================================ halo exchange
 static bool any_halo(const dslash_plan_t& p) { return p.halo[2] || p.halo[3]; }
 
-extern "C" dslash_status dslash_halo_start(dslash_t h, const void* in, int32_t src_parity, dslash_stream_t stream) {
-    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
-    if (!in || ((uintptr_t)in & 15)) return fail(h, DSLASH_ERR_ARG, "in is NULL or not 16-byte aligned");
-    if (src_parity & ~1) return fail(h, DSLASH_ERR_ARG, "src_parity %d not in {0,1}", src_parity);
+// Exchange the depth-3 faces of nrhs source vectors stored back to back ([nrhs][3][vh]).
+static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaStream_t s) {
     const dslash_plan_t& p = h->plan;
     if (!any_halo(p)) return DSLASH_OK;
-    cudaStream_t s = (cudaStream_t)stream;
-    const double2* src = (const double2*)in;
-    const int64_t vh = p.vh_local;
-    const int L0 = p.local_dims[0], L1 = p.local_dims[1], L2 = p.local_dims[2], L3 = p.local_dims[3];
-    const int lxh = L0 / 2;
+    if (nrhs > h->ghost_rhs) {
+        CU(h, cudaStreamSynchronize(h->comm));  // old ghosts may still be read by queued kernels
+        CU(h, cudaDeviceSynchronize());
+        dslash_status st = alloc_halo(h, nrhs);
+        if (st != DSLASH_OK) return st;
+    }
+    const size_t es = vec_elem(h);
+    const char* src = static_cast<const char*>(in);
+    const size_t vh = (size_t)p.vh_local;
+    const size_t L1 = p.local_dims[1], L2 = p.local_dims[2], L3 = p.local_dims[3];
+    const size_t lxh = p.local_dims[0] / 2;
+    const size_t rows = (size_t)3 * nrhs;  // (rhs, colour) rows of length vh
     CU(h, cudaEventRecord(h->ev_start, s));
     CU(h, cudaStreamWaitEvent(h->comm, h->ev_start, 0));
     bool nccl_work = false;
-    // --- local copies (neighbour == self) and z packing
+    const size_t tslab = 3 * lxh * L1 * L2;  // sites in 3 t-slices of one parity
     if (p.halo[3]) {
-        const size_t slab = (size_t)3 * lxh * L1 * L2;  // sites in 3 t-slices of one parity
         if (p.nbr_rank[3][0] == p.rank) {
             // minus ghost <- my top slices, plus ghost <- my bottom slices (periodic self-halo)
-            CU(h, cudaMemcpy2DAsync(h->ghost[3][0], slab * sizeof(double2), src + (size_t)(L3 - 3) * lxh * L1 * L2,
-                                    vh * sizeof(double2), slab * sizeof(double2), 3, cudaMemcpyDeviceToDevice, h->comm));
-            CU(h, cudaMemcpy2DAsync(h->ghost[3][1], slab * sizeof(double2), src, vh * sizeof(double2),
-                                    slab * sizeof(double2), 3, cudaMemcpyDeviceToDevice, h->comm));
+            CU(h, cudaMemcpy2DAsync(h->ghost[3][0], tslab * es, src + (vh - tslab) * es, vh * es, tslab * es, rows,
+                                    cudaMemcpyDeviceToDevice, h->comm));
+            CU(h, cudaMemcpy2DAsync(h->ghost[3][1], tslab * es, src, vh * es, tslab * es, rows,
+                                    cudaMemcpyDeviceToDevice, h->comm));
         } else {
             nccl_work = true;
         }
     }
     if (p.halo[2]) {
-        // [c][t][z0..z0+2][y][xh] -> [c][t][d][y][xh]: rows of 3 z-slices, one row per (c, t)
-        const size_t row = (size_t)lxh * L1;  // sites of one z-slice of one t
+        // [r][c][t][z0..z0+2][y][xh] -> [r][c][t][d][y][xh]: one row of 3 z-slices per (r, c, t)
+        const size_t zrow = lxh * L1;  // sites of one z-slice of one t
         const bool self = p.nbr_rank[2][0] == p.rank;
-        double2* to_minus = self ? h->ghost[2][1] : h->zsend[0];  // my bottom slices
-        double2* to_plus = self ? h->ghost[2][0] : h->zsend[1];   // my top slices
-        CU(h, cudaMemcpy2DAsync(to_minus, 3 * row * sizeof(double2), src, (size_t)L2 * row * sizeof(double2),
-                                3 * row * sizeof(double2), (size_t)3 * L3, cudaMemcpyDeviceToDevice, h->comm));
-        CU(h, cudaMemcpy2DAsync(to_plus, 3 * row * sizeof(double2), src + (size_t)(L2 - 3) * row,
-                                (size_t)L2 * row * sizeof(double2), 3 * row * sizeof(double2), (size_t)3 * L3,
+        char* to_minus = self ? h->ghost[2][1] : h->zsend[0];  // my bottom slices
+        char* to_plus = self ? h->ghost[2][0] : h->zsend[1];   // my top slices
+        CU(h, cudaMemcpy2DAsync(to_minus, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
                                 cudaMemcpyDeviceToDevice, h->comm));
+        CU(h, cudaMemcpy2DAsync(to_plus, 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es, 3 * zrow * es,
+                                rows * L3, cudaMemcpyDeviceToDevice, h->comm));
         if (!self) nccl_work = true;
     }
     if (nccl_work) {
@@ -483,34 +511,39 @@ extern "C" dslash_status dslash_halo_start(dslash_t h, const void* in, int32_t s
         // Per direction: sends (bottom -> minus, top -> plus) then receives (plus ghost <- plus,
         // minus ghost <- minus).  With P = 2 both neighbours are one rank and NCCL matches a pair's
         // messages in issue order: my first message (bottom) is the peer's first receive (its plus
-        // ghost, since I am its plus neighbour).
+        // ghost, since I am its plus neighbour).  Counts are bytes (ncclUint8).
         NC(h, ncclGroupStart());
         if (p.halo[3] && p.nbr_rank[3][0] != p.rank) {
-            const size_t slab = (size_t)3 * lxh * L1 * L2;
-            const size_t n = slab * 2;
-            for (int c = 0; c < 3; ++c)
-                NC(h, ncclSend(src + c * vh, n, ncclDouble, p.nbr_rank[3][0], h->nccl, h->comm));
-            for (int c = 0; c < 3; ++c)
-                NC(h, ncclSend(src + c * vh + (size_t)(L3 - 3) * lxh * L1 * L2, n, ncclDouble, p.nbr_rank[3][1], h->nccl,
-                               h->comm));
-            for (int c = 0; c < 3; ++c)
-                NC(h, ncclRecv(h->ghost[3][1] + c * slab, n, ncclDouble, p.nbr_rank[3][1], h->nccl, h->comm));
-            for (int c = 0; c < 3; ++c)
-                NC(h, ncclRecv(h->ghost[3][0] + c * slab, n, ncclDouble, p.nbr_rank[3][0], h->nccl, h->comm));
+            const size_t n = tslab * es;
+            for (size_t r = 0; r < rows; ++r)  // t-faces are contiguous in every (rhs, colour) row: zero copy
+                NC(h, ncclSend(src + r * vh * es, n, ncclUint8, p.nbr_rank[3][0], h->nccl, h->comm));
+            for (size_t r = 0; r < rows; ++r)
+                NC(h, ncclSend(src + (r * vh + vh - tslab) * es, n, ncclUint8, p.nbr_rank[3][1], h->nccl, h->comm));
+            for (size_t r = 0; r < rows; ++r)
+                NC(h, ncclRecv(h->ghost[3][1] + r * n, n, ncclUint8, p.nbr_rank[3][1], h->nccl, h->comm));
+            for (size_t r = 0; r < rows; ++r)
+                NC(h, ncclRecv(h->ghost[3][0] + r * n, n, ncclUint8, p.nbr_rank[3][0], h->nccl, h->comm));
         }
         if (p.halo[2] && p.nbr_rank[2][0] != p.rank) {
-            const size_t n = (size_t)3 * p.face_vh[2] * 2;
-            NC(h, ncclSend(h->zsend[0], n, ncclDouble, p.nbr_rank[2][0], h->nccl, h->comm));
-            NC(h, ncclSend(h->zsend[1], n, ncclDouble, p.nbr_rank[2][1], h->nccl, h->comm));
-            NC(h, ncclRecv(h->ghost[2][1], n, ncclDouble, p.nbr_rank[2][1], h->nccl, h->comm));
-            NC(h, ncclRecv(h->ghost[2][0], n, ncclDouble, p.nbr_rank[2][0], h->nccl, h->comm));
+            const size_t n = rows * p.face_vh[2] * es;
+            NC(h, ncclSend(h->zsend[0], n, ncclUint8, p.nbr_rank[2][0], h->nccl, h->comm));
+            NC(h, ncclSend(h->zsend[1], n, ncclUint8, p.nbr_rank[2][1], h->nccl, h->comm));
+            NC(h, ncclRecv(h->ghost[2][1], n, ncclUint8, p.nbr_rank[2][1], h->nccl, h->comm));
+            NC(h, ncclRecv(h->ghost[2][0], n, ncclUint8, p.nbr_rank[2][0], h->nccl, h->comm));
         }
         NC(h, ncclGroupEnd());
     }
-    (void)src_parity;  // faces are copied in the caller's cb order; parity only names the field
     CU(h, cudaEventRecord(h->ev_halo, h->comm));
     h->halo_pending = true;
     return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_halo_start(dslash_t h, const void* in, int32_t src_parity, dslash_stream_t stream) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (!in || ((uintptr_t)in & 15)) return fail(h, DSLASH_ERR_ARG, "in is NULL or not 16-byte aligned");
+    if (src_parity & ~1) return fail(h, DSLASH_ERR_ARG, "src_parity %d not in {0,1}", src_parity);
+    // faces are copied in the caller's cb order; the parity only names the field
+    return halo_start_impl(h, in, 1, (cudaStream_t)stream);
 }
 
 extern "C" dslash_status dslash_halo_wait(dslash_t h, dslash_stream_t stream) {
@@ -538,12 +571,47 @@ static void fill_boxes(StencilParams& K, const dslash_box_t* boxes, int n) {
     for (int b = n; b < kMaxBoxes; ++b) K.box_start[b + 1] = K.box_start[n];
 }
 
+typedef void (*StencilFn)(StencilParams);
+
+template <typename LR, typename VR, int LANES, bool GHOST>
+static StencilFn pick_minb(int minb) {
+    switch (minb) {
+        case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2>;
+        case 3: return dslash_kernel<LR, VR, LANES, GHOST, 3>;
+        default: return dslash_kernel<LR, VR, LANES, GHOST, 4>;
+    }
+}
+
+template <typename LR, typename VR, bool GHOST>
+static StencilFn pick_lanes(int lanes, int minb) {
+    switch (lanes) {
+        case 1: return pick_minb<LR, VR, 1, GHOST>(minb);
+        case 2: return pick_minb<LR, VR, 2, GHOST>(minb);
+        default: return pick_minb<LR, VR, 4, GHOST>(minb);
+    }
+}
+
+template <bool GHOST>
+static StencilFn pick_kernel(int precision, int lanes, int minb) {
+    switch (precision) {
+        case DSLASH_F32: return pick_lanes<float, float, GHOST>(lanes, minb);
+        case DSLASH_MIXED: return pick_lanes<float, double, GHOST>(lanes, minb);
+        default: return pick_lanes<double, double, GHOST>(lanes, minb);
+    }
+}
+
+// defaults chosen by measurement on B200 (tools/sweep.py; profiles/README.md): at 32^4 and 48^4
+// every mapping is best at <= 128 registers (min 2 blocks of 256), LANES 1/2 at 64-128 threads
+static int default_block(int lanes) { return lanes == 4 ? 64 : 64; }
+static int default_minb(int lanes) { return lanes == 4 ? 2 : 2; }
+
 static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int kind, cudaStream_t s) {
     const int64_t sites = K.box_start[K.nbox];
     if (sites == 0) return DSLASH_OK;
-    const bool dir4 = h->kernel == DSLASH_KERNEL_DIR4;
-    const int bs = h->block ? h->block : (dir4 ? 256 : 128);
-    const int64_t threads = dir4 ? sites * 4 : sites;
+    const int lanes = lanes_of(h->kernel);
+    const int bs = h->block ? h->block : default_block(lanes);
+    const int minb = h->min_blocks ? h->min_blocks : default_minb(lanes);
+    const int64_t threads = sites * lanes;
     const unsigned grid = (unsigned)((threads + bs - 1) / bs);
     dslash_s::TimedLaunch* tl = nullptr;
     if (h->timing) {
@@ -557,17 +625,8 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
         tl->kind = kind;
         CU(h, cudaEventRecord(tl->a, s));
     }
-    if (dir4) {
-        if (ghost)
-            dslash_dir4_kernel<true><<<grid, bs, 0, s>>>(K);
-        else
-            dslash_dir4_kernel<false><<<grid, bs, 0, s>>>(K);
-    } else {
-        if (ghost)
-            dslash_site_kernel<true><<<grid, bs, 0, s>>>(K);
-        else
-            dslash_site_kernel<false><<<grid, bs, 0, s>>>(K);
-    }
+    StencilFn fn = ghost ? pick_kernel<true>(h->precision, lanes, minb) : pick_kernel<false>(h->precision, lanes, minb);
+    fn<<<grid, bs, 0, s>>>(K);
     CU(h, cudaGetLastError());
     if (tl) CU(h, cudaEventRecord(tl->b, s));
     return DSLASH_OK;
@@ -576,7 +635,7 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
 static dslash_status check_vectors(dslash_t h, const void* out, const void* in) {
     if (!out || !in) return fail(h, DSLASH_ERR_ARG, "NULL vector pointer");
     if (((uintptr_t)out & 15) || ((uintptr_t)in & 15)) return fail(h, DSLASH_ERR_ARG, "vectors must be 16-byte aligned");
-    const uintptr_t n = (uintptr_t)(3 * h->plan.vh_local * sizeof(double2));
+    const uintptr_t n = (uintptr_t)(3 * h->plan.vh_local * vec_elem(h));
     const uintptr_t a = (uintptr_t)out, b = (uintptr_t)in;
     if (a < b + n && b < a + n) return fail(h, DSLASH_ERR_ARG, "in and out overlap");
     return DSLASH_OK;
@@ -594,8 +653,8 @@ extern "C" dslash_status dslash_apply(dslash_t h, void* out, const void* in, int
     const dslash_plan_t& p = h->plan;
     StencilParams K{};
     K.links = h->links[parity];
-    K.in = (const double2*)in;
-    K.out = (double2*)out;
+    K.in = in;
+    K.out = out;
     K.vh = p.vh_local;
     for (int d = 0; d < 4; ++d) {
         K.L[d] = p.local_dims[d];
@@ -610,7 +669,7 @@ extern "C" dslash_status dslash_apply(dslash_t h, void* out, const void* in, int
         fill_boxes(K, p.interior, p.n_interior);
         return launch(h, K, false, DSLASH_TIMING_INTERIOR, s);
     }
-    if ((st = dslash_halo_start(h, in, 1 - parity, stream)) != DSLASH_OK) return st;
+    if ((st = halo_start_impl(h, in, 1, s)) != DSLASH_OK) return st;
     if (h->overlap) {
         fill_boxes(K, p.interior, p.n_interior);
         if ((st = launch(h, K, false, DSLASH_TIMING_INTERIOR, s)) != DSLASH_OK) return st;
@@ -638,7 +697,7 @@ extern "C" dslash_status dslash_apply_host(dslash_t h, void* out_host, const voi
                                            dslash_stream_t stream) {
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!out_host || !in_host) return fail(h, DSLASH_ERR_ARG, "NULL host buffer");
-    const size_t bytes = 3 * (size_t)h->plan.vh_local * sizeof(double2);
+    const size_t bytes = 3 * (size_t)h->plan.vh_local * vec_elem(h);
     if (!h->stage_in) CU(h, cudaMalloc(&h->stage_in, bytes));
     if (!h->stage_out) CU(h, cudaMalloc(&h->stage_out, bytes));
     cudaStream_t s = (cudaStream_t)stream;
@@ -646,6 +705,59 @@ extern "C" dslash_status dslash_apply_host(dslash_t h, void* out_host, const voi
     dslash_status st = dslash_apply(h, h->stage_out, h->stage_in, parity, stream);
     if (st != DSLASH_OK) return st;
     CU(h, cudaMemcpyAsync(out_host, h->stage_out, bytes, cudaMemcpyDeviceToHost, s));
+    return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_apply_host_batch(dslash_t h, int32_t n, void* const* out_host,
+                                                 const void* const* in_host, int32_t parity,
+                                                 dslash_stream_t stream) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (n < 0 || (n > 0 && (!out_host || !in_host))) return fail(h, DSLASH_ERR_ARG, "bad batch arguments");
+    if (!h->loaded) return fail(h, DSLASH_ERR_STATE, "apply before load_links");
+    for (int32_t i = 0; i < n; ++i)
+        if (!out_host[i] || !in_host[i]) return fail(h, DSLASH_ERR_ARG, "NULL host buffer in batch entry %d", i);
+    if (n == 0) return DSLASH_OK;
+    const int S = dslash_s::kSlots;
+    const size_t bytes = 3 * (size_t)h->plan.vh_local * vec_elem(h);
+    if (!h->h2d) {
+        CU(h, cudaStreamCreateWithFlags(&h->h2d, cudaStreamNonBlocking));
+        CU(h, cudaStreamCreateWithFlags(&h->d2h, cudaStreamNonBlocking));
+        CU(h, cudaEventCreateWithFlags(&h->ev_batch, cudaEventDisableTiming));
+        for (int k = 0; k < S; ++k) {
+            CU(h, cudaMalloc(&h->slot_in[k], bytes));
+            CU(h, cudaMalloc(&h->slot_out[k], bytes));
+            CU(h, cudaEventCreateWithFlags(&h->ev_in_ready[k], cudaEventDisableTiming));
+            CU(h, cudaEventCreateWithFlags(&h->ev_in_free[k], cudaEventDisableTiming));
+            CU(h, cudaEventCreateWithFlags(&h->ev_out_ready[k], cudaEventDisableTiming));
+            CU(h, cudaEventCreateWithFlags(&h->ev_out_free[k], cudaEventDisableTiming));
+            // slots start free
+            CU(h, cudaEventRecord(h->ev_in_free[k], h->h2d));
+            CU(h, cudaEventRecord(h->ev_out_free[k], h->d2h));
+        }
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    CU(h, cudaEventRecord(h->ev_batch, s));
+    CU(h, cudaStreamWaitEvent(h->h2d, h->ev_batch, 0));
+    for (int32_t i = 0; i < n; ++i) {
+        const int k = i % S;
+        // H2D into slot k once the apply that last read it has finished
+        CU(h, cudaStreamWaitEvent(h->h2d, h->ev_in_free[k], 0));
+        CU(h, cudaMemcpyAsync(h->slot_in[k], in_host[i], bytes, cudaMemcpyHostToDevice, h->h2d));
+        CU(h, cudaEventRecord(h->ev_in_ready[k], h->h2d));
+        // apply on the caller's stream once the input landed and the output slot was drained
+        CU(h, cudaStreamWaitEvent(s, h->ev_in_ready[k], 0));
+        CU(h, cudaStreamWaitEvent(s, h->ev_out_free[k], 0));
+        dslash_status st = dslash_apply(h, h->slot_out[k], h->slot_in[k], parity, stream);
+        if (st != DSLASH_OK) return st;
+        CU(h, cudaEventRecord(h->ev_in_free[k], s));
+        CU(h, cudaEventRecord(h->ev_out_ready[k], s));
+        // D2H of the result
+        CU(h, cudaStreamWaitEvent(h->d2h, h->ev_out_ready[k], 0));
+        CU(h, cudaMemcpyAsync(out_host[i], h->slot_out[k], bytes, cudaMemcpyDeviceToHost, h->d2h));
+        CU(h, cudaEventRecord(h->ev_out_free[k], h->d2h));
+    }
+    CU(h, cudaEventRecord(h->ev_batch, h->d2h));
+    CU(h, cudaStreamWaitEvent(s, h->ev_batch, 0));
     return DSLASH_OK;
 }
 
@@ -705,6 +817,17 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
     free_halo(h);
     if (h->stage_in) cudaFree(h->stage_in);
     if (h->stage_out) cudaFree(h->stage_out);
+    if (h->h2d) cudaStreamSynchronize(h->h2d);
+    if (h->d2h) cudaStreamSynchronize(h->d2h);
+    for (int k = 0; k < dslash_s::kSlots; ++k) {
+        if (h->slot_in[k]) cudaFree(h->slot_in[k]);
+        if (h->slot_out[k]) cudaFree(h->slot_out[k]);
+        for (cudaEvent_t e : {h->ev_in_ready[k], h->ev_in_free[k], h->ev_out_ready[k], h->ev_out_free[k]})
+            if (e) cudaEventDestroy(e);
+    }
+    if (h->ev_batch) cudaEventDestroy(h->ev_batch);
+    if (h->h2d) cudaStreamDestroy(h->h2d);
+    if (h->d2h) cudaStreamDestroy(h->d2h);
     for (auto& t : h->tpool) {
         cudaEventDestroy(t.a);
         cudaEventDestroy(t.b);

@@ -21,13 +21,13 @@ struct LinkConvParams {
     const double2* lng;
     const double2* slab_fat[4];   // lower link slabs (halo directions only), see above
     const double2* slab_lng[4];
-    double2* links;               // internal layout (SITE or DIR4)
+    void* links;                  // internal layout: double2 (fp64) or float2 (fp32 / mixed)
     int64_t vh;
     int L[4];
     int lxh;
     int parity;
     int halo_mask;
-    int layout;                   // 0 = SITE, 1 = DIR4
+    int lanes;                    // layout of the kernel that will read the links: 1, 2 or 4
 };
 
 __device__ __forceinline__ const double2* canon_link(const LinkConvParams& P, bool is_long, int mu, int x, int y,
@@ -50,8 +50,10 @@ __device__ __forceinline__ const double2* canon_link(const LinkConvParams& P, bo
     return (is_long ? P.lng : P.fat) + (lex * 4 + mu) * 9;
 }
 
-// one thread per (target site, mu, l)
+// one thread per (target site, mu, l); LR = stored real type (fp64 input rounded to LR)
+template <typename LR>
 __global__ void convert_links_kernel(const LinkConvParams P) {
+    using L2 = cplx_t<LR>;
     const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (gid >= P.vh * 16) return;
     const int64_t cb = gid >> 4;
@@ -78,8 +80,10 @@ __global__ void convert_links_kernel(const LinkConvParams P) {
                 v = A[3 * i + j];
             }
             const int e = 3 * i + j;
-            const int64_t o = P.layout == 0 ? link_index_site(mu, l, e, P.vh, cb) : link_index_dir4(mu, l, e, P.vh, cb);
-            P.links[o] = v;
+            const int64_t o = P.lanes == 1   ? link_index<1>(mu, l, e, P.vh, cb)
+                              : P.lanes == 2 ? link_index<2>(mu, l, e, P.vh, cb)
+                                             : link_index<4>(mu, l, e, P.vh, cb);
+            static_cast<L2*>(P.links)[o] = to_cplx<L2>(v);
         }
 }
 

@@ -11,27 +11,29 @@
 // Links are read with L1::no_allocate + L2 evict_first, vectors with L2 evict_last, the
 // output with st.global.cs.
 //
-// Two mappings (chosen by measurement):
-//   SITE : one thread per target site (the paper's 1LP decomposition, L59-87);
-//   DIR4 : four consecutive lanes per site, lane = mu, each lane streams that direction's
-//          4 matrices and the partial sums meet in two __shfl_xor steps (the paper's 3LP-1
-//          "site x direction + reduction" idea, L101-142, with shuffles instead of local
-//          memory + barrier and without the row split, which replicates vector loads).
+// Mappings (chosen by measurement), one template dslash_kernel<LANES, ...>:
+//   SITE (LANES 1): one thread per target site (the paper's 1LP decomposition, L59-87);
+//   DIR2 (LANES 2): two lanes per site, two directions each, one __shfl_xor step;
+//   DIR4 (LANES 4): four consecutive lanes per site, lane = mu, each lane streams that
+//          direction's 4 matrices and the partial sums meet in two __shfl_xor steps (the
+//          paper's 3LP-1 "site x direction + reduction" idea, L101-142, with shuffles instead
+//          of local memory + barrier and without the row split, which replicates vector loads).
 #pragma once
 
 #include "common.cuh"
 
 namespace hisq {
 
-// Internal link layouts (double2 per complex element e = 3*i + j of a 3x3 matrix).
-// l: 0 = Ff (+1 hop), 1 = Fb (-1), 2 = Nf (+3), 3 = Nb (-3).
-//   SITE: links[((mu*4 + l)*9 + e) * vh + cb]       (16 x 9 coalesced streams per site block)
-//   DIR4: links[((l*9 + e) * vh + cb) * 4 + mu]     (lanes 4s..4s+3 read 64 contiguous bytes)
-__host__ __device__ __forceinline__ int64_t link_index_site(int mu, int l, int e, int64_t vh, int64_t cb) {
-    return ((int64_t)((mu * 4 + l) * 9 + e)) * vh + cb;
-}
-__host__ __device__ __forceinline__ int64_t link_index_dir4(int mu, int l, int e, int64_t vh, int64_t cb) {
-    return (((int64_t)(l * 9 + e)) * vh + cb) * 4 + mu;
+// Internal link layout, for a kernel with LANES lanes per site (lane j streams directions
+// mu = k*LANES + j, k < 4/LANES).  Element e = 3*i + j of 3x3 matrix l (0 = Ff (+1 hop),
+// 1 = Fb (-1), 2 = Nf (+3), 3 = Nb (-3)) in direction mu of target site cb lives at
+//   links[(((l*9 + e) * K + k) * vh + cb) * LANES + j],   K = 4 / LANES,
+// so at every load instruction the lanes of a warp read one contiguous 512-byte span, and the
+// 9 elements of a matrix are 4*vh double2 apart.
+template <int LANES>
+__host__ __device__ __forceinline__ int64_t link_index(int mu, int l, int e, int64_t vh, int64_t cb) {
+    constexpr int K = 4 / LANES;
+    return ((((int64_t)(l * 9 + e) * K + mu / LANES) * vh + cb) * LANES) + (mu % LANES);
 }
 
 struct Site {
@@ -62,16 +64,17 @@ __device__ __forceinline__ Site decode_site(const StencilParams& P, int64_t gid)
     return s;
 }
 
+template <typename V2>
 struct SrcRef {
-    const double2* p;  // colour component c at p[c * stride]
+    const V2* p;  // colour component c at p[c * stride]
     int64_t stride;
 };
 
 // Address of psi(x + h mu^).  GHOST: directions in P.halo_mask read the depth-3 ghost faces
 // outside [0, L); otherwise coordinates wrap periodically (two conditional steps suffice for
 // |h| <= 3 and L >= 2).
-template <bool GHOST>
-__device__ __forceinline__ SrcRef source(const StencilParams& P, int mu, int h, const Site& s) {
+template <typename V2, bool GHOST>
+__device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, int mu, int h, const Site& s) {
     const int c = mu == 0 ? s.x : mu == 1 ? s.y : mu == 2 ? s.z : s.t;
     const int L = P.L[mu];
     int cn = c + h;
@@ -83,7 +86,7 @@ __device__ __forceinline__ SrcRef source(const StencilParams& P, int mu, int h, 
             f = s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (s.z + (int64_t)P.L[2] * d));
         else
             f = s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (d + 3 * (int64_t)s.t));
-        return {P.ghost[mu][side] + f, P.face_vh[mu]};
+        return {static_cast<const V2*>(P.ghost[mu][side]) + f, P.face_vh[mu]};
     }
     if (cn < 0) cn += L;
     if (cn < 0) cn += L;
@@ -98,12 +101,12 @@ __device__ __forceinline__ SrcRef source(const StencilParams& P, int mu, int h, 
                                    : (int64_t)P.lxh * P.L[1] * P.L[2];
         idx = s.cb + (int64_t)(cn - c) * st;
     }
-    return {P.in + idx, P.vh};
+    return {static_cast<const V2*>(P.in) + idx, P.vh};
 }
 
 // acc (+/-)= U v for a 3x3 matrix whose 9 elements are U[e]
-template <bool SUB>
-__device__ __forceinline__ void matvec_acc(double2 acc[3], const double2 U[9], const double2 v[3]) {
+template <bool SUB, typename V2>
+__device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[3]) {
 #pragma unroll
     for (int i = 0; i < 3; ++i)
 #pragma unroll
@@ -115,80 +118,82 @@ __device__ __forceinline__ void matvec_acc(double2 acc[3], const double2 U[9], c
         }
 }
 
-// ---------------------------------------------------------------- SITE: one thread per site
-template <bool GHOST>
-__global__ void __launch_bounds__(256) dslash_site_kernel(const StencilParams P) {
+// ---------------------------------------------------------------- the stencil kernel
+// LANES consecutive threads per target site (1 = thread per site, the paper's 1LP mapping;
+// 4 = one lane per direction, the paper's 3LP-1 site x direction split with a shuffle
+// reduction instead of local memory + barrier).  MINB = minimum resident 256-thread blocks per
+// SM, which caps registers (2 -> 128, 3 -> 80, 4 -> 64) and so trades per-thread ILP against
+// occupancy.  GHOST selects the boundary variant that reads halo faces.  LR is the real type
+// of the stored links, VR that of the vectors and of the accumulation (double/double = fp64,
+// float/float = fp32, float/double = mixed: fp32 links widened to fp64 before the FMAs).
+template <typename LR, typename VR, int LANES, bool GHOST, int MINB>
+__global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P) {
+    static_assert(LANES == 1 || LANES == 2 || LANES == 4, "LANES must divide 4");
+    using L2 = cplx_t<LR>;
+    using V2 = cplx_t<VR>;
+    constexpr int K = 4 / LANES;
     const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (gid >= P.box_start[P.nbox]) return;
-    const uint64_t pol_stream = policy_evict_first();
-    const uint64_t pol_keep = policy_evict_last();
-    const Site s = decode_site(P, gid);
-    double2 acc[3] = {{0.0, 0.0}, {0.0, 0.0}, {0.0, 0.0}};
-#pragma unroll
-    for (int mu = 0; mu < 4; ++mu) {
-#pragma unroll
-        for (int l = 0; l < 4; ++l) {
-            const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
-            const SrcRef src = source<GHOST>(P, mu, h, s);
-            double2 v[3];
-#pragma unroll
-            for (int c = 0; c < 3; ++c) v[c] = ld_reuse(src.p + c * src.stride, pol_keep);
-            const double2* lp = P.links + link_index_site(mu, l, 0, P.vh, s.cb);
-            double2 U[9];
-#pragma unroll
-            for (int e = 0; e < 9; ++e) U[e] = ld_stream(lp + (int64_t)e * P.vh, pol_stream);
-            if (l & 1)
-                matvec_acc<true>(acc, U, v);
-            else
-                matvec_acc<false>(acc, U, v);
-        }
-    }
-#pragma unroll
-    for (int c = 0; c < 3; ++c) st_stream(P.out + c * P.vh + s.cb, acc[c]);
-}
-
-// ---------------------------------------------------------------- DIR4: four lanes per site
-template <bool GHOST>
-__global__ void __launch_bounds__(256) dslash_dir4_kernel(const StencilParams P) {
-    const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int mu = threadIdx.x & 3;
-    const int64_t site = gid >> 2;
+    const int lane = (LANES == 1) ? 0 : (int)(threadIdx.x & (LANES - 1));
+    const int64_t site = (LANES == 1) ? gid : (gid / LANES);
     const bool valid = site < P.box_start[P.nbox];
-    double2 acc[3] = {{0.0, 0.0}, {0.0, 0.0}, {0.0, 0.0}};
+    if (LANES == 1 && !valid) return;
+    V2 acc[3];
+#pragma unroll
+    for (int c = 0; c < 3; ++c) acc[c].x = acc[c].y = VR(0);
     Site s;
     if (valid) {
         const uint64_t pol_stream = policy_evict_first();
         const uint64_t pol_keep = policy_evict_last();
         s = decode_site(P, site);
+        const L2* links = static_cast<const L2*>(P.links);
 #pragma unroll
-        for (int l = 0; l < 4; ++l) {
-            const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
-            const SrcRef src = source<GHOST>(P, mu, h, s);
-            double2 v[3];
+        for (int k = 0; k < K; ++k) {
+            const int mu = k * LANES + lane;
 #pragma unroll
-            for (int c = 0; c < 3; ++c) v[c] = ld_reuse(src.p + c * src.stride, pol_keep);
-            const double2* lp = P.links + link_index_dir4(mu, l, 0, P.vh, s.cb);
-            double2 U[9];
+            for (int l = 0; l < 4; ++l) {
+                const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
+                const SrcRef<V2> src = source<V2, GHOST>(P, mu, h, s);
+                V2 v[3];
 #pragma unroll
-            for (int e = 0; e < 9; ++e) U[e] = ld_stream(lp + (int64_t)e * P.vh * 4, pol_stream);
-            if (l & 1)
-                matvec_acc<true>(acc, U, v);
-            else
-                matvec_acc<false>(acc, U, v);
+                for (int c = 0; c < 3; ++c) v[c] = ld_reuse(src.p + c * src.stride, pol_keep);
+                const L2* lp = links + link_index<LANES>(mu, l, 0, P.vh, s.cb);
+                V2 U[9];
+#pragma unroll
+                for (int e = 0; e < 9; ++e)
+                    U[e] = to_cplx<V2>(widen(ld_stream(lp + (int64_t)e * 4 * P.vh, pol_stream)));
+                if (l & 1)
+                    matvec_acc<true>(acc, U, v);
+                else
+                    matvec_acc<false>(acc, U, v);
+            }
         }
     }
-    // butterfly over the 4 lanes of a site: every lane ends with ((p0+p1)+(p2+p3)) bitwise
+    if (LANES > 1) {
+        // butterfly over the lanes of a site: every lane ends with the same bits
+        // (((p0+p1)+(p2+p3)) by commutativity of each pairwise add)
 #pragma unroll
-    for (int c = 0; c < 3; ++c) {
+        for (int c = 0; c < 3; ++c) {
 #pragma unroll
-        for (int off = 1; off <= 2; off <<= 1) {
-            acc[c].x += __shfl_xor_sync(0xffffffffu, acc[c].x, off);
-            acc[c].y += __shfl_xor_sync(0xffffffffu, acc[c].y, off);
+            for (int off = 1; off < LANES; off <<= 1) {
+                acc[c].x += __shfl_xor_sync(0xffffffffu, acc[c].x, off);
+                acc[c].y += __shfl_xor_sync(0xffffffffu, acc[c].y, off);
+            }
         }
     }
-    if (valid && mu < 3) {
-        const double2 r = mu == 0 ? acc[0] : mu == 1 ? acc[1] : acc[2];
-        st_stream(P.out + mu * P.vh + s.cb, r);
+    if (!valid) return;
+    V2* out = static_cast<V2*>(P.out);
+    if (LANES == 1) {
+#pragma unroll
+        for (int c = 0; c < 3; ++c) st_stream(out + c * P.vh + s.cb, acc[c]);
+    } else if (LANES == 2) {
+        if (lane == 0) {
+            st_stream(out + s.cb, acc[0]);
+            st_stream(out + P.vh + s.cb, acc[1]);
+        } else {
+            st_stream(out + 2 * P.vh + s.cb, acc[2]);
+        }
+    } else {
+        if (lane < 3) st_stream(out + lane * P.vh + s.cb, lane == 0 ? acc[0] : lane == 1 ? acc[1] : acc[2]);
     }
 }
 

@@ -14,7 +14,7 @@ import oracle
 pytestmark = pytest.mark.gpu
 
 TOL = 1e-12
-KERNELS = ["site", "dir4"]
+KERNELS = ["site", "dir2", "dir4"]
 
 
 @pytest.fixture(scope="module")
@@ -98,13 +98,19 @@ def test_self_halo_bitwise(torch_cuda, kernel, dims, mask, overlap):
         assert oracle.normwise_error(halo, ref) <= TOL
 
 
-def test_kernels_agree(torch_cuda):
+@pytest.mark.parametrize("kernel", KERNELS)
+@pytest.mark.parametrize("minb,block", [(2, 64), (3, 96), (4, 256), (2, 256)])
+def test_launch_configs_agree(torch_cuda, kernel, minb, block):
+    """Every register budget and block size gives the same bits for a given mapping (the
+    mapping fixes the summation order), and the mappings agree to rounding."""
     dims = (16, 16, 16, 16)
     fat, lng = fieldgen.workload_links(dims)
     src = fieldgen.vector_cb(dims, 7, 1)
-    a = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel="site")
-    b = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel="dir4")
-    assert oracle.normwise_error(a, b) < 1e-14
+    base = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel=kernel)
+    other = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel=kernel, min_blocks=minb, block=block)
+    assert np.array_equal(base, other)
+    ref = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel="site")
+    assert oracle.normwise_error(base, ref) < 1e-14
 
 
 @pytest.mark.parametrize("kernel", KERNELS)
@@ -170,6 +176,22 @@ def test_apply_host_and_determinism(torch_cuda):
         assert torch.equal(a.cpu(), hout)
 
 
+def test_apply_host_batch(torch_cuda):
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    torch = torch_cuda
+    dims = (8, 8, 8, 16)
+    fat, lng = fieldgen.workload_links(dims)
+    with Dslash(dims, force_halo=0x8) as D:
+        D.load_links(fat, lng)
+        ins = [torch.from_numpy(fieldgen.vector_cb(dims, 30 + i, 0)).pin_memory() for i in range(7)]
+        outs = [torch.empty_like(ins[0]).pin_memory() for _ in range(7)]
+        D.apply_host_batch(outs, ins, 1)
+        torch.cuda.synchronize()
+        for i in range(7):
+            assert torch.equal(outs[i], D(ins[i].cuda(), 1).cpu())
+        D.apply_host_batch([], [], 1)          # empty batch is a no-op
+
+
 def test_device_links_equal_host_links(torch_cuda):
     from paper_conf_sc_dufekgaad024_b200 import Dslash
     torch = torch_cuda
@@ -183,6 +205,44 @@ def test_device_links_equal_host_links(torch_cuda):
         b = D(src, 1)
         torch.cuda.synchronize()
         assert torch.equal(a, b)
+
+
+@pytest.mark.parametrize("precision,tol", [("f32", 1e-5), ("mixed", 1e-5)])
+@pytest.mark.parametrize("kernel", KERNELS)
+@pytest.mark.parametrize("dims", [(8, 10, 12, 14), (4, 4, 4, 4), (6, 8, 10, 12)])
+def test_reduced_precision_vs_fp64_oracle(torch_cuda, precision, tol, kernel, dims):
+    """§8(f)-1: fp32 and mixed paths against the fp64 oracle on the fp64 inputs, normwise 1e-5
+    (north star).  The fp32 input vector is the fp64 one rounded."""
+    import torch
+    fat, lng = fieldgen.workload_links(dims)
+    psi = fieldgen.vector(dims, fieldgen.SEED_PSI)
+    for parity in (0, 1):
+        ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, parity), parity)
+        src = torch.from_numpy(fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 1 - parity))
+        from paper_conf_sc_dufekgaad024_b200 import Dslash
+        with Dslash(dims, kernel=kernel, precision=precision) as D:
+            D.load_links(fat, lng)
+            out = D(src.to(D.dtype).cuda(), parity)
+            torch.cuda.synchronize()
+            got = out.cpu().numpy().astype(np.complex128)
+        err = oracle.normwise_error(got, ref)
+        assert err <= tol
+        assert err > 1e-12          # it really ran in reduced precision
+
+
+@pytest.mark.parametrize("precision", ["f32", "mixed"])
+def test_reduced_precision_self_halo_bitwise(torch_cuda, precision):
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 8, 8, 12)
+    fat, lng = fieldgen.workload_links(dims)
+    outs = []
+    for mask in (0, 0xC):
+        with Dslash(dims, precision=precision, force_halo=mask) as D:
+            D.load_links(fat, lng)
+            src = torch.from_numpy(fieldgen.vector_cb(dims, 3, 0)).to(D.dtype).cuda()
+            outs.append(D(src, 1).cpu())
+    assert torch.equal(outs[0], outs[1])
 
 
 def test_error_paths(torch_cuda):
