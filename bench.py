@@ -45,6 +45,12 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--kernel", default="dir2", choices=["site", "dir2", "dir4"])
     ap.add_argument("--min-blocks", type=int, default=0)
+    ap.add_argument("--nrhs", type=int, default=1, choices=[1, 2, 3, 4, 5, 6, 7, 8],
+                    help="right-hand sides per apply, one link pass (SURVEY §8(f)-4)")
+    ap.add_argument("--recon", type=int, default=18, choices=[18, 12],
+                    help="12: long links stored as 2 rows (SURVEY §8(f)-2, QUDA recon-12, PAPER.md L325)")
+    ap.add_argument("--precision", default="f64", choices=["f64", "f32", "mixed"],
+                    help="f64 is the paper's (L278) and the headline; f32/mixed are SURVEY §8(f)-1")
     ap.add_argument("--block", type=int, default=0)
     ap.add_argument("--local", default="32,32,32,32", help="per-GPU local extents x,y,z,t")
     ap.add_argument("--parity", type=int, default=0)
@@ -230,7 +236,7 @@ def main():
     import torch.distributed as dist
 
     import fieldgen
-    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    from paper_conf_sc_dufekgaad024_b200 import Dslash, algo_bytes
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -245,23 +251,34 @@ def main():
     gdims, grid, loc, name = workload(args, world)
     parity = args.parity
 
+    nrhs = args.nrhs
+    algo_bytes_site = algo_bytes(args.precision, args.recon, nrhs)
     D = Dslash(gdims, grid, parity_mask=parity, kernel=args.kernel, block=args.block, min_blocks=args.min_blocks,
+               precision=args.precision, recon=args.recon,
                overlap=not args.no_overlap, timing=True, rank=rank, world_size=world)
     origin, extent = D.origin, D.local_dims
     fat, lng = fieldgen.workload_links(gdims, origin=origin, extent=extent)
     D.load_links(fat, lng)
     del fat, lng
     vh = D.vh
-    vec_bytes = 3 * vh * 16
+    vec_bytes = 3 * vh * (8 if args.precision == "f32" else 16) * nrhs   # one step's source (or output)
     l2_bytes = torch.cuda.get_device_properties(local_rank).L2_cache_size
     R = max(2, int(np.ceil(2 * l2_bytes / (2 * vec_bytes))) + 1)
-    srcs = [torch.from_numpy(fieldgen.vector_cb(gdims, fieldgen.SEED_PSI + r, 1 - parity, origin=origin,
-                                                extent=extent)).cuda() for r in range(R)]
-    outs = [D.empty_vector() for _ in range(R)]
+
+    def make_src(r):
+        vs = [torch.from_numpy(fieldgen.vector_cb(gdims, fieldgen.SEED_PSI + r * nrhs + k, 1 - parity, origin=origin,
+                                                  extent=extent)).to(D.dtype) for k in range(nrhs)]
+        return (vs[0] if nrhs == 1 else torch.stack(vs)).contiguous()
+
+    srcs = [make_src(r).cuda() for r in range(R)]
+    outs = [torch.empty_like(srcs[0]) for _ in range(R)]
     stream = torch.cuda.current_stream()
 
     def step(i):
-        D.apply(outs[i % R], srcs[i % R], parity, stream)
+        if nrhs == 1:
+            D.apply(outs[i % R], srcs[i % R], parity, stream)
+        else:
+            D.apply_multi(outs[i % R], srcs[i % R], parity, stream)
 
     for i in range(args.warmup):
         step(i)
@@ -288,23 +305,26 @@ def main():
     if world > 1:
         dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
     ms_max = float(t_max.item())
-    total_sites = vh * world
+    total_sites = vh * world * nrhs      # site-RHS pairs per step
     gflops = FLOP_PER_SITE * total_sites * args.steps / (ms_max * 1e-3) / 1e9
-    algo_gbs = ALGO_BYTES_PER_SITE * total_sites * args.steps / (ms_max * 1e-3) / 1e9
+    algo_gbs = algo_bytes_site * vh * world * args.steps / (ms_max * 1e-3) / 1e9
 
     # dominant kernel: the full-lattice kernel at N = 1, the interior kernel at N > 1
     plan = D.plan
     dom_sites = int(plan.interior_sites) if plan.n_interior else int(plan.boundary_sites)
+    # algo_bytes_site already counts nrhs vectors per site; GB/s over sites, flop over site-RHS pairs
     peak, peak_src = measured_peak()
     kern_ms = t_int / max(1, n_int) if n_int else None
     roof = None
     if kern_ms:
-        achieved = ALGO_BYTES_PER_SITE * dom_sites / (kern_ms * 1e-3) / 1e9
+        achieved = algo_bytes_site * dom_sites / (kern_ms * 1e-3) / 1e9
         roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(achieved / peak, 4), "traffic": ncu_traffic(args.kernel, extent),
+                "frac": round(achieved / peak, 4),
+                "traffic": ncu_traffic(args.kernel + ("" if args.precision == "f64" else f"-{args.precision}")
+                                     + ("" if args.recon == 18 else f"-r{args.recon}"), extent),
                 "kernel": f"dslash_kernel<lanes={ {'site': 1, 'dir2': 2, 'dir4': 4}[args.kernel]}, ghost=false>"
                           + (" interior" if world > 1 else ""),
-                "bytes_per_launch": ALGO_BYTES_PER_SITE * dom_sites, "avg_launch_us": round(kern_ms * 1e3, 2),
+                "bytes_per_launch": algo_bytes_site * dom_sites, "bytes_per_site": algo_bytes_site, "avg_launch_us": round(kern_ms * 1e3, 2),
                 "launches": n_int, "peak_source": peak_src,
                 "frac_of_nominal_8TBs": round(achieved / NOMINAL_HBM_GBS, 4)}
 
@@ -312,10 +332,10 @@ def main():
     # and its chi device->host (dslash_apply_host_batch pipelines the copies of neighbouring steps
     # against the compute on 3 device slots)
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and nrhs == 1:
         RH = 4
         hins = [torch.from_numpy(fieldgen.vector_cb(gdims, fieldgen.SEED_PSI + r, 1 - parity, origin=origin,
-                                                    extent=extent)).pin_memory() for r in range(RH)]
+                                                    extent=extent)).to(D.dtype).pin_memory() for r in range(RH)]
         houts = [torch.empty_like(hins[0]).pin_memory() for _ in range(RH)]
         ke = max(12, min(args.steps, 600))
         seq_in = [hins[i % RH] for i in range(ke)]
@@ -346,13 +366,16 @@ def main():
     if rank == 0:
         line = {"metric": METRIC, "value": round(gflops, 2), "unit": "GFLOP/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
-                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "dtype": {"f64": "f64", "f32": "f32", "mixed": "f32 links, f64 vectors/accumulation"}[args.precision],
                 "data": "synthetic",
                 "config": {"workload": name, "global_dims": list(gdims), "local_dims": list(extent),
                            "proc_grid": list(grid), "parallelism": f"t{world}", "parity": parity,
-                           "kernel": args.kernel, "block": args.block or None,
+                           "kernel": args.kernel, "block": args.block or None, "precision": args.precision,
+                           "long_link_recon": args.recon, "nrhs": nrhs,
                            "overlap": not args.no_overlap,
-                           "l2": f"inputs > L2: 1.21 GB links/apply streamed; {R} rotating (psi, chi) pairs = "
+                           "l2": f"inputs > L2: {(algo_bytes_site - 2 * vec_bytes // (3 * vh) * 3) * vh / 1e9:.2f} GB "
+                                 f"links/apply streamed; {R} rotating (psi, chi) pairs = "
                                  f"{R * 2 * vec_bytes / 1e6:.0f} MB > {l2_bytes / 1e6:.0f} MB L2",
                            "links": "random SU(3) fat (seed 1), -1/24 random SU(3) long (seed 2)"},
                 "algorithmic_gbs": round(algo_gbs, 1),

@@ -58,7 +58,8 @@ typedef enum {
     DSLASH_ERR_CUDA = 3,        /* a CUDA runtime call failed (message carries cudaGetErrorString) */
     DSLASH_ERR_NCCL = 4,        /* an NCCL call failed */
     DSLASH_ERR_OOM = 5,         /* device allocation failed */
-    DSLASH_ERR_UNSUPPORTED = 6  /* valid but not implemented (x/y partitioning, fp32 before it exists) */
+    DSLASH_ERR_UNSUPPORTED = 6, /* valid but not implemented (x/y partitioning, an fp32 solver) */
+    DSLASH_ERR_NOT_CONVERGED = 7 /* dslash_cg reached max_iter (not sticky; results are still written) */
 } dslash_status;
 
 enum { DSLASH_EVEN = 0, DSLASH_ODD = 1, DSLASH_BOTH = 2 }; /* parity_mask */
@@ -84,6 +85,12 @@ enum {
     DSLASH_OPT_OVERLAP = 3,     /* 1 (default): interior kernel overlaps the halo exchange; 0: one
                                    kernel over all sites after the exchange                            */
     DSLASH_OPT_TIMING = 4,      /* 1: record CUDA events around every kernel (dslash_kernel_timing)   */
+    DSLASH_OPT_LONG_RECON = 6,  /* 18 (default): long links stored in full; 12: long links stored as
+                                   rows 0 and 1 only, row 2 rebuilt in registers as conj(r0 x r1)/s
+                                   (QUDA "recon-12").  Requires every long link
+                                   (and the link halo) to be s*W with W in SU(3) and one real s;
+                                   load_links verifies it and returns DSLASH_ERR_ARG otherwise.
+                                   Before load_links                                                  */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */
@@ -161,6 +168,14 @@ DSLASH_API dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
  * NULL, misaligned or overlapping buffers. */
 DSLASH_API dslash_status dslash_apply(dslash_t h, void* out, const void* in, int32_t parity, dslash_stream_t stream);
 
+/* nrhs applies sharing one pass over the links: out and in hold nrhs
+ * vectors back to back, [nrhs][3][Vh_local] (same element type and rules as dslash_apply),
+ * out[r] = D in[r].  Every link is read from HBM once per launch of up to 8 right-hand
+ * sides, so the algorithmic bytes per site are links + nrhs x (source + output).  The halo
+ * exchange (N > 1) moves all nrhs faces at once. */
+DSLASH_API dslash_status dslash_apply_multi(dslash_t h, int32_t nrhs, void* out, const void* in, int32_t parity,
+                                            dslash_stream_t stream);
+
 /* The same operation from HOST buffers (end-to-end path): copies in (host) to an
  * internal device buffer, applies, copies the result to out (host), all ordered on
  * `stream`; returns after enqueueing (synchronise the stream before reading out).
@@ -177,6 +192,26 @@ DSLASH_API dslash_status dslash_apply_host(dslash_t h, void* out_host, const voi
 DSLASH_API dslash_status dslash_apply_host_batch(dslash_t h, int32_t n, void* const* out_host,
                                                  const void* const* in_host, int32_t parity,
                                                  dslash_stream_t stream);
+
+/* The even-odd normal operator (the conjugate-gradient step of MILC's
+ * su3_rhmd_hisq):  out = A_p in,  A_p = m^2 - D_{p,1-p} D_{1-p,p}, where D_{a,b}
+ * is the Dslash from parity b to target parity a.  D is anti-Hermitian, so A_p = m^2 +
+ * D_{1-p,p}^dag D_{1-p,p} is Hermitian positive definite for m != 0.  in, out: fp64 [3][Vh]
+ * vectors on parity p.  Needs parity_mask DSLASH_BOTH and fp64 vectors (DSLASH_F64 or
+ * DSLASH_MIXED; DSLASH_F32 returns DSLASH_ERR_UNSUPPORTED).  Two applies + one fused
+ * m^2-subtraction kernel, stream-ordered. */
+DSLASH_API dslash_status dslash_normal_apply(dslash_t h, void* out, const void* in, int32_t parity, double mass,
+                                             dslash_stream_t stream);
+
+/* Conjugate gradient for A_p x = b (A_p as above), starting from x = 0, stopping when
+ * |r_k| <= rel_tol |b| or after max_iter iterations.  Dot products are reduced
+ * deterministically on each GPU and summed over ranks with ncclAllReduce.  Synchronous:
+ * returns after the solve (it reads each dot product on the host).  iters (may be NULL)
+ * receives the iteration count, rel_resid (may be NULL) the TRUE relative residual
+ * |b - A x| / |b| recomputed at the end.  Returns DSLASH_ERR_NOT_CONVERGED (not sticky) if the
+ * recursive residual did not reach rel_tol. */
+DSLASH_API dslash_status dslash_cg(dslash_t h, void* x, const void* b, int32_t parity, double mass, double rel_tol,
+                                   int32_t max_iter, int32_t* iters, double* rel_resid, dslash_stream_t stream);
 
 /* Halo exchange only: start sending the depth-3 faces of `in` (source parity
  * src_parity) after the work already queued on `stream`; dslash_halo_wait makes

@@ -21,6 +21,16 @@ ALGO_BYTES_PER_SITE = 2400    # + 48 B source (ideal reuse) + 48 B output (DESIG
 # algorithmic bytes per target site by precision: links + source + output
 ALGO_BYTES = {"f64": 2304 + 48 + 48, "f32": 1152 + 24 + 24, "mixed": 1152 + 48 + 48}
 
+
+def algo_bytes(precision="f64", recon=18, nrhs=1):
+    """Algorithmic bytes per target site for one launch over nrhs right-hand sides: links
+    (recon-12 stores 6 of 9 entries of the 8 long matrices) + nrhs x (source with ideal reuse +
+    output)."""
+    lb = 16 if precision == "f64" else 8
+    vb = 8 if precision == "f32" else 16
+    link_entries = 8 * 9 + 8 * (6 if recon == 12 else 9)
+    return link_entries * lb + nrhs * 2 * 3 * vb
+
 __all__ = ["Dslash", "DslashError", "dslash_plan", "FLOP_PER_SITE", "ALGO_BYTES_PER_SITE"]
 
 
@@ -44,7 +54,8 @@ class Dslash:
     """
 
     def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="dir2", block=0,
-                 force_halo=0, overlap=True, timing=False, rank=0, world_size=1, min_blocks=0, precision="f64"):
+                 force_halo=0, overlap=True, timing=False, rank=0, world_size=1, min_blocks=0, precision="f64",
+                 recon=18):
         import torch
         self.global_dims = tuple(int(d) for d in global_dims)
         self.precision = precision
@@ -67,6 +78,8 @@ class Dslash:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_BLOCK, block)
             if min_blocks:
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_MIN_BLOCKS, min_blocks)
+            if recon != 18:
+                _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_LONG_RECON, recon)
             if force_halo:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_FORCE_HALO, force_halo)
             _abi.dslash_set_option(self.h, DSLASH_OPT_OVERLAP, int(bool(overlap)))
@@ -117,6 +130,34 @@ class Dslash:
         self._check_vec(inp)
         _abi.dslash_apply(self.h, out.data_ptr(), inp.data_ptr(), int(parity), _stream_handle(stream))
         return out
+
+    def apply_multi(self, out, inp, parity, stream=None):
+        """out[r] = D inp[r] for tensors of shape (nrhs, 3, Vh), one pass over the links."""
+        for v in (out, inp):
+            if not (v.is_cuda and v.dtype == self.dtype and v.is_contiguous() and v.dim() == 3
+                    and tuple(v.shape[1:]) == (3, self.vh)):
+                raise ValueError(f"multi-RHS vectors must be contiguous {self.dtype} CUDA tensors (n, 3, {self.vh})")
+        if out.shape[0] != inp.shape[0]:
+            raise ValueError("out and inp hold different numbers of right-hand sides")
+        _abi.dslash_apply_multi(self.h, int(inp.shape[0]), out.data_ptr(), inp.data_ptr(), int(parity),
+                                _stream_handle(stream))
+        return out
+
+    def normal_apply(self, out, inp, parity, mass, stream=None):
+        """out = (m^2 - D_{p,1-p} D_{1-p,p}) inp on parity p (needs parity_mask BOTH, fp64 vectors)."""
+        self._check_vec(out)
+        self._check_vec(inp)
+        _abi.dslash_normal_apply(self.h, out.data_ptr(), inp.data_ptr(), int(parity), float(mass),
+                                 _stream_handle(stream))
+        return out
+
+    def cg(self, x, b, parity, mass, rel_tol=1e-10, max_iter=1000, stream=None):
+        """Solve (m^2 - D_{p,1-p} D_{1-p,p}) x = b by CG; returns (converged, iterations, true rel. residual)."""
+        self._check_vec(x)
+        self._check_vec(b)
+        st, it, res = _abi.dslash_cg(self.h, x.data_ptr(), b.data_ptr(), int(parity), float(mass), float(rel_tol),
+                                     int(max_iter), _stream_handle(stream))
+        return st == _abi.DSLASH_OK, it, res
 
     def __call__(self, inp, parity, stream=None):
         return self.apply(self.empty_vector(), inp, parity, stream)

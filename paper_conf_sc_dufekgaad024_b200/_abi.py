@@ -14,15 +14,16 @@ LIB_PATH = os.path.join(_HERE, "libhisq_dslash.so")
 HEADER = os.path.join(os.path.dirname(_HERE), "include", "hisq_dslash.h")
 
 DSLASH_OK, DSLASH_ERR_ARG, DSLASH_ERR_STATE, DSLASH_ERR_CUDA, DSLASH_ERR_NCCL, DSLASH_ERR_OOM, \
-    DSLASH_ERR_UNSUPPORTED = range(7)
+    DSLASH_ERR_UNSUPPORTED, DSLASH_ERR_NOT_CONVERGED = range(8)
 STATUS_NAMES = {0: "DSLASH_OK", 1: "DSLASH_ERR_ARG", 2: "DSLASH_ERR_STATE", 3: "DSLASH_ERR_CUDA",
-                4: "DSLASH_ERR_NCCL", 5: "DSLASH_ERR_OOM", 6: "DSLASH_ERR_UNSUPPORTED"}
+                4: "DSLASH_ERR_NCCL", 5: "DSLASH_ERR_OOM", 6: "DSLASH_ERR_UNSUPPORTED",
+                7: "DSLASH_ERR_NOT_CONVERGED"}
 DSLASH_EVEN, DSLASH_ODD, DSLASH_BOTH = 0, 1, 2
 DSLASH_F64, DSLASH_F32, DSLASH_MIXED = 0, 1, 2
 PRECISIONS = {"f64": DSLASH_F64, "f32": DSLASH_F32, "mixed": DSLASH_MIXED}
 DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_DIR2 = 0, 1, 2
 DSLASH_OPT_KERNEL, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_OVERLAP, DSLASH_OPT_TIMING, \
-    DSLASH_OPT_MIN_BLOCKS = range(6)
+    DSLASH_OPT_MIN_BLOCKS, DSLASH_OPT_LONG_RECON = range(7)
 DSLASH_TIMING_INTERIOR, DSLASH_TIMING_BOUNDARY, DSLASH_TIMING_ALL = range(3)
 KERNELS = {"site": DSLASH_KERNEL_SITE, "dir4": DSLASH_KERNEL_DIR4, "dir2": DSLASH_KERNEL_DIR2}
 
@@ -78,9 +79,13 @@ _SIGS = {
     "dslash_set_option": ([_h, ctypes.c_int32, ctypes.c_int64], ctypes.c_int),
     "dslash_load_links": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
+    "dslash_apply_multi": ([_h, ctypes.c_int32, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply_host": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply_host_batch": ([_h, ctypes.c_int32, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.c_int32,
                                  _vp], ctypes.c_int),
+    "dslash_normal_apply": ([_h, _vp, _vp, ctypes.c_int32, ctypes.c_double, _vp], ctypes.c_int),
+    "dslash_cg": ([_h, _vp, _vp, ctypes.c_int32, ctypes.c_double, ctypes.c_double, ctypes.c_int32,
+                   ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_double), _vp], ctypes.c_int),
     "dslash_halo_start": ([_h, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_halo_wait": ([_h, _vp], ctypes.c_int),
     "dslash_sync": ([_h], ctypes.c_int),
@@ -150,6 +155,10 @@ def dslash_apply(h, out_ptr, in_ptr, parity, stream=0):
     return check(lib.dslash_apply(h, out_ptr, in_ptr, parity, stream), h)
 
 
+def dslash_apply_multi(h, nrhs, out_ptr, in_ptr, parity, stream=0):
+    return check(lib.dslash_apply_multi(h, nrhs, out_ptr, in_ptr, parity, stream), h)
+
+
 def dslash_apply_host(h, out_ptr, in_ptr, parity, stream=0):
     return check(lib.dslash_apply_host(h, out_ptr, in_ptr, parity, stream), h)
 
@@ -161,6 +170,21 @@ def dslash_apply_host_batch(h, out_ptrs, in_ptrs, parity, stream=0):
     outs = (ctypes.c_void_p * max(n, 1))(*out_ptrs)
     ins = (ctypes.c_void_p * max(n, 1))(*in_ptrs)
     return check(lib.dslash_apply_host_batch(h, n, outs, ins, parity, stream), h)
+
+
+def dslash_normal_apply(h, out_ptr, in_ptr, parity, mass, stream=0):
+    return check(lib.dslash_normal_apply(h, out_ptr, in_ptr, parity, mass, stream), h)
+
+
+def dslash_cg(h, x_ptr, b_ptr, parity, mass, rel_tol, max_iter, stream=0):
+    """Returns (status, iterations, true relative residual); status is DSLASH_OK or
+    DSLASH_ERR_NOT_CONVERGED, anything else raises."""
+    it = ctypes.c_int32()
+    res = ctypes.c_double()
+    st = lib.dslash_cg(h, x_ptr, b_ptr, parity, mass, rel_tol, max_iter, ctypes.byref(it), ctypes.byref(res), stream)
+    if st not in (DSLASH_OK, DSLASH_ERR_NOT_CONVERGED):
+        check(st, h)
+    return st, it.value, res.value
 
 
 def dslash_halo_start(h, in_ptr, src_parity, stream=0):

@@ -19,22 +19,43 @@ def nccl_dir():
 
 def sources():
     return sorted(glob.glob(os.path.join(HERE, "csrc", "*.cu")) + glob.glob(os.path.join(HERE, "csrc", "*.cuh"))
-                  + [os.path.join(ROOT, "include", "hisq_dslash.h")])
+                  + glob.glob(os.path.join(HERE, "csrc", "*.h")) + [os.path.join(ROOT, "include", "hisq_dslash.h")])
+
+
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    """Compile every csrc/*.cu to an object in parallel (sm_100a, -lineinfo) and link the .so."""
     if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= max(os.path.getmtime(s) for s in sources()):
         return LIB
+    from concurrent.futures import ThreadPoolExecutor
+
     nccl = nccl_dir()
-    cmd = ["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
-           "-Xcompiler", "-fPIC,-fvisibility=hidden", "-shared",
-           "-I", os.path.join(nccl, "include"), "-I", os.path.join(ROOT, "include"),
-           "-o", LIB, os.path.join(HERE, "csrc", "dslash_lib.cu"),
-           "-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2", "-Xlinker", "-rpath=" + os.path.join(nccl, "lib")]
+    objdir = os.path.join(HERE, "build")
+    os.makedirs(objdir, exist_ok=True)
+    common = ["nvcc", *ARCH, "-lineinfo", "-O3", "-std=c++17", "-Xcompiler", "-fPIC,-fvisibility=hidden",
+              "-I", os.path.join(nccl, "include"), "-I", os.path.join(ROOT, "include")]
     if verbose:
-        cmd.insert(1, "-Xptxas=-v")
-        print(" ".join(cmd), file=sys.stderr)
-    subprocess.check_call(cmd)
+        common.append("-Xptxas=-v")
+    cus = sorted(glob.glob(os.path.join(HERE, "csrc", "*.cu")))
+    objs = [os.path.join(objdir, os.path.basename(c)[:-3] + ".o") for c in cus]
+
+    def compile_one(pair):
+        src, obj = pair
+        cmd = common + ["-c", src, "-o", obj]
+        if verbose:
+            print(" ".join(cmd), file=sys.stderr)
+        return subprocess.run(cmd, capture_output=not verbose, text=True)
+
+    with ThreadPoolExecutor(max_workers=min(len(cus), os.cpu_count() or 4)) as ex:
+        results = list(ex.map(compile_one, zip(cus, objs)))
+    for src, r in zip(cus, results):
+        if r.returncode != 0:
+            raise RuntimeError(f"nvcc failed on {src}:\n{r.stderr}")
+    link = ["nvcc", *ARCH, "-shared", "-o", LIB, *objs, "-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
+            "-Xlinker", "-rpath=" + os.path.join(nccl, "lib")]
+    subprocess.check_call(link)
     return LIB
 
 

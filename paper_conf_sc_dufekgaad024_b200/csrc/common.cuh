@@ -131,6 +131,7 @@ struct StencilParams {
     const void* ghost[4][2];   // [mu][side] -> [3][face_vh[mu]] (only where halo[mu])
     int64_t vh;
     int64_t face_vh[4];
+    double long_inv_scale;     // 1/s of the long links N = s W (recon-12 only)
     int L[4];                  // local extents
     int lxh;                   // L[0] / 2
     int parity;                // (target parity + origin sum) & 1, origin sum is even -> target parity

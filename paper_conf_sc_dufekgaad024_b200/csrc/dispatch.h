@@ -1,0 +1,19 @@
+// dispatch.h -- kernel selection across the per-precision translation units (kernels_*.cu).
+#pragma once
+
+#include "common.cuh"
+
+namespace hisq {
+
+typedef void (*StencilFn)(StencilParams);
+
+// Each returns the dslash_kernel instantiation for (ghost, lanes 1/2/4, min blocks 2/3/4,
+// right-hand sides per launch 1/2/4/8) of one (precision, long-link recon) pair.
+StencilFn pick_f64_r18(bool ghost, int lanes, int minb, int nrhs);
+StencilFn pick_f64_r12(bool ghost, int lanes, int minb, int nrhs);
+StencilFn pick_f32_r18(bool ghost, int lanes, int minb, int nrhs);
+StencilFn pick_f32_r12(bool ghost, int lanes, int minb, int nrhs);
+StencilFn pick_mixed_r18(bool ghost, int lanes, int minb, int nrhs);
+StencilFn pick_mixed_r12(bool ghost, int lanes, int minb, int nrhs);
+
+}  // namespace hisq

@@ -6,55 +6,25 @@
 // itself runs in the kernels of stencil.cuh / links.cuh.
 #include <nccl.h>
 
+#include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
 #include <string>
 #include <vector>
 
-#include "hisq_dslash.h"
+#include "handle.h"
 #include "common.cuh"
 #include "links.cuh"
 #include "stencil.cuh"
+#include "dispatch.h"
 
 using namespace hisq;
 
 // ============================================================================ errors
 static thread_local std::string g_last_error;
 
-struct dslash_s {
-    dslash_plan_t plan{};
-    int32_t global_dims[4]{}, proc_grid[4]{};
-    int parity_mask = 0, precision = 0, device = 0;
-    int kernel = DSLASH_KERNEL_DIR2, block = 0, force_halo = 0, overlap = 1, timing = 0, min_blocks = 0;
-    bool loaded = false;
-    void* links[2] = {nullptr, nullptr};
-    char* ghost[4][2] = {};        // source-vector ghost faces [nrhs][3][face_vh]
-    char* zsend[2] = {};           // packed z faces to send (NCCL path)
-    int ghost_rhs = 0;             // number of right-hand sides the ghost buffers hold
-    void* stage_in = nullptr;      // apply_host staging
-    void* stage_out = nullptr;
-    static constexpr int kSlots = 3;  // apply_host_batch pipeline depth
-    void* slot_in[kSlots] = {};
-    void* slot_out[kSlots] = {};
-    cudaStream_t h2d = nullptr, d2h = nullptr;
-    cudaEvent_t ev_in_ready[kSlots] = {}, ev_in_free[kSlots] = {}, ev_out_ready[kSlots] = {},
-                ev_out_free[kSlots] = {}, ev_batch = nullptr;
-    cudaStream_t comm = nullptr;
-    cudaEvent_t ev_start = nullptr, ev_halo = nullptr;
-    bool halo_pending = false;
-    ncclComm_t nccl = nullptr;
-    struct TimedLaunch {
-        cudaEvent_t a, b;
-        int kind;
-    };
-    std::vector<TimedLaunch> tpool;
-    size_t tused = 0;
-    dslash_status err = DSLASH_OK;
-    std::string msg;
-};
-
-static dslash_status fail(dslash_t h, dslash_status st, const char* fmt, ...) {
+dslash_status hisq_fail(dslash_t h, dslash_status st, const char* fmt, ...) {
     char buf[512];
     va_list ap;
     va_start(ap, fmt);
@@ -70,22 +40,7 @@ static dslash_status fail(dslash_t h, dslash_status st, const char* fmt, ...) {
     }
     return st;
 }
-
-#define CU(h, call)                                                                                   \
-    do {                                                                                              \
-        cudaError_t e_ = (call);                                                                      \
-        if (e_ != cudaSuccess)                                                                        \
-            return fail((h), e_ == cudaErrorMemoryAllocation ? DSLASH_ERR_OOM : DSLASH_ERR_CUDA,      \
-                        "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e_));           \
-    } while (0)
-
-#define NC(h, call)                                                                                   \
-    do {                                                                                              \
-        ncclResult_t r_ = (call);                                                                     \
-        if (r_ != ncclSuccess)                                                                        \
-            return fail((h), DSLASH_ERR_NCCL, "%s:%d %s: %s", __FILE__, __LINE__, #call,              \
-                        ncclGetErrorString(r_));                                                      \
-    } while (0)
+#define fail hisq_fail
 
 // ============================================================================ plan (host only)
 extern "C" dslash_status dslash_plan(const int32_t G[4], const int32_t P[4], int32_t rank, int32_t nranks,
@@ -310,6 +265,12 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
         case DSLASH_OPT_TIMING:
             h->timing = value != 0;
             return DSLASH_OK;
+        case DSLASH_OPT_LONG_RECON:
+            if (value != 18 && value != 12) return fail(h, DSLASH_ERR_ARG, "long-link recon %lld must be 18 or 12", (long long)value);
+            if (h->loaded && value != h->recon)
+                return fail(h, DSLASH_ERR_STATE, "long-link recon fixes the link layout: set it before load_links");
+            h->recon = (int)value;
+            return DSLASH_OK;
         case DSLASH_OPT_MIN_BLOCKS:
             if (value != 0 && (value < 2 || value > 4))
                 return fail(h, DSLASH_ERR_ARG, "min_blocks %lld must be 0, 2, 3 or 4", (long long)value);
@@ -372,6 +333,7 @@ extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
     C.lxh = p.local_dims[0] / 2;
     C.vh = p.vh_local;
     C.lanes = lanes_of(h->kernel);
+    C.recon = h->recon;
     int halo_mask = 0;
     for (int d = 2; d < 4; ++d)
         if (p.halo[d]) halo_mask |= 1 << d;
@@ -438,7 +400,53 @@ extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
         C.slab_fat[d] = slab[d][0];
         C.slab_lng[d] = slab[d][1];
     }
-    const size_t link_bytes = (size_t)p.vh_local * 144 * link_elem(h);
+    if (h->recon == 12) {
+        // s from the first local long link: det(s W) = s^3
+        double2 A[9];
+        CUL(cudaMemcpyAsync(A, dlng, sizeof A, cudaMemcpyDeviceToHost, s));
+        CUL(cudaStreamSynchronize(s));
+        auto cm = [](double2 a, double2 b) { return make_double2(a.x * b.x - a.y * b.y, a.x * b.y + a.y * b.x); };
+        auto sub = [](double2 a, double2 b) { return make_double2(a.x - b.x, a.y - b.y); };
+        const double2 m0 = sub(cm(A[4], A[8]), cm(A[5], A[7]));
+        const double2 m1 = sub(cm(A[3], A[8]), cm(A[5], A[6]));
+        const double2 m2 = sub(cm(A[3], A[7]), cm(A[4], A[6]));
+        const double det = cm(A[0], m0).x - cm(A[1], m1).x + cm(A[2], m2).x;
+        const double sc = std::cbrt(det);
+        if (!(std::fabs(sc) > 0.0)) {
+            cleanup();
+            return fail(h, DSLASH_ERR_ARG, "recon-12: first long link has zero determinant");
+        }
+        unsigned long long* dmax;
+        CUL(cudaMalloc(&dmax, sizeof *dmax));
+        tmp.push_back(dmax);
+        CUL(cudaMemsetAsync(dmax, 0, sizeof *dmax, s));
+        auto check = [&](const double2* arr, int64_t nmat) {
+            if (nmat > 0) recon_check_kernel<<<(unsigned)((nmat + 255) / 256), 256, 0, s>>>(arr, nmat, 1.0 / sc, dmax);
+        };
+        check(dlng, V * 4);
+        for (int d = 2; d < 4; ++d)
+            if (slab[d][1]) check(slab[d][1], 3 * (V / p.local_dims[d]) * 4);
+        CUL(cudaGetLastError());
+        unsigned long long bits = 0;
+        CUL(cudaMemcpyAsync(&bits, dmax, sizeof bits, cudaMemcpyDeviceToHost, s));
+        CUL(cudaStreamSynchronize(s));
+        double err;
+        memcpy(&err, &bits, sizeof err);
+        const double tol = (h->precision == DSLASH_F64 ? 1e-12 : 1e-6) * std::fabs(sc);
+        if (!(err <= tol)) {
+            cleanup();
+            return fail(h, DSLASH_ERR_ARG,
+                        "recon-12: long links are not s*SU(3) with one real s = %.17g (max row-2 deviation %.3e)", sc, err);
+        }
+        h->long_inv_scale = 1.0 / sc;
+    }
+    const size_t link_bytes = (size_t)p.vh_local * (h->recon == 12 ? 120 : 144) * link_elem(h);
+    for (int par = 0; par < 2; ++par)  // a recon change alters the size: reallocate
+        if (h->links[par] && h->link_bytes != link_bytes) {
+            cudaFree(h->links[par]);
+            h->links[par] = nullptr;
+        }
+    h->link_bytes = link_bytes;
     for (int par = 0; par < 2; ++par) {
         const bool want = h->parity_mask == DSLASH_BOTH || h->parity_mask == par;
         if (!want) continue;
@@ -571,32 +579,13 @@ static void fill_boxes(StencilParams& K, const dslash_box_t* boxes, int n) {
     for (int b = n; b < kMaxBoxes; ++b) K.box_start[b + 1] = K.box_start[n];
 }
 
-typedef void (*StencilFn)(StencilParams);
-
-template <typename LR, typename VR, int LANES, bool GHOST>
-static StencilFn pick_minb(int minb) {
-    switch (minb) {
-        case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2>;
-        case 3: return dslash_kernel<LR, VR, LANES, GHOST, 3>;
-        default: return dslash_kernel<LR, VR, LANES, GHOST, 4>;
-    }
-}
-
-template <typename LR, typename VR, bool GHOST>
-static StencilFn pick_lanes(int lanes, int minb) {
-    switch (lanes) {
-        case 1: return pick_minb<LR, VR, 1, GHOST>(minb);
-        case 2: return pick_minb<LR, VR, 2, GHOST>(minb);
-        default: return pick_minb<LR, VR, 4, GHOST>(minb);
-    }
-}
-
 template <bool GHOST>
-static StencilFn pick_kernel(int precision, int lanes, int minb) {
+static StencilFn pick_kernel(int precision, int recon, int lanes, int minb, int nrhs) {
+    const bool r12 = recon == 12;
     switch (precision) {
-        case DSLASH_F32: return pick_lanes<float, float, GHOST>(lanes, minb);
-        case DSLASH_MIXED: return pick_lanes<float, double, GHOST>(lanes, minb);
-        default: return pick_lanes<double, double, GHOST>(lanes, minb);
+        case DSLASH_F32: return r12 ? pick_f32_r12(GHOST, lanes, minb, nrhs) : pick_f32_r18(GHOST, lanes, minb, nrhs);
+        case DSLASH_MIXED: return r12 ? pick_mixed_r12(GHOST, lanes, minb, nrhs) : pick_mixed_r18(GHOST, lanes, minb, nrhs);
+        default: return r12 ? pick_f64_r12(GHOST, lanes, minb, nrhs) : pick_f64_r18(GHOST, lanes, minb, nrhs);
     }
 }
 
@@ -605,13 +594,14 @@ static StencilFn pick_kernel(int precision, int lanes, int minb) {
 static int default_block(int lanes) { return lanes == 4 ? 64 : 64; }
 static int default_minb(int lanes) { return lanes == 4 ? 2 : 2; }
 
-static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int kind, cudaStream_t s) {
+// one launch of the stencil over the boxes of K for nrhs (1, 2, 4 or 8) right-hand sides
+static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int kind, cudaStream_t s, int nrhs) {
     const int64_t sites = K.box_start[K.nbox];
     if (sites == 0) return DSLASH_OK;
     const int lanes = lanes_of(h->kernel);
     const int bs = h->block ? h->block : default_block(lanes);
     const int minb = h->min_blocks ? h->min_blocks : default_minb(lanes);
-    const int64_t threads = sites * lanes;
+    const int64_t threads = sites * lanes;  // right-hand sides are register-blocked per thread
     const unsigned grid = (unsigned)((threads + bs - 1) / bs);
     dslash_s::TimedLaunch* tl = nullptr;
     if (h->timing) {
@@ -625,29 +615,64 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
         tl->kind = kind;
         CU(h, cudaEventRecord(tl->a, s));
     }
-    StencilFn fn = ghost ? pick_kernel<true>(h->precision, lanes, minb) : pick_kernel<false>(h->precision, lanes, minb);
+    StencilFn fn = ghost ? pick_kernel<true>(h->precision, h->recon, lanes, minb, nrhs)
+                         : pick_kernel<false>(h->precision, h->recon, lanes, minb, nrhs);
     fn<<<grid, bs, 0, s>>>(K);
     CU(h, cudaGetLastError());
     if (tl) CU(h, cudaEventRecord(tl->b, s));
     return DSLASH_OK;
 }
 
-static dslash_status check_vectors(dslash_t h, const void* out, const void* in) {
+// launch over `boxes` for all nrhs right-hand sides, in chunks of 8, 4, 2, 1
+static dslash_status launch_rhs(dslash_t h, StencilParams K, const dslash_box_t* boxes, int nbox, bool ghost,
+                                int kind, cudaStream_t s, int nrhs) {
+    fill_boxes(K, boxes, nbox);
+    const size_t es = vec_elem(h);
+    const char* in0 = static_cast<const char*>(K.in);
+    char* out0 = static_cast<char*>(K.out);
+    const void* g0[4][2];
+    memcpy(g0, K.ghost, sizeof g0);
+    for (int r0 = 0; r0 < nrhs;) {
+        const int left = nrhs - r0;
+        const int nr = left >= 8 ? 8 : left >= 4 ? 4 : left >= 2 ? 2 : 1;
+        K.in = in0 + (size_t)r0 * 3 * K.vh * es;
+        K.out = out0 + (size_t)r0 * 3 * K.vh * es;
+        for (int d = 0; d < 4; ++d)
+            for (int side = 0; side < 2; ++side)
+                K.ghost[d][side] = g0[d][side] ? static_cast<const char*>(g0[d][side]) + (size_t)r0 * 3 * K.face_vh[d] * es
+                                               : nullptr;
+        dslash_status st = launch(h, K, ghost, kind, s, nr);
+        if (st != DSLASH_OK) return st;
+        r0 += nr;
+    }
+    return DSLASH_OK;
+}
+
+static dslash_status check_vectors(dslash_t h, const void* out, const void* in, int nrhs) {
     if (!out || !in) return fail(h, DSLASH_ERR_ARG, "NULL vector pointer");
     if (((uintptr_t)out & 15) || ((uintptr_t)in & 15)) return fail(h, DSLASH_ERR_ARG, "vectors must be 16-byte aligned");
-    const uintptr_t n = (uintptr_t)(3 * h->plan.vh_local * vec_elem(h));
+    const uintptr_t n = (uintptr_t)nrhs * 3 * h->plan.vh_local * vec_elem(h);
     const uintptr_t a = (uintptr_t)out, b = (uintptr_t)in;
     if (a < b + n && b < a + n) return fail(h, DSLASH_ERR_ARG, "in and out overlap");
     return DSLASH_OK;
 }
 
-extern "C" dslash_status dslash_apply(dslash_t h, void* out, const void* in, int32_t parity, dslash_stream_t stream) {
+static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs,
+                                dslash_stream_t stream);
+
+dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s) {
+    return apply_impl(h, out, in, parity, nrhs, (dslash_stream_t)s);
+}
+
+static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs,
+                                dslash_stream_t stream) {
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (parity & ~1) return fail(h, DSLASH_ERR_ARG, "parity %d not in {0,1}", parity);
+    if (nrhs < 1) return fail(h, DSLASH_ERR_ARG, "nrhs %d < 1", nrhs);
     if (h->parity_mask != DSLASH_BOTH && h->parity_mask != parity)
         return fail(h, DSLASH_ERR_ARG, "parity %d not prepared (parity_mask %d)", parity, h->parity_mask);
     if (!h->loaded) return fail(h, DSLASH_ERR_STATE, "apply before load_links");
-    dslash_status st = check_vectors(h, out, in);
+    dslash_status st = check_vectors(h, out, in, nrhs);
     if (st != DSLASH_OK) return st;
     cudaStream_t s = (cudaStream_t)stream;
     const dslash_plan_t& p = h->plan;
@@ -656,41 +681,47 @@ extern "C" dslash_status dslash_apply(dslash_t h, void* out, const void* in, int
     K.in = in;
     K.out = out;
     K.vh = p.vh_local;
+    K.lxh = p.local_dims[0] / 2;
+    K.parity = parity;
+    K.long_inv_scale = h->long_inv_scale;
     for (int d = 0; d < 4; ++d) {
         K.L[d] = p.local_dims[d];
         K.face_vh[d] = p.face_vh[d];
-        K.ghost[d][0] = h->ghost[d][0];
-        K.ghost[d][1] = h->ghost[d][1];
         if (p.halo[d]) K.halo_mask |= 1 << d;
     }
-    K.lxh = p.local_dims[0] / 2;
-    K.parity = parity;
-    if (!any_halo(p)) {
-        fill_boxes(K, p.interior, p.n_interior);
-        return launch(h, K, false, DSLASH_TIMING_INTERIOR, s);
+    if (!any_halo(p)) return launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
+    if ((st = halo_start_impl(h, in, nrhs, s)) != DSLASH_OK) return st;
+    for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
+        K.ghost[d][0] = h->ghost[d][0];
+        K.ghost[d][1] = h->ghost[d][1];
     }
-    if ((st = halo_start_impl(h, in, 1, s)) != DSLASH_OK) return st;
     if (h->overlap) {
-        fill_boxes(K, p.interior, p.n_interior);
-        if ((st = launch(h, K, false, DSLASH_TIMING_INTERIOR, s)) != DSLASH_OK) return st;
+        st = launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
+        if (st != DSLASH_OK) return st;
         if ((st = dslash_halo_wait(h, stream)) != DSLASH_OK) return st;
-        fill_boxes(K, p.boundary, p.n_boundary);
-        return launch(h, K, true, DSLASH_TIMING_BOUNDARY, s);
+        return launch_rhs(h, K, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, s, nrhs);
     }
     if ((st = dslash_halo_wait(h, stream)) != DSLASH_OK) return st;
+    if (p.n_interior + p.n_boundary > kMaxBoxes) {
+        // 5 boxes (t and z halo): launch the interior part first, then the boundary boxes
+        st = launch_rhs(h, K, p.interior, p.n_interior, true, DSLASH_TIMING_INTERIOR, s, nrhs);
+        if (st != DSLASH_OK) return st;
+        return launch_rhs(h, K, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, s, nrhs);
+    }
     dslash_box_t all[kMaxBoxes];
     int n = 0;
     for (int i = 0; i < p.n_interior; ++i) all[n++] = p.interior[i];
-    for (int i = 0; i < p.n_boundary && n < kMaxBoxes; ++i) all[n++] = p.boundary[i];
-    if (p.n_interior + p.n_boundary > kMaxBoxes) {
-        // 5 boxes (t and z halo): launch the interior part first, then the boundary boxes
-        fill_boxes(K, p.interior, p.n_interior);
-        if ((st = launch(h, K, true, DSLASH_TIMING_INTERIOR, s)) != DSLASH_OK) return st;
-        fill_boxes(K, p.boundary, p.n_boundary);
-        return launch(h, K, true, DSLASH_TIMING_BOUNDARY, s);
-    }
-    fill_boxes(K, all, n);
-    return launch(h, K, true, DSLASH_TIMING_ALL, s);
+    for (int i = 0; i < p.n_boundary; ++i) all[n++] = p.boundary[i];
+    return launch_rhs(h, K, all, n, true, DSLASH_TIMING_ALL, s, nrhs);
+}
+
+extern "C" dslash_status dslash_apply(dslash_t h, void* out, const void* in, int32_t parity, dslash_stream_t stream) {
+    return apply_impl(h, out, in, parity, 1, stream);
+}
+
+extern "C" dslash_status dslash_apply_multi(dslash_t h, int32_t nrhs, void* out, const void* in, int32_t parity,
+                                            dslash_stream_t stream) {
+    return apply_impl(h, out, in, parity, nrhs, stream);
 }
 
 extern "C" dslash_status dslash_apply_host(dslash_t h, void* out_host, const void* in_host, int32_t parity,
@@ -826,6 +857,10 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
             if (e) cudaEventDestroy(e);
     }
     if (h->ev_batch) cudaEventDestroy(h->ev_batch);
+    for (void* v : h->cg_vec)
+        if (v) cudaFree(v);
+    if (h->cg_partial) cudaFree(h->cg_partial);
+    if (h->cg_scalar) cudaFree(h->cg_scalar);
     if (h->h2d) cudaStreamDestroy(h->h2d);
     if (h->d2h) cudaStreamDestroy(h->d2h);
     for (auto& t : h->tpool) {

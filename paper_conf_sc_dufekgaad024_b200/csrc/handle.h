@@ -1,0 +1,73 @@
+// handle.h -- the library handle and the host-side helpers shared by dslash_lib.cu and solver.cu.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <string>
+#include <vector>
+
+#include "hisq_dslash.h"
+
+struct dslash_s {
+    dslash_plan_t plan{};
+    int32_t global_dims[4]{}, proc_grid[4]{};
+    int parity_mask = 0, precision = 0, device = 0;
+    int kernel = DSLASH_KERNEL_DIR2, block = 0, force_halo = 0, overlap = 1, timing = 0, min_blocks = 0;
+    int recon = 18;
+    double long_inv_scale = 1.0;
+    size_t link_bytes = 0;
+    bool loaded = false;
+    void* links[2] = {nullptr, nullptr};
+    char* ghost[4][2] = {};        // source-vector ghost faces [nrhs][3][face_vh]
+    char* zsend[2] = {};           // packed z faces to send (NCCL path)
+    int ghost_rhs = 0;             // number of right-hand sides the ghost buffers hold
+    void* stage_in = nullptr;      // apply_host staging
+    void* stage_out = nullptr;
+    static constexpr int kSlots = 3;  // apply_host_batch pipeline depth
+    void* slot_in[kSlots] = {};
+    void* slot_out[kSlots] = {};
+    cudaStream_t h2d = nullptr, d2h = nullptr;
+    cudaEvent_t ev_in_ready[kSlots] = {}, ev_in_free[kSlots] = {}, ev_out_ready[kSlots] = {},
+                ev_out_free[kSlots] = {}, ev_batch = nullptr;
+    cudaStream_t comm = nullptr;
+    cudaEvent_t ev_start = nullptr, ev_halo = nullptr;
+    bool halo_pending = false;
+    ncclComm_t nccl = nullptr;
+    struct TimedLaunch {
+        cudaEvent_t a, b;
+        int kind;
+    };
+    std::vector<TimedLaunch> tpool;
+    size_t tused = 0;
+    // conjugate-gradient scratch (solver.cu): r, p, q on the target parity, t on the other one,
+    // block partial sums and the reduced scalars
+    void* cg_vec[4] = {};
+    double* cg_partial = nullptr;
+    double* cg_scalar = nullptr;
+    dslash_status err = DSLASH_OK;
+    std::string msg;
+};
+
+// Record a failure on the handle (first error wins) or, with h == NULL, in the thread's last
+// error; returns st.
+dslash_status hisq_fail(dslash_t h, dslash_status st, const char* fmt, ...);
+
+#define CU(h, call)                                                                                   \
+    do {                                                                                              \
+        cudaError_t e_ = (call);                                                                      \
+        if (e_ != cudaSuccess)                                                                        \
+            return hisq_fail((h), e_ == cudaErrorMemoryAllocation ? DSLASH_ERR_OOM : DSLASH_ERR_CUDA, \
+                             "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e_));      \
+    } while (0)
+
+#define NC(h, call)                                                                                   \
+    do {                                                                                              \
+        ncclResult_t r_ = (call);                                                                     \
+        if (r_ != ncclSuccess)                                                                        \
+            return hisq_fail((h), DSLASH_ERR_NCCL, "%s:%d %s: %s", __FILE__, __LINE__, #call,         \
+                             ncclGetErrorString(r_));                                                 \
+    } while (0)
+
+// out = D in on target parity `parity` for nrhs back-to-back vectors (dslash_lib.cu)
+dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s);

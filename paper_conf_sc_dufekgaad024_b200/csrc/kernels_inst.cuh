@@ -1,0 +1,49 @@
+// kernels_inst.cuh -- instantiation table of dslash_kernel for one (LR, VR, RECON); included by
+// the kernels_*.cu translation units, which build in parallel.
+// Instantiated: every (lanes, ghost) with MINB 2/3/4 for one right-hand side, with MINB 2
+// (the measured best) for 2 and 4 right-hand sides per launch, and MINB 1 for 8 (24 complex
+// accumulators per thread do not fit 128 registers).
+#pragma once
+
+#include "dispatch.h"
+#include "stencil.cuh"
+
+namespace hisq {
+
+template <typename LR, typename VR, int LANES, bool GHOST, int RECON>
+StencilFn pick_minb(int minb, int nrhs) {
+    switch (nrhs) {
+        case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 2>;
+        case 4: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4>;
+        case 8: return dslash_kernel<LR, VR, LANES, GHOST, 1, RECON, 8>;  // 8 x 3 accumulators: <= 255 regs
+        default: break;
+    }
+    switch (minb) {
+        case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON>;
+        case 3: return dslash_kernel<LR, VR, LANES, GHOST, 3, RECON>;
+        default: return dslash_kernel<LR, VR, LANES, GHOST, 4, RECON>;
+    }
+}
+
+template <typename LR, typename VR, bool GHOST, int RECON>
+StencilFn pick_lanes(int lanes, int minb, int nrhs) {
+    switch (lanes) {
+        case 1: return pick_minb<LR, VR, 1, GHOST, RECON>(minb, nrhs);
+        case 2: return pick_minb<LR, VR, 2, GHOST, RECON>(minb, nrhs);
+        default: return pick_minb<LR, VR, 4, GHOST, RECON>(minb, nrhs);
+    }
+}
+
+template <typename LR, typename VR, int RECON>
+StencilFn pick_any(bool ghost, int lanes, int minb, int nrhs) {
+    return ghost ? pick_lanes<LR, VR, true, RECON>(lanes, minb, nrhs) : pick_lanes<LR, VR, false, RECON>(lanes, minb, nrhs);
+}
+
+}  // namespace hisq
+
+#define HISQ_DEFINE_PICK(NAME, LR, VR, RECON)                                  \
+    namespace hisq {                                                           \
+    StencilFn NAME(bool ghost, int lanes, int minb, int nrhs) {                \
+        return pick_any<LR, VR, RECON>(ghost, lanes, minb, nrhs);              \
+    }                                                                          \
+    }

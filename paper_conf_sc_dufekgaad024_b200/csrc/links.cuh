@@ -28,6 +28,7 @@ struct LinkConvParams {
     int parity;
     int halo_mask;
     int lanes;                    // layout of the kernel that will read the links: 1, 2 or 4
+    int recon;                    // 18 = full matrices, 12 = long links keep rows 0 and 1 only
 };
 
 __device__ __forceinline__ const double2* canon_link(const LinkConvParams& P, bool is_long, int mu, int x, int y,
@@ -70,7 +71,8 @@ __global__ void convert_links_kernel(const LinkConvParams P) {
     const bool is_long = l >= 2;
     const int back = (l == 1) ? 1 : (l == 3) ? 3 : 0;
     const double2* A = canon_link(P, is_long, mu, x, y, z, t, back);
-    for (int i = 0; i < 3; ++i)
+    const int rows = (P.recon == 12 && is_long) ? 2 : 3;
+    for (int i = 0; i < rows; ++i)
         for (int j = 0; j < 3; ++j) {
             double2 v;
             if (back) {  // (A^dag)_{ij} = conj(A_{ji})
@@ -80,11 +82,37 @@ __global__ void convert_links_kernel(const LinkConvParams P) {
                 v = A[3 * i + j];
             }
             const int e = 3 * i + j;
-            const int64_t o = P.lanes == 1   ? link_index<1>(mu, l, e, P.vh, cb)
-                              : P.lanes == 2 ? link_index<2>(mu, l, e, P.vh, cb)
-                                             : link_index<4>(mu, l, e, P.vh, cb);
+            int64_t o;
+            if (P.recon == 12)
+                o = P.lanes == 1 ? link_index<1, 12>(mu, l, e, P.vh, cb)
+                  : P.lanes == 2 ? link_index<2, 12>(mu, l, e, P.vh, cb)
+                                 : link_index<4, 12>(mu, l, e, P.vh, cb);
+            else
+                o = P.lanes == 1 ? link_index<1>(mu, l, e, P.vh, cb)
+                  : P.lanes == 2 ? link_index<2>(mu, l, e, P.vh, cb)
+                                 : link_index<4>(mu, l, e, P.vh, cb);
             static_cast<L2*>(P.links)[o] = to_cplx<L2>(v);
         }
+}
+
+// recon-12 admissibility: for every canonical long link N (fp64 input), the largest deviation
+// |row2 - conj(row0 x row1)/s| over its 3 entries, as a non-negative double whose bit pattern
+// orders like an unsigned integer (atomicMax on the bits).
+__global__ void recon_check_kernel(const double2* lng, int64_t nmat, double inv_s, unsigned long long* max_bits) {
+    const int64_t m = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    double err = 0.0;
+    if (m < nmat) {
+        const double2* A = lng + m * 9;
+        double2 U[9];
+        for (int e = 0; e < 9; ++e) U[e] = A[e];
+        double2 R[9];
+        for (int e = 0; e < 9; ++e) R[e] = U[e];
+        reconstruct_row2(R, inv_s);
+        for (int j = 0; j < 3; ++j) err = fmax(err, fmax(fabs(R[6 + j].x - U[6 + j].x), fabs(R[6 + j].y - U[6 + j].y)));
+    }
+    // warp max, then one atomic per warp
+    for (int off = 16; off; off >>= 1) err = fmax(err, __shfl_xor_sync(0xffffffffu, err, off));
+    if ((threadIdx.x & 31) == 0) atomicMax(max_bits, (unsigned long long)__double_as_longlong(err));
 }
 
 }  // namespace hisq

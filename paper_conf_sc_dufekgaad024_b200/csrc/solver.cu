@@ -1,0 +1,234 @@
+// solver.cu -- the even-odd normal operator and a conjugate-gradient solver on top of the
+// single-parity Dslash ("both-parity D^dag D = -D_oe D_eo, plus CG", the step
+// downstream of the Dslash in su3_rhmd_hisq).
+//
+// With D anti-Hermitian (D_{p,1-p} = -D_{1-p,p}^dag, pin P3), the operator
+//     A_p = m^2 - D_{p,1-p} D_{1-p,p} = m^2 + D_{1-p,p}^dag D_{1-p,p}
+// is Hermitian positive definite on parity p for m != 0, and CG solves A_p x = b.
+// Dot products are reduced deterministically (fixed block partition, fixed final order) and,
+// with several ranks, summed with ncclAllReduce: the solver's one true collective.
+#include <cmath>
+
+#include "common.cuh"
+#include "handle.h"
+
+namespace {
+
+constexpr int kRedThreads = 256;
+constexpr int kRedBlocks = 592;  // 4 x 148 SMs; fixed, so the summation order never changes
+
+// block-level sum of v (all threads call); result valid in thread 0
+__device__ double block_sum(double v) {
+    __shared__ double warp_part[kRedThreads / 32];
+#pragma unroll
+    for (int off = 16; off; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+    if ((threadIdx.x & 31) == 0) warp_part[threadIdx.x >> 5] = v;
+    __syncthreads();
+    double s = 0.0;
+    if (threadIdx.x == 0)
+        for (int w = 0; w < kRedThreads / 32; ++w) s += warp_part[w];
+    return s;
+}
+
+// q = m2 p - q ; partial[block] = sum Re(conj(p) q)
+__global__ void __launch_bounds__(kRedThreads) k_normal_finish(const double2* __restrict__ p, double2* __restrict__ q,
+                                                               double m2, int64_t n, double* __restrict__ partial) {
+    double acc = 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double2 a = p[i];
+        double2 b = q[i];
+        b.x = m2 * a.x - b.x;
+        b.y = m2 * a.y - b.y;
+        q[i] = b;
+        acc += a.x * b.x + a.y * b.y;
+    }
+    const double s = block_sum(acc);
+    if (partial && threadIdx.x == 0) partial[blockIdx.x] = s;
+}
+
+// partial[block] = sum |v|^2
+__global__ void __launch_bounds__(kRedThreads) k_norm2(const double2* __restrict__ v, int64_t n,
+                                                       double* __restrict__ partial) {
+    double acc = 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double2 a = v[i];
+        acc += a.x * a.x + a.y * a.y;
+    }
+    const double s = block_sum(acc);
+    if (threadIdx.x == 0) partial[blockIdx.x] = s;
+}
+
+// x += alpha p ; r -= alpha q ; partial[block] = sum |r|^2
+__global__ void __launch_bounds__(kRedThreads) k_cg_update(double2* __restrict__ x, double2* __restrict__ r,
+                                                           const double2* __restrict__ p, const double2* __restrict__ q,
+                                                           double alpha, int64_t n, double* __restrict__ partial) {
+    double acc = 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        double2 xi = x[i], ri = r[i];
+        const double2 pi = p[i], qi = q[i];
+        xi.x = fma(alpha, pi.x, xi.x);
+        xi.y = fma(alpha, pi.y, xi.y);
+        ri.x = fma(-alpha, qi.x, ri.x);
+        ri.y = fma(-alpha, qi.y, ri.y);
+        x[i] = xi;
+        r[i] = ri;
+        acc += ri.x * ri.x + ri.y * ri.y;
+    }
+    const double s = block_sum(acc);
+    if (threadIdx.x == 0) partial[blockIdx.x] = s;
+}
+
+// p = r + beta p
+__global__ void k_cg_direction(double2* __restrict__ p, const double2* __restrict__ r, double beta, int64_t n) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double2 ri = r[i];
+        double2 pi = p[i];
+        pi.x = fma(beta, pi.x, ri.x);
+        pi.y = fma(beta, pi.y, ri.y);
+        p[i] = pi;
+    }
+}
+
+// r = b - r  (true residual from r = A x)
+__global__ void k_sub_from(double2* __restrict__ r, const double2* __restrict__ b, int64_t n) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double2 bi = b[i];
+        double2 ri = r[i];
+        ri.x = bi.x - ri.x;
+        ri.y = bi.y - ri.y;
+        r[i] = ri;
+    }
+}
+
+// out[0] = sum_{k < n} partial[k] in index order (one thread: deterministic)
+__global__ void k_finalize(const double* __restrict__ partial, int n, double* __restrict__ out) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) {
+        double s = 0.0;
+        for (int k = 0; k < n; ++k) s += partial[k];
+        out[0] = s;
+    }
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------------------- host helpers
+static dslash_status need_scratch(dslash_t h) {
+    const size_t bytes = 3 * (size_t)h->plan.vh_local * sizeof(double2);
+    for (void*& v : h->cg_vec)
+        if (!v) CU(h, cudaMalloc(&v, bytes));
+    if (!h->cg_partial) CU(h, cudaMalloc(&h->cg_partial, kRedBlocks * sizeof(double)));
+    if (!h->cg_scalar) CU(h, cudaMalloc(&h->cg_scalar, 2 * sizeof(double)));
+    return DSLASH_OK;
+}
+
+// the partials of one reduction -> global sum (all ranks) -> host value
+static dslash_status reduce_to_host(dslash_t h, cudaStream_t s, double* value) {
+    k_finalize<<<1, 32, 0, s>>>(h->cg_partial, kRedBlocks, h->cg_scalar);
+    CU(h, cudaGetLastError());
+    if (h->nccl) NC(h, ncclAllReduce(h->cg_scalar, h->cg_scalar, 1, ncclDouble, ncclSum, h->nccl, s));
+    CU(h, cudaMemcpyAsync(value, h->cg_scalar, sizeof(double), cudaMemcpyDeviceToHost, s));
+    CU(h, cudaStreamSynchronize(s));
+    return DSLASH_OK;
+}
+
+static dslash_status check_solver_args(dslash_t h, const void* a, const void* b, int32_t parity) {
+    if (!h) return hisq_fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (parity & ~1) return hisq_fail(h, DSLASH_ERR_ARG, "parity %d not in {0,1}", parity);
+    if (h->parity_mask != DSLASH_BOTH)
+        return hisq_fail(h, DSLASH_ERR_ARG, "the normal operator applies both parities: create with DSLASH_BOTH");
+    if (h->precision == DSLASH_F32)
+        return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the solver works on fp64 vectors (DSLASH_F64 or DSLASH_MIXED)");
+    if (!h->loaded) return hisq_fail(h, DSLASH_ERR_STATE, "solver before load_links");
+    if (!a || !b || ((uintptr_t)a & 15) || ((uintptr_t)b & 15))
+        return hisq_fail(h, DSLASH_ERR_ARG, "NULL or misaligned vector");
+    const uintptr_t n = 3 * (uintptr_t)h->plan.vh_local * sizeof(double2);
+    if ((uintptr_t)a < (uintptr_t)b + n && (uintptr_t)b < (uintptr_t)a + n)
+        return hisq_fail(h, DSLASH_ERR_ARG, "vectors overlap");
+    return DSLASH_OK;
+}
+
+// q = A p, and (if partial) the block partials of Re<p, q>
+static dslash_status normal_apply(dslash_t h, double2* q, const double2* p, int32_t parity, double m2,
+                                  double2* tmp, cudaStream_t s, bool dot) {
+    dslash_status st = hisq_apply(h, tmp, p, 1 - parity, 1, s);  // t = D_{1-p,p} p
+    if (st != DSLASH_OK) return st;
+    if ((st = hisq_apply(h, q, tmp, parity, 1, s)) != DSLASH_OK) return st;  // q = D_{p,1-p} t
+    const int64_t n = 3 * h->plan.vh_local;
+    k_normal_finish<<<kRedBlocks, kRedThreads, 0, s>>>(p, q, m2, n, dot ? h->cg_partial : nullptr);
+    CU(h, cudaGetLastError());
+    return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_normal_apply(dslash_t h, void* out, const void* in, int32_t parity, double mass,
+                                             dslash_stream_t stream) {
+    dslash_status st = check_solver_args(h, out, in, parity);
+    if (st != DSLASH_OK) return st;
+    if ((st = need_scratch(h)) != DSLASH_OK) return st;
+    return normal_apply(h, (double2*)out, (const double2*)in, parity, mass * mass, (double2*)h->cg_vec[3],
+                        (cudaStream_t)stream, false);
+}
+
+extern "C" dslash_status dslash_cg(dslash_t h, void* x_out, const void* b_in, int32_t parity, double mass,
+                                   double rel_tol, int32_t max_iter, int32_t* iters, double* rel_resid,
+                                   dslash_stream_t stream) {
+    dslash_status st = check_solver_args(h, x_out, b_in, parity);
+    if (st != DSLASH_OK) return st;
+    if (!(rel_tol > 0.0) || max_iter < 1) return hisq_fail(h, DSLASH_ERR_ARG, "rel_tol must be > 0 and max_iter >= 1");
+    if (!(mass != 0.0)) return hisq_fail(h, DSLASH_ERR_ARG, "mass must be nonzero (A is then positive definite)");
+    if ((st = need_scratch(h)) != DSLASH_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t n = 3 * h->plan.vh_local;
+    const size_t bytes = n * sizeof(double2);
+    const double m2 = mass * mass;
+    double2* x = (double2*)x_out;
+    const double2* b = (const double2*)b_in;
+    double2* r = (double2*)h->cg_vec[0];
+    double2* p = (double2*)h->cg_vec[1];
+    double2* q = (double2*)h->cg_vec[2];
+    double2* t = (double2*)h->cg_vec[3];
+    // x = 0, r = b, p = b
+    CU(h, cudaMemsetAsync(x, 0, bytes, s));
+    CU(h, cudaMemcpyAsync(r, b, bytes, cudaMemcpyDeviceToDevice, s));
+    CU(h, cudaMemcpyAsync(p, b, bytes, cudaMemcpyDeviceToDevice, s));
+    double bb = 0.0, rr = 0.0, pq = 0.0;
+    k_norm2<<<kRedBlocks, kRedThreads, 0, s>>>(b, n, h->cg_partial);
+    CU(h, cudaGetLastError());
+    if ((st = reduce_to_host(h, s, &bb)) != DSLASH_OK) return st;
+    int k = 0;
+    if (bb > 0.0) {
+        rr = bb;
+        const double stop = rel_tol * rel_tol * bb;
+        for (k = 1; k <= max_iter; ++k) {
+            if ((st = normal_apply(h, q, p, parity, m2, t, s, true)) != DSLASH_OK) return st;  // q = A p
+            if ((st = reduce_to_host(h, s, &pq)) != DSLASH_OK) return st;
+            const double alpha = rr / pq;
+            k_cg_update<<<kRedBlocks, kRedThreads, 0, s>>>(x, r, p, q, alpha, n, h->cg_partial);
+            CU(h, cudaGetLastError());
+            double rr_new = 0.0;
+            if ((st = reduce_to_host(h, s, &rr_new)) != DSLASH_OK) return st;
+            if (rr_new <= stop) {
+                rr = rr_new;
+                break;
+            }
+            k_cg_direction<<<kRedBlocks, kRedThreads, 0, s>>>(p, r, rr_new / rr, n);
+            CU(h, cudaGetLastError());
+            rr = rr_new;
+        }
+        if (k > max_iter) k = max_iter;
+    }
+    // true residual |b - A x| / |b|
+    double res = 0.0;
+    if (bb > 0.0) {
+        if ((st = normal_apply(h, r, x, parity, m2, t, s, false)) != DSLASH_OK) return st;
+        k_sub_from<<<kRedBlocks, kRedThreads, 0, s>>>(r, b, n);
+        k_norm2<<<kRedBlocks, kRedThreads, 0, s>>>(r, n, h->cg_partial);
+        CU(h, cudaGetLastError());
+        double rt = 0.0;
+        if ((st = reduce_to_host(h, s, &rt)) != DSLASH_OK) return st;
+        res = std::sqrt(rt / bb);
+    }
+    if (iters) *iters = k;
+    if (rel_resid) *rel_resid = res;
+    // not converged: reported, but not a sticky handle error
+    return (bb > 0.0 && !(rr <= rel_tol * rel_tol * bb)) ? DSLASH_ERR_NOT_CONVERGED : DSLASH_OK;
+}

@@ -25,15 +25,41 @@
 namespace hisq {
 
 // Internal link layout, for a kernel with LANES lanes per site (lane j streams directions
-// mu = k*LANES + j, k < 4/LANES).  Element e = 3*i + j of 3x3 matrix l (0 = Ff (+1 hop),
-// 1 = Fb (-1), 2 = Nf (+3), 3 = Nb (-3)) in direction mu of target site cb lives at
-//   links[(((l*9 + e) * K + k) * vh + cb) * LANES + j],   K = 4 / LANES,
-// so at every load instruction the lanes of a warp read one contiguous 512-byte span, and the
-// 9 elements of a matrix are 4*vh double2 apart.
-template <int LANES>
+// mu = k*LANES + j, k < 4/LANES).  Matrix l (0 = Ff (+1 hop), 1 = Fb (-1), 2 = Nf (+3),
+// 3 = Nb (-3)) of direction mu at target site cb stores its elements e (row-major 3*i + j) at
+//   links[(((base(l) + e) * K + k) * vh + cb) * LANES + j],   K = 4 / LANES,
+// base(l) = 9 l without compression; with RECON = 12 the long matrices keep only rows 0 and 1
+// (e < 6), base(2) = 18, base(3) = 24.  At every load instruction the lanes of a warp read one
+// contiguous span, and consecutive elements of a matrix are 4*vh complex apart.
+template <int RECON>
+__host__ __device__ __forceinline__ int elem_base(int l) {
+    return (RECON == 12 && l >= 2) ? 18 + (l - 2) * 6 : l * 9;
+}
+template <int RECON>
+__host__ __device__ __forceinline__ int elems_of(int l) {
+    return (RECON == 12 && l >= 2) ? 6 : 9;
+}
+template <int LANES, int RECON = 18>
 __host__ __device__ __forceinline__ int64_t link_index(int mu, int l, int e, int64_t vh, int64_t cb) {
     constexpr int K = 4 / LANES;
-    return ((((int64_t)(l * 9 + e) * K + mu / LANES) * vh + cb) * LANES) + (mu % LANES);
+    return ((((int64_t)(elem_base<RECON>(l) + e) * K + mu / LANES) * vh + cb) * LANES) + (mu % LANES);
+}
+
+// Row 2 of s*W, W in SU(3), from rows 0 and 1: conj(r0 x r1) / s  (QUDA/MILC "recon-12";
+// the back-link N(x-3mu)^dag = s W^dag has the same form).  inv_s = 1/s.
+template <typename V2, typename R>
+__device__ __forceinline__ void reconstruct_row2(V2 U[9], R inv_s) {
+#pragma unroll
+    for (int j = 0; j < 3; ++j) {
+        const int j1 = (j + 1) % 3, j2 = (j + 2) % 3;
+        // x = r0[j1] r1[j2] - r0[j2] r1[j1]
+        R xr = U[j1].x * U[3 + j2].x - U[j1].y * U[3 + j2].y;
+        R xi = U[j1].x * U[3 + j2].y + U[j1].y * U[3 + j2].x;
+        xr -= U[j2].x * U[3 + j1].x - U[j2].y * U[3 + j1].y;
+        xi -= U[j2].x * U[3 + j1].y + U[j2].y * U[3 + j1].x;
+        U[6 + j].x = xr * inv_s;
+        U[6 + j].y = -xi * inv_s;
+    }
 }
 
 struct Site {
@@ -74,7 +100,7 @@ struct SrcRef {
 // outside [0, L); otherwise coordinates wrap periodically (two conditional steps suffice for
 // |h| <= 3 and L >= 2).
 template <typename V2, bool GHOST>
-__device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, int mu, int h, const Site& s) {
+__device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, int mu, int h, const Site& s, int rhs) {
     const int c = mu == 0 ? s.x : mu == 1 ? s.y : mu == 2 ? s.z : s.t;
     const int L = P.L[mu];
     int cn = c + h;
@@ -86,7 +112,7 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, int mu, int
             f = s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (s.z + (int64_t)P.L[2] * d));
         else
             f = s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (d + 3 * (int64_t)s.t));
-        return {static_cast<const V2*>(P.ghost[mu][side]) + f, P.face_vh[mu]};
+        return {static_cast<const V2*>(P.ghost[mu][side]) + (int64_t)rhs * 3 * P.face_vh[mu] + f, P.face_vh[mu]};
     }
     if (cn < 0) cn += L;
     if (cn < 0) cn += L;
@@ -101,7 +127,7 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, int mu, int
                                    : (int64_t)P.lxh * P.L[1] * P.L[2];
         idx = s.cb + (int64_t)(cn - c) * st;
     }
-    return {static_cast<const V2*>(P.in) + idx, P.vh};
+    return {static_cast<const V2*>(P.in) + (int64_t)rhs * 3 * P.vh + idx, P.vh};
 }
 
 // acc (+/-)= U v for a 3x3 matrix whose 9 elements are U[e]
@@ -123,10 +149,14 @@ __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[
 // 4 = one lane per direction, the paper's 3LP-1 site x direction split with a shuffle
 // reduction instead of local memory + barrier).  MINB = minimum resident 256-thread blocks per
 // SM, which caps registers (2 -> 128, 3 -> 80, 4 -> 64) and so trades per-thread ILP against
-// occupancy.  GHOST selects the boundary variant that reads halo faces.  LR is the real type
-// of the stored links, VR that of the vectors and of the accumulation (double/double = fp64,
-// float/float = fp32, float/double = mixed: fp32 links widened to fp64 before the FMAs).
-template <typename LR, typename VR, int LANES, bool GHOST, int MINB>
+// occupancy.  NRHS right-hand sides ([NRHS][3][vh] vectors) are register-blocked: each thread
+// loads a link matrix once and applies it to NRHS vectors, so the link stream is shared
+// (the L25 Domain-Wall intensity argument).  GHOST selects the boundary
+// variant that reads halo faces.  LR is the real type of the stored links, VR that of the
+// vectors and of the accumulation (double/double = fp64, float/float = fp32, float/double =
+// mixed: fp32 links widened to fp64 before the FMAs).  RECON 12 rebuilds row 2 of the long
+// links.  The summation order per (site, rhs) is the same for every NRHS, MINB and block size.
+template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1>
 __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P) {
     static_assert(LANES == 1 || LANES == 2 || LANES == 4, "LANES must divide 4");
     using L2 = cplx_t<LR>;
@@ -134,12 +164,14 @@ __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P
     constexpr int K = 4 / LANES;
     const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int lane = (LANES == 1) ? 0 : (int)(threadIdx.x & (LANES - 1));
-    const int64_t site = (LANES == 1) ? gid : (gid / LANES);
+    const int64_t site = gid / LANES;
     const bool valid = site < P.box_start[P.nbox];
     if (LANES == 1 && !valid) return;
-    V2 acc[3];
+    V2 acc[NRHS][3];
 #pragma unroll
-    for (int c = 0; c < 3; ++c) acc[c].x = acc[c].y = VR(0);
+    for (int r = 0; r < NRHS; ++r)
+#pragma unroll
+        for (int c = 0; c < 3; ++c) acc[r][c].x = acc[r][c].y = VR(0);
     Site s;
     if (valid) {
         const uint64_t pol_stream = policy_evict_first();
@@ -152,19 +184,24 @@ __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P
 #pragma unroll
             for (int l = 0; l < 4; ++l) {
                 const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
-                const SrcRef<V2> src = source<V2, GHOST>(P, mu, h, s);
-                V2 v[3];
-#pragma unroll
-                for (int c = 0; c < 3; ++c) v[c] = ld_reuse(src.p + c * src.stride, pol_keep);
-                const L2* lp = links + link_index<LANES>(mu, l, 0, P.vh, s.cb);
+                const SrcRef<V2> src = source<V2, GHOST>(P, mu, h, s, 0);
+                const L2* lp = links + link_index<LANES, RECON>(mu, l, 0, P.vh, s.cb);
                 V2 U[9];
 #pragma unroll
-                for (int e = 0; e < 9; ++e)
+                for (int e = 0; e < elems_of<RECON>(l); ++e)
                     U[e] = to_cplx<V2>(widen(ld_stream(lp + (int64_t)e * 4 * P.vh, pol_stream)));
-                if (l & 1)
-                    matvec_acc<true>(acc, U, v);
-                else
-                    matvec_acc<false>(acc, U, v);
+                if (elems_of<RECON>(l) == 6) reconstruct_row2(U, (VR)P.long_inv_scale);
+#pragma unroll
+                for (int r = 0; r < NRHS; ++r) {
+                    const int64_t roff = (int64_t)r * 3 * src.stride;  // [rhs][3][vh or face_vh]
+                    V2 v[3];
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) v[c] = ld_reuse(src.p + roff + c * src.stride, pol_keep);
+                    if (l & 1)
+                        matvec_acc<true>(acc[r], U, v);
+                    else
+                        matvec_acc<false>(acc[r], U, v);
+                }
             }
         }
     }
@@ -172,28 +209,33 @@ __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P
         // butterfly over the lanes of a site: every lane ends with the same bits
         // (((p0+p1)+(p2+p3)) by commutativity of each pairwise add)
 #pragma unroll
-        for (int c = 0; c < 3; ++c) {
+        for (int r = 0; r < NRHS; ++r)
 #pragma unroll
-            for (int off = 1; off < LANES; off <<= 1) {
-                acc[c].x += __shfl_xor_sync(0xffffffffu, acc[c].x, off);
-                acc[c].y += __shfl_xor_sync(0xffffffffu, acc[c].y, off);
+            for (int c = 0; c < 3; ++c) {
+#pragma unroll
+                for (int off = 1; off < LANES; off <<= 1) {
+                    acc[r][c].x += __shfl_xor_sync(0xffffffffu, acc[r][c].x, off);
+                    acc[r][c].y += __shfl_xor_sync(0xffffffffu, acc[r][c].y, off);
+                }
             }
-        }
     }
     if (!valid) return;
-    V2* out = static_cast<V2*>(P.out);
-    if (LANES == 1) {
 #pragma unroll
-        for (int c = 0; c < 3; ++c) st_stream(out + c * P.vh + s.cb, acc[c]);
-    } else if (LANES == 2) {
-        if (lane == 0) {
-            st_stream(out + s.cb, acc[0]);
-            st_stream(out + P.vh + s.cb, acc[1]);
+    for (int r = 0; r < NRHS; ++r) {
+        V2* out = static_cast<V2*>(P.out) + (int64_t)r * 3 * P.vh;
+        if (LANES == 1) {
+#pragma unroll
+            for (int c = 0; c < 3; ++c) st_stream(out + c * P.vh + s.cb, acc[r][c]);
+        } else if (LANES == 2) {
+            if (lane == 0) {
+                st_stream(out + s.cb, acc[r][0]);
+                st_stream(out + P.vh + s.cb, acc[r][1]);
+            } else {
+                st_stream(out + 2 * P.vh + s.cb, acc[r][2]);
+            }
         } else {
-            st_stream(out + 2 * P.vh + s.cb, acc[2]);
+            if (lane < 3) st_stream(out + lane * P.vh + s.cb, lane == 0 ? acc[r][0] : lane == 1 ? acc[r][1] : acc[r][2]);
         }
-    } else {
-        if (lane < 3) st_stream(out + lane * P.vh + s.cb, lane == 0 ? acc[0] : lane == 1 ? acc[1] : acc[2]);
     }
 }
 

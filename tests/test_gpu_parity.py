@@ -245,6 +245,101 @@ def test_reduced_precision_self_halo_bitwise(torch_cuda, precision):
     assert torch.equal(outs[0], outs[1])
 
 
+@pytest.mark.parametrize("kernel", KERNELS)
+@pytest.mark.parametrize("precision,tol", [("f64", 1e-12), ("mixed", 1e-5), ("f32", 1e-5)])
+@pytest.mark.parametrize("dims", [(8, 10, 12, 14), (4, 4, 4, 4)])
+def test_recon12_vs_oracle(torch_cuda, kernel, precision, tol, dims):
+    """§8(f)-2: long links stored as two rows, row 2 rebuilt as conj(r0 x r1)/s in registers."""
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    fat, lng = fieldgen.workload_links(dims)
+    psi = fieldgen.vector(dims, fieldgen.SEED_PSI)
+    for parity in (0, 1):
+        ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, parity), parity)
+        src = torch.from_numpy(fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 1 - parity))
+        with Dslash(dims, kernel=kernel, precision=precision, recon=12) as D:
+            D.load_links(fat, lng)
+            got = D(src.to(D.dtype).cuda(), parity).cpu().numpy().astype(np.complex128)
+        assert oracle.normwise_error(got, ref) <= tol
+
+
+def test_recon12_self_halo_and_scale(torch_cuda):
+    """recon-12 through the halo path is bitwise the unpartitioned recon-12 result; a long-link
+    scale other than -1/24 is found from det(N) = s^3."""
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 8, 8, 12)
+    fat = fieldgen.links(dims, 1)
+    lng = fieldgen.links(dims, 2, scale=0.37)
+    psi = fieldgen.vector(dims, 3)
+    src = torch.from_numpy(fieldgen.vector_cb(dims, 3, 0)).cuda()
+    outs = []
+    for mask in (0, 0xC):
+        with Dslash(dims, recon=12, force_halo=mask) as D:
+            D.load_links(fat, lng)
+            outs.append(D(src, 1).cpu())
+    assert torch.equal(outs[0], outs[1])
+    ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, 1), 1)
+    assert oracle.normwise_error(outs[0].numpy(), ref) <= 1e-12
+
+
+def test_recon12_rejects_non_su3_long_links(torch_cuda):
+    from paper_conf_sc_dufekgaad024_b200 import Dslash, _abi
+    dims = (8, 8, 8, 8)
+    fat = fieldgen.links(dims, 1)
+    with Dslash(dims, recon=12) as D:
+        with pytest.raises(_abi.DslashError) as e:
+            D.load_links(fat, fieldgen.links(dims, 2, "gauss"))          # not unitary
+        assert e.value.status == _abi.DSLASH_ERR_ARG
+    lng = fieldgen.links(dims, 2, scale=-1 / 24)
+    lng[1, 2, 3, 4, 2] *= -1                                              # one link with the other sign
+    with Dslash(dims, recon=12) as D:
+        with pytest.raises(_abi.DslashError) as e:
+            D.load_links(fat, lng)
+        assert e.value.status == _abi.DSLASH_ERR_ARG
+
+
+@pytest.mark.parametrize("kernel", KERNELS)
+@pytest.mark.parametrize("nrhs", [1, 2, 3, 5, 8, 11])
+@pytest.mark.parametrize("mask", [0, 0xC])
+def test_multi_rhs_bitwise_and_oracle(torch_cuda, kernel, nrhs, mask):
+    """§8(f)-4: one link pass for nrhs vectors gives, for every right-hand side, the bits of the
+    single-vector apply (same per-thread arithmetic) and matches the oracle."""
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 10, 12, 14) if mask == 0 else (8, 8, 8, 12)
+    fat, lng = fieldgen.workload_links(dims)
+    parity = 1
+    src = torch.stack([torch.from_numpy(fieldgen.vector_cb(dims, 40 + r, 0)) for r in range(nrhs)]).cuda()
+    with Dslash(dims, kernel=kernel, force_halo=mask) as D:
+        D.load_links(fat, lng)
+        out = torch.empty_like(src)
+        D.apply_multi(out, src, parity)
+        singles = torch.stack([D(src[r].contiguous(), parity) for r in range(nrhs)])
+        torch.cuda.synchronize()
+    assert torch.equal(out, singles)
+    for r in (0, nrhs - 1):
+        psi = fieldgen.vector(dims, 40 + r)
+        ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, parity), parity)
+        assert oracle.normwise_error(out[r].cpu().numpy(), ref) <= TOL
+
+
+@pytest.mark.parametrize("precision,recon", [("f32", 18), ("mixed", 12), ("f64", 12)])
+def test_multi_rhs_precisions(torch_cuda, precision, recon):
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 10, 12, 14)
+    fat, lng = fieldgen.workload_links(dims)
+    with Dslash(dims, precision=precision, recon=recon) as D:
+        D.load_links(fat, lng)
+        src = torch.stack([torch.from_numpy(fieldgen.vector_cb(dims, 50 + r, 1)) for r in range(4)]).to(D.dtype).cuda()
+        out = torch.empty_like(src)
+        D.apply_multi(out, src, 0)
+        singles = torch.stack([D(src[r].contiguous(), 0) for r in range(4)])
+        torch.cuda.synchronize()
+    assert torch.equal(out, singles)
+
+
 def test_error_paths(torch_cuda):
     from paper_conf_sc_dufekgaad024_b200 import Dslash, _abi
     torch = torch_cuda

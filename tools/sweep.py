@@ -14,7 +14,7 @@ import numpy as np
 import torch
 
 import fieldgen
-from paper_conf_sc_dufekgaad024_b200 import ALGO_BYTES_PER_SITE, FLOP_PER_SITE, Dslash, _abi
+from paper_conf_sc_dufekgaad024_b200 import ALGO_BYTES, FLOP_PER_SITE, Dslash, _abi
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--dims", default="32,32,32,32")
@@ -23,16 +23,17 @@ ap.add_argument("--blocks", default="64,128,256")
 ap.add_argument("--minb", default="2,3,4")
 ap.add_argument("--steps", type=int, default=500)
 ap.add_argument("--halo", type=int, default=0)
+ap.add_argument("--precision", default="f64")
 a = ap.parse_args()
 dims = tuple(int(v) for v in a.dims.split(","))
 fat, lng = fieldgen.workload_links(dims)
 l2 = torch.cuda.get_device_properties(0).L2_cache_size
 for kern in a.kernels.split(","):
-    D = Dslash(dims, parity_mask=0, kernel=kern, force_halo=a.halo, timing=True)
+    D = Dslash(dims, parity_mask=0, kernel=kern, force_halo=a.halo, timing=True, precision=a.precision)
     D.load_links(fat, lng)
     vb = 3 * D.vh * 16
     R = max(2, int(np.ceil(2 * l2 / (2 * vb))) + 1)
-    srcs = [torch.from_numpy(fieldgen.vector_cb(dims, 3 + r, 1)).cuda() for r in range(R)]
+    srcs = [torch.from_numpy(fieldgen.vector_cb(dims, 3 + r, 1)).to(D.dtype).cuda() for r in range(R)]
     outs = [D.empty_vector() for _ in range(R)]
     for bs, mb in [(int(b), int(m)) for b in a.blocks.split(",") for m in a.minb.split(",")]:
         try:
@@ -55,6 +56,6 @@ for kern in a.kernels.split(","):
         D.kernel_timing_reset()
         print(json.dumps({"dims": dims, "kernel": kern, "block": bs, "minb": mb, "us_per_apply": round(ms * 1e3, 2),
                           "kernel_us": round(kms / max(n, 1) * 1e3, 2),
-                          "algo_gbs": round(ALGO_BYTES_PER_SITE * D.vh / (ms * 1e-3) / 1e9, 1),
+                          "precision": a.precision, "algo_gbs": round(ALGO_BYTES[a.precision] * D.vh / (ms * 1e-3) / 1e9, 1),
                           "gflops": round(FLOP_PER_SITE * D.vh / (ms * 1e-3) / 1e9, 1)}), flush=True)
     D.close()
