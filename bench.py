@@ -43,7 +43,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=2000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--kernel", default="dir2", choices=["site", "dir2", "dir4"])
+    ap.add_argument("--kernel", default="dir2", choices=["site", "dir2", "dir4", "bulk"])
     ap.add_argument("--min-blocks", type=int, default=0)
     ap.add_argument("--nrhs", type=int, default=1, choices=[1, 2, 3, 4, 5, 6, 7, 8],
                     help="right-hand sides per apply, one link pass (SURVEY §8(f)-4)")
@@ -52,7 +52,12 @@ def parse():
     ap.add_argument("--precision", default="f64", choices=["f64", "f32", "mixed"],
                     help="f64 is the paper's (L278) and the headline; f32/mixed are SURVEY §8(f)-1")
     ap.add_argument("--block", type=int, default=0)
-    ap.add_argument("--local", default="32,32,32,32", help="per-GPU local extents x,y,z,t")
+    ap.add_argument("--local", default="32,32,32,32", help="per-GPU local extents x,y,z,t (weak scaling)")
+    ap.add_argument("--global-dims", default=None,
+                    help="strong scaling: fixed global lattice x,y,z,t (e.g. 48,48,48,48, configs[3])")
+    ap.add_argument("--grid", default=None, help="process grid x,y,z,t (default 1,1,1,N: t-partitioned)")
+    ap.add_argument("--force-halo", type=int, default=0,
+                    help="bitmask of directions run through the halo path with neighbour = self (1 GPU)")
     ap.add_argument("--parity", type=int, default=0)
     ap.add_argument("--no-overlap", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -62,9 +67,15 @@ def parse():
 
 
 def workload(args, world):
+    grid = tuple(int(v) for v in args.grid.split(",")) if args.grid else (1, 1, 1, world)
+    if args.global_dims:
+        gdims = tuple(int(v) for v in args.global_dims.split(","))
+        loc = tuple(g // p for g, p in zip(gdims, grid))
+        name = (f"{gdims[0]}x{gdims[1]}x{gdims[2]}x{gdims[3]} fp64 single-parity HISQ Dslash, strong scaling, "
+                f"grid {'x'.join(map(str, grid))} (configs[3] shape)")
+        return gdims, grid, loc, name
     loc = tuple(int(v) for v in args.local.split(","))
-    gdims = (loc[0], loc[1], loc[2], loc[3] * world)
-    grid = (1, 1, 1, world)
+    gdims = tuple(l * p for l, p in zip(loc, grid))
     if world == 1 and loc == (32, 32, 32, 32):
         name = "32^4 fp64 single-parity HISQ Dslash, 1 GPU (BASELINE.json configs[2])"
     else:
@@ -255,7 +266,7 @@ def main():
     algo_bytes_site = algo_bytes(args.precision, args.recon, nrhs)
     D = Dslash(gdims, grid, parity_mask=parity, kernel=args.kernel, block=args.block, min_blocks=args.min_blocks,
                precision=args.precision, recon=args.recon,
-               overlap=not args.no_overlap, timing=True, rank=rank, world_size=world)
+               overlap=not args.no_overlap, timing=True, rank=rank, world_size=world, force_halo=args.force_halo)
     origin, extent = D.origin, D.local_dims
     fat, lng = fieldgen.workload_links(gdims, origin=origin, extent=extent)
     D.load_links(fat, lng)
@@ -300,7 +311,10 @@ def main():
     ms = ev0.elapsed_time(ev1)
     t_int, n_int = D.kernel_timing(0)
     t_bnd, n_bnd = D.kernel_timing(1)
+    t_all, n_all = D.kernel_timing(2)
     D.kernel_timing_reset()
+    if n_int == 0 and n_all > n_bnd:      # --no-overlap: one launch over all sites
+        t_int, n_int = t_all - t_bnd, n_all - n_bnd
     t_max = torch.tensor([ms], dtype=torch.float64, device="cuda")
     if world > 1:
         dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
@@ -312,6 +326,8 @@ def main():
     # dominant kernel: the full-lattice kernel at N = 1, the interior kernel at N > 1
     plan = D.plan
     dom_sites = int(plan.interior_sites) if plan.n_interior else int(plan.boundary_sites)
+    if args.no_overlap and any(plan.halo):
+        dom_sites = int(plan.vh_local)
     # algo_bytes_site already counts nrhs vectors per site; GB/s over sites, flop over site-RHS pairs
     peak, peak_src = measured_peak()
     kern_ms = t_int / max(1, n_int) if n_int else None
@@ -322,10 +338,12 @@ def main():
                 "frac": round(achieved / peak, 4),
                 "traffic": ncu_traffic(args.kernel + ("" if args.precision == "f64" else f"-{args.precision}")
                                      + ("" if args.recon == 18 else f"-r{args.recon}"), extent),
-                "kernel": f"dslash_kernel<lanes={ {'site': 1, 'dir2': 2, 'dir4': 4}[args.kernel]}, ghost=false>"
+                "kernel": ("dslash_bulk_kernel<ghost=false> (TMA)" if args.kernel == "bulk" else
+                           f"dslash_kernel<lanes={ {'site': 1, 'dir2': 2, 'dir4': 4}[args.kernel]}, ghost=false>")
                           + (" interior" if world > 1 else ""),
                 "bytes_per_launch": algo_bytes_site * dom_sites, "bytes_per_site": algo_bytes_site, "avg_launch_us": round(kern_ms * 1e3, 2),
                 "launches": n_int, "peak_source": peak_src,
+                "boundary_kernel_us": round(t_bnd / n_bnd * 1e3, 2) if n_bnd else None,
                 "frac_of_nominal_8TBs": round(achieved / NOMINAL_HBM_GBS, 4)}
 
     # end to end through the C ABI from pinned host buffers: every step copies its psi host->device
@@ -359,18 +377,20 @@ def main():
                        "device -> pinned host chi; copies of neighbouring steps overlap the compute"}
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.global_dims:
         cpu, _ = run_oracle_baseline(gdims, parity, args.cpu_seconds)
 
     launches_per_step = (1 if not any(plan.halo) else (int(plan.n_interior > 0) + 1))
     if rank == 0:
         line = {"metric": METRIC, "value": round(gflops, 2), "unit": "GFLOP/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
-                "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "higher_is_better": True, "scaling": "strong" if args.global_dims else "weak", "vs_baseline": None,
                 "dtype": {"f64": "f64", "f32": "f32", "mixed": "f32 links, f64 vectors/accumulation"}[args.precision],
                 "data": "synthetic",
                 "config": {"workload": name, "global_dims": list(gdims), "local_dims": list(extent),
-                           "proc_grid": list(grid), "parallelism": f"t{world}", "parity": parity,
+                           "proc_grid": list(grid),
+                           "parallelism": (f"t{grid[3]}" if grid[2] == 1 else f"z{grid[2]}t{grid[3]}")
+                           + (f" self-halo mask {args.force_halo}" if args.force_halo else ""), "parity": parity,
                            "kernel": args.kernel, "block": args.block or None, "precision": args.precision,
                            "long_link_recon": args.recon, "nrhs": nrhs,
                            "overlap": not args.no_overlap,

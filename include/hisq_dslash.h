@@ -72,7 +72,10 @@ enum { DSLASH_F64 = 0, DSLASH_F32 = 1, DSLASH_MIXED = 2 };
 enum {
     DSLASH_KERNEL_SITE = 0, /* one thread per target site, 16 link matrices streamed per thread   */
     DSLASH_KERNEL_DIR4 = 1, /* four lanes per site (one per mu), 2-step shuffle reduction ("3LP") */
-    DSLASH_KERNEL_DIR2 = 2  /* two lanes per site (two directions each), 1-step shuffle reduction  */
+    DSLASH_KERNEL_DIR2 = 2, /* two lanes per site (two directions each), 1-step shuffle reduction  */
+    DSLASH_KERNEL_BULK = 3  /* persistent TMA pipeline: cp.async.bulk link tiles into shared memory,
+                               one producer thread, 8 consumer warps (DIR4 mapping); needs Lx/2 to
+                               be a multiple of 8; one right-hand side per launch                  */
 };
 
 /* Options (dslash_set_option). */

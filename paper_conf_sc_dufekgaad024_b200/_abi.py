@@ -21,11 +21,12 @@ STATUS_NAMES = {0: "DSLASH_OK", 1: "DSLASH_ERR_ARG", 2: "DSLASH_ERR_STATE", 3: "
 DSLASH_EVEN, DSLASH_ODD, DSLASH_BOTH = 0, 1, 2
 DSLASH_F64, DSLASH_F32, DSLASH_MIXED = 0, 1, 2
 PRECISIONS = {"f64": DSLASH_F64, "f32": DSLASH_F32, "mixed": DSLASH_MIXED}
-DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_DIR2 = 0, 1, 2
+DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_DIR2, DSLASH_KERNEL_BULK = 0, 1, 2, 3
 DSLASH_OPT_KERNEL, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_OVERLAP, DSLASH_OPT_TIMING, \
     DSLASH_OPT_MIN_BLOCKS, DSLASH_OPT_LONG_RECON = range(7)
 DSLASH_TIMING_INTERIOR, DSLASH_TIMING_BOUNDARY, DSLASH_TIMING_ALL = range(3)
-KERNELS = {"site": DSLASH_KERNEL_SITE, "dir4": DSLASH_KERNEL_DIR4, "dir2": DSLASH_KERNEL_DIR2}
+KERNELS = {"site": DSLASH_KERNEL_SITE, "dir4": DSLASH_KERNEL_DIR4, "dir2": DSLASH_KERNEL_DIR2,
+           "bulk": DSLASH_KERNEL_BULK}
 
 
 class dslash_box_t(ctypes.Structure):

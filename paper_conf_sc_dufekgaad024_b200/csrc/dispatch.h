@@ -16,4 +16,15 @@ StencilFn pick_f32_r12(bool ghost, int lanes, int minb, int nrhs);
 StencilFn pick_mixed_r18(bool ghost, int lanes, int minb, int nrhs);
 StencilFn pick_mixed_r12(bool ghost, int lanes, int minb, int nrhs);
 
+// The TMA-staged persistent kernel (bulk.cuh): function, dynamic shared memory, threads per CTA,
+// sites per tile.  precision: 0 fp64, 1 fp32, 2 mixed (DSLASH_F64/F32/MIXED).
+typedef void (*BulkFn)(StencilParams, unsigned long long*, unsigned long long);
+struct BulkKernel {
+    BulkFn fn;
+    size_t smem;
+    int threads;
+    int tile;
+};
+BulkKernel pick_bulk(int precision, int recon, bool ghost);
+
 }  // namespace hisq

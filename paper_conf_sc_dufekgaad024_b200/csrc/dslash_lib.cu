@@ -17,6 +17,7 @@
 #include "common.cuh"
 #include "links.cuh"
 #include "stencil.cuh"
+#include "bulk.cuh"
 #include "dispatch.h"
 
 using namespace hisq;
@@ -238,8 +239,11 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     switch (key) {
         case DSLASH_OPT_KERNEL:
-            if (value != DSLASH_KERNEL_SITE && value != DSLASH_KERNEL_DIR4 && value != DSLASH_KERNEL_DIR2)
+            if (value != DSLASH_KERNEL_SITE && value != DSLASH_KERNEL_DIR4 && value != DSLASH_KERNEL_DIR2 &&
+                value != DSLASH_KERNEL_BULK)
                 return fail(h, DSLASH_ERR_ARG, "unknown kernel variant %lld", (long long)value);
+            if (value == DSLASH_KERNEL_BULK && (h->plan.local_dims[0] / 2) % kBulkTile)
+                return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel needs Lx/2 to be a multiple of %d", kBulkTile);
             if (h->loaded && value != h->kernel)
                 return fail(h, DSLASH_ERR_STATE, "kernel variant fixes the link layout: set it before load_links");
             h->kernel = (int)value;
@@ -286,7 +290,7 @@ static size_t vec_elem(const dslash_s* h) { return h->precision == DSLASH_F32 ? 
 static size_t link_elem(const dslash_s* h) { return h->precision == DSLASH_F64 ? 16 : 8; }
 
 static int lanes_of(int kernel) {
-    return kernel == DSLASH_KERNEL_DIR4 ? 4 : kernel == DSLASH_KERNEL_DIR2 ? 2 : 1;
+    return (kernel == DSLASH_KERNEL_DIR4 || kernel == DSLASH_KERNEL_BULK) ? 4 : kernel == DSLASH_KERNEL_DIR2 ? 2 : 1;
 }
 
 // ============================================================================ link loading
@@ -332,7 +336,7 @@ extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
     for (int d = 0; d < 4; ++d) C.L[d] = p.local_dims[d];
     C.lxh = p.local_dims[0] / 2;
     C.vh = p.vh_local;
-    C.lanes = lanes_of(h->kernel);
+    C.lanes = h->kernel == DSLASH_KERNEL_BULK ? 0 : lanes_of(h->kernel);
     C.recon = h->recon;
     int halo_mask = 0;
     for (int d = 2; d < 4; ++d)
@@ -595,9 +599,42 @@ static int default_block(int lanes) { return lanes == 4 ? 64 : 64; }
 static int default_minb(int lanes) { return lanes == 4 ? 2 : 2; }
 
 // one launch of the stencil over the boxes of K for nrhs (1, 2, 4 or 8) right-hand sides
+static int num_sms(dslash_t h) {
+    static int n = 0;
+    if (!n && cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, h->device) != cudaSuccess) n = 148;
+    return n;
+}
+
 static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int kind, cudaStream_t s, int nrhs) {
     const int64_t sites = K.box_start[K.nbox];
     if (sites == 0) return DSLASH_OK;
+    if (h->kernel == DSLASH_KERNEL_BULK) {
+        const BulkKernel bk = pick_bulk(h->precision, h->recon, ghost);
+        const int64_t ntiles = sites / bk.tile;
+        const unsigned grid = (unsigned)(ntiles < num_sms(h) ? ntiles : num_sms(h));
+        dslash_s::TimedLaunch* tl = nullptr;
+        if (h->timing) {
+            if (h->tused == h->tpool.size()) {
+                dslash_s::TimedLaunch t{};
+                CU(h, cudaEventCreate(&t.a));
+                CU(h, cudaEventCreate(&t.b));
+                h->tpool.push_back(t);
+            }
+            tl = &h->tpool[h->tused++];
+            tl->kind = kind;
+            CU(h, cudaEventRecord(tl->a, s));
+        }
+        if (!h->sched) CU(h, cudaMalloc(&h->sched, sizeof(unsigned long long)));
+        if (!h->sched_init) {
+            CU(h, cudaMemsetAsync(h->sched, 0, sizeof(unsigned long long), s));
+            h->sched_init = true;
+        }
+        bk.fn<<<grid, bk.threads, bk.smem, s>>>(K, h->sched, h->sched_next);
+        h->sched_next += (unsigned long long)ntiles + grid;  // tickets this launch consumes
+        CU(h, cudaGetLastError());
+        if (tl) CU(h, cudaEventRecord(tl->b, s));
+        return DSLASH_OK;
+    }
     const int lanes = lanes_of(h->kernel);
     const int bs = h->block ? h->block : default_block(lanes);
     const int minb = h->min_blocks ? h->min_blocks : default_minb(lanes);
@@ -634,7 +671,8 @@ static dslash_status launch_rhs(dslash_t h, StencilParams K, const dslash_box_t*
     memcpy(g0, K.ghost, sizeof g0);
     for (int r0 = 0; r0 < nrhs;) {
         const int left = nrhs - r0;
-        const int nr = left >= 8 ? 8 : left >= 4 ? 4 : left >= 2 ? 2 : 1;
+        int nr = left >= 8 ? 8 : left >= 4 ? 4 : left >= 2 ? 2 : 1;
+        if (h->kernel == DSLASH_KERNEL_BULK) nr = 1;  // the TMA kernel streams one right-hand side
         K.in = in0 + (size_t)r0 * 3 * K.vh * es;
         K.out = out0 + (size_t)r0 * 3 * K.vh * es;
         for (int d = 0; d < 4; ++d)
@@ -857,6 +895,7 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
             if (e) cudaEventDestroy(e);
     }
     if (h->ev_batch) cudaEventDestroy(h->ev_batch);
+    if (h->sched) cudaFree(h->sched);
     for (void* v : h->cg_vec)
         if (v) cudaFree(v);
     if (h->cg_partial) cudaFree(h->cg_partial);

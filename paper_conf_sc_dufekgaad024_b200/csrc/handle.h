@@ -45,6 +45,10 @@ struct dslash_s {
     void* cg_vec[4] = {};
     double* cg_partial = nullptr;
     double* cg_scalar = nullptr;
+    // tile scheduler of the TMA kernel: a ticket counter and the first ticket of the next launch
+    unsigned long long* sched = nullptr;
+    unsigned long long sched_next = 0;
+    bool sched_init = false;
     dslash_status err = DSLASH_OK;
     std::string msg;
 };

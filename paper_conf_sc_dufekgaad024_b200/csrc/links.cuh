@@ -13,6 +13,7 @@
 
 #include "common.cuh"
 #include "stencil.cuh"
+#include "bulk.cuh"
 
 namespace hisq {
 
@@ -27,7 +28,8 @@ struct LinkConvParams {
     int lxh;
     int parity;
     int halo_mask;
-    int lanes;                    // layout of the kernel that will read the links: 1, 2 or 4
+    int lanes;                    // layout of the kernel that will read the links: 1, 2 or 4,
+                                  // or 0 = tiled (the TMA kernel, bulk.cuh)
     int recon;                    // 18 = full matrices, 12 = long links keep rows 0 and 1 only
 };
 
@@ -83,7 +85,9 @@ __global__ void convert_links_kernel(const LinkConvParams P) {
             }
             const int e = 3 * i + j;
             int64_t o;
-            if (P.recon == 12)
+            if (P.lanes == 0)
+                o = P.recon == 12 ? link_index_tiled<12>(mu, l, e, cb) : link_index_tiled<18>(mu, l, e, cb);
+            else if (P.recon == 12)
                 o = P.lanes == 1 ? link_index<1, 12>(mu, l, e, P.vh, cb)
                   : P.lanes == 2 ? link_index<2, 12>(mu, l, e, P.vh, cb)
                                  : link_index<4, 12>(mu, l, e, P.vh, cb);

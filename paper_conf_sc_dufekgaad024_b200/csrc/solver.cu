@@ -58,10 +58,13 @@ __global__ void __launch_bounds__(kRedThreads) k_norm2(const double2* __restrict
     if (threadIdx.x == 0) partial[blockIdx.x] = s;
 }
 
-// x += alpha p ; r -= alpha q ; partial[block] = sum |r|^2
+// x += alpha p ; r -= alpha q ; partial[block] = sum |r|^2, alpha = rr / pq read on the device
+// (0 when pq == 0: an exactly converged iterate stays put)
 __global__ void __launch_bounds__(kRedThreads) k_cg_update(double2* __restrict__ x, double2* __restrict__ r,
                                                            const double2* __restrict__ p, const double2* __restrict__ q,
-                                                           double alpha, int64_t n, double* __restrict__ partial) {
+                                                           const double* __restrict__ rr, const double* __restrict__ pq,
+                                                           int64_t n, double* __restrict__ partial) {
+    const double alpha = (*pq != 0.0) ? *rr / *pq : 0.0;
     double acc = 0.0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         double2 xi = x[i], ri = r[i];
@@ -78,8 +81,10 @@ __global__ void __launch_bounds__(kRedThreads) k_cg_update(double2* __restrict__
     if (threadIdx.x == 0) partial[blockIdx.x] = s;
 }
 
-// p = r + beta p
-__global__ void k_cg_direction(double2* __restrict__ p, const double2* __restrict__ r, double beta, int64_t n) {
+// p = r + beta p, beta = rr_new / rr read on the device (0 when rr == 0)
+__global__ void k_cg_direction(double2* __restrict__ p, const double2* __restrict__ r, const double* __restrict__ rr_new,
+                               const double* __restrict__ rr, int64_t n) {
+    const double beta = (*rr != 0.0) ? *rr_new / *rr : 0.0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const double2 ri = r[i];
         double2 pi = p[i];
@@ -100,13 +105,14 @@ __global__ void k_sub_from(double2* __restrict__ r, const double2* __restrict__ 
     }
 }
 
-// out[0] = sum_{k < n} partial[k] in index order (one thread: deterministic)
-__global__ void k_finalize(const double* __restrict__ partial, int n, double* __restrict__ out) {
-    if (threadIdx.x == 0 && blockIdx.x == 0) {
-        double s = 0.0;
-        for (int k = 0; k < n; ++k) s += partial[k];
-        out[0] = s;
-    }
+// out[0] = sum_{k < n} partial[k]: thread t sums k = t, t + 256, ... in order, then the fixed
+// shuffle tree of block_sum (one block: deterministic)
+__global__ void __launch_bounds__(kRedThreads) k_finalize(const double* __restrict__ partial, int n,
+                                                          double* __restrict__ out) {
+    double acc = 0.0;
+    for (int k = threadIdx.x; k < n; k += kRedThreads) acc += partial[k];
+    const double s = block_sum(acc);
+    if (threadIdx.x == 0) out[0] = s;
 }
 
 }  // namespace
@@ -117,15 +123,22 @@ static dslash_status need_scratch(dslash_t h) {
     for (void*& v : h->cg_vec)
         if (!v) CU(h, cudaMalloc(&v, bytes));
     if (!h->cg_partial) CU(h, cudaMalloc(&h->cg_partial, kRedBlocks * sizeof(double)));
-    if (!h->cg_scalar) CU(h, cudaMalloc(&h->cg_scalar, 2 * sizeof(double)));
+    if (!h->cg_scalar) CU(h, cudaMalloc(&h->cg_scalar, 4 * sizeof(double)));
     return DSLASH_OK;
 }
 
-// the partials of one reduction -> global sum (all ranks) -> host value
-static dslash_status reduce_to_host(dslash_t h, cudaStream_t s, double* value) {
-    k_finalize<<<1, 32, 0, s>>>(h->cg_partial, kRedBlocks, h->cg_scalar);
+// the partials of one reduction -> global sum over all ranks in device scalar `slot`
+static dslash_status reduce_to_slot(dslash_t h, cudaStream_t s, double* slot) {
+    k_finalize<<<1, kRedThreads, 0, s>>>(h->cg_partial, kRedBlocks, slot);
     CU(h, cudaGetLastError());
-    if (h->nccl) NC(h, ncclAllReduce(h->cg_scalar, h->cg_scalar, 1, ncclDouble, ncclSum, h->nccl, s));
+    if (h->nccl) NC(h, ncclAllReduce(slot, slot, 1, ncclDouble, ncclSum, h->nccl, s));
+    return DSLASH_OK;
+}
+
+// ... and to the host (synchronous)
+static dslash_status reduce_to_host(dslash_t h, cudaStream_t s, double* value) {
+    dslash_status st = reduce_to_slot(h, s, h->cg_scalar);
+    if (st != DSLASH_OK) return st;
     CU(h, cudaMemcpyAsync(value, h->cg_scalar, sizeof(double), cudaMemcpyDeviceToHost, s));
     CU(h, cudaStreamSynchronize(s));
     return DSLASH_OK;
@@ -190,31 +203,69 @@ extern "C" dslash_status dslash_cg(dslash_t h, void* x_out, const void* b_in, in
     CU(h, cudaMemsetAsync(x, 0, bytes, s));
     CU(h, cudaMemcpyAsync(r, b, bytes, cudaMemcpyDeviceToDevice, s));
     CU(h, cudaMemcpyAsync(p, b, bytes, cudaMemcpyDeviceToDevice, s));
-    double bb = 0.0, rr = 0.0, pq = 0.0;
+    // Device scalars: sc[0], sc[1] = <r,r> of alternate iterations (ping-pong, so no kernel
+    // overwrites a value another block may still read), sc[2] = <p, A p>, sc[3] = scratch.
+    // The host learns <r,r> through pinned memory one iteration late, so the GPU never waits
+    // for the host; the solve can run one iteration past convergence, which only refines x.
+    double* sc = h->cg_scalar;
+    double bb = 0.0, rr_last = 0.0;
     k_norm2<<<kRedBlocks, kRedThreads, 0, s>>>(b, n, h->cg_partial);
     CU(h, cudaGetLastError());
     if ((st = reduce_to_host(h, s, &bb)) != DSLASH_OK) return st;
     int k = 0;
+    bool converged = !(bb > 0.0);
     if (bb > 0.0) {
-        rr = bb;
+        CU(h, cudaMemcpyAsync(&sc[0], &bb, sizeof(double), cudaMemcpyHostToDevice, s));
         const double stop = rel_tol * rel_tol * bb;
+        double* host_rr = nullptr;
+        cudaEvent_t ev[2] = {nullptr, nullptr};
+        CU(h, cudaMallocHost(&host_rr, 2 * sizeof(double)));
+        auto release = [&]() {
+            for (cudaEvent_t e : ev)
+                if (e) cudaEventDestroy(e);
+            cudaFreeHost(host_rr);
+        };
+#define CUR(call)                                                                                    \
+    do {                                                                                             \
+        cudaError_t e_ = (call);                                                                     \
+        if (e_ != cudaSuccess) {                                                                     \
+            release();                                                                               \
+            return hisq_fail(h, DSLASH_ERR_CUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call,          \
+                             cudaGetErrorString(e_));                                                \
+        }                                                                                            \
+    } while (0)
+        CUR(cudaEventCreateWithFlags(&ev[0], cudaEventDisableTiming));
+        CUR(cudaEventCreateWithFlags(&ev[1], cudaEventDisableTiming));
         for (k = 1; k <= max_iter; ++k) {
-            if ((st = normal_apply(h, q, p, parity, m2, t, s, true)) != DSLASH_OK) return st;  // q = A p
-            if ((st = reduce_to_host(h, s, &pq)) != DSLASH_OK) return st;
-            const double alpha = rr / pq;
-            k_cg_update<<<kRedBlocks, kRedThreads, 0, s>>>(x, r, p, q, alpha, n, h->cg_partial);
-            CU(h, cudaGetLastError());
-            double rr_new = 0.0;
-            if ((st = reduce_to_host(h, s, &rr_new)) != DSLASH_OK) return st;
-            if (rr_new <= stop) {
-                rr = rr_new;
-                break;
+            double* rr_cur = &sc[(k - 1) & 1];
+            double* rr_new = &sc[k & 1];
+            if ((st = normal_apply(h, q, p, parity, m2, t, s, true)) != DSLASH_OK) break;  // q = A p
+            if ((st = reduce_to_slot(h, s, &sc[2])) != DSLASH_OK) break;                 // <p, q>
+            k_cg_update<<<kRedBlocks, kRedThreads, 0, s>>>(x, r, p, q, rr_cur, &sc[2], n, h->cg_partial);
+            CUR(cudaGetLastError());
+            if ((st = reduce_to_slot(h, s, rr_new)) != DSLASH_OK) break;                  // <r, r>
+            k_cg_direction<<<kRedBlocks, kRedThreads, 0, s>>>(p, r, rr_new, rr_cur, n);
+            CUR(cudaGetLastError());
+            CUR(cudaMemcpyAsync(&host_rr[k & 1], rr_new, sizeof(double), cudaMemcpyDeviceToHost, s));
+            CUR(cudaEventRecord(ev[k & 1], s));
+            // check iteration k-1 (already complete or nearly) while iteration k runs
+            if (k >= 2) {
+                CUR(cudaEventSynchronize(ev[(k - 1) & 1]));
+                if (host_rr[(k - 1) & 1] <= stop) {
+                    converged = true;
+                    break;
+                }
             }
-            k_cg_direction<<<kRedBlocks, kRedThreads, 0, s>>>(p, r, rr_new / rr, n);
-            CU(h, cudaGetLastError());
-            rr = rr_new;
         }
-        if (k > max_iter) k = max_iter;
+        if (st == DSLASH_OK) {
+            if (k > max_iter) k = max_iter;
+            CUR(cudaEventSynchronize(ev[k & 1]));
+            rr_last = host_rr[k & 1];
+            if (rr_last <= stop) converged = true;
+        }
+        release();
+#undef CUR
+        if (st != DSLASH_OK) return st;
     }
     // true residual |b - A x| / |b|
     double res = 0.0;
@@ -230,5 +281,5 @@ extern "C" dslash_status dslash_cg(dslash_t h, void* x_out, const void* b_in, in
     if (iters) *iters = k;
     if (rel_resid) *rel_resid = res;
     // not converged: reported, but not a sticky handle error
-    return (bb > 0.0 && !(rr <= rel_tol * rel_tol * bb)) ? DSLASH_ERR_NOT_CONVERGED : DSLASH_OK;
+    return converged ? DSLASH_OK : DSLASH_ERR_NOT_CONVERGED;
 }

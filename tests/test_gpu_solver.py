@@ -98,7 +98,9 @@ def test_cg_free_field_closed_form(torch_cuda):
         D.load_links(fat, lng)
         x = D.empty_vector()
         ok, it, res = D.cg(x, torch.from_numpy(oracle.full_to_cb(psi, 0)).cuda(), 0, m, rel_tol=1e-13)
-    assert ok and it == 1
+    # converges in one iteration; the host learns it one iteration late (lagged check), so the
+    # solver may run one more, which must leave the exact solution in place
+    assert ok and it <= 2
     assert oracle.normwise_error(x.cpu().numpy(), oracle.full_to_cb(psi / lam, 0)) < 1e-13
 
 
