@@ -26,6 +26,7 @@ namespace hisq {
 constexpr int kBulkTile = 8;       // target sites per tile (lxh must be a multiple)
 constexpr int kBulkConsumers = 8;  // consumer warps per CTA
 constexpr int kBulkStages = 8;     // stage ring depth: one stage per consumer warp
+constexpr int kBulkBatch = 4;      // tiles per scheduler ticket draw
 
 template <int RECON>
 __host__ __device__ constexpr int bulk_elems() { return RECON == 12 ? 30 : 36; }
@@ -79,9 +80,11 @@ __device__ __forceinline__ float2 lds(const float2* p) {
 }
 
 // ---------------------------------------------------------------- the kernel
-// sched: a 64-bit counter shared by the launches of one handle; this launch owns the tickets
-// [sched_base, sched_base + ntiles + gridDim.x): every CTA's producer takes tickets until it
-// draws one past the pool, so exactly ntiles + gridDim.x tickets are consumed per launch.
+// sched: a 64-bit counter shared by the launches of one handle.  A producer draws batches of
+// kBulkBatch tiles and always has the next draw in flight (its latency overlaps the current
+// batch); it stops at the first batch past the pool, so every CTA makes exactly 2 draws that
+// process nothing and a launch consumes (ceil(ntiles / B) + 2 gridDim.x) * B tickets, starting
+// at sched_base.
 template <typename LR, typename VR, bool GHOST, int RECON>
 __global__ void __launch_bounds__(32 * (kBulkConsumers + 1), 1)
     dslash_bulk_kernel(const StencilParams P, unsigned long long* sched, unsigned long long sched_base) {
@@ -114,24 +117,29 @@ __global__ void __launch_bounds__(32 * (kBulkConsumers + 1), 1)
             const uint64_t pol = policy_evict_first();
             const unsigned char* links = static_cast<const unsigned char*>(P.links);
             long long k = 0;
-            for (;; ++k) {
-                const int st = (int)(k % kBulkStages);
-                const uint32_t phase = (uint32_t)(k / kBulkStages) & 1u;
-                const long long tile = (long long)(atomicAdd(sched, 1ull) - sched_base);
-                mbar_wait(&empty[st], phase ^ 1u);  // fresh barrier: passes immediately
-                if (tile >= ntiles) break;
-                tile_of[st] = tile;
-                // tile index in the box enumeration -> checkerboard tile (boxes hold whole x-rows)
-                const Site s0 = decode_site(P, tile * kBulkTile);
-                mbar_arrive_expect_tx(&full[st], kTileBytes);  // release: publishes tile_of[st]
-                bulk_g2s(stage_base + (size_t)st * (kTileBytes / sizeof(L2)),
-                         links + (size_t)(s0.cb / kBulkTile) * kTileBytes, kTileBytes, &full[st], pol);
+            long long batch = (long long)(atomicAdd(sched, (unsigned long long)kBulkBatch) - sched_base);
+            for (;;) {
+                const long long next = (long long)(atomicAdd(sched, (unsigned long long)kBulkBatch) - sched_base);
+                if (batch >= ntiles) break;
+                const long long end = batch + kBulkBatch < ntiles ? batch + kBulkBatch : ntiles;
+                for (long long tile = batch; tile < end; ++tile, ++k) {
+                    const int st = (int)(k % kBulkStages);
+                    const uint32_t phase = (uint32_t)(k / kBulkStages) & 1u;
+                    mbar_wait(&empty[st], phase ^ 1u);  // fresh barrier: passes immediately
+                    tile_of[st] = tile;
+                    // tile index in the box enumeration -> checkerboard tile (boxes hold whole x-rows)
+                    const Site s0 = decode_site(P, tile * kBulkTile);
+                    mbar_arrive_expect_tx(&full[st], kTileBytes);  // release: publishes tile_of[st]
+                    bulk_g2s(stage_base + (size_t)st * (kTileBytes / sizeof(L2)),
+                             links + (size_t)(s0.cb / kBulkTile) * kTileBytes, kTileBytes, &full[st], pol);
+                }
+                batch = next;
             }
             // stop every consumer: a sentinel in the next stage of each warp
             for (int j = 0; j < kBulkStages; ++j, ++k) {
                 const int st = (int)(k % kBulkStages);
                 const uint32_t phase = (uint32_t)(k / kBulkStages) & 1u;
-                if (j > 0) mbar_wait(&empty[st], phase ^ 1u);
+                mbar_wait(&empty[st], phase ^ 1u);
                 tile_of[st] = -1;
                 mbar_arrive(&full[st]);
             }

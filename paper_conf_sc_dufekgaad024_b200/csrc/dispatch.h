@@ -24,6 +24,7 @@ struct BulkKernel {
     size_t smem;
     int threads;
     int tile;
+    int batch;  // tiles per scheduler draw
 };
 BulkKernel pick_bulk(int precision, int recon, bool ghost);
 

@@ -630,7 +630,8 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
             h->sched_init = true;
         }
         bk.fn<<<grid, bk.threads, bk.smem, s>>>(K, h->sched, h->sched_next);
-        h->sched_next += (unsigned long long)ntiles + grid;  // tickets this launch consumes
+        // tickets this launch consumes (bulk.cuh): (ceil(ntiles / B) + 2 grid) * B
+        h->sched_next += ((unsigned long long)((ntiles + bk.batch - 1) / bk.batch) + 2ull * grid) * bk.batch;
         CU(h, cudaGetLastError());
         if (tl) CU(h, cudaEventRecord(tl->b, s));
         return DSLASH_OK;

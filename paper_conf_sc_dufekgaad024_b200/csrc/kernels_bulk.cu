@@ -11,6 +11,7 @@ static BulkKernel pick_bulk_t(bool ghost) {
     k.smem = bulk_smem_bytes<LR, RECON>();
     k.threads = 32 * (kBulkConsumers + 1);
     k.tile = kBulkTile;
+    k.batch = kBulkBatch;
     // opt in to > 48 KB of dynamic shared memory (idempotent)
     cudaFuncSetAttribute(k.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k.smem);
     return k;
