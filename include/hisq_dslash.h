@@ -94,9 +94,29 @@ enum {
                                    (and the link halo) to be s*W with W in SU(3) and one real s;
                                    load_links verifies it and returns DSLASH_ERR_ARG otherwise.
                                    Before load_links                                                  */
+    DSLASH_OPT_PERSISTENT = 7,  /* 1 (default): one persistent launch per apply; blocks draw tiles from
+                                   ticket counters, interior first; a block out of interior tiles
+                                   looks once at the halo flag and takes boundary tiles only if the
+                                   faces have landed (never waits, so it cannot starve the exchange);
+                                   a stream-ordered clean-up launch takes the rest.  0: separate
+                                   interior / boundary launches.  Single-RHS applies only; any time */
+    DSLASH_OPT_TRANSPORT = 8,   /* DSLASH_TRANSPORT_NCCL / _P2P; before load_links                    */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */
+};
+
+/* Halo transports (DSLASH_OPT_TRANSPORT). */
+enum {
+    DSLASH_TRANSPORT_NCCL = 0, /* grouped ncclSend/ncclRecv on the communication stream (default when
+                                  dslash_create got an NCCL unique id)                               */
+    DSLASH_TRANSPORT_P2P = 1   /* SM-free: faces are copied by the copy engines straight into the
+                                  neighbours' CUDA-IPC-mapped ghost buffers (NVLink within a node),
+                                  and cuStreamWriteValue32/WaitValue32 epoch flags order producers and
+                                  consumers.  Needs dslash_get_ipc_blob / dslash_open_ipc_blobs, and
+                                  dslash_load_links_halo when neighbours are other ranks.  Also works
+                                  for several ranks on ONE GPU (NCCL refuses that).  At most 8
+                                  right-hand sides per apply                                         */
 };
 
 /* Kernel classes for dslash_kernel_timing. */
@@ -139,12 +159,22 @@ DSLASH_API dslash_status dslash_plan(const int32_t global_dims[4], const int32_t
  * parities links are prepared (DSLASH_BOTH doubles link memory).  precision: DSLASH_F64,
  * DSLASH_F32 or DSLASH_MIXED (it fixes the stored link type and the vector type).
  * nccl_unique_id: the 128-byte ncclUniqueId from dslash_get_unique_id() on rank 0,
- * broadcast to all ranks by the caller; NULL when nranks == 1.  On success *out owns
+ * broadcast to all ranks by the caller; NULL when nranks == 1, or when the ranks will use
+ * DSLASH_TRANSPORT_P2P (then no NCCL communicator is created).  On success *out owns
  * a CUDA communication stream, events, ghost buffers and (nranks > 1) an NCCL
  * communicator; release it with dslash_destroy.  On failure *out is NULL. */
 DSLASH_API dslash_status dslash_create(const int32_t global_dims[4], const int32_t proc_grid[4], int32_t parity_mask,
                             int32_t precision, const void* nccl_unique_id, int32_t nranks, int32_t rank,
                             dslash_t* out);
+
+/* P2P transport setup.  dslash_ipc_blob_size() bytes describe one rank's halo buffers (CUDA IPC
+ * handles of its ghost buffers and epoch flags).  Every rank writes its blob with
+ * dslash_get_ipc_blob, the caller all-gathers them (blobs of rank r at r * size) and every rank
+ * calls dslash_open_ipc_blobs.  Both need DSLASH_OPT_TRANSPORT = P2P first.  Ranks must be on
+ * GPUs of one node (or the same GPU). */
+DSLASH_API int64_t dslash_ipc_blob_size(void);
+DSLASH_API dslash_status dslash_get_ipc_blob(dslash_t h, void* blob);
+DSLASH_API dslash_status dslash_open_ipc_blobs(dslash_t h, const void* blobs);
 
 /* Write a fresh ncclUniqueId (128 bytes) to id_out.  Call on rank 0 only. */
 DSLASH_API dslash_status dslash_get_unique_id(void* id_out);
@@ -162,6 +192,16 @@ DSLASH_API dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
  * the links. */
 DSLASH_API dslash_status dslash_load_links(dslash_t h, const void* fat, const void* lng, int32_t on_device,
                                 dslash_stream_t stream);
+
+/* load_links with caller-provided link halo: for every halo direction d whose neighbour is
+ * another rank, slab_fat[d] / slab_lng[d] hold the 3 coordinate slices just below the local
+ * origin, taken from the minus neighbour's canonical links (its top 3 slices): layout
+ * [d][z][y][x][mu][3][3] for d = t (3), [t][d][y][x][mu][3][3] for d = z (2).  Entries of other
+ * directions are ignored (may be NULL).  Same device-ness as fat and lng (on_device).  This is
+ * how the P2P transport (no NCCL communicator) loads links. */
+DSLASH_API dslash_status dslash_load_links_halo(dslash_t h, const void* fat, const void* lng,
+                                                const void* const slab_fat[4], const void* const slab_lng[4],
+                                                int32_t on_device, dslash_stream_t stream);
 
 /* chi = D psi on target parity `parity`.  out: device [3][Vh_local] complex on parity
  * `parity`; in: device [3][Vh_local] complex on parity 1-parity.  Both caller-owned,

@@ -55,14 +55,15 @@ class Dslash:
 
     def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="dir2", block=0,
                  force_halo=0, overlap=True, timing=False, rank=0, world_size=1, min_blocks=0, precision="f64",
-                 recon=18):
+                 recon=18, persistent=True, transport="nccl"):
         import torch
         self.global_dims = tuple(int(d) for d in global_dims)
         self.precision = precision
         self.dtype = torch.complex64 if precision == "f32" else torch.complex128
         self.proc_grid = tuple(int(p) for p in proc_grid)
         uid = None
-        if world_size > 1:
+        self.world_size, self.rank, self.transport = world_size, rank, transport
+        if world_size > 1 and transport == "nccl":
             import torch
             import torch.distributed as dist
             t = torch.zeros(128, dtype=torch.uint8, device="cuda" if dist.get_backend() == "nccl" else "cpu")
@@ -80,6 +81,14 @@ class Dslash:
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_MIN_BLOCKS, min_blocks)
             if recon != 18:
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_LONG_RECON, recon)
+            if transport == "p2p":
+                _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_TRANSPORT, _abi.DSLASH_TRANSPORT_P2P)
+                if world_size > 1:      # exchange CUDA IPC handles through torch.distributed
+                    import torch.distributed as dist
+                    blobs = [None] * world_size
+                    dist.all_gather_object(blobs, _abi.dslash_get_ipc_blob(self.h))
+                    _abi.dslash_open_ipc_blobs(self.h, b"".join(blobs))
+            _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_PERSISTENT, int(bool(persistent)))
             if force_halo:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_FORCE_HALO, force_halo)
             _abi.dslash_set_option(self.h, DSLASH_OPT_OVERLAP, int(bool(overlap)))
@@ -96,6 +105,8 @@ class Dslash:
     # -- links
     def load_links(self, fat, lng, stream=None):
         import numpy as np
+        if self.transport == "p2p" and self.world_size > 1:
+            return self._load_links_p2p(np.asarray(fat), np.asarray(lng), stream)
         if isinstance(fat, np.ndarray):
             fat = np.ascontiguousarray(fat, dtype=np.complex128)
             lng = np.ascontiguousarray(lng, dtype=np.complex128)
@@ -107,6 +118,40 @@ class Dslash:
             assert lng.is_cuda and lng.dtype == torch.complex128 and lng.is_contiguous()
             self._check_links(tuple(fat.shape), tuple(lng.shape))
             _abi.dslash_load_links(self.h, fat.data_ptr(), lng.data_ptr(), 1, _stream_handle(stream))
+
+    def _load_links_p2p(self, fat, lng, stream):
+        """Link halo through torch.distributed: send my top 3 slices (t, then z) to the plus
+        neighbour, receive the 3 slices below my origin from the minus neighbour."""
+        import numpy as np
+        import torch
+        import torch.distributed as dist
+        fat = np.ascontiguousarray(fat, dtype=np.complex128)
+        lng = np.ascontiguousarray(lng, dtype=np.complex128)
+        self._check_links(fat.shape, lng.shape)
+        dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+        slabs = {2: [None, None], 3: [None, None]}
+        keep = []
+        for d, axis in ((3, 0), (2, 1)):
+            if not self.plan.halo[d]:
+                continue
+            plus, minus = self.plan.nbr_rank[d][1], self.plan.nbr_rank[d][0]
+            for k, arr in enumerate((fat, lng)):
+                top = np.ascontiguousarray(np.take(arr, range(arr.shape[axis] - 3, arr.shape[axis]), axis=axis))
+                if plus == self.rank:
+                    slabs[d][k] = top
+                    continue
+                send = torch.from_numpy(top.view(np.float64)).to(dev)
+                recv = torch.empty_like(send)
+                reqs = [dist.isend(send, plus), dist.irecv(recv, minus)]
+                for r in reqs:
+                    r.wait()
+                slabs[d][k] = np.ascontiguousarray(recv.cpu().numpy()).view(np.complex128)
+        for d in (2, 3):
+            keep += [s for s in slabs[d] if s is not None]
+        sf = [slabs[d][0].ctypes.data if d in slabs and slabs[d][0] is not None else 0 for d in range(4)]
+        sl = [slabs[d][1].ctypes.data if d in slabs and slabs[d][1] is not None else 0 for d in range(4)]
+        _abi.dslash_load_links_halo(self.h, fat.ctypes.data, lng.ctypes.data, sf, sl, 0, _stream_handle(stream))
+        del keep
 
     def _check_links(self, a, b):
         lx, ly, lz, lt = self.local_dims

@@ -23,7 +23,9 @@ DSLASH_F64, DSLASH_F32, DSLASH_MIXED = 0, 1, 2
 PRECISIONS = {"f64": DSLASH_F64, "f32": DSLASH_F32, "mixed": DSLASH_MIXED}
 DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_DIR2, DSLASH_KERNEL_BULK = 0, 1, 2, 3
 DSLASH_OPT_KERNEL, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_OVERLAP, DSLASH_OPT_TIMING, \
-    DSLASH_OPT_MIN_BLOCKS, DSLASH_OPT_LONG_RECON = range(7)
+    DSLASH_OPT_MIN_BLOCKS, DSLASH_OPT_LONG_RECON, DSLASH_OPT_PERSISTENT, DSLASH_OPT_TRANSPORT = range(9)
+DSLASH_TRANSPORT_NCCL, DSLASH_TRANSPORT_P2P = 0, 1
+TRANSPORTS = {"nccl": DSLASH_TRANSPORT_NCCL, "p2p": DSLASH_TRANSPORT_P2P}
 DSLASH_TIMING_INTERIOR, DSLASH_TIMING_BOUNDARY, DSLASH_TIMING_ALL = range(3)
 KERNELS = {"site": DSLASH_KERNEL_SITE, "dir4": DSLASH_KERNEL_DIR4, "dir2": DSLASH_KERNEL_DIR2,
            "bulk": DSLASH_KERNEL_BULK}
@@ -77,6 +79,11 @@ _SIGS = {
     "dslash_create": ([_i4, _i4, ctypes.c_int32, ctypes.c_int32, _vp, ctypes.c_int32, ctypes.c_int32,
                        ctypes.POINTER(_h)], ctypes.c_int),
     "dslash_get_unique_id": ([_vp], ctypes.c_int),
+    "dslash_ipc_blob_size": ([], ctypes.c_int64),
+    "dslash_get_ipc_blob": ([_h, _vp], ctypes.c_int),
+    "dslash_open_ipc_blobs": ([_h, _vp], ctypes.c_int),
+    "dslash_load_links_halo": ([_h, _vp, _vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.c_int32, _vp],
+                               ctypes.c_int),
     "dslash_set_option": ([_h, ctypes.c_int32, ctypes.c_int64], ctypes.c_int),
     "dslash_load_links": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
@@ -142,6 +149,27 @@ def dslash_create(global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, 
     check(lib.dslash_create(i4(global_dims), i4(proc_grid), parity_mask, precision, uid, nranks, rank,
                             ctypes.byref(h)))
     return h
+
+
+def dslash_ipc_blob_size() -> int:
+    return int(lib.dslash_ipc_blob_size())
+
+
+def dslash_get_ipc_blob(h) -> bytes:
+    buf = ctypes.create_string_buffer(dslash_ipc_blob_size())
+    check(lib.dslash_get_ipc_blob(h, buf), h)
+    return buf.raw
+
+
+def dslash_open_ipc_blobs(h, blobs: bytes):
+    buf = ctypes.create_string_buffer(blobs, len(blobs))
+    return check(lib.dslash_open_ipc_blobs(h, buf), h)
+
+
+def dslash_load_links_halo(h, fat_ptr, lng_ptr, slab_fat_ptrs, slab_lng_ptrs, on_device, stream=0):
+    sf = (ctypes.c_void_p * 4)(*[p or None for p in slab_fat_ptrs])
+    sl = (ctypes.c_void_p * 4)(*[p or None for p in slab_lng_ptrs])
+    return check(lib.dslash_load_links_halo(h, fat_ptr, lng_ptr, sf, sl, on_device, stream), h)
 
 
 def dslash_set_option(h, key, value):

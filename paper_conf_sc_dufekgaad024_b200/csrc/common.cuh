@@ -115,7 +115,7 @@ __device__ __forceinline__ void cmsub(float2& acc, float2 a, float2 b) {
 }
 
 // ---------------------------------------------------------------- kernel parameters
-constexpr int kMaxBoxes = 4;
+constexpr int kMaxBoxes = 5;  // interior + up to 4 boundary slabs (t and z halo)
 
 struct Box {
     int lo[4];

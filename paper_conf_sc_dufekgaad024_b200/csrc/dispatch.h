@@ -2,10 +2,13 @@
 #pragma once
 
 #include "common.cuh"
+#include "stencil.cuh"
 
 namespace hisq {
 
 typedef void (*StencilFn)(StencilParams);
+
+typedef void (*PersistFn)(StencilParams, PersistArgs);
 
 // Each returns the dslash_kernel instantiation for (ghost, lanes 1/2/4, min blocks 2/3/4,
 // right-hand sides per launch 1/2/4/8) of one (precision, long-link recon) pair.
@@ -15,6 +18,15 @@ StencilFn pick_f32_r18(bool ghost, int lanes, int minb, int nrhs);
 StencilFn pick_f32_r12(bool ghost, int lanes, int minb, int nrhs);
 StencilFn pick_mixed_r18(bool ghost, int lanes, int minb, int nrhs);
 StencilFn pick_mixed_r12(bool ghost, int lanes, int minb, int nrhs);
+
+// the persistent fused kernel (stencil.cuh) of one (precision, recon): lanes 1/2/4; mode 0 = no
+// halo, 1 = halo (interior, then boundary tiles if the faces have landed), 2 = boundary clean-up
+PersistFn persist_f64_r18(int mode, int lanes);
+PersistFn persist_f64_r12(int mode, int lanes);
+PersistFn persist_f32_r18(int mode, int lanes);
+PersistFn persist_f32_r12(int mode, int lanes);
+PersistFn persist_mixed_r18(int mode, int lanes);
+PersistFn persist_mixed_r12(int mode, int lanes);
 
 // The TMA-staged persistent kernel (bulk.cuh): function, dynamic shared memory, threads per CTA,
 // sites per tile.  precision: 0 fp64, 1 fp32, 2 mixed (DSLASH_F64/F32/MIXED).

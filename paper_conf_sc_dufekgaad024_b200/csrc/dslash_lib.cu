@@ -186,6 +186,16 @@ static dslash_status alloc_halo(dslash_t h, int nrhs) {
     return DSLASH_OK;
 }
 
+static constexpr int kP2PMaxRhs = 8;  // ghost capacity with the P2P transport (IPC-exported once)
+
+static dslash_status alloc_flags(dslash_t h) {
+    if (!h->flags) {
+        CU(h, cudaMalloc(&h->flags, 16 * sizeof(unsigned int)));
+        CU(h, cudaMemset(h->flags, 0, 16 * sizeof(unsigned int)));
+    }
+    return DSLASH_OK;
+}
+
 extern "C" dslash_status dslash_create(const int32_t G[4], const int32_t P[4], int32_t parity_mask, int32_t precision,
                                        const void* nccl_unique_id, int32_t nranks, int32_t rank, dslash_t* out) {
     if (!out) return fail(nullptr, DSLASH_ERR_ARG, "NULL out");
@@ -194,7 +204,6 @@ extern "C" dslash_status dslash_create(const int32_t G[4], const int32_t P[4], i
         return fail(nullptr, DSLASH_ERR_ARG, "parity_mask %d not in {0,1,2}", parity_mask);
     if (precision != DSLASH_F64 && precision != DSLASH_F32 && precision != DSLASH_MIXED)
         return fail(nullptr, DSLASH_ERR_ARG, "precision %d unknown", precision);
-    if (nranks > 1 && !nccl_unique_id) return fail(nullptr, DSLASH_ERR_ARG, "nranks > 1 needs an NCCL unique id");
     dslash_plan_t plan;
     dslash_status st = dslash_plan(G, P, rank, nranks, 0, &plan);
     if (st != DSLASH_OK) return st;
@@ -215,12 +224,15 @@ extern "C" dslash_status dslash_create(const int32_t G[4], const int32_t P[4], i
         return bail(DSLASH_ERR_CUDA);
     }
     if ((e = cudaStreamCreateWithFlags(&h->comm, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaStreamCreateWithFlags(&h->bstream, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&h->ev_bdone, cudaEventDisableTiming)) != cudaSuccess ||
         (e = cudaEventCreateWithFlags(&h->ev_start, cudaEventDisableTiming)) != cudaSuccess ||
         (e = cudaEventCreateWithFlags(&h->ev_halo, cudaEventDisableTiming)) != cudaSuccess) {
         fail(h, DSLASH_ERR_CUDA, "stream/event creation: %s", cudaGetErrorString(e));
         return bail(DSLASH_ERR_CUDA);
     }
-    if (nranks > 1) {
+    h->transport = (nranks > 1 && !nccl_unique_id) ? DSLASH_TRANSPORT_P2P : DSLASH_TRANSPORT_NCCL;
+    if (nranks > 1 && nccl_unique_id) {
         ncclUniqueId id;
         memcpy(&id, nccl_unique_id, sizeof id);
         ncclResult_t r = ncclCommInitRank(&h->nccl, nranks, id, rank);
@@ -230,7 +242,8 @@ extern "C" dslash_status dslash_create(const int32_t G[4], const int32_t P[4], i
             return bail(DSLASH_ERR_NCCL);
         }
     }
-    if ((st = alloc_halo(h, 1)) != DSLASH_OK) return bail(st);
+    if ((st = alloc_halo(h, h->transport == DSLASH_TRANSPORT_P2P ? kP2PMaxRhs : 1)) != DSLASH_OK) return bail(st);
+    if (h->transport == DSLASH_TRANSPORT_P2P && (st = alloc_flags(h)) != DSLASH_OK) return bail(st);
     *out = h;
     return DSLASH_OK;
 }
@@ -261,13 +274,28 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             if (st != DSLASH_OK) return fail(h, st, "%s", g_last_error.c_str());
             h->plan = p;
             h->force_halo = (int)value;
-            return alloc_halo(h, 1);
+            return alloc_halo(h, h->transport == DSLASH_TRANSPORT_P2P ? kP2PMaxRhs : 1);
         }
         case DSLASH_OPT_OVERLAP:
             h->overlap = value != 0;
             return DSLASH_OK;
         case DSLASH_OPT_TIMING:
             h->timing = value != 0;
+            return DSLASH_OK;
+        case DSLASH_OPT_TRANSPORT: {
+            if (value != DSLASH_TRANSPORT_NCCL && value != DSLASH_TRANSPORT_P2P)
+                return fail(h, DSLASH_ERR_ARG, "unknown transport %lld", (long long)value);
+            if (h->loaded || h->p2p_ready)
+                return fail(h, DSLASH_ERR_STATE, "the transport must be chosen before load_links / IPC setup");
+            if (value == DSLASH_TRANSPORT_NCCL && h->plan.nranks > 1 && !h->nccl)
+                return fail(h, DSLASH_ERR_STATE, "NCCL transport needs dslash_create with an NCCL unique id");
+            h->transport = (int)value;
+            dslash_status st = alloc_halo(h, value == DSLASH_TRANSPORT_P2P ? kP2PMaxRhs : 1);
+            if (st == DSLASH_OK && value == DSLASH_TRANSPORT_P2P) st = alloc_flags(h);
+            return st;
+        }
+        case DSLASH_OPT_PERSISTENT:
+            h->persistent = value != 0;
             return DSLASH_OK;
         case DSLASH_OPT_LONG_RECON:
             if (value != 18 && value != 12) return fail(h, DSLASH_ERR_ARG, "long-link recon %lld must be 18 or 12", (long long)value);
@@ -294,8 +322,10 @@ static int lanes_of(int kernel) {
 }
 
 // ============================================================================ link loading
-extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const void* lng, int32_t on_device,
-                                           dslash_stream_t stream) {
+// slab_fat / slab_lng (may be NULL): caller-provided lower link slabs per direction (same device-ness
+// as fat / lng); where absent for a halo direction with another rank as neighbour, NCCL fetches them
+static dslash_status load_links_impl(dslash_t h, const void* fat, const void* lng, const void* const* slab_fat_in,
+                                     const void* const* slab_lng_in, int32_t on_device, dslash_stream_t stream) {
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!fat || !lng) return fail(h, DSLASH_ERR_ARG, "NULL link pointer");
     cudaStream_t s = (cudaStream_t)stream;
@@ -355,12 +385,28 @@ extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
     // Exchange: rank sends its top 3 slices to its plus neighbour, receives into its lower
     // slab from its minus neighbour.  All ranks issue t then z, fat then long (same order).
     bool need_nccl = false;
-    for (int d = 3; d >= 2; --d)
-        if (p.halo[d] && p.nbr_rank[d][1] != p.rank) need_nccl = true;
+    bool given[4] = {false, false, false, false};
+    for (int d = 3; d >= 2; --d) {
+        if (!p.halo[d]) continue;
+        given[d] = slab_fat_in && slab_lng_in && slab_fat_in[d] && slab_lng_in[d];
+        if (!given[d] && p.nbr_rank[d][1] != p.rank) need_nccl = true;
+    }
+    if (need_nccl && !h->nccl) {
+        cleanup();
+        return fail(h, DSLASH_ERR_STATE,
+                    "no NCCL communicator for the link halo: pass the slabs with dslash_load_links_halo");
+    }
     const int L0 = p.local_dims[0], L1 = p.local_dims[1], L2 = p.local_dims[2], L3 = p.local_dims[3];
     const size_t row = (size_t)L0 * L1 * 36 * sizeof(double2);  // one z-slice of one t
     for (int d = 3; d >= 2; --d) {
         if (!p.halo[d]) continue;
+        if (given[d]) {
+            const size_t bytes = (size_t)3 * (V / p.local_dims[d]) * 36 * sizeof(double2);
+            const cudaMemcpyKind kind = on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+            CUL(cudaMemcpyAsync(slab[d][0], slab_fat_in[d], bytes, kind, s));
+            CUL(cudaMemcpyAsync(slab[d][1], slab_lng_in[d], bytes, kind, s));
+            continue;
+        }
         for (int k = 0; k < 2; ++k) {
             const double2* src = k ? dlng : dfat;
             if (d == 3) {
@@ -386,7 +432,7 @@ extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
         CUL(cudaStreamSynchronize(s));
         ncclResult_t r = ncclGroupStart();
         for (int d = 3; d >= 2 && r == ncclSuccess; --d) {
-            if (!p.halo[d] || p.nbr_rank[d][1] == p.rank) continue;
+            if (!p.halo[d] || p.nbr_rank[d][1] == p.rank || given[d]) continue;
             const size_t n = (size_t)3 * (V / p.local_dims[d]) * 36 * 2;  // doubles
             for (int k = 0; k < 2 && r == ncclSuccess; ++k) {
                 r = ncclSend(send[d][k], n, ncclDouble, p.nbr_rank[d][1], h->nccl, s);
@@ -472,13 +518,210 @@ extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
     return DSLASH_OK;
 }
 
+extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const void* lng, int32_t on_device,
+                                           dslash_stream_t stream) {
+    return load_links_impl(h, fat, lng, nullptr, nullptr, on_device, stream);
+}
+
+extern "C" dslash_status dslash_load_links_halo(dslash_t h, const void* fat, const void* lng,
+                                                const void* const slab_fat[4], const void* const slab_lng[4],
+                                                int32_t on_device, dslash_stream_t stream) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (!slab_fat || !slab_lng) return fail(h, DSLASH_ERR_ARG, "NULL slab arrays");
+    for (int d = 2; d < 4; ++d)
+        if (h->plan.halo[d] && h->plan.nbr_rank[d][1] != h->plan.rank && (!slab_fat[d] || !slab_lng[d]))
+            return fail(h, DSLASH_ERR_ARG, "missing link slab for halo direction %d", d);
+    return load_links_impl(h, fat, lng, slab_fat, slab_lng, on_device, stream);
+}
+
+// cuStreamWriteValue32 through the runtime's driver entry point (no link-time libcuda): the halo
+// stream's front end writes the epoch flag the persistent kernel waits on, without an SM.
+typedef int (*WriteValue32Fn)(cudaStream_t, unsigned long long, unsigned int, unsigned int);
+static WriteValue32Fn write_value_fn() {
+    static WriteValue32Fn fn = nullptr;
+    static bool tried = false;
+    if (!tried) {
+        tried = true;
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuStreamWriteValue32", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (WriteValue32Fn)p;
+        else
+            cudaGetLastError();
+    }
+    return fn;
+}
+
+// cuStreamWaitValue32 (flags 0 = CU_STREAM_WAIT_VALUE_GEQ: wait until (int32)(*addr - value) >= 0)
+typedef int (*WaitValue32Fn)(cudaStream_t, unsigned long long, unsigned int, unsigned int);
+static WaitValue32Fn wait_value_fn() {
+    static WaitValue32Fn fn = nullptr;
+    static bool tried = false;
+    if (!tried) {
+        tried = true;
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuStreamWaitValue32", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (WaitValue32Fn)p;
+        else
+            cudaGetLastError();
+    }
+    return fn;
+}
+
+
+// ---------------------------------------------------------------------------- P2P transport
+struct IpcBlob {
+    int32_t magic, rank, device, reserved;
+    cudaIpcMemHandle_t ghost[4][2];
+    cudaIpcMemHandle_t flags;
+};
+static constexpr int32_t kIpcMagic = 0x48495351;  // "HISQ"
+
+extern "C" int64_t dslash_ipc_blob_size(void) { return (int64_t)sizeof(IpcBlob); }
+
+extern "C" dslash_status dslash_get_ipc_blob(dslash_t h, void* blob) {
+    if (!h || !blob) return fail(h, DSLASH_ERR_ARG, "NULL argument");
+    if (h->transport != DSLASH_TRANSPORT_P2P) return fail(h, DSLASH_ERR_STATE, "set DSLASH_TRANSPORT_P2P first");
+    IpcBlob b;
+    memset(&b, 0, sizeof b);
+    b.magic = kIpcMagic;
+    b.rank = h->plan.rank;
+    b.device = h->device;
+    for (int d = 2; d < 4; ++d)
+        for (int side = 0; side < 2; ++side)
+            if (h->ghost[d][side]) CU(h, cudaIpcGetMemHandle(&b.ghost[d][side], h->ghost[d][side]));
+    CU(h, cudaIpcGetMemHandle(&b.flags, h->flags));
+    memcpy(blob, &b, sizeof b);
+    return DSLASH_OK;
+}
+
+// my bottom face (side 0) fills the minus neighbour's PLUS ghost, my top face (side 1) the plus
+// neighbour's MINUS ghost; after consuming my ghost[d][side] I release it to the rank that filled it
+static void set_peer(dslash_t h, int d, int side, char* nbr_ghost_other_side, unsigned int* nbr_flags) {
+    const int other = 1 - side;
+    h->peer_ghost[d][side] = nbr_ghost_other_side;
+    h->peer_ready[d][side] = nbr_flags + 2 * d + other;
+    h->peer_free[d][side] = nbr_flags + 8 + 2 * d + other;
+}
+
+extern "C" dslash_status dslash_open_ipc_blobs(dslash_t h, const void* blobs) {
+    if (!h || !blobs) return fail(h, DSLASH_ERR_ARG, "NULL argument");
+    if (h->transport != DSLASH_TRANSPORT_P2P) return fail(h, DSLASH_ERR_STATE, "set DSLASH_TRANSPORT_P2P first");
+    const dslash_plan_t& p = h->plan;
+    const IpcBlob* all = static_cast<const IpcBlob*>(blobs);
+    std::vector<unsigned int*> flags_of(p.nranks, nullptr);
+    for (int d = 2; d < 4; ++d) {
+        if (!p.halo[d]) continue;
+        for (int side = 0; side < 2; ++side) {
+            const int nbr = p.nbr_rank[d][side];
+            if (nbr == p.rank) {
+                set_peer(h, d, side, h->ghost[d][1 - side], h->flags);
+                continue;
+            }
+            const IpcBlob& b = all[nbr];
+            if (b.magic != kIpcMagic || b.rank != nbr)
+                return fail(h, DSLASH_ERR_ARG, "IPC blob of rank %d is malformed or out of order", nbr);
+            if (!flags_of[nbr]) {
+                void* fp = nullptr;
+                CU(h, cudaIpcOpenMemHandle(&fp, b.flags, cudaIpcMemLazyEnablePeerAccess));
+                h->ipc_opened.push_back(fp);
+                flags_of[nbr] = static_cast<unsigned int*>(fp);
+            }
+            void* gp = nullptr;
+            CU(h, cudaIpcOpenMemHandle(&gp, b.ghost[d][1 - side], cudaIpcMemLazyEnablePeerAccess));
+            h->ipc_opened.push_back(gp);
+            set_peer(h, d, side, static_cast<char*>(gp), flags_of[nbr]);
+        }
+    }
+    h->p2p_ready = true;
+    return DSLASH_OK;
+}
+
+// pointer setup when every neighbour is this rank (self-halo): no IPC needed
+static dslash_status p2p_prepare(dslash_t h) {
+    if (h->p2p_ready) return DSLASH_OK;
+    const dslash_plan_t& p = h->plan;
+    for (int d = 2; d < 4; ++d)
+        if (p.halo[d] && (p.nbr_rank[d][0] != p.rank || p.nbr_rank[d][1] != p.rank))
+            return fail(h, DSLASH_ERR_STATE, "P2P transport: call dslash_open_ipc_blobs first");
+    for (int d = 2; d < 4; ++d)
+        if (p.halo[d])
+            for (int side = 0; side < 2; ++side) set_peer(h, d, side, h->ghost[d][1 - side], h->flags);
+    h->p2p_ready = true;
+    return DSLASH_OK;
+}
+
 // ============================================================================ halo exchange
 static bool any_halo(const dslash_plan_t& p) { return p.halo[2] || p.halo[3]; }
+
+// P2P exchange of epoch e on the communication stream (copy engines + stream memory operations):
+//   1. release my ghosts of epoch e-1 to the ranks that filled them (every kernel that read them
+//      precedes ev_start),
+//   2. wait until the ghosts my faces go to were released by their consumers (epoch e-1),
+//   3. copy my bottom / top faces straight into the neighbours' ghosts (IPC-mapped),
+//   4. raise their ready flags to e.
+// Consumers wait for their own ready flags (halo_landed).  Every rank releases before it waits, so
+// the ring of waits always resolves.
+static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaStream_t s) {
+    const dslash_plan_t& p = h->plan;
+    if (nrhs > kP2PMaxRhs)
+        return fail(h, DSLASH_ERR_UNSUPPORTED, "P2P transport: at most %d right-hand sides per apply", kP2PMaxRhs);
+    dslash_status st = p2p_prepare(h);
+    if (st != DSLASH_OK) return st;
+    WriteValue32Fn wr = write_value_fn();
+    WaitValue32Fn wt = wait_value_fn();
+    if (!wr || !wt) return fail(h, DSLASH_ERR_UNSUPPORTED, "stream memory operations unavailable");
+    const unsigned int e = ++h->epoch;
+    const size_t es = vec_elem(h);
+    const char* src = static_cast<const char*>(in);
+    const size_t vh = (size_t)p.vh_local;
+    const size_t L1 = p.local_dims[1], L2 = p.local_dims[2], L3 = p.local_dims[3];
+    const size_t lxh = p.local_dims[0] / 2;
+    const size_t rows = (size_t)3 * nrhs;
+    CU(h, cudaEventRecord(h->ev_start, s));
+    CU(h, cudaStreamWaitEvent(h->comm, h->ev_start, 0));
+    for (int d = 3; d >= 2; --d)
+        if (p.halo[d])
+            for (int side = 0; side < 2; ++side)
+                if (wr(h->comm, (unsigned long long)(uintptr_t)h->peer_free[d][side], e - 1, 0) != 0)
+                    return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 (release) failed");
+    for (int d = 3; d >= 2; --d)
+        if (p.halo[d])
+            for (int side = 0; side < 2; ++side)
+                if (wt(h->comm, (unsigned long long)(uintptr_t)(h->flags + 8 + 2 * d + side), e - 1, 0) != 0)
+                    return fail(h, DSLASH_ERR_CUDA, "cuStreamWaitValue32 (free) failed");
+    if (p.halo[3]) {
+        const size_t tslab = 3 * lxh * L1 * L2;
+        CU(h, cudaMemcpy2DAsync(h->peer_ghost[3][0], tslab * es, src, vh * es, tslab * es, rows,
+                                cudaMemcpyDeviceToDevice, h->comm));
+        CU(h, cudaMemcpy2DAsync(h->peer_ghost[3][1], tslab * es, src + (vh - tslab) * es, vh * es, tslab * es, rows,
+                                cudaMemcpyDeviceToDevice, h->comm));
+    }
+    if (p.halo[2]) {
+        const size_t zrow = lxh * L1;
+        CU(h, cudaMemcpy2DAsync(h->peer_ghost[2][0], 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
+                                cudaMemcpyDeviceToDevice, h->comm));
+        CU(h, cudaMemcpy2DAsync(h->peer_ghost[2][1], 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es,
+                                3 * zrow * es, rows * L3, cudaMemcpyDeviceToDevice, h->comm));
+    }
+    for (int d = 3; d >= 2; --d)
+        if (p.halo[d])
+            for (int side = 0; side < 2; ++side)
+                if (wr(h->comm, (unsigned long long)(uintptr_t)h->peer_ready[d][side], e, 0) != 0)
+                    return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 (ready) failed");
+    CU(h, cudaEventRecord(h->ev_halo, h->comm));
+    h->halo_pending = true;
+    return DSLASH_OK;
+}
 
 // Exchange the depth-3 faces of nrhs source vectors stored back to back ([nrhs][3][vh]).
 static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaStream_t s) {
     const dslash_plan_t& p = h->plan;
     if (!any_halo(p)) return DSLASH_OK;
+    if (h->transport == DSLASH_TRANSPORT_P2P) return halo_start_p2p(h, in, nrhs, s);
     if (nrhs > h->ghost_rhs) {
         CU(h, cudaStreamSynchronize(h->comm));  // old ghosts may still be read by queued kernels
         CU(h, cudaDeviceSynchronize());
@@ -558,9 +801,19 @@ extern "C" dslash_status dslash_halo_start(dslash_t h, const void* in, int32_t s
     return halo_start_impl(h, in, 1, (cudaStream_t)stream);
 }
 
+// `stream` waits until this rank's ghosts hold the current epoch's faces and its own sends are
+// done (P2P: my ready flags, raised by the neighbours; NCCL / self copies: the comm event).
 extern "C" dslash_status dslash_halo_wait(dslash_t h, dslash_stream_t stream) {
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!h->halo_pending) return DSLASH_OK;
+    if (h->transport == DSLASH_TRANSPORT_P2P) {
+        WaitValue32Fn wt = wait_value_fn();
+        for (int d = 3; d >= 2; --d)
+            if (h->plan.halo[d])
+                for (int side = 0; side < 2; ++side)
+                    if (wt((cudaStream_t)stream, (unsigned long long)(uintptr_t)(h->flags + 2 * d + side), h->epoch, 0) != 0)
+                        return fail(h, DSLASH_ERR_CUDA, "cuStreamWaitValue32 (ready) failed");
+    }
     CU(h, cudaStreamWaitEvent((cudaStream_t)stream, h->ev_halo, 0));
     h->halo_pending = false;
     return DSLASH_OK;
@@ -624,14 +877,16 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
             tl->kind = kind;
             CU(h, cudaEventRecord(tl->a, s));
         }
-        if (!h->sched) CU(h, cudaMalloc(&h->sched, sizeof(unsigned long long)));
-        if (!h->sched_init) {
-            CU(h, cudaMemsetAsync(h->sched, 0, sizeof(unsigned long long), s));
-            h->sched_init = true;
+        // one ticket counter per kernel class: interior and boundary launches may run concurrently
+        if (!h->sched) {
+            CU(h, cudaMalloc(&h->sched, 4 * sizeof(unsigned long long)));
+            CU(h, cudaMemset(h->sched, 0, 4 * sizeof(unsigned long long)));
         }
-        bk.fn<<<grid, bk.threads, bk.smem, s>>>(K, h->sched, h->sched_next);
+        const int slot = ghost ? 1 : 0;
+        bk.fn<<<grid, bk.threads, bk.smem, s>>>(K, h->sched + slot, h->sched_next[slot]);
         // tickets this launch consumes (bulk.cuh): (ceil(ntiles / B) + 2 grid) * B
-        h->sched_next += ((unsigned long long)((ntiles + bk.batch - 1) / bk.batch) + 2ull * grid) * bk.batch;
+        h->sched_next[slot] +=
+            ((unsigned long long)((ntiles + bk.batch - 1) / bk.batch) + 2ull * grid) * bk.batch;
         CU(h, cudaGetLastError());
         if (tl) CU(h, cudaEventRecord(tl->b, s));
         return DSLASH_OK;
@@ -687,6 +942,112 @@ static dslash_status launch_rhs(dslash_t h, StencilParams K, const dslash_box_t*
     return DSLASH_OK;
 }
 
+// ---------------------------------------------------------------------------- persistent path
+static int persist_occupancy(dslash_t h, PersistFn fn, int bs) {
+    static PersistFn last_fn = nullptr;
+    static int last_bs = 0, last_occ = 1;
+    if (fn != last_fn || bs != last_bs) {
+        int occ = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, bs, 0) != cudaSuccess || occ < 1) occ = 1;
+        last_fn = fn;
+        last_bs = bs;
+        last_occ = occ;
+    }
+    (void)h;
+    return last_occ;
+}
+
+static PersistFn pick_persist(int precision, int recon, int mode, int lanes) {
+    const bool r12 = recon == 12;
+    switch (precision) {
+        case DSLASH_F32: return r12 ? persist_f32_r12(mode, lanes) : persist_f32_r18(mode, lanes);
+        case DSLASH_MIXED: return r12 ? persist_mixed_r12(mode, lanes) : persist_mixed_r18(mode, lanes);
+        default: return r12 ? persist_f64_r12(mode, lanes) : persist_f64_r18(mode, lanes);
+    }
+}
+
+// One persistent launch per apply (stencil.cuh, dslash_persistent_kernel): interior boxes
+// first; with a halo, blocks continue with boundary tiles if the faces have landed, and a
+// stream-ordered clean-up launch after the halo event takes the boundary tiles left over.
+static dslash_status apply_persistent(dslash_t h, StencilParams K, cudaStream_t s) {
+    const dslash_plan_t& p = h->plan;
+    const bool halo = any_halo(p);
+    dslash_box_t all[kMaxBoxes];
+    int n = 0;
+    for (int i = 0; i < p.n_interior; ++i) all[n++] = p.interior[i];
+    for (int i = 0; i < p.n_boundary; ++i) all[n++] = p.boundary[i];
+    fill_boxes(K, all, n);
+    if (!h->sched) {
+        CU(h, cudaMalloc(&h->sched, 4 * sizeof(unsigned long long)));
+        CU(h, cudaMemset(h->sched, 0, 4 * sizeof(unsigned long long)));
+    }
+    const int lanes = lanes_of(h->kernel);
+    const int bs = h->block ? h->block : default_block(lanes);
+    const int64_t sites = K.box_start[K.nbox];
+    const int64_t isites = halo ? p.interior_sites : sites;
+    PersistArgs A{};
+    A.sched = h->sched + 2;
+    A.base = h->sched_next[2];
+    A.interior_sites = isites;
+    A.ntiles_int = (isites * lanes + bs - 1) / bs;
+    A.ntiles_bnd = ((sites - isites) * lanes + bs - 1) / bs;
+    dslash_s::TimedLaunch* tl = nullptr;
+    if (h->timing) {
+        if (h->tused == h->tpool.size()) {
+            dslash_s::TimedLaunch t{};
+            CU(h, cudaEventCreate(&t.a));
+            CU(h, cudaEventCreate(&t.b));
+            h->tpool.push_back(t);
+        }
+        tl = &h->tpool[h->tused++];
+        tl->kind = DSLASH_TIMING_ALL;
+    }
+    if (halo) {
+        if (!h->halo_flag) {
+            CU(h, cudaMalloc(&h->halo_flag, sizeof(unsigned int)));
+            CU(h, cudaMemset(h->halo_flag, 0, sizeof(unsigned int)));
+            h->epoch = 0;
+        }
+        CU(h, cudaMemsetAsync(A.sched + 1, 0, sizeof(unsigned long long), s));  // boundary tickets
+        dslash_status st = halo_start_impl(h, K.in, 1, s);
+        if (st != DSLASH_OK) return st;
+        for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
+            K.ghost[d][0] = h->ghost[d][0];
+            K.ghost[d][1] = h->ghost[d][1];
+        }
+        if (h->transport == DSLASH_TRANSPORT_P2P) {
+            // the faces have landed when the neighbours raised my ready flags (halo_start_p2p)
+            for (int d = 3; d >= 2; --d)
+                if (p.halo[d])
+                    for (int side = 0; side < 2; ++side) A.flags[A.nflags++] = h->flags + 2 * d + side;
+        } else {
+            ++h->epoch;
+            if (write_value_fn()(h->comm, (unsigned long long)(uintptr_t)h->halo_flag, h->epoch, 0) != 0)
+                return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 failed");
+            A.flags[A.nflags++] = h->halo_flag;
+        }
+        A.epoch = h->epoch;
+    }
+    const PersistFn fn = pick_persist(h->precision, h->recon, halo ? 1 : 0, lanes);
+    const int64_t cap = (int64_t)persist_occupancy(h, fn, bs) * num_sms(h);
+    const int64_t want = A.ntiles_int + (halo ? A.ntiles_bnd : 0);
+    const unsigned grid = (unsigned)(want < cap ? (want > 0 ? want : 1) : cap);
+    if (tl) CU(h, cudaEventRecord(tl->a, s));
+    fn<<<grid, bs, 0, s>>>(K, A);
+    CU(h, cudaGetLastError());
+    h->sched_next[2] += (unsigned long long)A.ntiles_int + 2ull * grid;
+    if (halo) {
+        dslash_status st = dslash_halo_wait(h, (dslash_stream_t)s);  // the faces are in the ghosts
+        if (st != DSLASH_OK) return st;
+        const PersistFn clean = pick_persist(h->precision, h->recon, 2, lanes);
+        const unsigned g2 = (unsigned)(A.ntiles_bnd < cap ? (A.ntiles_bnd > 0 ? A.ntiles_bnd : 1) : cap);
+        clean<<<g2, bs, 0, s>>>(K, A);
+        CU(h, cudaGetLastError());
+    }
+    if (tl) CU(h, cudaEventRecord(tl->b, s));
+    return DSLASH_OK;
+}
+
 static dslash_status check_vectors(dslash_t h, const void* out, const void* in, int nrhs) {
     if (!out || !in) return fail(h, DSLASH_ERR_ARG, "NULL vector pointer");
     if (((uintptr_t)out & 15) || ((uintptr_t)in & 15)) return fail(h, DSLASH_ERR_ARG, "vectors must be 16-byte aligned");
@@ -728,6 +1089,8 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         K.face_vh[d] = p.face_vh[d];
         if (p.halo[d]) K.halo_mask |= 1 << d;
     }
+    if (h->persistent && nrhs == 1 && h->kernel != DSLASH_KERNEL_BULK && write_value_fn())
+        return apply_persistent(h, K, s);
     if (!any_halo(p)) return launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
     if ((st = halo_start_impl(h, in, nrhs, s)) != DSLASH_OK) return st;
     for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
@@ -735,10 +1098,17 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         K.ghost[d][1] = h->ghost[d][1];
     }
     if (h->overlap) {
+        // interior on the caller's stream; boundary on the handle's boundary stream as soon as the
+        // halo lands, so it fills the SMs the interior kernel's tail leaves idle; then the caller's
+        // stream joins (the two kernels write disjoint sites of out)
         st = launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
         if (st != DSLASH_OK) return st;
-        if ((st = dslash_halo_wait(h, stream)) != DSLASH_OK) return st;
-        return launch_rhs(h, K, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, s, nrhs);
+        if ((st = dslash_halo_wait(h, (dslash_stream_t)h->bstream)) != DSLASH_OK) return st;
+        st = launch_rhs(h, K, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, h->bstream, nrhs);
+        if (st != DSLASH_OK) return st;
+        CU(h, cudaEventRecord(h->ev_bdone, h->bstream));
+        CU(h, cudaStreamWaitEvent(s, h->ev_bdone, 0));
+        return DSLASH_OK;
     }
     if ((st = dslash_halo_wait(h, stream)) != DSLASH_OK) return st;
     if (p.n_interior + p.n_boundary > kMaxBoxes) {
@@ -897,6 +1267,9 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
     }
     if (h->ev_batch) cudaEventDestroy(h->ev_batch);
     if (h->sched) cudaFree(h->sched);
+    if (h->halo_flag) cudaFree(h->halo_flag);
+    for (void* q : h->ipc_opened) cudaIpcCloseMemHandle(q);
+    if (h->flags) cudaFree(h->flags);
     for (void* v : h->cg_vec)
         if (v) cudaFree(v);
     if (h->cg_partial) cudaFree(h->cg_partial);
@@ -911,6 +1284,8 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
     if (h->ev_start) cudaEventDestroy(h->ev_start);
     if (h->ev_halo) cudaEventDestroy(h->ev_halo);
     if (h->comm) cudaStreamDestroy(h->comm);
+    if (h->bstream) cudaStreamDestroy(h->bstream);
+    if (h->ev_bdone) cudaEventDestroy(h->ev_bdone);
     delete h;
     return DSLASH_OK;
 }

@@ -8,6 +8,7 @@
 #include <vector>
 
 #include "hisq_dslash.h"
+#include "dispatch.h"
 
 struct dslash_s {
     dslash_plan_t plan{};
@@ -31,7 +32,8 @@ struct dslash_s {
     cudaEvent_t ev_in_ready[kSlots] = {}, ev_in_free[kSlots] = {}, ev_out_ready[kSlots] = {},
                 ev_out_free[kSlots] = {}, ev_batch = nullptr;
     cudaStream_t comm = nullptr;
-    cudaEvent_t ev_start = nullptr, ev_halo = nullptr;
+    cudaStream_t bstream = nullptr;  // boundary kernels (overlap the interior kernel's tail)
+    cudaEvent_t ev_start = nullptr, ev_halo = nullptr, ev_bdone = nullptr;
     bool halo_pending = false;
     ncclComm_t nccl = nullptr;
     struct TimedLaunch {
@@ -45,10 +47,26 @@ struct dslash_s {
     void* cg_vec[4] = {};
     double* cg_partial = nullptr;
     double* cg_scalar = nullptr;
-    // tile scheduler of the TMA kernel: a ticket counter and the first ticket of the next launch
-    unsigned long long* sched = nullptr;
-    unsigned long long sched_next = 0;
-    bool sched_init = false;
+    // tile scheduler of the TMA kernel: ticket counters ([0] interior, [0/1] boundary launches,
+    // which may overlap) and the first ticket of each counter's next launch
+    unsigned long long* sched = nullptr;   // [0] TMA interior, [1] TMA boundary, [2] persistent
+                                           // interior (monotonic), [3] persistent boundary (reset)
+    unsigned long long sched_next[3] = {0, 0, 0};
+    // persistent fused kernel (DSLASH_OPT_PERSISTENT): the halo epoch flag it looks at
+    int persistent = 1;
+    unsigned int* halo_flag = nullptr;
+    unsigned int epoch = 0;             // halo exchanges started so far
+    // P2P transport (DSLASH_TRANSPORT_P2P): CUDA-IPC-mapped neighbour buffers, copy engines and
+    // stream memory operations.  flags (device, IPC-exported): [0..7] ready[d][side] (written by the
+    // neighbour that fills my ghost[d][side]), [8..15] free_from[d][side] (written by the neighbour
+    // whose ghost my bottom (side 0) / top (side 1) face fills, once it consumed it).
+    int transport = DSLASH_TRANSPORT_NCCL;
+    unsigned int* flags = nullptr;
+    char* peer_ghost[4][2] = {};        // [d][0]: minus nbr's plus ghost; [d][1]: plus nbr's minus ghost
+    unsigned int* peer_ready[4][2] = {};  // the ready flag of that ghost
+    unsigned int* peer_free[4][2] = {};   // [d][0]: minus nbr's free_from[d][1]; [d][1]: plus nbr's free_from[d][0]
+    std::vector<void*> ipc_opened;
+    bool p2p_ready = false;
     dslash_status err = DSLASH_OK;
     std::string msg;
 };

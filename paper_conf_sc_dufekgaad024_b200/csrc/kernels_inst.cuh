@@ -39,11 +39,30 @@ StencilFn pick_any(bool ghost, int lanes, int minb, int nrhs) {
     return ghost ? pick_lanes<LR, VR, true, RECON>(lanes, minb, nrhs) : pick_lanes<LR, VR, false, RECON>(lanes, minb, nrhs);
 }
 
+template <typename LR, typename VR, int LANES, int RECON>
+PersistFn pick_persist_l(int mode) {
+    switch (mode) {
+        case 0: return dslash_persistent_kernel<LR, VR, LANES, false, RECON, false>;  // no halo
+        case 1: return dslash_persistent_kernel<LR, VR, LANES, true, RECON, false>;   // halo, main
+        default: return dslash_persistent_kernel<LR, VR, LANES, true, RECON, true>;   // halo, clean-up
+    }
+}
+
+template <typename LR, typename VR, int RECON>
+PersistFn pick_persist(int mode, int lanes) {
+    switch (lanes) {
+        case 1: return pick_persist_l<LR, VR, 1, RECON>(mode);
+        case 2: return pick_persist_l<LR, VR, 2, RECON>(mode);
+        default: return pick_persist_l<LR, VR, 4, RECON>(mode);
+    }
+}
+
 }  // namespace hisq
 
-#define HISQ_DEFINE_PICK(NAME, LR, VR, RECON)                                  \
+#define HISQ_DEFINE_PICK(NAME, PNAME, LR, VR, RECON)                           \
     namespace hisq {                                                           \
     StencilFn NAME(bool ghost, int lanes, int minb, int nrhs) {                \
         return pick_any<LR, VR, RECON>(ghost, lanes, minb, nrhs);              \
     }                                                                          \
+    PersistFn PNAME(int mode, int lanes) { return pick_persist<LR, VR, RECON>(mode, lanes); } \
     }

@@ -152,6 +152,8 @@ static dslash_status check_solver_args(dslash_t h, const void* a, const void* b,
     if (h->precision == DSLASH_F32)
         return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the solver works on fp64 vectors (DSLASH_F64 or DSLASH_MIXED)");
     if (!h->loaded) return hisq_fail(h, DSLASH_ERR_STATE, "solver before load_links");
+    if (h->plan.nranks > 1 && !h->nccl)
+        return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "dot products across ranks need an NCCL communicator");
     if (!a || !b || ((uintptr_t)a & 15) || ((uintptr_t)b & 15))
         return hisq_fail(h, DSLASH_ERR_ARG, "NULL or misaligned vector");
     const uintptr_t n = 3 * (uintptr_t)h->plan.vh_local * sizeof(double2);

@@ -156,16 +156,17 @@ __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[
 // vectors and of the accumulation (double/double = fp64, float/float = fp32, float/double =
 // mixed: fp32 links widened to fp64 before the FMAs).  RECON 12 rebuilds row 2 of the long
 // links.  The summation order per (site, rhs) is the same for every NRHS, MINB and block size.
-template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1>
-__global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P) {
+// The per-thread body: thread gid of the box enumeration (LANES consecutive gids per site).  All
+// LANES threads of a site must call it together (shuffle reduction).
+template <typename LR, typename VR, int LANES, bool GHOST, int RECON, int NRHS>
+__device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_t gid, const int64_t site_end) {
     static_assert(LANES == 1 || LANES == 2 || LANES == 4, "LANES must divide 4");
     using L2 = cplx_t<LR>;
     using V2 = cplx_t<VR>;
     constexpr int K = 4 / LANES;
-    const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int lane = (LANES == 1) ? 0 : (int)(threadIdx.x & (LANES - 1));
+    const int lane = (LANES == 1) ? 0 : (int)(gid & (LANES - 1));
     const int64_t site = gid / LANES;
-    const bool valid = site < P.box_start[P.nbox];
+    const bool valid = site < site_end;
     if (LANES == 1 && !valid) return;
     V2 acc[NRHS][3];
 #pragma unroll
@@ -236,6 +237,80 @@ __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P
         } else {
             if (lane < 3) st_stream(out + lane * P.vh + s.cb, lane == 0 ? acc[r][0] : lane == 1 ? acc[r][1] : acc[r][2]);
         }
+    }
+}
+
+template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1>
+__global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P) {
+    dslash_body<LR, VR, LANES, GHOST, RECON, NRHS>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                                                   P.box_start[P.nbox]);
+}
+
+// ---------------------------------------------------------------- persistent fused kernel
+// One launch per apply (DSLASH_OPT_PERSISTENT): blocks stay resident and draw tiles of
+// blockDim.x threads from ticket counters.  Interior sites (the first `interior_sites` of the
+// box enumeration) come from counter sched[0]: a launch consumes exactly ntiles_int + 2
+// gridDim.x tickets from `base` (each block draws one ahead, so the atomic's latency overlaps a
+// tile).  With a halo, a block that runs out of interior tiles looks ONCE at the halo epoch
+// flag, which the halo stream sets after the exchange (cuStreamWriteValue32, no SM involved):
+// if the faces have landed it goes on with boundary tiles from counter sched[1] (reset to 0
+// before the launch), otherwise it exits.  No block ever waits, so the kernel cannot starve the
+// exchange of SMs (NCCL's send/recv kernels, or a copy kernel); a stream-ordered clean-up launch
+// after the halo event (BOUNDARY_ONLY) takes whatever boundary tiles are left.  Interior work
+// and the exchange thus overlap inside one kernel, and dynamic tiles end every SM together.
+struct PersistArgs {
+    unsigned long long* sched;  // [0] interior tickets (monotonic), [1] boundary tickets (reset per apply)
+    unsigned long long base;    // first interior ticket of this launch
+    int64_t interior_sites;     // sites [0, interior_sites) are interior
+    int64_t ntiles_int;         // ceil(interior_sites * LANES / blockDim.x)
+    int64_t ntiles_bnd;         // ceil(boundary sites * LANES / blockDim.x)
+    const unsigned int* flags[4];  // halo epoch flags that must all reach `epoch` (none: no halo)
+    int nflags;
+    unsigned int epoch;
+};
+
+template <typename LR, typename VR, int LANES, bool GHOST, int RECON, bool BOUNDARY_ONLY>
+__global__ void __launch_bounds__(256, 2) dslash_persistent_kernel(const StencilParams P, const PersistArgs A) {
+    __shared__ long long s_tile;
+    const int64_t total = P.box_start[P.nbox];
+    if (!BOUNDARY_ONLY) {
+        long long next = 0;
+        if (threadIdx.x == 0) next = (long long)(atomicAdd(A.sched, 1ull) - A.base);
+        for (;;) {
+            if (threadIdx.x == 0) {
+                s_tile = next;
+                next = (long long)(atomicAdd(A.sched, 1ull) - A.base);  // in flight while this tile runs
+            }
+            __syncthreads();
+            const long long t = s_tile;
+            __syncthreads();  // all threads hold t before thread 0 publishes the next tile
+            if (t >= A.ntiles_int) break;
+            dslash_body<LR, VR, LANES, GHOST, RECON, 1>(P, t * blockDim.x + threadIdx.x, A.interior_sites);
+        }
+        if (!GHOST) return;
+        // boundary tiles only if the halo has already landed: one look, never a wait
+        if (threadIdx.x == 0) {
+            long long ok = 1;
+            for (int f = 0; f < A.nflags; ++f) {
+                unsigned int v;
+                asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(A.flags[f]) : "memory");
+                if ((int)(v - A.epoch) < 0) ok = 0;
+            }
+            s_tile = ok;
+        }
+        __syncthreads();
+        const bool ready = s_tile != 0;
+        __syncthreads();
+        if (!ready) return;
+    }
+    const int64_t bnd0 = A.interior_sites * LANES;  // first boundary thread index
+    for (;;) {
+        if (threadIdx.x == 0) s_tile = (long long)atomicAdd(A.sched + 1, 1ull);
+        __syncthreads();
+        const long long t = s_tile;
+        __syncthreads();
+        if (t >= A.ntiles_bnd) break;
+        dslash_body<LR, VR, LANES, GHOST, RECON, 1>(P, bnd0 + t * blockDim.x + threadIdx.x, total);
     }
 }
 

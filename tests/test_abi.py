@@ -108,8 +108,11 @@ def test_create_argument_errors_precede_cuda():
     assert rc == _abi.DSLASH_ERR_ARG and not h.value
     rc = _abi.lib.dslash_create(_abi.i4((8, 8, 8, 8)), _abi.i4((1, 1, 1, 1)), 5, 0, None, 1, 0, ctypes.byref(h))
     assert rc == _abi.DSLASH_ERR_ARG
-    rc = _abi.lib.dslash_create(_abi.i4((8, 8, 8, 8)), _abi.i4((1, 1, 1, 2)), 2, 0, None, 2, 0, ctypes.byref(h))
-    assert rc == _abi.DSLASH_ERR_ARG           # nranks > 1 without an NCCL id
+    rc = _abi.lib.dslash_create(_abi.i4((8, 8, 8, 8)), _abi.i4((1, 1, 1, 2)), 2, 0, None, 4, 0, ctypes.byref(h))
+    assert rc == _abi.DSLASH_ERR_ARG           # prod(proc_grid) != nranks
+    rc = _abi.lib.dslash_create(_abi.i4((8, 8, 8, 8)), _abi.i4((1, 1, 1, 1)), 0, 7, None, 1, 0, ctypes.byref(h))
+    assert rc == _abi.DSLASH_ERR_ARG           # unknown precision
     assert _abi.lib.dslash_apply(None, None, None, 0, None) == _abi.DSLASH_ERR_ARG
     assert _abi.lib.dslash_local_half_volume(None) == -1
     assert _abi.lib.dslash_destroy(None) == _abi.DSLASH_OK
+    assert _abi.dslash_ipc_blob_size() > 9 * 64          # 9 CUDA IPC handles + header

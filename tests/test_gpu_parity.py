@@ -83,31 +83,35 @@ def test_point_source_exact(torch_cuda, kernel):
 @pytest.mark.parametrize("kernel", KERNELS)
 @pytest.mark.parametrize("dims,mask", [((8, 8, 8, 8), 0x8), ((8, 8, 8, 8), 0x4), ((8, 8, 8, 8), 0xC),
                                        ((8, 10, 12, 14), 0xC), ((4, 4, 4, 4), 0xC), ((6, 8, 10, 12), 0x8)])
-@pytest.mark.parametrize("overlap", [True, False])
-def test_self_halo_bitwise(torch_cuda, kernel, dims, mask, overlap):
-    """The halo path with neighbour = self (ghost faces, interior/boundary split) must give the
-    unpartitioned result bit for bit (same per-site device function), and match the oracle."""
+@pytest.mark.parametrize("overlap,persistent", [(True, True), (True, False), (False, False)])
+def test_self_halo_bitwise(torch_cuda, kernel, dims, mask, overlap, persistent):
+    """The halo path with neighbour = self (ghost faces; the persistent fused kernel waiting on
+    the halo flag, or separate interior/boundary launches) must give the unpartitioned result
+    bit for bit (same per-site device function), and match the oracle."""
     fat, lng = fieldgen.workload_links(dims)
     psi = fieldgen.vector(dims, fieldgen.SEED_PSI)
     for parity in (0, 1):
         src = fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 1 - parity)
-        plain = _gpu_apply(torch_cuda, dims, fat, lng, src, parity, kernel=kernel)
-        halo = _gpu_apply(torch_cuda, dims, fat, lng, src, parity, kernel=kernel, force_halo=mask, overlap=overlap)
+        plain = _gpu_apply(torch_cuda, dims, fat, lng, src, parity, kernel=kernel, persistent=False)
+        halo = _gpu_apply(torch_cuda, dims, fat, lng, src, parity, kernel=kernel, force_halo=mask, overlap=overlap,
+                          persistent=persistent)
         assert np.array_equal(plain, halo)
         ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, parity), parity)
         assert oracle.normwise_error(halo, ref) <= TOL
 
 
 @pytest.mark.parametrize("kernel", KERNELS)
-@pytest.mark.parametrize("minb,block", [(2, 64), (3, 96), (4, 256), (2, 256)])
-def test_launch_configs_agree(torch_cuda, kernel, minb, block):
+@pytest.mark.parametrize("minb,block,persistent", [(2, 64, False), (3, 96, False), (4, 256, False), (2, 256, False),
+                                                   (2, 64, True), (2, 96, True), (2, 256, True)])
+def test_launch_configs_agree(torch_cuda, kernel, minb, block, persistent):
     """Every register budget and block size gives the same bits for a given mapping (the
     mapping fixes the summation order), and the mappings agree to rounding."""
     dims = (16, 16, 16, 16)
     fat, lng = fieldgen.workload_links(dims)
     src = fieldgen.vector_cb(dims, 7, 1)
     base = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel=kernel)
-    other = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel=kernel, min_blocks=minb, block=block)
+    other = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel=kernel, min_blocks=minb, block=block,
+                       persistent=persistent)
     assert np.array_equal(base, other)
     ref = _gpu_apply(torch_cuda, dims, fat, lng, src, 0, kernel="site")
     assert oracle.normwise_error(base, ref) < 1e-14
@@ -138,6 +142,49 @@ def test_sampled_48(torch_cuda):
     pick = np.sort(rng.choice(lex.size, 4096, replace=False))
     pick = np.concatenate([[0, 1, lex.size - 1], pick])          # first/last sites (wrap in every dim)
     ref = oracle.dslash_sites(fat, lng, psi, lex[pick])           # (n, 3)
+    assert oracle.normwise_error(got[:, pick].T, ref) <= TOL
+
+
+@pytest.mark.parametrize("mask", [0x8, 0xC])
+def test_full_size_32_halo_path(torch_cuda, mask):
+    """The per-GPU launch configuration of the weak-scaling bench (local 32^4, t-halo; plus z):
+    interior + boundary kernels on two streams with the self-halo, bitwise equal to the
+    unpartitioned apply at full size."""
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash, _abi
+    dims = (32, 32, 32, 32)
+    fat, lng = fieldgen.workload_links(dims)
+    src = torch.from_numpy(fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 1)).cuda()
+    outs = []
+    for m, pers in ((0, False), (mask, True), (mask, False)):
+        with Dslash(dims, parity_mask=_abi.DSLASH_EVEN, force_halo=m, persistent=pers) as D:
+            D.load_links(fat, lng)
+            o = D.empty_vector()
+            for _ in range(3):                       # repeated applies reuse the ghost buffers
+                D.apply(o, src, 0)
+            torch.cuda.synchronize()
+            outs.append(o.cpu())
+    assert torch.equal(outs[0], outs[1]) and torch.equal(outs[0], outs[2])
+
+
+def test_large_lattice_64x64x64x32(torch_cuda):
+    """A large local volume (Vh = 4.2M, 9.7 GB of links per parity): 64-bit indexing and grid
+    sizes; 2048 sampled sites vs the oracle (first/last sites included)."""
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash, _abi
+    dims = (64, 64, 64, 32)
+    fat, lng = fieldgen.workload_links(dims)
+    psi = fieldgen.vector(dims, fieldgen.SEED_PSI)
+    parity = 0
+    with Dslash(dims, parity_mask=_abi.DSLASH_EVEN) as D:
+        D.load_links(fat, lng)
+        out = D(torch.from_numpy(fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 1)).cuda(), parity)
+        torch.cuda.synchronize()
+        got = out.cpu().numpy()
+    lex = oracle.lex_sites_of_parity(dims, parity)
+    pick = np.concatenate([[0, 1, lex.size - 2, lex.size - 1],
+                           np.sort(np.random.default_rng(64).choice(lex.size, 2048, replace=False))])
+    ref = oracle.dslash_sites(fat, lng, psi, lex[pick])
     assert oracle.normwise_error(got[:, pick].T, ref) <= TOL
 
 
@@ -429,7 +476,40 @@ def test_kernel_timing_records(torch_cuda):
         for _ in range(3):
             D.apply(out, src, 0)
         ms, n = D.kernel_timing()
+        assert n == 3 and ms > 0   # one persistent launch per apply
+        D.kernel_timing_reset()
+        _abi = __import__("paper_conf_sc_dufekgaad024_b200")._abi
+        _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_PERSISTENT, 0)
+        for _ in range(3):
+            D.apply(out, src, 0)
+        ms, n = D.kernel_timing()
         assert n == 6 and ms > 0   # interior + boundary per apply
         assert D.kernel_timing(0)[1] == 3 and D.kernel_timing(1)[1] == 3
         D.kernel_timing_reset()
         assert D.kernel_timing()[1] == 0
+
+
+@pytest.mark.parametrize("mask", [0x8, 0x4, 0xC])
+@pytest.mark.parametrize("persistent", [True, False])
+def test_p2p_transport_self_halo(torch_cuda, mask, persistent):
+    """The P2P transport (copy-engine face puts + stream-memory epoch flags) with neighbour =
+    self: several epochs through the same ghosts, single and multi-RHS, bitwise equal to the
+    unpartitioned apply."""
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 8, 8, 12)
+    fat, lng = fieldgen.workload_links(dims)
+    srcs = torch.stack([torch.from_numpy(fieldgen.vector_cb(dims, 60 + r, 0)) for r in range(3)]).cuda()
+    with Dslash(dims, persistent=False) as D:
+        D.load_links(fat, lng)
+        ref = torch.stack([D(srcs[r].contiguous(), 1) for r in range(3)]).cpu()
+    with Dslash(dims, force_halo=mask, transport="p2p", persistent=persistent) as D:
+        D.load_links(fat, lng)
+        for it in range(4):
+            for r in range(3):
+                out = D(srcs[r].contiguous(), 1)
+                assert torch.equal(out.cpu(), ref[r]), (it, r)
+        multi = torch.empty_like(srcs)
+        D.apply_multi(multi, srcs, 1)
+        torch.cuda.synchronize()
+        assert torch.equal(multi.cpu(), ref)

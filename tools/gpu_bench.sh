@@ -1,7 +1,7 @@
 # full bench (default config) + ncu launch list + ncu --set full of the default kernel
 set -x
 mkdir -p gpurun_out
-python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -2
+timeout 600 python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -2
 timeout 1200 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
 nvidia-smi --query-gpu=index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active --format=csv -lms 200 > gpurun_out/clocks.csv &
 SMI=$!

@@ -1,6 +1,6 @@
 set -x
 mkdir -p gpurun_out
-python -c "import __graft_entry__ as g; g.build()" 2>&1 | tail -2
+timeout 600 python -c "import __graft_entry__ as g; g.build()" 2>&1 | tail -2
 timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -k "bulk" 2>&1 | tail -8
 run() { name=$1; shift; python bench.py --steps 1000 --no-cpu-baseline --no-e2e "$@" > gpurun_out/bench_$name.json 2> gpurun_out/bench_$name.err; python -c "
 import json,sys; d=json.load(open('gpurun_out/bench_$name.json')); r=d['roofline']

@@ -1,6 +1,6 @@
 set -x
 mkdir -p gpurun_out
-python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -2
+timeout 600 python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -2
 timeout 1200 python -m pytest tests -m gpu -x -q 2>&1 | tail -4
 for p in f32 mixed; do
   python bench.py --precision $p --steps 1000 --no-cpu-baseline > gpurun_out/bench_$p.json 2> gpurun_out/bench_$p.err

@@ -1,7 +1,7 @@
 # ncu launch list + full capture of both kernel variants (run on the GPU box from the repo root)
 set -x
 mkdir -p gpurun_out
-python -c "import __graft_entry__ as g; g.build()"
+timeout 600 python -c "import __graft_entry__ as g; g.build()"
 python tools/sweep.py --dims 32,32,32,32 > gpurun_out/sweep_32.jsonl 2>&1
 python tools/sweep.py --dims 16,16,16,16 --blocks 64,128,256 > gpurun_out/sweep_16.jsonl 2>&1
 python tools/sweep.py --dims 48,48,48,48 --blocks 128,256 --steps 100 > gpurun_out/sweep_48.jsonl 2>&1

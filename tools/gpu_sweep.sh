@@ -1,6 +1,6 @@
 set -x
 mkdir -p gpurun_out
-python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -2
+timeout 600 python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -2
 python tools/sweep.py --dims 32,32,32,32 --steps 400 > gpurun_out/sweep2_32.jsonl 2>&1
 python tools/sweep.py --dims 48,48,48,48 --steps 60 --blocks 128,256 > gpurun_out/sweep2_48.jsonl 2>&1
 cat gpurun_out/sweep2_*.jsonl
