@@ -63,8 +63,13 @@ def parse():
                     help="bitmask of directions run through the halo path with neighbour = self (1 GPU)")
     ap.add_argument("--parity", type=int, default=0)
     ap.add_argument("--no-overlap", action="store_true")
-    ap.add_argument("--no-persistent", action="store_true",
-                    help="separate interior/boundary launches instead of the persistent fused kernel")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"],
+                    help="halo transport for N > 1: NCCL send/recv, or copy-engine puts into IPC-mapped ghosts")
+    ap.add_argument("--persistent", action="store_true",
+                    help="one persistent launch per apply when a halo is exchanged (default: separate "
+                         "interior / boundary launches, measured faster)")
+    ap.add_argument("--persistent-always", action="store_true",
+                    help="the persistent kernel also without a halo")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="oracle CPU-baseline budget")
@@ -272,7 +277,7 @@ def main():
     D = Dslash(gdims, grid, parity_mask=parity, kernel=args.kernel, block=args.block, min_blocks=args.min_blocks,
                precision=args.precision, recon=args.recon,
                overlap=not args.no_overlap, timing=True, rank=rank, world_size=world, force_halo=args.force_halo,
-               persistent=not args.no_persistent)
+               persistent=("always" if args.persistent_always else args.persistent), transport=args.transport if world > 1 or args.force_halo else "nccl")
     origin, extent = D.origin, D.local_dims
     fat, lng = fieldgen.workload_links(gdims, origin=origin, extent=extent)
     D.load_links(fat, lng)
@@ -350,7 +355,8 @@ def main():
         roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4),
                 "traffic": ncu_traffic(args.kernel + ("" if args.precision == "f64" else f"-{args.precision}")
-                                     + ("" if args.recon == 18 else f"-r{args.recon}"), extent),
+                                     + ("" if args.recon == 18 else f"-r{args.recon}")
+                                     + ("-persistent" if one_kernel and not args.no_overlap else ""), extent),
                 "kernel": ("dslash_bulk_kernel (TMA)" if args.kernel == "bulk" else
                            (f"dslash_persistent_kernel<lanes={ {'site': 1, 'dir2': 2, 'dir4': 4}[args.kernel]}, "
                             f"ghost={str(any(plan.halo)).lower()}> (all sites, one launch)") if one_kernel else
@@ -407,7 +413,8 @@ def main():
                            + (f" self-halo mask {args.force_halo}" if args.force_halo else ""), "parity": parity,
                            "kernel": args.kernel, "block": args.block or None, "precision": args.precision,
                            "long_link_recon": args.recon, "nrhs": nrhs,
-                           "overlap": not args.no_overlap,
+                           "overlap": not args.no_overlap, "persistent": "always" if args.persistent_always else args.persistent,
+                           "transport": args.transport if world > 1 else None,
                            "l2": ("L2 flushed between steps (2x L2 buffer write); time = summed kernel events; "
                                   if args.flush_l2 else "") + f"inputs > L2: {(algo_bytes_site - 2 * vec_bytes // (3 * vh) * 3) * vh / 1e9:.2f} GB "
                                  f"links/apply streamed; {R} rotating (psi, chi) pairs = "

@@ -94,12 +94,15 @@ enum {
                                    (and the link halo) to be s*W with W in SU(3) and one real s;
                                    load_links verifies it and returns DSLASH_ERR_ARG otherwise.
                                    Before load_links                                                  */
-    DSLASH_OPT_PERSISTENT = 7,  /* 1 (default): one persistent launch per apply; blocks draw tiles from
-                                   ticket counters, interior first; a block out of interior tiles
-                                   looks once at the halo flag and takes boundary tiles only if the
-                                   faces have landed (never waits, so it cannot starve the exchange);
-                                   a stream-ordered clean-up launch takes the rest.  0: separate
-                                   interior / boundary launches.  Single-RHS applies only; any time */
+    DSLASH_OPT_PERSISTENT = 7,  /* 0 (default): separate interior / boundary launches (measured faster
+                                   on B200, profiles/README.md).  1: when a halo is exchanged, one
+                                   persistent launch per
+                                   apply; blocks draw tiles from ticket counters, interior first; a
+                                   block out of interior tiles looks once at the halo flag and takes
+                                   boundary tiles only if the faces have landed (never waits, so it
+                                   cannot starve the exchange); a stream-ordered clean-up launch takes
+                                   the rest.  2: persistent also without a halo.  Single-RHS applies
+                                   only; any time                                                     */
     DSLASH_OPT_TRANSPORT = 8,   /* DSLASH_TRANSPORT_NCCL / _P2P; before load_links                    */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
@@ -202,6 +205,13 @@ DSLASH_API dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
 DSLASH_API dslash_status dslash_load_links_halo(dslash_t h, const void* fat, const void* lng,
                                                 const void* const slab_fat[4], const void* const slab_lng[4],
                                                 int32_t on_device, dslash_stream_t stream);
+
+/* Read back the internal link arrays of target parity `parity` (debugging / verification of
+ * load_links): out_host[cb][mu][l][3][3] complex fp64, Vh_local x 144 complex, with
+ * l = 0 F(x,mu), 1 F(x-mu,mu)^dag, 2 N(x,mu), 3 N(x-3mu,mu)^dag (PAPER.md L51's |l| = 4 arrays)
+ * for the target site x of checkerboard index cb.  Values as stored (fp32 widened); with
+ * recon-12 row 2 of the long matrices is not stored and reads as 0.  Synchronous. */
+DSLASH_API dslash_status dslash_get_links(dslash_t h, int32_t parity, void* out_host);
 
 /* chi = D psi on target parity `parity`.  out: device [3][Vh_local] complex on parity
  * `parity`; in: device [3][Vh_local] complex on parity 1-parity.  Both caller-owned,

@@ -55,7 +55,7 @@ class Dslash:
 
     def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="dir2", block=0,
                  force_halo=0, overlap=True, timing=False, rank=0, world_size=1, min_blocks=0, precision="f64",
-                 recon=18, persistent=True, transport="nccl"):
+                 recon=18, persistent=False, transport="nccl"):
         import torch
         self.global_dims = tuple(int(d) for d in global_dims)
         self.precision = precision
@@ -88,7 +88,9 @@ class Dslash:
                     blobs = [None] * world_size
                     dist.all_gather_object(blobs, _abi.dslash_get_ipc_blob(self.h))
                     _abi.dslash_open_ipc_blobs(self.h, b"".join(blobs))
-            _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_PERSISTENT, int(bool(persistent)))
+            # True -> 1 (persistent when a halo is exchanged), "always" -> 2, False -> 0
+            _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_PERSISTENT,
+                                   2 if persistent == "always" else int(bool(persistent)))
             if force_halo:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_FORCE_HALO, force_halo)
             _abi.dslash_set_option(self.h, DSLASH_OPT_OVERLAP, int(bool(overlap)))
@@ -118,6 +120,14 @@ class Dslash:
             assert lng.is_cuda and lng.dtype == torch.complex128 and lng.is_contiguous()
             self._check_links(tuple(fat.shape), tuple(lng.shape))
             _abi.dslash_load_links(self.h, fat.data_ptr(), lng.data_ptr(), 1, _stream_handle(stream))
+
+    def get_links(self, parity):
+        """Internal link arrays of target parity as numpy (Vh, 4 mu, 4 l, 3, 3) complex128,
+        l = F(x,mu), F(x-mu,mu)^dag, N(x,mu), N(x-3mu,mu)^dag (verification of load_links)."""
+        import numpy as np
+        out = np.empty((self.vh, 4, 4, 3, 3), np.complex128)
+        _abi.dslash_get_links(self.h, int(parity), out.ctypes.data)
+        return out
 
     def _load_links_p2p(self, fat, lng, stream):
         """Link halo through torch.distributed: send my top 3 slices (t, then z) to the plus

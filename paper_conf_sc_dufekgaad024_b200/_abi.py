@@ -82,6 +82,7 @@ _SIGS = {
     "dslash_ipc_blob_size": ([], ctypes.c_int64),
     "dslash_get_ipc_blob": ([_h, _vp], ctypes.c_int),
     "dslash_open_ipc_blobs": ([_h, _vp], ctypes.c_int),
+    "dslash_get_links": ([_h, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_load_links_halo": ([_h, _vp, _vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.c_int32, _vp],
                                ctypes.c_int),
     "dslash_set_option": ([_h, ctypes.c_int32, ctypes.c_int64], ctypes.c_int),
@@ -170,6 +171,10 @@ def dslash_load_links_halo(h, fat_ptr, lng_ptr, slab_fat_ptrs, slab_lng_ptrs, on
     sf = (ctypes.c_void_p * 4)(*[p or None for p in slab_fat_ptrs])
     sl = (ctypes.c_void_p * 4)(*[p or None for p in slab_lng_ptrs])
     return check(lib.dslash_load_links_halo(h, fat_ptr, lng_ptr, sf, sl, on_device, stream), h)
+
+
+def dslash_get_links(h, parity, out_ptr):
+    return check(lib.dslash_get_links(h, parity, out_ptr), h)
 
 
 def dslash_set_option(h, key, value):

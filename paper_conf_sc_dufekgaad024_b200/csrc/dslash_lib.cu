@@ -295,7 +295,8 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             return st;
         }
         case DSLASH_OPT_PERSISTENT:
-            h->persistent = value != 0;
+            if (value < 0 || value > 2) return fail(h, DSLASH_ERR_ARG, "persistent mode %lld not in {0,1,2}", (long long)value);
+            h->persistent = (int)value;
             return DSLASH_OK;
         case DSLASH_OPT_LONG_RECON:
             if (value != 18 && value != 12) return fail(h, DSLASH_ERR_ARG, "long-link recon %lld must be 18 or 12", (long long)value);
@@ -521,6 +522,31 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
 extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const void* lng, int32_t on_device,
                                            dslash_stream_t stream) {
     return load_links_impl(h, fat, lng, nullptr, nullptr, on_device, stream);
+}
+
+extern "C" dslash_status dslash_get_links(dslash_t h, int32_t parity, void* out_host) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (!out_host || (parity & ~1)) return fail(h, DSLASH_ERR_ARG, "NULL output or bad parity");
+    if (!h->loaded || !h->links[parity]) return fail(h, DSLASH_ERR_STATE, "links of parity %d not loaded", parity);
+    const dslash_plan_t& p = h->plan;
+    LinkConvParams C{};
+    C.links = h->links[parity];
+    C.vh = p.vh_local;
+    C.lanes = h->kernel == DSLASH_KERNEL_BULK ? 0 : lanes_of(h->kernel);
+    C.recon = h->recon;
+    const size_t bytes = (size_t)p.vh_local * 144 * sizeof(double2);
+    void* tmp = nullptr;
+    CU(h, cudaMalloc(&tmp, bytes));
+    const int64_t n = p.vh_local * 16;
+    if (h->precision == DSLASH_F64)
+        export_links_kernel<double><<<(unsigned)((n + 255) / 256), 256>>>(C, (double2*)tmp);
+    else
+        export_links_kernel<float><<<(unsigned)((n + 255) / 256), 256>>>(C, (double2*)tmp);
+    cudaError_t e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaMemcpy(out_host, tmp, bytes, cudaMemcpyDeviceToHost);
+    cudaFree(tmp);
+    if (e != cudaSuccess) return fail(h, DSLASH_ERR_CUDA, "dslash_get_links: %s", cudaGetErrorString(e));
+    return DSLASH_OK;
 }
 
 extern "C" dslash_status dslash_load_links_halo(dslash_t h, const void* fat, const void* lng,
@@ -1089,7 +1115,9 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         K.face_vh[d] = p.face_vh[d];
         if (p.halo[d]) K.halo_mask |= 1 << d;
     }
-    if (h->persistent && nrhs == 1 && h->kernel != DSLASH_KERNEL_BULK && write_value_fn())
+    // persistent: 1 = when a halo is exchanged (default), 2 = always
+    if (h->persistent && (h->persistent == 2 || any_halo(p)) && nrhs == 1 && h->kernel != DSLASH_KERNEL_BULK &&
+        write_value_fn())
         return apply_persistent(h, K, s);
     if (!any_halo(p)) return launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
     if ((st = halo_start_impl(h, in, nrhs, s)) != DSLASH_OK) return st;

@@ -99,6 +99,38 @@ __global__ void convert_links_kernel(const LinkConvParams P) {
         }
 }
 
+// Export (dslash_get_links): internal layout -> out[cb][mu][l][e] (double2), l = Ff, Fb, Nf, Nb.
+// With recon-12 the long matrices' row 2 is not stored: exported as zeros.
+template <typename LR>
+__global__ void export_links_kernel(const LinkConvParams P, double2* out) {
+    using L2 = cplx_t<LR>;
+    const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (gid >= P.vh * 16) return;
+    const int64_t cb = gid >> 4;
+    const int mu = (int)(gid >> 2) & 3;
+    const int l = (int)gid & 3;
+    const L2* links = static_cast<const L2*>(P.links);
+    const int stored = (P.recon == 12 && l >= 2) ? 6 : 9;
+    for (int e = 0; e < 9; ++e) {
+        double2 v = make_double2(0.0, 0.0);
+        if (e < stored) {
+            int64_t o;
+            if (P.lanes == 0)
+                o = P.recon == 12 ? link_index_tiled<12>(mu, l, e, cb) : link_index_tiled<18>(mu, l, e, cb);
+            else if (P.recon == 12)
+                o = P.lanes == 1 ? link_index<1, 12>(mu, l, e, P.vh, cb)
+                  : P.lanes == 2 ? link_index<2, 12>(mu, l, e, P.vh, cb)
+                                 : link_index<4, 12>(mu, l, e, P.vh, cb);
+            else
+                o = P.lanes == 1 ? link_index<1>(mu, l, e, P.vh, cb)
+                  : P.lanes == 2 ? link_index<2>(mu, l, e, P.vh, cb)
+                                 : link_index<4>(mu, l, e, P.vh, cb);
+            v = widen(links[o]);
+        }
+        out[((cb * 4 + mu) * 4 + l) * 9 + e] = v;
+    }
+}
+
 // recon-12 admissibility: for every canonical long link N (fp64 input), the largest deviation
 // |row2 - conj(row0 x row1)/s| over its 3 entries, as a non-negative double whose bit pattern
 // orders like an unsigned integer (atomicMax on the bits).

@@ -285,7 +285,8 @@ __global__ void __launch_bounds__(256, 2) dslash_persistent_kernel(const Stencil
             const long long t = s_tile;
             __syncthreads();  // all threads hold t before thread 0 publishes the next tile
             if (t >= A.ntiles_int) break;
-            dslash_body<LR, VR, LANES, GHOST, RECON, 1>(P, t * blockDim.x + threadIdx.x, A.interior_sites);
+            // interior sites never reach a ghost face: the ghost-free addressing suffices
+            dslash_body<LR, VR, LANES, false, RECON, 1>(P, t * blockDim.x + threadIdx.x, A.interior_sites);
         }
         if (!GHOST) return;
         // boundary tiles only if the halo has already landed: one look, never a wait

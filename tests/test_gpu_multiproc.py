@@ -99,7 +99,7 @@ def _single(gdims, kw, parity, nrhs=1):
 @pytest.mark.parametrize("gdims,grid", [((8, 8, 8, 16), (1, 1, 1, 2)), ((8, 8, 16, 8), (1, 1, 2, 1)),
                                         ((8, 8, 8, 8), (1, 1, 2, 2)), ((8, 8, 8, 24), (1, 1, 1, 3))])
 @pytest.mark.parametrize("persistent", [True, False])
-def test_multirank_p2p_bitwise(gdims, grid, persistent):
+def test_multirank_p2p_bitwise(gdims, grid, persistent):   # True = persistent kernel when a halo exists
     world = grid[2] * grid[3]
     kw = {"persistent": persistent}
     for parity in (0, 1):

@@ -102,7 +102,7 @@ def test_self_halo_bitwise(torch_cuda, kernel, dims, mask, overlap, persistent):
 
 @pytest.mark.parametrize("kernel", KERNELS)
 @pytest.mark.parametrize("minb,block,persistent", [(2, 64, False), (3, 96, False), (4, 256, False), (2, 256, False),
-                                                   (2, 64, True), (2, 96, True), (2, 256, True)])
+                                                   (2, 64, "always"), (2, 96, "always"), (2, 256, "always")])
 def test_launch_configs_agree(torch_cuda, kernel, minb, block, persistent):
     """Every register budget and block size gives the same bits for a given mapping (the
     mapping fixes the summation order), and the mappings agree to rounding."""
@@ -469,14 +469,14 @@ def test_kernel_timing_records(torch_cuda):
     torch = torch_cuda
     dims = (8, 8, 8, 16)
     fat, lng = fieldgen.workload_links(dims)
-    with Dslash(dims, timing=True, force_halo=0x8) as D:
+    with Dslash(dims, timing=True, force_halo=0x8, persistent=True) as D:
         D.load_links(fat, lng)
         src = torch.from_numpy(fieldgen.vector_cb(dims, 3, 1)).cuda()
         out = D.empty_vector()
         for _ in range(3):
             D.apply(out, src, 0)
         ms, n = D.kernel_timing()
-        assert n == 3 and ms > 0   # one persistent launch per apply
+        assert n == 3 and ms > 0   # one persistent launch (+ clean-up) per apply
         D.kernel_timing_reset()
         _abi = __import__("paper_conf_sc_dufekgaad024_b200")._abi
         _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_PERSISTENT, 0)
@@ -513,3 +513,27 @@ def test_p2p_transport_self_halo(torch_cuda, mask, persistent):
         D.apply_multi(multi, srcs, 1)
         torch.cuda.synchronize()
         assert torch.equal(multi.cpu(), ref)
+
+
+@pytest.mark.parametrize("kernel", ["site", "dir2", "dir4", "bulk"])
+@pytest.mark.parametrize("mask", [0, 0xC])
+def test_load_links_layout_roundtrip(torch_cuda, kernel, mask):
+    """Row a0 bitwise: the internal arrays hold exactly F(x,mu), F(x-mu,mu)^dag, N(x,mu) and
+    N(x-3mu,mu)^dag for every target site (built here with numpy rolls of the canonical input),
+    in every kernel layout, through the local and the halo-slab paths."""
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (16, 8, 8, 12)
+    fat = fieldgen.links(dims, 81, "gauss")
+    lng = fieldgen.links(dims, 82, "gauss")
+    AX = {0: 3, 1: 2, 2: 1, 3: 0}
+    dag = lambda m: np.conj(np.swapaxes(m, -1, -2))
+    with Dslash(dims, kernel=kernel, force_halo=mask) as D:
+        D.load_links(fat, lng)
+        for parity in (0, 1):
+            got = D.get_links(parity)                       # (Vh, mu, l, 3, 3)
+            lex = oracle.lex_sites_of_parity(dims, parity)
+            for mu in range(4):
+                fb = dag(np.roll(fat[..., mu, :, :], 1, axis=AX[mu]))
+                nb = dag(np.roll(lng[..., mu, :, :], 3, axis=AX[mu]))
+                for l, arr in enumerate((fat[..., mu, :, :], fb, lng[..., mu, :, :], nb)):
+                    assert np.array_equal(got[:, mu, l], arr.reshape(-1, 3, 3)[lex]), (parity, mu, l)
