@@ -63,6 +63,9 @@ def parse():
                     help="bitmask of directions run through the halo path with neighbour = self (1 GPU)")
     ap.add_argument("--parity", type=int, default=0)
     ap.add_argument("--no-overlap", action="store_true")
+    ap.add_argument("--colocate", action="store_true",
+                    help="testing aid: every rank on GPU 0 (gloo process group, P2P transport); checks the N > 1 "
+                         "code path on a one-GPU box -- its timings are not scaling numbers")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"],
                     help="halo transport for N > 1: NCCL send/recv, or copy-engine puts into IPC-mapped ghosts")
     ap.add_argument("--persistent", action="store_true",
@@ -266,9 +269,15 @@ def main():
         if world == 1 and args.gpus > 1:
             print(json.dumps({"error": f"--gpus {args.gpus} needs torchrun with {args.gpus} ranks"}))
             return 2
+    if args.colocate:
+        local_rank = 0
+        args.transport = "p2p"
     torch.cuda.set_device(local_rank)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if args.colocate:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     gdims, grid, loc, name = workload(args, world)
     parity = args.parity
 
@@ -334,7 +343,8 @@ def main():
     one_kernel = n_one > 0                # persistent fused kernel (or --no-overlap)
     if one_kernel:
         t_int, n_int = t_one, n_one
-    t_max = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    red_dev = "cpu" if args.colocate else "cuda"
+    t_max = torch.tensor([ms], dtype=torch.float64, device=red_dev)
     if world > 1:
         dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
     ms_max = float(t_max.item())
@@ -387,7 +397,7 @@ def main():
         ev1.record(stream)
         torch.cuda.synchronize()
         D.kernel_timing_reset()
-        te = torch.tensor([ev0.elapsed_time(ev1)], dtype=torch.float64, device="cuda")
+        te = torch.tensor([ev0.elapsed_time(ev1)], dtype=torch.float64, device=red_dev)
         if world > 1:
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
         e2e = {"value": round(FLOP_PER_SITE * total_sites * ke / (float(te.item()) * 1e-3) / 1e9, 2),
@@ -415,6 +425,7 @@ def main():
                            "long_link_recon": args.recon, "nrhs": nrhs,
                            "overlap": not args.no_overlap, "persistent": "always" if args.persistent_always else args.persistent,
                            "transport": args.transport if world > 1 else None,
+                           "colocated_ranks_on_one_gpu": bool(args.colocate) or None,
                            "l2": ("L2 flushed between steps (2x L2 buffer write); time = summed kernel events; "
                                   if args.flush_l2 else "") + f"inputs > L2: {(algo_bytes_site - 2 * vec_bytes // (3 * vh) * 3) * vh / 1e9:.2f} GB "
                                  f"links/apply streamed; {R} rotating (psi, chi) pairs = "

@@ -920,7 +920,8 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
     const int lanes = lanes_of(h->kernel);
     const int bs = h->block ? h->block : default_block(lanes);
     const int minb = h->min_blocks ? h->min_blocks : default_minb(lanes);
-    const int64_t threads = sites * lanes;  // right-hand sides are register-blocked per thread
+    // right-hand sides are register-blocked per thread; 8 of them use 2 thread groups of 4
+    const int64_t threads = sites * lanes * (nrhs == 8 ? 2 : 1);
     const unsigned grid = (unsigned)((threads + bs - 1) / bs);
     dslash_s::TimedLaunch* tl = nullptr;
     if (h->timing) {

@@ -1,8 +1,9 @@
 // kernels_inst.cuh -- instantiation table of dslash_kernel for one (LR, VR, RECON); included by
 // the kernels_*.cu translation units, which build in parallel.
 // Instantiated: every (lanes, ghost) with MINB 2/3/4 for one right-hand side, with MINB 2
-// (the measured best) for 2 and 4 right-hand sides per launch, and MINB 1 for 8 (24 complex
-// accumulators per thread do not fit 128 registers).
+// (the measured best) for 2 and 4 right-hand sides per launch; 8 right-hand sides run as two
+// adjacent thread groups of 4 register-blocked ones (8 per thread needs 255 registers and ran at
+// 12% occupancy).
 #pragma once
 
 #include "dispatch.h"
@@ -15,7 +16,7 @@ StencilFn pick_minb(int minb, int nrhs) {
     switch (nrhs) {
         case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 2>;
         case 4: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4>;
-        case 8: return dslash_kernel<LR, VR, LANES, GHOST, 1, RECON, 8>;  // 8 x 3 accumulators: <= 255 regs
+        case 8: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2>;  // 2 thread groups x 4 RHS each
         default: break;
     }
     switch (minb) {

@@ -158,14 +158,18 @@ __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[
 // links.  The summation order per (site, rhs) is the same for every NRHS, MINB and block size.
 // The per-thread body: thread gid of the box enumeration (LANES consecutive gids per site).  All
 // LANES threads of a site must call it together (shuffle reduction).
-template <typename LR, typename VR, int LANES, bool GHOST, int RECON, int NRHS>
+// RHSL > 1: the site's right-hand sides are split over RHSL adjacent thread groups, each
+// register-blocking NRHS of them (rhs = rl * NRHS + r); the groups of a site issue identical link
+// addresses in one warp instruction, so each sector is fetched once.
+template <typename LR, typename VR, int LANES, bool GHOST, int RECON, int NRHS, int RHSL = 1>
 __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_t gid, const int64_t site_end) {
     static_assert(LANES == 1 || LANES == 2 || LANES == 4, "LANES must divide 4");
     using L2 = cplx_t<LR>;
     using V2 = cplx_t<VR>;
     constexpr int K = 4 / LANES;
     const int lane = (LANES == 1) ? 0 : (int)(gid & (LANES - 1));
-    const int64_t site = gid / LANES;
+    const int rl = (RHSL == 1) ? 0 : (int)((gid / LANES) % RHSL);
+    const int64_t site = gid / (LANES * RHSL);
     const bool valid = site < site_end;
     if (LANES == 1 && !valid) return;
     V2 acc[NRHS][3];
@@ -185,7 +189,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 #pragma unroll
             for (int l = 0; l < 4; ++l) {
                 const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
-                const SrcRef<V2> src = source<V2, GHOST>(P, mu, h, s, 0);
+                const SrcRef<V2> src = source<V2, GHOST>(P, mu, h, s, rl * NRHS);
                 const L2* lp = links + link_index<LANES, RECON>(mu, l, 0, P.vh, s.cb);
                 V2 U[9];
 #pragma unroll
@@ -223,7 +227,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
     if (!valid) return;
 #pragma unroll
     for (int r = 0; r < NRHS; ++r) {
-        V2* out = static_cast<V2*>(P.out) + (int64_t)r * 3 * P.vh;
+        V2* out = static_cast<V2*>(P.out) + (int64_t)(rl * NRHS + r) * 3 * P.vh;
         if (LANES == 1) {
 #pragma unroll
             for (int c = 0; c < 3; ++c) st_stream(out + c * P.vh + s.cb, acc[r][c]);
@@ -240,10 +244,10 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
     }
 }
 
-template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1>
+template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1, int RHSL = 1>
 __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P) {
-    dslash_body<LR, VR, LANES, GHOST, RECON, NRHS>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
-                                                   P.box_start[P.nbox]);
+    dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                                                         P.box_start[P.nbox]);
 }
 
 // ---------------------------------------------------------------- persistent fused kernel
