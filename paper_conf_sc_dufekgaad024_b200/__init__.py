@@ -63,7 +63,13 @@ class Dslash:
         self.proc_grid = tuple(int(p) for p in proc_grid)
         uid = None
         self.world_size, self.rank, self.transport = world_size, rank, transport
-        if world_size > 1 and transport == "nccl":
+        # an NCCL communicator for the halo (transport "nccl") and, on an NCCL process group, for
+        # the solver's cross-rank dot products even when the halo goes through P2P
+        use_nccl = False
+        if world_size > 1:
+            import torch.distributed as dist
+            use_nccl = transport == "nccl" or dist.get_backend() == "nccl"
+        if use_nccl:
             import torch
             import torch.distributed as dist
             t = torch.zeros(128, dtype=torch.uint8, device="cuda" if dist.get_backend() == "nccl" else "cpu")
@@ -81,8 +87,9 @@ class Dslash:
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_MIN_BLOCKS, min_blocks)
             if recon != 18:
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_LONG_RECON, recon)
-            if transport == "p2p":
+            if transport == "p2p" and (world_size == 1 or use_nccl):
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_TRANSPORT, _abi.DSLASH_TRANSPORT_P2P)
+            if transport == "p2p":
                 if world_size > 1:      # exchange CUDA IPC handles through torch.distributed
                     import torch.distributed as dist
                     blobs = [None] * world_size

@@ -268,7 +268,8 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             h->block = (int)value;
             return DSLASH_OK;
         case DSLASH_OPT_FORCE_HALO: {
-            if (h->loaded) return fail(h, DSLASH_ERR_STATE, "FORCE_HALO must be set before load_links");
+            if (h->loaded || h->p2p_ready)
+                return fail(h, DSLASH_ERR_STATE, "FORCE_HALO must be set before load_links and the IPC setup");
             dslash_plan_t p;
             dslash_status st = dslash_plan(h->global_dims, h->proc_grid, h->plan.rank, h->plan.nranks, (int)value, &p);
             if (st != DSLASH_OK) return fail(h, st, "%s", g_last_error.c_str());
