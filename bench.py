@@ -370,7 +370,8 @@ def main():
                 "kernel": ("dslash_bulk_kernel (TMA)" if args.kernel == "bulk" else
                            (f"dslash_persistent_kernel<lanes={ {'site': 1, 'dir2': 2, 'dir4': 4}[args.kernel]}, "
                             f"ghost={str(any(plan.halo)).lower()}> (all sites, one launch)") if one_kernel else
-                           f"dslash_kernel<lanes={ {'site': 1, 'dir2': 2, 'dir4': 4}[args.kernel]}, ghost=false> interior"),
+                           f"dslash_kernel<lanes={ {'site': 1, 'dir2': 2, 'dir4': 4}[args.kernel]}, ghost=false>"
+                           + (" interior" if any(plan.halo) else " (all sites)")),
                 "bytes_per_launch": algo_bytes_site * dom_sites, "bytes_per_site": algo_bytes_site, "avg_launch_us": round(kern_ms * 1e3, 2),
                 "launches": n_int, "peak_source": peak_src,
                 "boundary_kernel_us": round(t_bnd / n_bnd * 1e3, 2) if n_bnd else None,
