@@ -122,8 +122,10 @@ enum {
                                   right-hand sides per apply                                         */
 };
 
-/* Kernel classes for dslash_kernel_timing. */
-enum { DSLASH_TIMING_INTERIOR = 0, DSLASH_TIMING_BOUNDARY = 1, DSLASH_TIMING_ALL = 2 };
+/* Kernel classes for dslash_kernel_timing.  SPAN: with a halo and the classic split, the time
+ * from the interior kernel's start to the join after the (overlapping, higher-priority) boundary
+ * kernel, i.e. the duration of the apply's stencil work; ALL sums the kernel launches only. */
+enum { DSLASH_TIMING_INTERIOR = 0, DSLASH_TIMING_BOUNDARY = 1, DSLASH_TIMING_ALL = 2, DSLASH_TIMING_SPAN = 3 };
 
 /* Host-only decomposition of the local lattice (no CUDA calls).  A "box" is
  * [lo[d], hi[d]) per dimension in local coordinates; the target-parity sites of a

@@ -26,7 +26,7 @@ DSLASH_OPT_KERNEL, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_OVERLAP, 
     DSLASH_OPT_MIN_BLOCKS, DSLASH_OPT_LONG_RECON, DSLASH_OPT_PERSISTENT, DSLASH_OPT_TRANSPORT = range(9)
 DSLASH_TRANSPORT_NCCL, DSLASH_TRANSPORT_P2P = 0, 1
 TRANSPORTS = {"nccl": DSLASH_TRANSPORT_NCCL, "p2p": DSLASH_TRANSPORT_P2P}
-DSLASH_TIMING_INTERIOR, DSLASH_TIMING_BOUNDARY, DSLASH_TIMING_ALL = range(3)
+DSLASH_TIMING_INTERIOR, DSLASH_TIMING_BOUNDARY, DSLASH_TIMING_ALL, DSLASH_TIMING_SPAN = range(4)
 KERNELS = {"site": DSLASH_KERNEL_SITE, "dir4": DSLASH_KERNEL_DIR4, "dir2": DSLASH_KERNEL_DIR2,
            "bulk": DSLASH_KERNEL_BULK}
 

@@ -482,9 +482,13 @@ def test_kernel_timing_records(torch_cuda):
         _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_PERSISTENT, 0)
         for _ in range(3):
             D.apply(out, src, 0)
+        for _ in range(40):        # enough timed launches to grow the event pool repeatedly
+            D.apply(out, src, 0)
         ms, n = D.kernel_timing()
-        assert n == 6 and ms > 0   # interior + boundary per apply
-        assert D.kernel_timing(0)[1] == 3 and D.kernel_timing(1)[1] == 3
+        assert n == 86 and ms > 0  # interior + boundary per apply
+        assert D.kernel_timing(0)[1] == 43 and D.kernel_timing(1)[1] == 43
+        span_ms, n_span = D.kernel_timing(3)
+        assert n_span == 43 and span_ms > 0
         D.kernel_timing_reset()
         assert D.kernel_timing()[1] == 0
 
