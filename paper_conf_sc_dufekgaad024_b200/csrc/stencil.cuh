@@ -103,31 +103,33 @@ template <typename V2, bool GHOST>
 __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, int mu, int h, const Site& s, int rhs) {
     const int c = mu == 0 ? s.x : mu == 1 ? s.y : mu == 2 ? s.z : s.t;
     const int L = P.L[mu];
-    int cn = c + h;
-    if (GHOST && mu >= 2 && ((P.halo_mask >> mu) & 1) && (cn < 0 || cn >= L)) {
-        const int side = cn >= L;
-        const int d = side ? cn - L : cn + 3;
-        int64_t f;
-        if (mu == 3)
-            f = s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (s.z + (int64_t)P.L[2] * d));
-        else
-            f = s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (d + 3 * (int64_t)s.t));
-        return {static_cast<const V2*>(P.ghost[mu][side]) + (int64_t)rhs * 3 * P.face_vh[mu] + f, P.face_vh[mu]};
-    }
-    if (cn < 0) cn += L;
-    if (cn < 0) cn += L;
-    if (cn >= L) cn -= L;
-    if (cn >= L) cn -= L;
+    const int cn = c + h;
+    int cw = cn;
+    if (cw < 0) cw += L;
+    if (cw < 0) cw += L;
+    if (cw >= L) cw -= L;
+    if (cw >= L) cw -= L;
     int64_t idx;
     if (mu == 0) {
-        idx = s.cb - s.xh + (cn >> 1);
+        idx = s.cb - s.xh + (cw >> 1);
     } else {
         const int64_t st = mu == 1 ? (int64_t)P.lxh
                          : mu == 2 ? (int64_t)P.lxh * P.L[1]
                                    : (int64_t)P.lxh * P.L[1] * P.L[2];
-        idx = s.cb + (int64_t)(cn - c) * st;
+        idx = s.cb + (int64_t)(cw - c) * st;
     }
-    return {static_cast<const V2*>(P.in) + (int64_t)rhs * 3 * P.vh + idx, P.vh};
+    const V2* local = static_cast<const V2*>(P.in) + (int64_t)rhs * 3 * P.vh + idx;
+    if (!GHOST || mu < 2) return {local, P.vh};
+    // branch-free choice between the local site and the ghost face: the lanes of a site walk
+    // different directions, so a branch here would diverge within the warp
+    const bool ghost = ((P.halo_mask >> mu) & 1) && (cn < 0 || cn >= L);
+    const int side = cn >= L;
+    const int d = side ? cn - L : cn + 3;
+    const int64_t f = (mu == 3) ? s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (s.z + (int64_t)P.L[2] * d))
+                                : s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (d + 3 * (int64_t)s.t));
+    const int64_t fv = P.face_vh[mu];
+    const V2* gp = static_cast<const V2*>(P.ghost[mu][side]) + (int64_t)rhs * 3 * fv + f;
+    return {ghost ? gp : local, ghost ? fv : P.vh};
 }
 
 // acc (+/-)= U v for a 3x3 matrix whose 9 elements are U[e]
