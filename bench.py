@@ -211,10 +211,14 @@ def run_oracle_baseline(gdims, parity, budget_s, steps=None, warmup=0):
             el = time.perf_counter() - t0
             if el >= budget_s:
                 break
+        t0 = time.perf_counter()
+        oracle.dslash(fat, lng, psi, parity, 1)                  # one single-threaded apply
+        t1 = time.perf_counter() - t0
         return {"value": FLOP_PER_SITE * vh * n / el / 1e9, "unit": "GFLOP/s", "cores": cores,
                 "kind": "oracle", "cpu": cpu_model(),
+                "value_1_thread": FLOP_PER_SITE * vh / t1 / 1e9,
                 "sample": f"{n} full {gdims[0]}x{gdims[1]}x{gdims[2]}x{gdims[3]} applies (parity {parity}), "
-                          f"{el:.1f} s, OpenMP over target sites"}, el / n
+                          f"{el:.1f} s, OpenMP over target sites; value_1_thread: one apply on 1 thread"}, el / n
     sites_all = oracle.lex_sites_of_parity(gdims, parity)
     frac = min(1.0, budget_s / max(1, steps + warmup) / t_full)
     stride = max(1, int(round(1.0 / frac)))

@@ -56,7 +56,18 @@ def build(force: bool = False, verbose: bool = False) -> str:
     link = ["nvcc", *ARCH, "-shared", "-o", LIB, *objs, "-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
             "-Xlinker", "-rpath=" + os.path.join(nccl, "lib")]
     subprocess.check_call(link)
+    build_c_demo()
     return LIB
+
+
+def build_c_demo() -> str:
+    """examples/c_api_demo: the library used from plain C (the boundary is a C ABI)."""
+    src = os.path.join(ROOT, "examples", "c_api_demo.c")
+    exe = os.path.join(ROOT, "examples", "c_api_demo")
+    if os.path.exists(src):
+        subprocess.check_call(["gcc", "-std=c99", "-O2", src, "-I", os.path.join(ROOT, "include"), "-L", HERE,
+                               "-lhisq_dslash", "-Wl,-rpath," + HERE, "-lm", "-o", exe])
+    return exe
 
 
 if __name__ == "__main__":

@@ -116,3 +116,12 @@ def test_create_argument_errors_precede_cuda():
     assert _abi.lib.dslash_local_half_volume(None) == -1
     assert _abi.lib.dslash_destroy(None) == _abi.DSLASH_OK
     assert _abi.dslash_ipc_blob_size() > 9 * 64          # 9 CUDA IPC handles + header
+
+
+def test_c_demo_builds_and_links():
+    """The boundary is a plain C ABI: examples/c_api_demo.c compiles against include/ and links
+    the library with gcc (it runs on the GPU in tests/test_gpu_parity.py)."""
+    import os
+    from paper_conf_sc_dufekgaad024_b200 import build
+    exe = build.build_c_demo()
+    assert os.path.exists(exe)

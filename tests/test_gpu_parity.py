@@ -541,3 +541,16 @@ def test_load_links_layout_roundtrip(torch_cuda, kernel, mask):
                 nb = dag(np.roll(lng[..., mu, :, :], 3, axis=AX[mu]))
                 for l, arr in enumerate((fat[..., mu, :, :], fb, lng[..., mu, :, :], nb)):
                     assert np.array_equal(got[:, mu, l], arr.reshape(-1, 3, 3)[lex]), (parity, mu, l)
+
+
+def test_c_api_demo_runs(torch_cuda):
+    """examples/c_api_demo (plain C, no Python binding): create / load_links / apply_host / sync /
+    destroy, anti-Hermiticity to 1e-12."""
+    import os
+    import subprocess
+    from paper_conf_sc_dufekgaad024_b200 import build
+    exe = build.build_c_demo()
+    for dims in (["8", "8", "8", "16"], ["8", "10", "12", "14"]):
+        r = subprocess.run([exe, *dims], capture_output=True, text=True, timeout=120)
+        assert r.returncode == 0, r.stdout + r.stderr
+        assert "rel.diff" in r.stdout
