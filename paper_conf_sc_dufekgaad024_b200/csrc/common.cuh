@@ -61,6 +61,14 @@ __device__ __forceinline__ float2 ld_stream(const float2* p, uint64_t pol) {
     return r;
 }
 
+__device__ __forceinline__ float4 ld_stream(const float4* p, uint64_t pol) {
+    float4 r;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+        : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+        : "l"(p), "l"(pol));
+    return r;
+}
+
 __device__ __forceinline__ float2 ld_reuse(const float2* p, uint64_t pol) {
     float2 r;
     asm("ld.global.nc.L2::cache_hint.v2.f32 {%0, %1}, [%2], %3;" : "=f"(r.x), "=f"(r.y) : "l"(p), "l"(pol));

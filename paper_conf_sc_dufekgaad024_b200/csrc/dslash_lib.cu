@@ -374,6 +374,7 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
     C.vh = p.vh_local;
     C.lanes = h->kernel == DSLASH_KERNEL_BULK ? 0 : lanes_of(h->kernel);
     C.recon = h->recon;
+    C.paired = h->precision != DSLASH_F64 && h->kernel != DSLASH_KERNEL_BULK;
     int halo_mask = 0;
     for (int d = 2; d < 4; ++d)
         if (p.halo[d]) halo_mask |= 1 << d;
@@ -539,6 +540,7 @@ extern "C" dslash_status dslash_get_links(dslash_t h, int32_t parity, void* out_
     C.vh = p.vh_local;
     C.lanes = h->kernel == DSLASH_KERNEL_BULK ? 0 : lanes_of(h->kernel);
     C.recon = h->recon;
+    C.paired = h->precision != DSLASH_F64 && h->kernel != DSLASH_KERNEL_BULK;
     const size_t bytes = (size_t)p.vh_local * 144 * sizeof(double2);
     void* tmp = nullptr;
     CU(h, cudaMalloc(&tmp, bytes));

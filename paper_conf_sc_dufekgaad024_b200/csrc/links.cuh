@@ -31,7 +31,27 @@ struct LinkConvParams {
     int lanes;                    // layout of the kernel that will read the links: 1, 2 or 4,
                                   // or 0 = tiled (the TMA kernel, bulk.cuh)
     int recon;                    // 18 = full matrices, 12 = long links keep rows 0 and 1 only
+    int paired;                   // 1: fp32 paired layout (link_index_paired), register kernels only
 };
+
+// float2 offset of entry (mu, l, e) of site cb in the layout selected by P
+__host__ __device__ __forceinline__ int64_t conv_index(const LinkConvParams& P, int mu, int l, int e, int64_t cb) {
+    if (P.lanes == 0)
+        return P.recon == 12 ? link_index_tiled<12>(mu, l, e, cb) : link_index_tiled<18>(mu, l, e, cb);
+    if (P.paired) {
+        const int64_t o4 = P.lanes == 1   ? link_index_paired<1>(mu, l >> 1, e, P.vh, cb)
+                           : P.lanes == 2 ? link_index_paired<2>(mu, l >> 1, e, P.vh, cb)
+                                          : link_index_paired<4>(mu, l >> 1, e, P.vh, cb);
+        return o4 * 2 + (l & 1);
+    }
+    if (P.recon == 12)
+        return P.lanes == 1 ? link_index<1, 12>(mu, l, e, P.vh, cb)
+             : P.lanes == 2 ? link_index<2, 12>(mu, l, e, P.vh, cb)
+                            : link_index<4, 12>(mu, l, e, P.vh, cb);
+    return P.lanes == 1 ? link_index<1>(mu, l, e, P.vh, cb)
+         : P.lanes == 2 ? link_index<2>(mu, l, e, P.vh, cb)
+                        : link_index<4>(mu, l, e, P.vh, cb);
+}
 
 __device__ __forceinline__ const double2* canon_link(const LinkConvParams& P, bool is_long, int mu, int x, int y,
                                                      int z, int t, int back) {
@@ -84,18 +104,7 @@ __global__ void convert_links_kernel(const LinkConvParams P) {
                 v = A[3 * i + j];
             }
             const int e = 3 * i + j;
-            int64_t o;
-            if (P.lanes == 0)
-                o = P.recon == 12 ? link_index_tiled<12>(mu, l, e, cb) : link_index_tiled<18>(mu, l, e, cb);
-            else if (P.recon == 12)
-                o = P.lanes == 1 ? link_index<1, 12>(mu, l, e, P.vh, cb)
-                  : P.lanes == 2 ? link_index<2, 12>(mu, l, e, P.vh, cb)
-                                 : link_index<4, 12>(mu, l, e, P.vh, cb);
-            else
-                o = P.lanes == 1 ? link_index<1>(mu, l, e, P.vh, cb)
-                  : P.lanes == 2 ? link_index<2>(mu, l, e, P.vh, cb)
-                                 : link_index<4>(mu, l, e, P.vh, cb);
-            static_cast<L2*>(P.links)[o] = to_cplx<L2>(v);
+            static_cast<L2*>(P.links)[conv_index(P, mu, l, e, cb)] = to_cplx<L2>(v);
         }
 }
 
@@ -113,20 +122,7 @@ __global__ void export_links_kernel(const LinkConvParams P, double2* out) {
     const int stored = (P.recon == 12 && l >= 2) ? 6 : 9;
     for (int e = 0; e < 9; ++e) {
         double2 v = make_double2(0.0, 0.0);
-        if (e < stored) {
-            int64_t o;
-            if (P.lanes == 0)
-                o = P.recon == 12 ? link_index_tiled<12>(mu, l, e, cb) : link_index_tiled<18>(mu, l, e, cb);
-            else if (P.recon == 12)
-                o = P.lanes == 1 ? link_index<1, 12>(mu, l, e, P.vh, cb)
-                  : P.lanes == 2 ? link_index<2, 12>(mu, l, e, P.vh, cb)
-                                 : link_index<4, 12>(mu, l, e, P.vh, cb);
-            else
-                o = P.lanes == 1 ? link_index<1>(mu, l, e, P.vh, cb)
-                  : P.lanes == 2 ? link_index<2>(mu, l, e, P.vh, cb)
-                                 : link_index<4>(mu, l, e, P.vh, cb);
-            v = widen(links[o]);
-        }
+        if (e < stored) v = widen(links[conv_index(P, mu, l, e, cb)]);
         out[((cb * 4 + mu) * 4 + l) * 9 + e] = v;
     }
 }

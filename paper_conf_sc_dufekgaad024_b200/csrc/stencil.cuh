@@ -45,6 +45,16 @@ __host__ __device__ __forceinline__ int64_t link_index(int mu, int l, int e, int
     return ((((int64_t)(elem_base<RECON>(l) + e) * K + mu / LANES) * vh + cb) * LANES) + (mu % LANES);
 }
 
+// fp32 links ("paired" layout): entry e of the forward and the backward matrix of one kind
+// (Ff, Fb: pair j = 0; Nf, Nb: j = 1) share one 16-byte float4, so every lane issues 16-byte
+// loads as in fp64 (no padding: a matrix pair is 2 x 72 B):
+//   links4[(((pbase(j) + e) * K + k) * vh + cb) * LANES + lane],  pbase(0) = 0, pbase(1) = 9.
+template <int LANES>
+__host__ __device__ __forceinline__ int64_t link_index_paired(int mu, int j, int e, int64_t vh, int64_t cb) {
+    constexpr int K = 4 / LANES;
+    return ((((int64_t)(j * 9 + e) * K + mu / LANES) * vh + cb) * LANES) + (mu % LANES);
+}
+
 // Row 2 of s*W, W in SU(3), from rows 0 and 1: conj(r0 x r1) / s  (QUDA/MILC "recon-12";
 // the back-link N(x-3mu)^dag = s W^dag has the same form).  inv_s = 1/s.
 template <typename V2, typename R>
@@ -188,6 +198,43 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 #pragma unroll
         for (int k = 0; k < K; ++k) {
             const int mu = k * LANES + lane;
+            if constexpr (sizeof(LR) == 4) {
+                // fp32 links, paired layout: one 16-byte load feeds the forward and the backward
+                // matrix of a kind; the FMA order is that of the unpaired loop (l = 0, 1, 2, 3)
+                const float4* links4 = static_cast<const float4*>(P.links);
+#pragma unroll
+                for (int j = 0; j < 2; ++j) {
+                    const int hop = j ? 3 : 1;
+                    const float4* lp = links4 + link_index_paired<LANES>(mu, j, 0, P.vh, s.cb);
+                    V2 Ua[9], Ub[9];
+#pragma unroll
+                    for (int e = 0; e < elems_of<RECON>(2 * j); ++e) {
+                        const float4 w = ld_stream(lp + (int64_t)e * 4 * P.vh, pol_stream);
+                        Ua[e] = to_cplx<V2>(widen(make_float2(w.x, w.y)));
+                        Ub[e] = to_cplx<V2>(widen(make_float2(w.z, w.w)));
+                    }
+                    if (elems_of<RECON>(2 * j) == 6) {
+                        reconstruct_row2(Ua, (VR)P.long_inv_scale);
+                        reconstruct_row2(Ub, (VR)P.long_inv_scale);
+                    }
+#pragma unroll
+                    for (int sub = 0; sub < 2; ++sub) {
+                        const SrcRef<V2> src = source<V2, GHOST>(P, mu, sub ? -hop : hop, s, rl * NRHS);
+#pragma unroll
+                        for (int r = 0; r < NRHS; ++r) {
+                            const int64_t roff = (int64_t)r * 3 * src.stride;
+                            V2 v[3];
+#pragma unroll
+                            for (int c = 0; c < 3; ++c) v[c] = ld_reuse(src.p + roff + c * src.stride, pol_keep);
+                            if (sub)
+                                matvec_acc<true>(acc[r], Ub, v);
+                            else
+                                matvec_acc<false>(acc[r], Ua, v);
+                        }
+                    }
+                }
+                continue;
+            }
 #pragma unroll
             for (int l = 0; l < 4; ++l) {
                 const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
