@@ -68,6 +68,11 @@ def parse():
                          "code path on a one-GPU box -- its timings are not scaling numbers")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"],
                     help="halo transport for N > 1: NCCL send/recv, or copy-engine puts into IPC-mapped ghosts")
+    ap.add_argument("--no-pdl", action="store_true",
+                    help="ordinary launches instead of programmatic dependent launch (DSLASH_OPT_PDL)")
+    ap.add_argument("--kernel-timing", action="store_true",
+                    help="per-kernel events even with one stencil launch per step (they cost ~3%% of the "
+                         "step and block PDL overlap); always on with a halo (span) or --flush-l2")
     ap.add_argument("--persistent", action="store_true",
                     help="one persistent launch per apply when a halo is exchanged (default: separate "
                          "interior / boundary launches, measured faster)")
@@ -287,10 +292,13 @@ def main():
 
     nrhs = args.nrhs
     algo_bytes_site = algo_bytes(args.precision, args.recon, nrhs)
+    # per-kernel events only where one step holds several launches or foreign kernels
+    kernel_timing = bool(args.kernel_timing or world > 1 or args.force_halo or args.flush_l2)
     D = Dslash(gdims, grid, parity_mask=parity, kernel=args.kernel, block=args.block, min_blocks=args.min_blocks,
+               timing=kernel_timing,
                precision=args.precision, recon=args.recon,
-               overlap=not args.no_overlap, timing=True, rank=rank, world_size=world, force_halo=args.force_halo,
-               persistent=("always" if args.persistent_always else args.persistent), transport=args.transport if world > 1 or args.force_halo else "nccl")
+               overlap=not args.no_overlap, rank=rank, world_size=world, force_halo=args.force_halo,
+               pdl=not args.no_pdl, persistent=("always" if args.persistent_always else args.persistent), transport=args.transport if world > 1 or args.force_halo else "nccl")
     origin, extent = D.origin, D.local_dims
     fat, lng = fieldgen.workload_links(gdims, origin=origin, extent=extent)
     D.load_links(fat, lng)
@@ -367,9 +375,17 @@ def main():
     # algo_bytes_site already counts nrhs vectors per site; GB/s over sites, flop over site-RHS pairs
     peak, peak_src = measured_peak()
     kern_ms = t_int / max(1, n_int) if n_int else None
+    if kern_ms is None and not kernel_timing:
+        # one stencil launch per step and nothing else on the stream: the events around the timed
+        # region / launches is the average launch duration (it includes the launch gaps)
+        kern_ms, n_int = ms_max / args.steps, args.steps
+        dom_sites = int(plan.vh_local)
     lanes_n = {"site": 1, "dir2": 2, "dir4": 4, "bulk": 4}[args.kernel]
     if args.kernel == "bulk":
         kname = "dslash_bulk_kernel (TMA)"
+    elif not kernel_timing:
+        kname = (f"dslash_kernel<lanes={lanes_n}, ghost=false> (all sites): duration = CUDA events around the "
+                 f"timed region / launches (1 stencil launch per step{', PDL' if not args.no_pdl else ''})")
     elif overlapped:
         kname = f"dslash_kernel<lanes={lanes_n}> interior + boundary (high-priority stream): span per apply"
     elif one_kernel:
@@ -438,7 +454,8 @@ def main():
                            + (f" self-halo mask {args.force_halo}" if args.force_halo else ""), "parity": parity,
                            "kernel": args.kernel, "block": args.block or None, "precision": args.precision,
                            "long_link_recon": args.recon, "nrhs": nrhs,
-                           "overlap": not args.no_overlap, "persistent": "always" if args.persistent_always else args.persistent,
+                           "overlap": not args.no_overlap, "pdl": not args.no_pdl,
+                           "per_kernel_events": kernel_timing, "persistent": "always" if args.persistent_always else args.persistent,
                            "transport": args.transport if world > 1 else None,
                            "colocated_ranks_on_one_gpu": bool(args.colocate) or None,
                            "l2": ("L2 flushed between steps (2x L2 buffer write); time = summed kernel events; "

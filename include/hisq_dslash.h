@@ -104,6 +104,11 @@ enum {
                                    the rest.  2: persistent also without a halo.  Single-RHS applies
                                    only; any time                                                     */
     DSLASH_OPT_TRANSPORT = 8,   /* DSLASH_TRANSPORT_NCCL / _P2P; before load_links                    */
+    DSLASH_OPT_PDL = 9,         /* 1 (default): launch the stencil kernels with programmatic stream
+                                   serialization, so an apply's blocks start (and prefetch their
+                                   first read-only link matrix) while the previous kernel on the
+                                   stream drains; psi / chi are touched only after
+                                   griddepcontrol.wait.  0: ordinary launches; any time              */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */

@@ -55,7 +55,7 @@ class Dslash:
 
     def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="dir2", block=0,
                  force_halo=0, overlap=True, timing=False, rank=0, world_size=1, min_blocks=0, precision="f64",
-                 recon=18, persistent=False, transport="nccl"):
+                 recon=18, persistent=False, transport="nccl", pdl=True):
         import torch
         self.global_dims = tuple(int(d) for d in global_dims)
         self.precision = precision
@@ -87,6 +87,7 @@ class Dslash:
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_MIN_BLOCKS, min_blocks)
             if recon != 18:
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_LONG_RECON, recon)
+            _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_PDL, int(bool(pdl)))
             if transport == "p2p" and (world_size == 1 or use_nccl):
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_TRANSPORT, _abi.DSLASH_TRANSPORT_P2P)
             if transport == "p2p":

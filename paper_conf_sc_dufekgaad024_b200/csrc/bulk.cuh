@@ -163,7 +163,7 @@ __global__ void __launch_bounds__(32 * (kBulkConsumers + 1), 1)
 #pragma unroll
         for (int l = 0; l < 4; ++l) {
             const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
-            const SrcRef<V2> src = source<V2, GHOST>(P, mu, h, s, 0);
+            const SrcRef<V2> src = source<V2, GHOST>(P, P.in, mu, h, s, 0);
 #pragma unroll
             for (int c = 0; c < 3; ++c) v[l][c] = ld_reuse(src.p + c * src.stride, pol_keep);
         }

@@ -299,6 +299,9 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             if (st == DSLASH_OK && value == DSLASH_TRANSPORT_P2P) st = alloc_flags(h);
             return st;
         }
+        case DSLASH_OPT_PDL:
+            h->pdl = value != 0;
+            return DSLASH_OK;
         case DSLASH_OPT_PERSISTENT:
             if (value < 0 || value > 2) return fail(h, DSLASH_ERR_ARG, "persistent mode %lld not in {0,1,2}", (long long)value);
             h->persistent = (int)value;
@@ -944,7 +947,22 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
     }
     StencilFn fn = ghost ? pick_kernel<true>(h->precision, h->recon, lanes, minb, nrhs)
                          : pick_kernel<false>(h->precision, h->recon, lanes, minb, nrhs);
-    fn<<<grid, bs, 0, s>>>(K);
+    if (h->pdl) {
+        // programmatic dependent launch: may start while the previous kernel on `s` drains; the
+        // kernel waits (griddepcontrol.wait) before touching psi or chi (stencil.cuh)
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(grid);
+        cfg.blockDim = dim3(bs);
+        cfg.stream = s;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        CU(h, cudaLaunchKernelEx(&cfg, fn, K));
+    } else {
+        fn<<<grid, bs, 0, s>>>(K);
+    }
     CU(h, cudaGetLastError());
     if (tl) CU(h, cudaEventRecord(tl->b, s));
     return DSLASH_OK;

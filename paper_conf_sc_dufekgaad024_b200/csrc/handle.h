@@ -54,6 +54,7 @@ struct dslash_s {
     unsigned long long sched_next[3] = {0, 0, 0};
     // persistent fused kernel (DSLASH_OPT_PERSISTENT): the halo epoch flag it looks at
     int persistent = 0;
+    int pdl = 1;                        // programmatic dependent launch of the stencil kernels
     unsigned int* halo_flag = nullptr;
     unsigned int epoch = 0;             // halo exchanges started so far
     // P2P transport (DSLASH_TRANSPORT_P2P): CUDA-IPC-mapped neighbour buffers, copy engines and

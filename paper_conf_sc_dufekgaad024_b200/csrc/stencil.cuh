@@ -110,7 +110,8 @@ struct SrcRef {
 // outside [0, L); otherwise coordinates wrap periodically (two conditional steps suffice for
 // |h| <= 3 and L >= 2).
 template <typename V2, bool GHOST>
-__device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, int mu, int h, const Site& s, int rhs) {
+__device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, const void* in, int mu, int h, const Site& s,
+                                             int rhs) {
     const int c = mu == 0 ? s.x : mu == 1 ? s.y : mu == 2 ? s.z : s.t;
     const int L = P.L[mu];
     const int cn = c + h;
@@ -128,7 +129,7 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, int mu, int
                                    : (int64_t)P.lxh * P.L[1] * P.L[2];
         idx = s.cb + (int64_t)(cw - c) * st;
     }
-    const V2* local = static_cast<const V2*>(P.in) + (int64_t)rhs * 3 * P.vh + idx;
+    const V2* local = static_cast<const V2*>(in) + (int64_t)rhs * 3 * P.vh + idx;
     if (!GHOST || mu < 2) return {local, P.vh};
     // branch-free choice between the local site and the ghost face: the lanes of a site walk
     // different directions, so a branch here would diverge within the warp
@@ -195,6 +196,19 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
         const uint64_t pol_keep = policy_evict_last();
         s = decode_site(P, site);
         const L2* links = static_cast<const L2*>(P.links);
+        // Programmatic dependent launch (DSLASH_OPT_PDL): the links are read-only, so the first
+        // matrix (unpaired layouts) is fetched before waiting for the previous grid; psi (and the
+        // ghosts) are read, and chi written, only after griddepcontrol.wait, whose asm yields the
+        // psi base pointer so no psi load can be hoisted above it.  Without a PDL launch the wait
+        // returns at once.
+        V2 U0[9];
+        if constexpr (sizeof(LR) != 4) {
+            const L2* lp0 = links + link_index<LANES, RECON>(lane, 0, 0, P.vh, s.cb);
+#pragma unroll
+            for (int e = 0; e < 9; ++e) U0[e] = to_cplx<V2>(widen(ld_stream(lp0 + (int64_t)e * 4 * P.vh, pol_stream)));
+        }
+        const void* in;
+        asm volatile("griddepcontrol.wait;\n\tmov.b64 %0, %1;" : "=l"(in) : "l"(P.in) : "memory");
 #pragma unroll
         for (int k = 0; k < K; ++k) {
             const int mu = k * LANES + lane;
@@ -219,7 +233,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     }
 #pragma unroll
                     for (int sub = 0; sub < 2; ++sub) {
-                        const SrcRef<V2> src = source<V2, GHOST>(P, mu, sub ? -hop : hop, s, rl * NRHS);
+                        const SrcRef<V2> src = source<V2, GHOST>(P, in, mu, sub ? -hop : hop, s, rl * NRHS);
 #pragma unroll
                         for (int r = 0; r < NRHS; ++r) {
                             const int64_t roff = (int64_t)r * 3 * src.stride;
@@ -238,12 +252,17 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 #pragma unroll
             for (int l = 0; l < 4; ++l) {
                 const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
-                const SrcRef<V2> src = source<V2, GHOST>(P, mu, h, s, rl * NRHS);
+                const SrcRef<V2> src = source<V2, GHOST>(P, in, mu, h, s, rl * NRHS);
                 const L2* lp = links + link_index<LANES, RECON>(mu, l, 0, P.vh, s.cb);
                 V2 U[9];
+                if (k == 0 && l == 0) {
 #pragma unroll
-                for (int e = 0; e < elems_of<RECON>(l); ++e)
-                    U[e] = to_cplx<V2>(widen(ld_stream(lp + (int64_t)e * 4 * P.vh, pol_stream)));
+                    for (int e = 0; e < 9; ++e) U[e] = U0[e];
+                } else {
+#pragma unroll
+                    for (int e = 0; e < elems_of<RECON>(l); ++e)
+                        U[e] = to_cplx<V2>(widen(ld_stream(lp + (int64_t)e * 4 * P.vh, pol_stream)));
+                }
                 if (elems_of<RECON>(l) == 6) reconstruct_row2(U, (VR)P.long_inv_scale);
 #pragma unroll
                 for (int r = 0; r < NRHS; ++r) {
@@ -295,6 +314,8 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 
 template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1, int RHSL = 1>
 __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P) {
+    // every block has started: the next PDL-launched apply may begin filling freed SMs
+    asm volatile("griddepcontrol.launch_dependents;");
     dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
                                                          P.box_start[P.nbox]);
 }
