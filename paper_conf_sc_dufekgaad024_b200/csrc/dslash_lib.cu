@@ -919,10 +919,8 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
             CU(h, cudaMemset(h->sched, 0, 4 * sizeof(unsigned long long)));
         }
         const int slot = ghost ? 1 : 0;
-        bk.fn<<<grid, bk.threads, bk.smem, s>>>(K, h->sched + slot, h->sched_next[slot]);
-        // tickets this launch consumes (bulk.cuh): (ceil(ntiles / B) + 2 grid) * B
-        h->sched_next[slot] +=
-            ((unsigned long long)((ntiles + bk.batch - 1) / bk.batch) + 2ull * grid) * bk.batch;
+        CU(h, cudaMemsetAsync(h->sched + slot, 0, sizeof(unsigned long long), s));  // fresh tickets
+        bk.fn<<<grid, bk.threads, bk.smem, s>>>(K, h->sched + slot, 0ull);
         CU(h, cudaGetLastError());
         if (tl) CU(h, cudaEventRecord(tl->b, s));
         return DSLASH_OK;

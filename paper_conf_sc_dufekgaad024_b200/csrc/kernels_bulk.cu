@@ -9,9 +9,9 @@ static BulkKernel pick_bulk_t(bool ghost) {
     BulkKernel k;
     k.fn = ghost ? dslash_bulk_kernel<LR, VR, true, RECON> : dslash_bulk_kernel<LR, VR, false, RECON>;
     k.smem = bulk_smem_bytes<LR, RECON>();
-    k.threads = 32 * (kBulkConsumers + 1);
+    k.threads = 32 * kBulkWarps;
     k.tile = kBulkTile;
-    k.batch = kBulkBatch;
+    k.batch = 1;
     // opt in to > 48 KB of dynamic shared memory (idempotent)
     cudaFuncSetAttribute(k.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k.smem);
     return k;

@@ -247,8 +247,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                         }
                     }
                 }
-                continue;
-            }
+            } else {
 #pragma unroll
             for (int l = 0; l < 4; ++l) {
                 const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
@@ -276,6 +275,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                         matvec_acc<false>(acc[r], U, v);
                 }
             }
+            }  // unpaired links
         }
     }
     if (LANES > 1) {

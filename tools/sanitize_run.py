@@ -1,0 +1,44 @@
+"""Small applies through every kernel family, for compute-sanitizer (memcheck / racecheck /
+synccheck / initcheck).  python tools/sanitize_run.py  -> exits 0 if every result matches."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import numpy as np
+import torch
+
+import fieldgen
+from paper_conf_sc_dufekgaad024_b200 import Dslash
+
+torch.cuda.set_device(0)
+dims = (16, 8, 8, 8)
+fat, lng = fieldgen.workload_links(dims)
+src = {p: torch.from_numpy(fieldgen.vector_cb(dims, 3, p)).cuda() for p in (0, 1)}
+ref = None
+cases = [dict(kernel=k) for k in ("site", "dir2", "dir4", "bulk")]
+cases += [dict(force_halo=m, persistent=pers) for m in (0x8, 0xC) for pers in (False, True)]
+cases += [dict(force_halo=0xC, transport="p2p"), dict(recon=12), dict(precision="mixed"), dict(pdl=False)]
+n = 0
+for kw in cases:
+    with Dslash(dims, **kw) as D:
+        D.load_links(fat, lng)
+        out = D(src[1].to(D.dtype), 0)
+        o2 = D.empty_vector()
+        D.apply(o2, out.to(D.dtype), 1)
+        multi = torch.stack([src[1], src[1]]).to(D.dtype)
+        mo = torch.empty_like(multi)
+        D.apply_multi(mo, multi, 0)
+        if D.precision != "f32" and kw.get("kernel") != "bulk":
+            x = D.empty_vector()
+            D.cg(x, src[0], 0, 0.5, rel_tol=1e-8, max_iter=50)
+        torch.cuda.synchronize()
+        r = out.cpu().numpy().astype(np.complex128)
+        if ref is None:
+            ref = r
+        tol = 1e-5 if kw.get("precision") == "mixed" else 1e-12
+        err = np.abs(r - ref).max() / np.abs(ref).max()
+        assert err <= tol, (kw, err)
+        assert torch.equal(mo[0], mo[1])
+        n += 1
+print(f"sanitize_run: {n} configurations OK")

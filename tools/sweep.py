@@ -24,12 +24,15 @@ ap.add_argument("--minb", default="2,3,4")
 ap.add_argument("--steps", type=int, default=500)
 ap.add_argument("--halo", type=int, default=0)
 ap.add_argument("--precision", default="f64")
+ap.add_argument("--kernel-events", action="store_true", help="per-kernel events (cost ~3%%, block PDL overlap)")
+ap.add_argument("--no-pdl", action="store_true")
 a = ap.parse_args()
 dims = tuple(int(v) for v in a.dims.split(","))
 fat, lng = fieldgen.workload_links(dims)
 l2 = torch.cuda.get_device_properties(0).L2_cache_size
 for kern in a.kernels.split(","):
-    D = Dslash(dims, parity_mask=0, kernel=kern, force_halo=a.halo, timing=True, precision=a.precision)
+    D = Dslash(dims, parity_mask=0, kernel=kern, force_halo=a.halo, timing=a.kernel_events, precision=a.precision,
+               pdl=not a.no_pdl)
     D.load_links(fat, lng)
     vb = 3 * D.vh * 16
     R = max(2, int(np.ceil(2 * l2 / (2 * vb))) + 1)
@@ -52,7 +55,7 @@ for kern in a.kernels.split(","):
         e1.record()
         torch.cuda.synchronize()
         ms = e0.elapsed_time(e1) / a.steps
-        kms, n = D.kernel_timing()
+        kms, n = D.kernel_timing() if a.kernel_events else (ms * a.steps, a.steps)
         D.kernel_timing_reset()
         print(json.dumps({"dims": dims, "kernel": kern, "block": bs, "minb": mb, "us_per_apply": round(ms * 1e3, 2),
                           "kernel_us": round(kms / max(n, 1) * 1e3, 2),
