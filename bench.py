@@ -66,6 +66,9 @@ def parse():
     ap.add_argument("--colocate", action="store_true",
                     help="testing aid: every rank on GPU 0 (gloo process group, P2P transport); checks the N > 1 "
                          "code path on a one-GPU box -- its timings are not scaling numbers")
+    ap.add_argument("--self-nccl", action="store_true",
+                    help="with --force-halo at N = 1: self-neighbour faces through NCCL send/recv to this rank "
+                         "(one-rank communicator; the P = 2 message pattern)")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"],
                     help="halo transport for N > 1: NCCL send/recv, or copy-engine puts into IPC-mapped ghosts")
     ap.add_argument("--no-pdl", action="store_true",
@@ -263,6 +266,9 @@ def main():
     args = parse()
     if args.impl == "reference":
         return reference_arm(args)
+    # NCCL writes its log (incl. the "NCCL version" banner rank 0 prints at communicator init) to
+    # stdout by default; the bench's stdout is the one JSON line, so the log goes to stderr
+    os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
 
     import numpy as np
     import torch
@@ -298,7 +304,8 @@ def main():
                timing=kernel_timing,
                precision=args.precision, recon=args.recon,
                overlap=not args.no_overlap, rank=rank, world_size=world, force_halo=args.force_halo,
-               pdl=not args.no_pdl, persistent=("always" if args.persistent_always else args.persistent), transport=args.transport if world > 1 or args.force_halo else "nccl")
+               pdl=not args.no_pdl, persistent=("always" if args.persistent_always else args.persistent), transport=args.transport if world > 1 or args.force_halo else "nccl",
+               self_nccl=bool(args.self_nccl and world == 1 and args.force_halo and args.transport == "nccl"))
     origin, extent = D.origin, D.local_dims
     fat, lng = fieldgen.workload_links(gdims, origin=origin, extent=extent)
     D.load_links(fat, lng)
@@ -451,7 +458,9 @@ def main():
                 "config": {"workload": name, "global_dims": list(gdims), "local_dims": list(extent),
                            "proc_grid": list(grid),
                            "parallelism": (f"t{grid[3]}" if grid[2] == 1 else f"z{grid[2]}t{grid[3]}")
-                           + (f" self-halo mask {args.force_halo}" if args.force_halo else ""), "parity": parity,
+                           + (f" self-halo mask {args.force_halo}" if args.force_halo else "")
+                           + (" via NCCL send/recv to self" if args.force_halo and args.self_nccl else ""),
+                           "parity": parity,
                            "kernel": args.kernel, "block": args.block or None, "precision": args.precision,
                            "long_link_recon": args.recon, "nrhs": nrhs,
                            "overlap": not args.no_overlap, "pdl": not args.no_pdl,

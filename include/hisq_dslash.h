@@ -109,6 +109,12 @@ enum {
                                    first read-only link matrix) while the previous kernel on the
                                    stream drains; psi / chi are touched only after
                                    griddepcontrol.wait.  0: ordinary launches; any time              */
+    DSLASH_OPT_SELF_NCCL = 10,  /* 1: directions whose neighbour is this rank (FORCE_HALO with Pmu == 1)
+                                   exchange their faces (and load_links its link slabs) with NCCL
+                                   send/recv to this rank instead of device copies: the message
+                                   pattern of Pmu == 2, run on one GPU.  Needs the NCCL transport
+                                   and a communicator (dslash_create with an id, also for
+                                   nranks == 1); before load_links; 0 (default) = device copies    */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */
@@ -170,7 +176,9 @@ DSLASH_API dslash_status dslash_plan(const int32_t global_dims[4], const int32_t
  * DSLASH_F32 or DSLASH_MIXED (it fixes the stored link type and the vector type).
  * nccl_unique_id: the 128-byte ncclUniqueId from dslash_get_unique_id() on rank 0,
  * broadcast to all ranks by the caller; NULL when nranks == 1, or when the ranks will use
- * DSLASH_TRANSPORT_P2P (then no NCCL communicator is created).  On success *out owns
+ * DSLASH_TRANSPORT_P2P (then no NCCL communicator is created).  With nranks == 1 an id
+ * creates a one-rank communicator (for DSLASH_OPT_SELF_NCCL; the solver's sums then also
+ * pass through ncclAllReduce).  On success *out owns
  * a CUDA communication stream, events, ghost buffers and (nranks > 1) an NCCL
  * communicator; release it with dslash_destroy.  On failure *out is NULL. */
 DSLASH_API dslash_status dslash_create(const int32_t global_dims[4], const int32_t proc_grid[4], int32_t parity_mask,

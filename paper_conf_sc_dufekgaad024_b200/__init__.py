@@ -55,7 +55,7 @@ class Dslash:
 
     def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="dir2", block=0,
                  force_halo=0, overlap=True, timing=False, rank=0, world_size=1, min_blocks=0, precision="f64",
-                 recon=18, persistent=False, transport="nccl", pdl=True):
+                 recon=18, persistent=False, transport="nccl", pdl=True, self_nccl=False):
         import torch
         self.global_dims = tuple(int(d) for d in global_dims)
         self.precision = precision
@@ -77,6 +77,11 @@ class Dslash:
                 t.copy_(torch.frombuffer(bytearray(_abi.dslash_get_unique_id()), dtype=torch.uint8))
             dist.broadcast(t, 0)
             uid = bytes(t.cpu().numpy().tobytes())
+        elif self_nccl:
+            # one rank: a one-rank communicator, and the self-neighbour faces go through NCCL
+            # send/recv to this rank (the P = 2 message pattern on one GPU)
+            assert world_size == 1 and transport == "nccl", "self_nccl is a one-rank NCCL-transport option"
+            uid = _abi.dslash_get_unique_id()
         self.h = _abi.dslash_create(self.global_dims, self.proc_grid, parity_mask, _abi.PRECISIONS[precision], uid,
                                     world_size, rank)
         try:
@@ -101,6 +106,8 @@ class Dslash:
                                    2 if persistent == "always" else int(bool(persistent)))
             if force_halo:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_FORCE_HALO, force_halo)
+            if self_nccl:
+                _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_SELF_NCCL, 1)
             _abi.dslash_set_option(self.h, DSLASH_OPT_OVERLAP, int(bool(overlap)))
             if timing:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_TIMING, 1)

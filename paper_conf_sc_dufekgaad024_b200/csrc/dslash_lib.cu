@@ -158,6 +158,14 @@ static void free_links(dslash_t h) {
     h->loaded = false;
 }
 
+// Does direction d's exchange go through NCCL (or, under the P2P transport, the peers)?  A
+// neighbour on another rank always does; a self-neighbour (P_d = 1 with FORCE_HALO) is served by
+// device copies unless DSLASH_OPT_SELF_NCCL routes it through NCCL send/recv to this rank, the
+// message pattern of P_d = 2 (both neighbours one peer, messages matched in issue order).
+static bool exch_remote(const dslash_s* h, int d) {
+    return h->plan.nbr_rank[d][0] != h->plan.rank || h->self_nccl;
+}
+
 static void free_halo(dslash_t h) {
     for (int d = 0; d < 4; ++d)
         for (int s = 0; s < 2; ++s)
@@ -180,7 +188,7 @@ static dslash_status alloc_halo(dslash_t h, int nrhs) {
         if (!p.halo[d]) continue;
         for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->ghost[d][s], (size_t)nrhs * 3 * p.face_vh[d] * es));
     }
-    if (p.halo[2] && p.nbr_rank[2][0] != p.rank)
+    if (p.halo[2] && exch_remote(h, 2))
         for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->zsend[s], (size_t)nrhs * 3 * p.face_vh[2] * es));
     h->ghost_rhs = nrhs;
     return DSLASH_OK;
@@ -236,7 +244,7 @@ extern "C" dslash_status dslash_create(const int32_t G[4], const int32_t P[4], i
         return bail(DSLASH_ERR_CUDA);
     }
     h->transport = (nranks > 1 && !nccl_unique_id) ? DSLASH_TRANSPORT_P2P : DSLASH_TRANSPORT_NCCL;
-    if (nranks > 1 && nccl_unique_id) {
+    if (nccl_unique_id) {  // nranks == 1: a one-rank communicator (DSLASH_OPT_SELF_NCCL, solver sums)
         ncclUniqueId id;
         memcpy(&id, nccl_unique_id, sizeof id);
         ncclResult_t r = ncclCommInitRank(&h->nccl, nranks, id, rank);
@@ -280,6 +288,15 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             h->plan = p;
             h->force_halo = (int)value;
             return alloc_halo(h, h->transport == DSLASH_TRANSPORT_P2P ? kP2PMaxRhs : 1);
+        }
+        case DSLASH_OPT_SELF_NCCL: {
+            if (h->loaded || h->p2p_ready)
+                return fail(h, DSLASH_ERR_STATE, "SELF_NCCL must be set before load_links");
+            if (value && (h->transport != DSLASH_TRANSPORT_NCCL || !h->nccl))
+                return fail(h, DSLASH_ERR_STATE,
+                            "SELF_NCCL needs the NCCL transport and a communicator (dslash_create with an id)");
+            h->self_nccl = value != 0;
+            return alloc_halo(h, 1);
         }
         case DSLASH_OPT_OVERLAP:
             h->overlap = value != 0;
@@ -399,7 +416,7 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
     for (int d = 3; d >= 2; --d) {
         if (!p.halo[d]) continue;
         given[d] = slab_fat_in && slab_lng_in && slab_fat_in[d] && slab_lng_in[d];
-        if (!given[d] && p.nbr_rank[d][1] != p.rank) need_nccl = true;
+        if (!given[d] && exch_remote(h, d)) need_nccl = true;
     }
     if (need_nccl && !h->nccl) {
         cleanup();
@@ -421,13 +438,13 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
             const double2* src = k ? dlng : dfat;
             if (d == 3) {
                 const double2* top = src + (size_t)(L3 - 3) * L2 * L1 * L0 * 36;
-                if (p.nbr_rank[3][1] == p.rank)
+                if (!exch_remote(h, 3))
                     CUL(cudaMemcpyAsync(slab[3][k], top, 3 * (size_t)L2 * row, cudaMemcpyDeviceToDevice, s));
                 else
                     send[3][k] = (double2*)top;  // contiguous: zero copy
             } else {
                 double2* dst = slab[2][k];
-                if (p.nbr_rank[2][1] != p.rank) {
+                if (exch_remote(h, 2)) {
                     CUL(cudaMalloc(&send[2][k], 3 * (size_t)L3 * row));
                     tmp.push_back(send[2][k]);
                     dst = send[2][k];
@@ -442,7 +459,7 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
         CUL(cudaStreamSynchronize(s));
         ncclResult_t r = ncclGroupStart();
         for (int d = 3; d >= 2 && r == ncclSuccess; --d) {
-            if (!p.halo[d] || p.nbr_rank[d][1] == p.rank || given[d]) continue;
+            if (!p.halo[d] || !exch_remote(h, d) || given[d]) continue;
             const size_t n = (size_t)3 * (V / p.local_dims[d]) * 36 * 2;  // doubles
             for (int k = 0; k < 2 && r == ncclSuccess; ++k) {
                 r = ncclSend(send[d][k], n, ncclDouble, p.nbr_rank[d][1], h->nccl, s);
@@ -775,7 +792,7 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
     bool nccl_work = false;
     const size_t tslab = 3 * lxh * L1 * L2;  // sites in 3 t-slices of one parity
     if (p.halo[3]) {
-        if (p.nbr_rank[3][0] == p.rank) {
+        if (!exch_remote(h, 3)) {
             // minus ghost <- my top slices, plus ghost <- my bottom slices (periodic self-halo)
             CU(h, cudaMemcpy2DAsync(h->ghost[3][0], tslab * es, src + (vh - tslab) * es, vh * es, tslab * es, rows,
                                     cudaMemcpyDeviceToDevice, h->comm));
@@ -788,7 +805,7 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
     if (p.halo[2]) {
         // [r][c][t][z0..z0+2][y][xh] -> [r][c][t][d][y][xh]: one row of 3 z-slices per (r, c, t)
         const size_t zrow = lxh * L1;  // sites of one z-slice of one t
-        const bool self = p.nbr_rank[2][0] == p.rank;
+        const bool self = !exch_remote(h, 2);
         char* to_minus = self ? h->ghost[2][1] : h->zsend[0];  // my bottom slices
         char* to_plus = self ? h->ghost[2][0] : h->zsend[1];   // my top slices
         CU(h, cudaMemcpy2DAsync(to_minus, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
@@ -804,7 +821,7 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
         // messages in issue order: my first message (bottom) is the peer's first receive (its plus
         // ghost, since I am its plus neighbour).  Counts are bytes (ncclUint8).
         NC(h, ncclGroupStart());
-        if (p.halo[3] && p.nbr_rank[3][0] != p.rank) {
+        if (p.halo[3] && exch_remote(h, 3)) {
             const size_t n = tslab * es;
             for (size_t r = 0; r < rows; ++r)  // t-faces are contiguous in every (rhs, colour) row: zero copy
                 NC(h, ncclSend(src + r * vh * es, n, ncclUint8, p.nbr_rank[3][0], h->nccl, h->comm));
@@ -815,7 +832,7 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
             for (size_t r = 0; r < rows; ++r)
                 NC(h, ncclRecv(h->ghost[3][0] + r * n, n, ncclUint8, p.nbr_rank[3][0], h->nccl, h->comm));
         }
-        if (p.halo[2] && p.nbr_rank[2][0] != p.rank) {
+        if (p.halo[2] && exch_remote(h, 2)) {
             const size_t n = rows * p.face_vh[2] * es;
             NC(h, ncclSend(h->zsend[0], n, ncclUint8, p.nbr_rank[2][0], h->nccl, h->comm));
             NC(h, ncclSend(h->zsend[1], n, ncclUint8, p.nbr_rank[2][1], h->nccl, h->comm));

@@ -577,3 +577,48 @@ def test_pdl_chained_applies_bitwise(torch_cuda, kernel):
             torch.cuda.synchronize()
             res.append(torch.stack([x.cpu() for x in xs]))
     assert torch.equal(res[0], res[1])
+
+
+@pytest.mark.parametrize("mask", [0x8, 0x4, 0xC])
+@pytest.mark.parametrize("kernel", ["dir2", "site"])
+def test_nccl_transport_self_halo(torch_cuda, mask, kernel):
+    """The NCCL transport run for real on one GPU (DSLASH_OPT_SELF_NCCL): a one-rank
+    communicator, faces and link slabs sent with ncclSend/ncclRecv to this rank in the P = 2
+    message pattern (both neighbours one peer, matched in issue order).  Several epochs, single
+    and multi-RHS, bitwise equal to the unpartitioned apply; the NCCL face order and the ghost
+    layout are the ones a 2-rank t / z partition uses."""
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 8, 8, 12)
+    fat, lng = fieldgen.workload_links(dims)
+    srcs = torch.stack([torch.from_numpy(fieldgen.vector_cb(dims, 90 + r, 1)) for r in range(3)]).cuda()
+    with Dslash(dims, kernel=kernel) as D:
+        D.load_links(fat, lng)
+        ref = torch.stack([D(srcs[r].contiguous(), 0) for r in range(3)]).cpu()
+    with Dslash(dims, kernel=kernel, force_halo=mask, self_nccl=True) as D:
+        D.load_links(fat, lng)
+        for it in range(3):
+            for r in range(3):
+                out = D(srcs[r].contiguous(), 0)
+                assert torch.equal(out.cpu(), ref[r]), (it, r)
+        multi = torch.empty_like(srcs)
+        D.apply_multi(multi, srcs, 0)
+        torch.cuda.synchronize()
+        assert torch.equal(multi.cpu(), ref)
+    # the oracle as well, so a consistently wrong face (both paths) cannot pass
+    psi = fieldgen.vector(dims, 90)
+    want = oracle.full_to_cb(oracle.dslash(fat, lng, psi, 0), 0)
+    assert oracle.normwise_error(ref[0].numpy(), want) <= TOL
+
+
+def test_nccl_self_option_errors(torch_cuda):
+    from paper_conf_sc_dufekgaad024_b200 import Dslash, DslashError, _abi
+    dims = (8, 8, 8, 12)
+    with Dslash(dims, force_halo=0x8) as D:     # no communicator
+        with pytest.raises(DslashError):
+            _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_SELF_NCCL, 1)
+    fat, lng = fieldgen.workload_links(dims)
+    with Dslash(dims, force_halo=0x8, self_nccl=True) as D:
+        D.load_links(fat, lng)
+        with pytest.raises(DslashError):           # after load_links
+            _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_SELF_NCCL, 0)

@@ -68,13 +68,16 @@ def test_cg_self_halo_bitwise(torch_cuda):
     fat, lng = fieldgen.workload_links(dims)
     b = torch.from_numpy(fieldgen.vector_cb(dims, 73, 0)).cuda()
     sols = []
-    for mask in (0, 0xC):
-        with Dslash(dims, force_halo=mask) as D:
+    # unpartitioned; self-halo by device copies; self-halo through NCCL send/recv to this rank
+    # with the dot products through a one-rank ncclAllReduce (DSLASH_OPT_SELF_NCCL)
+    for mask, self_nccl in ((0, False), (0xC, False), (0xC, True)):
+        with Dslash(dims, force_halo=mask, self_nccl=self_nccl) as D:
             D.load_links(fat, lng)
             x = D.empty_vector()
             ok, it, res = D.cg(x, b, 0, 0.3, rel_tol=1e-10)
             sols.append((x.cpu(), it, res))
-    assert torch.equal(sols[0][0], sols[1][0]) and sols[0][1] == sols[1][1]
+    for k in (1, 2):
+        assert torch.equal(sols[0][0], sols[k][0]) and sols[0][1] == sols[k][1], k
 
 
 def test_cg_free_field_closed_form(torch_cuda):
