@@ -66,6 +66,9 @@ def parse():
     ap.add_argument("--colocate", action="store_true",
                     help="testing aid: every rank on GPU 0 (gloo process group, P2P transport); checks the N > 1 "
                          "code path on a one-GPU box -- its timings are not scaling numbers")
+    ap.add_argument("--stage", action="store_true",
+                    help="neighbour-staged kernel: x/y source rows of a tile copied to shared memory by TMA "
+                         "(site / dir2 variants)")
     ap.add_argument("--self-nccl", action="store_true",
                     help="with --force-halo at N = 1: self-neighbour faces through NCCL send/recv to this rank "
                          "(one-rank communicator; the P = 2 message pattern)")
@@ -305,7 +308,8 @@ def main():
                precision=args.precision, recon=args.recon,
                overlap=not args.no_overlap, rank=rank, world_size=world, force_halo=args.force_halo,
                pdl=not args.no_pdl, persistent=("always" if args.persistent_always else args.persistent), transport=args.transport if world > 1 or args.force_halo else "nccl",
-               self_nccl=bool(args.self_nccl and world == 1 and args.force_halo and args.transport == "nccl"))
+               self_nccl=bool(args.self_nccl and world == 1 and args.force_halo and args.transport == "nccl"),
+               stage=args.stage)
     origin, extent = D.origin, D.local_dims
     fat, lng = fieldgen.workload_links(gdims, origin=origin, extent=extent)
     D.load_links(fat, lng)
@@ -400,12 +404,15 @@ def main():
                  if not args.no_overlap else f"dslash_kernel<lanes={lanes_n}, ghost=true> (all sites, after the halo)")
     else:
         kname = f"dslash_kernel<lanes={lanes_n}, ghost=false>" + (" interior" if any(plan.halo) else " (all sites)")
+    if args.stage and args.kernel != "bulk":
+        kname = kname.replace("dslash_kernel<", "dslash_stage_kernel<")
     roof = None
     if kern_ms:
         achieved = algo_bytes_site * dom_sites / (kern_ms * 1e-3) / 1e9
         roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4),
-                "traffic": ncu_traffic(args.kernel + ("" if args.precision == "f64" else f"-{args.precision}")
+                "traffic": ncu_traffic(args.kernel + ("-stage" if args.stage else "")
+                                     + ("" if args.precision == "f64" else f"-{args.precision}")
                                      + ("" if args.recon == 18 else f"-r{args.recon}")
                                      + ("-persistent" if one_kernel and not args.no_overlap else ""), extent),
                 "kernel": kname,
@@ -461,7 +468,7 @@ def main():
                            + (f" self-halo mask {args.force_halo}" if args.force_halo else "")
                            + (" via NCCL send/recv to self" if args.force_halo and args.self_nccl else ""),
                            "parity": parity,
-                           "kernel": args.kernel, "block": args.block or None, "precision": args.precision,
+                           "kernel": args.kernel, "stage": bool(args.stage), "block": args.block or None, "precision": args.precision,
                            "long_link_recon": args.recon, "nrhs": nrhs,
                            "overlap": not args.no_overlap, "pdl": not args.no_pdl,
                            "per_kernel_events": kernel_timing, "persistent": "always" if args.persistent_always else args.persistent,

@@ -115,6 +115,13 @@ enum {
                                    pattern of Pmu == 2, run on one GPU.  Needs the NCCL transport
                                    and a communicator (dslash_create with an id, also for
                                    nranks == 1); before load_links; 0 (default) = device copies    */
+    DSLASH_OPT_STAGE = 11,      /* 1: neighbour-staged kernel for the site / dir2 variants (PAPER.md L321,
+                                   the 3LP-1 local-memory staging): a block owns TY full x-rows of one
+                                   (z, t); the TMA engine copies the source rows y0-3 .. y0+TY+2 into
+                                   shared memory once (cp.async.bulk + mbarrier) and the 8 x/y hops
+                                   per site read them there; z/t hops stay global loads.  Same link
+                                   layout (any time).  fp32 needs Lx/2 even; the persistent path
+                                   (DSLASH_OPT_PERSISTENT) does not stage.  0 (default): off        */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */

@@ -55,7 +55,7 @@ class Dslash:
 
     def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="dir2", block=0,
                  force_halo=0, overlap=True, timing=False, rank=0, world_size=1, min_blocks=0, precision="f64",
-                 recon=18, persistent=False, transport="nccl", pdl=True, self_nccl=False):
+                 recon=18, persistent=False, transport="nccl", pdl=True, self_nccl=False, stage=False):
         import torch
         self.global_dims = tuple(int(d) for d in global_dims)
         self.precision = precision
@@ -108,6 +108,8 @@ class Dslash:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_FORCE_HALO, force_halo)
             if self_nccl:
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_SELF_NCCL, 1)
+            if stage:
+                _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_STAGE, 1)
             _abi.dslash_set_option(self.h, DSLASH_OPT_OVERLAP, int(bool(overlap)))
             if timing:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_TIMING, 1)

@@ -19,6 +19,14 @@ StencilFn pick_f32_r12(bool ghost, int lanes, int minb, int nrhs);
 StencilFn pick_mixed_r18(bool ghost, int lanes, int minb, int nrhs);
 StencilFn pick_mixed_r12(bool ghost, int lanes, int minb, int nrhs);
 
+// the neighbour-staged kernel (stencil.cuh dslash_stage_kernel) of one (precision, recon): lanes 1/2
+StencilFn pick_f64_r18_stage(bool ghost, int lanes, int nrhs);
+StencilFn pick_f64_r12_stage(bool ghost, int lanes, int nrhs);
+StencilFn pick_f32_r18_stage(bool ghost, int lanes, int nrhs);
+StencilFn pick_f32_r12_stage(bool ghost, int lanes, int nrhs);
+StencilFn pick_mixed_r18_stage(bool ghost, int lanes, int nrhs);
+StencilFn pick_mixed_r12_stage(bool ghost, int lanes, int nrhs);
+
 // the persistent fused kernel (stencil.cuh) of one (precision, recon): lanes 1/2/4; mode 0 = no
 // halo, 1 = halo (interior, then boundary tiles if the faces have landed), 2 = boundary clean-up
 PersistFn persist_f64_r18(int mode, int lanes);

@@ -271,6 +271,8 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
                 return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel needs Lx/2 to be a multiple of %d", kBulkTile);
             if (h->loaded && value != h->kernel)
                 return fail(h, DSLASH_ERR_STATE, "kernel variant fixes the link layout: set it before load_links");
+            if (h->stage && value != DSLASH_KERNEL_SITE && value != DSLASH_KERNEL_DIR2)
+                return fail(h, DSLASH_ERR_UNSUPPORTED, "the neighbour-staged kernel serves the site and dir2 variants");
             h->kernel = (int)value;
             return DSLASH_OK;
         case DSLASH_OPT_BLOCK:
@@ -298,6 +300,13 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             h->self_nccl = value != 0;
             return alloc_halo(h, 1);
         }
+        case DSLASH_OPT_STAGE:
+            if (value && h->kernel != DSLASH_KERNEL_SITE && h->kernel != DSLASH_KERNEL_DIR2)
+                return fail(h, DSLASH_ERR_UNSUPPORTED, "the neighbour-staged kernel serves the site and dir2 variants");
+            if (value && h->precision == DSLASH_F32 && (h->plan.local_dims[0] / 2) % 2)
+                return fail(h, DSLASH_ERR_UNSUPPORTED, "staged fp32 rows need Lx/2 even (16-byte bulk copies)");
+            h->stage = value != 0;
+            return DSLASH_OK;
         case DSLASH_OPT_OVERLAP:
             h->overlap = value != 0;
             return DSLASH_OK;
@@ -904,6 +913,97 @@ static StencilFn pick_kernel(int precision, int recon, int lanes, int minb, int 
 static int default_block(int lanes) { return lanes == 4 ? 64 : 64; }
 static int default_minb(int lanes) { return lanes == 4 ? 2 : 2; }
 
+static StencilFn pick_stage_kernel(int precision, int recon, bool ghost, int lanes, int nrhs) {
+    const bool r12 = recon == 12;
+    switch (precision) {
+        case DSLASH_F32:
+            return r12 ? pick_f32_r12_stage(ghost, lanes, nrhs) : pick_f32_r18_stage(ghost, lanes, nrhs);
+        case DSLASH_MIXED:
+            return r12 ? pick_mixed_r12_stage(ghost, lanes, nrhs) : pick_mixed_r18_stage(ghost, lanes, nrhs);
+        default: return r12 ? pick_f64_r12_stage(ghost, lanes, nrhs) : pick_f64_r18_stage(ghost, lanes, nrhs);
+    }
+}
+
+// rows per tile of the neighbour-staged kernel: the largest divisor TY of Ly with
+// lxh * TY * threads_per_site <= 256 (0: an x-row alone exceeds a block)
+static int stage_rows(const dslash_s* h, int threads_per_site) {
+    const int lxh = h->plan.local_dims[0] / 2, Ly = h->plan.local_dims[1];
+    for (int ty = Ly; ty >= 1; --ty)
+        if (Ly % ty == 0 && lxh * ty * threads_per_site <= 256) return ty;
+    return 0;
+}
+
+// events around one timed launch (DSLASH_OPT_TIMING); *out = NULL when timing is off
+static dslash_status timing_begin(dslash_t h, int kind, cudaStream_t s, dslash_s::TimedLaunch** out) {
+    *out = nullptr;
+    if (!h->timing) return DSLASH_OK;
+    if (h->tused == h->tpool.size()) {
+        dslash_s::TimedLaunch t{};
+        CU(h, cudaEventCreate(&t.a));
+        CU(h, cudaEventCreate(&t.b));
+        h->tpool.push_back(t);
+    }
+    dslash_s::TimedLaunch* tl = &h->tpool[h->tused++];
+    tl->kind = kind;
+    CU(h, cudaEventRecord(tl->a, s));
+    *out = tl;
+    return DSLASH_OK;
+}
+
+// launch with programmatic stream serialization (the kernels wait with griddepcontrol.wait before
+// touching psi or chi, stencil.cuh) or as an ordinary launch
+static cudaError_t launch_pdl(bool pdl, StencilFn fn, const StencilParams& K, unsigned grid, int bs, size_t smem,
+                              cudaStream_t s) {
+    if (!pdl) {
+        fn<<<grid, bs, smem, s>>>(K);
+        return cudaGetLastError();
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(bs);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, fn, K);
+}
+
+// the neighbour-staged kernel over the boxes of K: one block per tile of TY full x-rows
+static dslash_status launch_stage(dslash_t h, StencilParams K, bool ghost, int kind, cudaStream_t s, int nrhs,
+                                  int lanes) {
+    const int64_t sites = K.box_start[K.nbox];
+    const int rhsl = nrhs == 8 ? 2 : 1;
+    const int ty = stage_rows(h, lanes * rhsl);
+    if (!ty)
+        return fail(h, DSLASH_ERR_UNSUPPORTED, "staged kernel: an x-row of %d sites x %d threads exceeds a block",
+                    K.lxh, lanes * rhsl);
+    K.stage_ty = ty;
+    const int64_t tile = (int64_t)K.lxh * ty;  // every box holds whole tiles (full x and y extents)
+    const unsigned grid = (unsigned)(sites / tile);
+    const int bs = (int)(tile * lanes * rhsl);
+    const size_t smem = (size_t)nrhs * 3 * (ty + 6) * K.lxh * vec_elem(h);
+    StencilFn fn = pick_stage_kernel(h->precision, h->recon, ghost, lanes, nrhs);
+    static std::vector<std::pair<StencilFn, size_t>> smem_set;  // opt-in above 48 KB, once per size
+    if (smem > 48 * 1024) {
+        bool done = false;
+        for (auto& e : smem_set)
+            if (e.first == fn && e.second >= smem) done = true;
+        if (!done) {
+            CU(h, cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            smem_set.push_back({fn, smem});
+        }
+    }
+    dslash_s::TimedLaunch* tl = nullptr;
+    dslash_status st = timing_begin(h, kind, s, &tl);
+    if (st != DSLASH_OK) return st;
+    CU(h, launch_pdl(h->pdl, fn, K, grid, bs, smem, s));
+    if (tl) CU(h, cudaEventRecord(tl->b, s));
+    return DSLASH_OK;
+}
+
 // one launch of the stencil over the boxes of K for nrhs (1, 2, 4 or 8) right-hand sides
 static int num_sms(dslash_t h) {
     static int n = 0;
@@ -919,17 +1019,8 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
         const int64_t ntiles = sites / bk.tile;
         const unsigned grid = (unsigned)(ntiles < num_sms(h) ? ntiles : num_sms(h));
         dslash_s::TimedLaunch* tl = nullptr;
-        if (h->timing) {
-            if (h->tused == h->tpool.size()) {
-                dslash_s::TimedLaunch t{};
-                CU(h, cudaEventCreate(&t.a));
-                CU(h, cudaEventCreate(&t.b));
-                h->tpool.push_back(t);
-            }
-            tl = &h->tpool[h->tused++];
-            tl->kind = kind;
-            CU(h, cudaEventRecord(tl->a, s));
-        }
+        dslash_status st = timing_begin(h, kind, s, &tl);
+        if (st != DSLASH_OK) return st;
         // one ticket counter per kernel class: interior and boundary launches may run concurrently
         if (!h->sched) {
             CU(h, cudaMalloc(&h->sched, 4 * sizeof(unsigned long long)));
@@ -943,42 +1034,19 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
         return DSLASH_OK;
     }
     const int lanes = lanes_of(h->kernel);
+    if (h->stage) return launch_stage(h, K, ghost, kind, s, nrhs, lanes);
     const int bs = h->block ? h->block : default_block(lanes);
     const int minb = h->min_blocks ? h->min_blocks : default_minb(lanes);
     // right-hand sides are register-blocked per thread; 8 of them use 2 thread groups of 4
     const int64_t threads = sites * lanes * (nrhs == 8 ? 2 : 1);
     const unsigned grid = (unsigned)((threads + bs - 1) / bs);
     dslash_s::TimedLaunch* tl = nullptr;
-    if (h->timing) {
-        if (h->tused == h->tpool.size()) {
-            dslash_s::TimedLaunch t{};
-            CU(h, cudaEventCreate(&t.a));
-            CU(h, cudaEventCreate(&t.b));
-            h->tpool.push_back(t);
-        }
-        tl = &h->tpool[h->tused++];
-        tl->kind = kind;
-        CU(h, cudaEventRecord(tl->a, s));
-    }
+    dslash_status st = timing_begin(h, kind, s, &tl);
+    if (st != DSLASH_OK) return st;
     StencilFn fn = ghost ? pick_kernel<true>(h->precision, h->recon, lanes, minb, nrhs)
                          : pick_kernel<false>(h->precision, h->recon, lanes, minb, nrhs);
-    if (h->pdl) {
-        // programmatic dependent launch: may start while the previous kernel on `s` drains; the
-        // kernel waits (griddepcontrol.wait) before touching psi or chi (stencil.cuh)
-        cudaLaunchConfig_t cfg = {};
-        cfg.gridDim = dim3(grid);
-        cfg.blockDim = dim3(bs);
-        cfg.stream = s;
-        cudaLaunchAttribute attr[1];
-        attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-        attr[0].val.programmaticStreamSerializationAllowed = 1;
-        cfg.attrs = attr;
-        cfg.numAttrs = 1;
-        CU(h, cudaLaunchKernelEx(&cfg, fn, K));
-    } else {
-        fn<<<grid, bs, 0, s>>>(K);
-    }
-    CU(h, cudaGetLastError());
+    // programmatic dependent launch: may start while the previous kernel on `s` drains
+    CU(h, launch_pdl(h->pdl, fn, K, grid, bs, 0, s));
     if (tl) CU(h, cudaEventRecord(tl->b, s));
     return DSLASH_OK;
 }

@@ -62,6 +62,7 @@ struct dslash_s {
     // neighbour that fills my ghost[d][side]), [8..15] free_from[d][side] (written by the neighbour
     // whose ghost my bottom (side 0) / top (side 1) face fills, once it consumed it).
     int transport = DSLASH_TRANSPORT_NCCL;
+    int stage = 0;                      // DSLASH_OPT_STAGE: neighbour-staged kernel (x/y rows in smem by TMA)
     int self_nccl = 0;                  // DSLASH_OPT_SELF_NCCL: self-neighbour faces via NCCL
     unsigned int* flags = nullptr;
     char* peer_ghost[4][2] = {};        // [d][0]: minus nbr's plus ghost; [d][1]: plus nbr's minus ghost

@@ -40,6 +40,24 @@ StencilFn pick_any(bool ghost, int lanes, int minb, int nrhs) {
     return ghost ? pick_lanes<LR, VR, true, RECON>(lanes, minb, nrhs) : pick_lanes<LR, VR, false, RECON>(lanes, minb, nrhs);
 }
 
+// the neighbour-staged kernel (DSLASH_OPT_STAGE): LANES 1 and 2, MINB 2, 1/2/4/8 right-hand sides
+template <typename LR, typename VR, int LANES, bool GHOST, int RECON>
+StencilFn pick_stage_n(int nrhs) {
+    switch (nrhs) {
+        case 2: return dslash_stage_kernel<LR, VR, LANES, GHOST, RECON, 2>;
+        case 4: return dslash_stage_kernel<LR, VR, LANES, GHOST, RECON, 4>;
+        case 8: return dslash_stage_kernel<LR, VR, LANES, GHOST, RECON, 4, 2>;
+        default: return dslash_stage_kernel<LR, VR, LANES, GHOST, RECON, 1>;
+    }
+}
+
+template <typename LR, typename VR, int RECON>
+StencilFn pick_stage(bool ghost, int lanes, int nrhs) {
+    if (lanes == 1)
+        return ghost ? pick_stage_n<LR, VR, 1, true, RECON>(nrhs) : pick_stage_n<LR, VR, 1, false, RECON>(nrhs);
+    return ghost ? pick_stage_n<LR, VR, 2, true, RECON>(nrhs) : pick_stage_n<LR, VR, 2, false, RECON>(nrhs);
+}
+
 template <typename LR, typename VR, int LANES, int RECON>
 PersistFn pick_persist_l(int mode) {
     switch (mode) {
@@ -66,4 +84,5 @@ PersistFn pick_persist(int mode, int lanes) {
         return pick_any<LR, VR, RECON>(ghost, lanes, minb, nrhs);              \
     }                                                                          \
     PersistFn PNAME(int mode, int lanes) { return pick_persist<LR, VR, RECON>(mode, lanes); } \
+    StencilFn NAME##_stage(bool ghost, int lanes, int nrhs) { return pick_stage<LR, VR, RECON>(ghost, lanes, nrhs); } \
     }

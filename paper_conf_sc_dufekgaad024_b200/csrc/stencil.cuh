@@ -143,6 +143,94 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, const void*
     return {ghost ? gp : local, ghost ? fv : P.vh};
 }
 
+// ---------------------------------------------------------------- staged neighbour tile
+// DSLASH_OPT_STAGE (the 3LP-1 kernel's local-memory staging):
+// a block owns one tile = TY full x-rows y0 .. y0+TY-1 at one (z, t).  Its 8 x- and y-hops per
+// site read source rows y0-3 .. y0+TY+2 of that (z, t) plane, which the TMA engine copies into
+// shared memory once per tile (cp.async.bulk, one copy per contiguous run of rows and
+// (rhs, colour)), instead of 8 gathers per site from L1/L2.  z and t hops, whose sources no
+// other site of the tile reads, stay global loads.  x and y are never partitioned, so every
+// staged row is local.  Layout: sv[((r * 3 + c) * rows + i) * lxh + xh], row i <-> y = y0-3+i.
+template <typename V2>
+struct StageTile {
+    V2* sv;          // shared-memory tile
+    uint64_t* bar;   // mbarrier: the tile's bulk copies complete on it (phase 0)
+    int y0;          // first row of the tile
+    int rows;        // TY + 6
+    int64_t plane0;  // cb offset of (xh = 0, y = 0) in the tile's (z, t) plane
+    uint32_t sbase;  // shared-state-space address of sv
+};
+
+// thread 0: one bulk copy per (rhs, colour) and contiguous run of rows (the y wrap splits it)
+template <typename V2>
+__device__ __forceinline__ void stage_tile_issue(const StencilParams& P, const void* in, const StageTile<V2>& T, int nr,
+                                                 uint64_t pol) {
+    const int Ly = P.L[1], lxh = P.lxh, rows = T.rows;
+    const uint32_t row_bytes = (uint32_t)(lxh * sizeof(V2));
+    mbar_arrive_expect_tx(T.bar, (uint32_t)(nr * 3 * rows) * row_bytes);
+    const V2* src = static_cast<const V2*>(in);
+    for (int i = 0; i < rows;) {
+        int y = (T.y0 - 3 + i) % Ly;
+        if (y < 0) y += Ly;
+        const int n = min(rows - i, Ly - y);
+        for (int rc = 0; rc < nr * 3; ++rc)
+            bulk_g2s(T.sv + ((int64_t)rc * rows + i) * lxh, src + (int64_t)rc * P.vh + T.plane0 + (int64_t)y * lxh,
+                     (uint32_t)n * row_bytes, T.bar, pol);
+        i += n;
+    }
+}
+
+// shared address of psi(x + h mu^), colour 0, right-hand side `rhs`, for mu = 0 (x) or 1 (y);
+// colour c / rhs r lie c (3 r) planes of rows * lxh complex further
+template <typename V2>
+__device__ __forceinline__ uint32_t staged_addr(const StencilParams& P, const StageTile<V2>& T, uint32_t sbase, int mu,
+                                                int h, const Site& s, int rhs) {
+    const int L = P.L[0];
+    int cw = s.x + h;
+    if (cw < 0) cw += L;
+    if (cw < 0) cw += L;
+    if (cw >= L) cw -= L;
+    if (cw >= L) cw -= L;
+    const bool ymove = mu != 0;
+    const int row = s.y - T.y0 + 3 + (ymove ? h : 0);
+    const int xh = ymove ? s.xh : (cw >> 1);
+    return sbase + (uint32_t)((rhs * 3 * T.rows + row) * P.lxh + xh) * (uint32_t)sizeof(V2);
+}
+
+// Wait for the tile's bulk copies; the returned base address comes out of the waiting asm, so no
+// shared load addressed from it can be scheduled above the wait (the loads below need not be
+// volatile and can be batched freely).
+__device__ __forceinline__ uint32_t stage_wait(uint64_t* bar, uint32_t sbase) {
+    uint32_t b;
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "SWAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n\t"
+        "@!p bra SWAIT_%=;\n\t"
+        "mov.b32 %0, %2;\n}"
+        : "=r"(b)
+        : "r"(smem_addr(bar)), "r"(sbase)
+        : "memory");
+    return b;
+}
+
+__device__ __forceinline__ double2 lds_at(uint32_t a, double2*) {
+    double2 r;
+    asm("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(r.x), "=d"(r.y) : "r"(a));
+    return r;
+}
+__device__ __forceinline__ float2 lds_at(uint32_t a, float2*) {
+    float2 r;
+    asm("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(r.x), "=f"(r.y) : "r"(a));
+    return r;
+}
+
+// one neighbour colour component: from the staged tile (shared address sa + off_b) or from global
+template <typename V2>
+__device__ __forceinline__ V2 ld_src(bool staged, uint32_t sa, uint32_t off_b, const V2* p, uint64_t pol) {
+    return staged ? lds_at(sa + off_b, (V2*)nullptr) : ld_reuse(p, pol);
+}
+
 // acc (+/-)= U v for a 3x3 matrix whose 9 elements are U[e]
 template <bool SUB, typename V2>
 __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[3]) {
@@ -174,12 +262,19 @@ __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[
 // RHSL > 1: the site's right-hand sides are split over RHSL adjacent thread groups, each
 // register-blocking NRHS of them (rhs = rl * NRHS + r); the groups of a site issue identical link
 // addresses in one warp instruction, so each sector is fetched once.
-template <typename LR, typename VR, int LANES, bool GHOST, int RECON, int NRHS, int RHSL = 1>
-__device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_t gid, const int64_t site_end) {
+// STAGED: x/y neighbours come from the block's shared-memory tile T (dslash_stage_kernel).  The
+// staged kernel visits the global (z, t) directions first and the tile's (x, y) ones last, so
+// the tile's bulk copies land while the z/t links and neighbours stream (a different summation
+// order from the unstaged kernel: equal within the fp64 tolerance, not bitwise).
+template <typename LR, typename VR, int LANES, bool GHOST, int RECON, int NRHS, int RHSL = 1, bool STAGED = false>
+__device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_t gid, const int64_t site_end,
+                                            const StageTile<cplx_t<VR>> T = {}) {
     static_assert(LANES == 1 || LANES == 2 || LANES == 4, "LANES must divide 4");
+    static_assert(!STAGED || LANES <= 2, "the staged tile serves LANES 1 and 2");
     using L2 = cplx_t<LR>;
     using V2 = cplx_t<VR>;
     constexpr int K = 4 / LANES;
+    constexpr int kFirstStaged = LANES == 1 ? 2 : 1;  // first loop step that reads the tile
     const int lane = (LANES == 1) ? 0 : (int)(gid & (LANES - 1));
     const int rl = (RHSL == 1) ? 0 : (int)((gid / LANES) % RHSL);
     const int64_t site = gid / (LANES * RHSL);
@@ -201,17 +296,31 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
         // ghosts) are read, and chi written, only after griddepcontrol.wait, whose asm yields the
         // psi base pointer so no psi load can be hoisted above it.  Without a PDL launch the wait
         // returns at once.
+        // (staged: thread 0 issues the tile's bulk copies right after the wait, before any link is
+        // in flight, so the issue loop's registers never coexist with a held matrix)
+        const void* in = nullptr;
+        if constexpr (STAGED) {
+            asm volatile("griddepcontrol.wait;\n\tmov.b64 %0, %1;" : "=l"(in) : "l"(P.in) : "memory");
+            if (threadIdx.x == 0) stage_tile_issue(P, in, T, NRHS * RHSL, pol_keep);
+        }
         V2 U0[9];
         if constexpr (sizeof(LR) != 4) {
-            const L2* lp0 = links + link_index<LANES, RECON>(lane, 0, 0, P.vh, s.cb);
+            const L2* lp0 = links + link_index<LANES, RECON>((STAGED ? K - 1 : 0) * LANES + lane, 0, 0, P.vh, s.cb);
 #pragma unroll
             for (int e = 0; e < 9; ++e) U0[e] = to_cplx<V2>(widen(ld_stream(lp0 + (int64_t)e * 4 * P.vh, pol_stream)));
         }
-        const void* in;
-        asm volatile("griddepcontrol.wait;\n\tmov.b64 %0, %1;" : "=l"(in) : "l"(P.in) : "memory");
+        if constexpr (!STAGED) asm volatile("griddepcontrol.wait;\n\tmov.b64 %0, %1;" : "=l"(in) : "l"(P.in) : "memory");
+        const uint32_t plane_b = STAGED ? (uint32_t)(T.rows * P.lxh * sizeof(V2)) : 0u;  // bytes per staged plane
+        uint32_t sbase = 0;  // the tile's shared address, valid once stage_wait returned it
 #pragma unroll
-        for (int k = 0; k < K; ++k) {
+        for (int kk = 0; kk < K; ++kk) {
+            const int k = STAGED ? K - 1 - kk : kk;
             const int mu = k * LANES + lane;
+            // compile-time after unrolling: LANES 1 -> mu = k; LANES 2 -> k == 0 is (x, y)
+            const bool stg = STAGED && (LANES == 1 ? k < 2 : k == 0);
+            if constexpr (STAGED) {
+                if (kk == kFirstStaged) sbase = stage_wait(T.bar, T.sbase);
+            }
             if constexpr (sizeof(LR) == 4) {
                 // fp32 links, paired layout: one 16-byte load feeds the forward and the backward
                 // matrix of a kind; the FMA order is that of the unpaired loop (l = 0, 1, 2, 3)
@@ -233,13 +342,17 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     }
 #pragma unroll
                     for (int sub = 0; sub < 2; ++sub) {
-                        const SrcRef<V2> src = source<V2, GHOST>(P, in, mu, sub ? -hop : hop, s, rl * NRHS);
+                        const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0}
+                                                   : source<V2, GHOST>(P, in, mu, sub ? -hop : hop, s, rl * NRHS);
+                        const uint32_t sa = stg ? staged_addr<V2>(P, T, sbase, mu, sub ? -hop : hop, s, rl * NRHS) : 0u;
 #pragma unroll
                         for (int r = 0; r < NRHS; ++r) {
                             const int64_t roff = (int64_t)r * 3 * src.stride;
                             V2 v[3];
 #pragma unroll
-                            for (int c = 0; c < 3; ++c) v[c] = ld_reuse(src.p + roff + c * src.stride, pol_keep);
+                            for (int c = 0; c < 3; ++c)
+                                v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride,
+                                              pol_keep);
                             if (sub)
                                 matvec_acc<true>(acc[r], Ub, v);
                             else
@@ -251,10 +364,11 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 #pragma unroll
             for (int l = 0; l < 4; ++l) {
                 const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
-                const SrcRef<V2> src = source<V2, GHOST>(P, in, mu, h, s, rl * NRHS);
+                const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0} : source<V2, GHOST>(P, in, mu, h, s, rl * NRHS);
+                const uint32_t sa = stg ? staged_addr<V2>(P, T, sbase, mu, h, s, rl * NRHS) : 0u;
                 const L2* lp = links + link_index<LANES, RECON>(mu, l, 0, P.vh, s.cb);
                 V2 U[9];
-                if (k == 0 && l == 0) {
+                if (kk == 0 && l == 0) {
 #pragma unroll
                     for (int e = 0; e < 9; ++e) U[e] = U0[e];
                 } else {
@@ -268,7 +382,8 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     const int64_t roff = (int64_t)r * 3 * src.stride;  // [rhs][3][vh or face_vh]
                     V2 v[3];
 #pragma unroll
-                    for (int c = 0; c < 3; ++c) v[c] = ld_reuse(src.p + roff + c * src.stride, pol_keep);
+                    for (int c = 0; c < 3; ++c)
+                        v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride, pol_keep);
                     if (l & 1)
                         matvec_acc<true>(acc[r], U, v);
                     else
@@ -318,6 +433,34 @@ __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P
     asm volatile("griddepcontrol.launch_dependents;");
     dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
                                                          P.box_start[P.nbox]);
+}
+
+// The neighbour-staged variant (DSLASH_OPT_STAGE): one tile of P.stage_ty full x-rows per block
+// (blockDim = lxh * stage_ty * LANES * RHSL threads), the tile's source rows y0-3 .. y0+TY+2 in
+// dynamic shared memory (NRHS * RHSL * 3 * (TY + 6) * lxh complex).  Boxes span full x and y, so
+// tiles never straddle a box and every thread is valid.
+template <typename LR, typename VR, int LANES, bool GHOST, int RECON, int NRHS = 1, int RHSL = 1>
+__global__ void __launch_bounds__(256, 2) dslash_stage_kernel(const StencilParams P) {
+    using V2 = cplx_t<VR>;
+    asm volatile("griddepcontrol.launch_dependents;");
+    __shared__ uint64_t bar;
+    extern __shared__ __align__(128) unsigned char stage_smem[];
+    if (threadIdx.x == 0) {
+        mbar_init(&bar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const int64_t tile_sites = (int64_t)P.lxh * P.stage_ty;
+    const Site s0 = decode_site(P, (int64_t)blockIdx.x * tile_sites);
+    StageTile<V2> T;
+    T.sv = reinterpret_cast<V2*>(stage_smem);
+    T.bar = &bar;
+    T.y0 = s0.y;
+    T.rows = P.stage_ty + 6;
+    T.plane0 = s0.cb - s0.xh - (int64_t)P.lxh * s0.y;
+    T.sbase = smem_addr(stage_smem);
+    dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL, true>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                                                               P.box_start[P.nbox], T);
 }
 
 // ---------------------------------------------------------------- persistent fused kernel
