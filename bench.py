@@ -63,6 +63,10 @@ def parse():
                     help="bitmask of directions run through the halo path with neighbour = self (1 GPU)")
     ap.add_argument("--parity", type=int, default=0)
     ap.add_argument("--no-overlap", action="store_true")
+    ap.add_argument("--overlap", default="sites", choices=["sites", "dirs"],
+                    help="with a halo: split by sites (interior box during the exchange, boundary slabs "
+                         "after) or by direction (local hops of every site during the exchange, ghost hops "
+                         "after)")
     ap.add_argument("--colocate", action="store_true",
                     help="testing aid: every rank on GPU 0 (gloo process group, P2P transport); checks the N > 1 "
                          "code path on a one-GPU box -- its timings are not scaling numbers")
@@ -306,7 +310,7 @@ def main():
     D = Dslash(gdims, grid, parity_mask=parity, kernel=args.kernel, block=args.block, min_blocks=args.min_blocks,
                timing=kernel_timing,
                precision=args.precision, recon=args.recon,
-               overlap=not args.no_overlap, rank=rank, world_size=world, force_halo=args.force_halo,
+               overlap="none" if args.no_overlap else args.overlap, rank=rank, world_size=world, force_halo=args.force_halo,
                pdl=not args.no_pdl, persistent=("always" if args.persistent_always else args.persistent), transport=args.transport if world > 1 or args.force_halo else "nccl",
                self_nccl=bool(args.self_nccl and world == 1 and args.force_halo and args.transport == "nccl"),
                stage=args.stage)
@@ -398,7 +402,9 @@ def main():
         kname = (f"dslash_kernel<lanes={lanes_n}, ghost=false> (all sites): duration = CUDA events around the "
                  f"timed region / launches (1 stencil launch per step{', PDL' if not args.no_pdl else ''})")
     elif overlapped:
-        kname = f"dslash_kernel<lanes={lanes_n}> interior + boundary (high-priority stream): span per apply"
+        kname = (f"dslash_kernel<lanes={lanes_n}, ghost=true> local pass (all sites) + ghost pass (boundary): "
+                 "span per apply" if args.overlap == "dirs" else
+                 f"dslash_kernel<lanes={lanes_n}> interior + boundary (high-priority stream): span per apply")
     elif one_kernel:
         kname = (f"dslash_persistent_kernel<lanes={lanes_n}, ghost={str(any(plan.halo)).lower()}> (all sites)"
                  if not args.no_overlap else f"dslash_kernel<lanes={lanes_n}, ghost=true> (all sites, after the halo)")
@@ -470,7 +476,7 @@ def main():
                            "parity": parity,
                            "kernel": args.kernel, "stage": bool(args.stage), "block": args.block or None, "precision": args.precision,
                            "long_link_recon": args.recon, "nrhs": nrhs,
-                           "overlap": not args.no_overlap, "pdl": not args.no_pdl,
+                           "overlap": "none" if args.no_overlap else args.overlap, "pdl": not args.no_pdl,
                            "per_kernel_events": kernel_timing, "persistent": "always" if args.persistent_always else args.persistent,
                            "transport": args.transport if world > 1 else None,
                            "colocated_ranks_on_one_gpu": bool(args.colocate) or None,

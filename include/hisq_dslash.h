@@ -85,8 +85,8 @@ enum {
     DSLASH_OPT_BLOCK = 1,       /* threads per block (multiple of 32, <= 256), 0 = default; any time   */
     DSLASH_OPT_FORCE_HALO = 2,  /* bitmask of directions (bit mu) exchanged through the halo path even
                                    when Pmu == 1 (self-halo: neighbour = self); before load_links      */
-    DSLASH_OPT_OVERLAP = 3,     /* 1 (default): interior kernel overlaps the halo exchange; 0: one
-                                   kernel over all sites after the exchange                            */
+    DSLASH_OPT_OVERLAP = 3,     /* how an apply with a halo overlaps the exchange (DSLASH_OVERLAP_*);
+                                   any time                                                           */
     DSLASH_OPT_TIMING = 4,      /* 1: record CUDA events around every kernel (dslash_kernel_timing)   */
     DSLASH_OPT_LONG_RECON = 6,  /* 18 (default): long links stored in full; 12: long links stored as
                                    rows 0 and 1 only, row 2 rebuilt in registers as conj(r0 x r1)/s
@@ -125,6 +125,22 @@ enum {
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */
+};
+
+/* Overlap modes (DSLASH_OPT_OVERLAP) of an apply that exchanges a halo. */
+enum {
+    DSLASH_OVERLAP_NONE = 0,   /* one kernel over all sites after the exchange                        */
+    DSLASH_OVERLAP_SITES = 1,  /* (default) split by sites: the interior box (no ghost source) runs
+                                  during the exchange; the boundary slabs run on a high-priority
+                                  stream once the faces land                                        */
+    DSLASH_OVERLAP_DIRS = 2    /* split by direction: a local pass over every site during the
+                                  exchange skips the hops into ghost faces; a ghost pass over the
+                                  boundary slabs then adds exactly those hops to the stored partial
+                                  sums (+96 B per boundary site).  Hides the exchange even when no
+                                  site is interior (local extent 6 with a depth-3 halo).  Boundary
+                                  sites sum their terms in another order than DSLASH_OVERLAP_NONE:
+                                  equal within the fp64 tolerance, not bitwise.  Not for the TMA
+                                  kernel                                                             */
 };
 
 /* Halo transports (DSLASH_OPT_TRANSPORT). */

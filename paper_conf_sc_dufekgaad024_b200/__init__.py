@@ -110,7 +110,9 @@ class Dslash:
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_SELF_NCCL, 1)
             if stage:
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_STAGE, 1)
-            _abi.dslash_set_option(self.h, DSLASH_OPT_OVERLAP, int(bool(overlap)))
+            # True / "sites": split by sites (default); "dirs": split by direction; False / "none"
+            _abi.dslash_set_option(self.h, DSLASH_OPT_OVERLAP,
+                                   _abi.OVERLAPS[overlap] if isinstance(overlap, str) else int(overlap))
             if timing:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_TIMING, 1)
         except Exception:

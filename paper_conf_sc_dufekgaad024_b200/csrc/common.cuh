@@ -191,6 +191,13 @@ struct StencilParams {
     int64_t box_start[kMaxBoxes + 1];  // prefix sum of target sites per box
     FastDiv div_xh[kMaxBoxes], div_y[kMaxBoxes], div_z[kMaxBoxes];
     int stage_ty;              // rows per tile of the neighbour-staged kernel (DSLASH_OPT_STAGE)
+    int halo_pass;             // GHOST kernels: kPassAll, or one pass of the split-by-direction overlap
 };
+
+// Passes of a GHOST kernel (StencilParams::halo_pass).  kPassAll reads local sources and ghost
+// faces alike.  The split-by-direction overlap (DSLASH_OVERLAP_DIRS) runs kPassLocal over every
+// site while the faces are in flight (hops into a ghost face are skipped, link and vector), then
+// kPassGhost over the boundary sites: only the skipped hops, added to the stored partial sum.
+constexpr int kPassAll = 0, kPassLocal = 1, kPassGhost = 2;
 
 }  // namespace hisq

@@ -267,6 +267,8 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             if (value != DSLASH_KERNEL_SITE && value != DSLASH_KERNEL_DIR4 && value != DSLASH_KERNEL_DIR2 &&
                 value != DSLASH_KERNEL_BULK)
                 return fail(h, DSLASH_ERR_ARG, "unknown kernel variant %lld", (long long)value);
+            if (value == DSLASH_KERNEL_BULK && h->overlap == DSLASH_OVERLAP_DIRS)
+                return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel has no split-by-direction passes");
             if (value == DSLASH_KERNEL_BULK && (h->plan.local_dims[0] / 2) % kBulkTile)
                 return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel needs Lx/2 to be a multiple of %d", kBulkTile);
             if (h->loaded && value != h->kernel)
@@ -308,7 +310,11 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             h->stage = value != 0;
             return DSLASH_OK;
         case DSLASH_OPT_OVERLAP:
-            h->overlap = value != 0;
+            if (value < 0 || value > DSLASH_OVERLAP_DIRS)
+                return fail(h, DSLASH_ERR_ARG, "overlap mode %lld not in {0, 1, 2}", (long long)value);
+            if (value == DSLASH_OVERLAP_DIRS && h->kernel == DSLASH_KERNEL_BULK)
+                return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel has no split-by-direction passes");
+            h->overlap = (int)value;
             return DSLASH_OK;
         case DSLASH_OPT_TIMING:
             h->timing = value != 0;
@@ -1233,6 +1239,37 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
     for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
         K.ghost[d][0] = h->ghost[d][0];
         K.ghost[d][1] = h->ghost[d][1];
+    }
+    if (h->overlap == DSLASH_OVERLAP_DIRS) {
+        // split by direction: the local pass runs over EVERY site while the faces are in flight,
+        // skipping the hops into ghost faces; once they landed, the ghost pass adds exactly those
+        // hops to the boundary sites' partial sums (QUDA-style interior / exterior kernels).  Both
+        // on the caller's stream; the bench reports their span.
+        size_t span = (size_t)-1;
+        if (h->timing) {
+            dslash_s::TimedLaunch* tl = nullptr;
+            if ((st = timing_begin(h, DSLASH_TIMING_SPAN, s, &tl)) != DSLASH_OK) return st;
+            span = (size_t)(tl - h->tpool.data());
+        }
+        K.halo_pass = kPassLocal;
+        if (p.n_interior + p.n_boundary > kMaxBoxes) {
+            st = launch_rhs(h, K, p.interior, p.n_interior, true, DSLASH_TIMING_INTERIOR, s, nrhs);
+            if (st == DSLASH_OK)
+                st = launch_rhs(h, K, p.boundary, p.n_boundary, true, DSLASH_TIMING_INTERIOR, s, nrhs);
+        } else {
+            dslash_box_t all[kMaxBoxes];
+            int n = 0;
+            for (int i = 0; i < p.n_interior; ++i) all[n++] = p.interior[i];
+            for (int i = 0; i < p.n_boundary; ++i) all[n++] = p.boundary[i];
+            st = launch_rhs(h, K, all, n, true, DSLASH_TIMING_INTERIOR, s, nrhs);
+        }
+        if (st != DSLASH_OK) return st;
+        if ((st = dslash_halo_wait(h, stream)) != DSLASH_OK) return st;
+        K.halo_pass = kPassGhost;
+        if ((st = launch_rhs(h, K, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, s, nrhs)) != DSLASH_OK)
+            return st;
+        if (span != (size_t)-1) CU(h, cudaEventRecord(h->tpool[span].b, s));
+        return DSLASH_OK;
     }
     if (h->overlap) {
         // interior on the caller's stream; boundary on the handle's boundary stream as soon as the

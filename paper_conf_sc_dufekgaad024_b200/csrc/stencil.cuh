@@ -104,6 +104,7 @@ template <typename V2>
 struct SrcRef {
     const V2* p;  // colour component c at p[c * stride]
     int64_t stride;
+    bool ghost;   // the source lies in a ghost face (GHOST kernels only)
 };
 
 // Address of psi(x + h mu^).  GHOST: directions in P.halo_mask read the depth-3 ghost faces
@@ -130,7 +131,7 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, const void*
         idx = s.cb + (int64_t)(cw - c) * st;
     }
     const V2* local = static_cast<const V2*>(in) + (int64_t)rhs * 3 * P.vh + idx;
-    if (!GHOST || mu < 2) return {local, P.vh};
+    if (!GHOST || mu < 2) return {local, P.vh, false};
     // branch-free choice between the local site and the ghost face: the lanes of a site walk
     // different directions, so a branch here would diverge within the warp
     const bool ghost = ((P.halo_mask >> mu) & 1) && (cn < 0 || cn >= L);
@@ -140,7 +141,10 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, const void*
                                 : s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (d + 3 * (int64_t)s.t));
     const int64_t fv = P.face_vh[mu];
     const V2* gp = static_cast<const V2*>(P.ghost[mu][side]) + (int64_t)rhs * 3 * fv + f;
-    return {ghost ? gp : local, ghost ? fv : P.vh};
+    // local pass of the split-by-direction overlap: the face is still in flight, so a ghost hop
+    // reads the (valid) wrapped local address and the caller zeroes the vector
+    const bool use_face = ghost && P.halo_pass != kPassLocal;
+    return {use_face ? gp : local, use_face ? fv : P.vh, ghost};
 }
 
 // ---------------------------------------------------------------- staged neighbour tile
@@ -231,6 +235,13 @@ __device__ __forceinline__ V2 ld_src(bool staged, uint32_t sa, uint32_t off_b, c
     return staged ? lds_at(sa + off_b, (V2*)nullptr) : ld_reuse(p, pol);
 }
 
+// v = 0 when z (a select, so acc + U * 0 leaves acc's value unchanged without a branch)
+template <typename V2>
+__device__ __forceinline__ void zero_if(V2& v, bool z) {
+    v.x = z ? decltype(v.x)(0) : v.x;
+    v.y = z ? decltype(v.y)(0) : v.y;
+}
+
 // acc (+/-)= U v for a 3x3 matrix whose 9 elements are U[e]
 template <bool SUB, typename V2>
 __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[3]) {
@@ -304,7 +315,8 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
             if (threadIdx.x == 0) stage_tile_issue(P, in, T, NRHS * RHSL, pol_keep);
         }
         V2 U0[9];
-        if constexpr (sizeof(LR) != 4) {
+        // (not in the ghost pass, whose first hop is never a ghost hop for LANES 1 / 2)
+        if (sizeof(LR) != 4 && !(GHOST && P.halo_pass == kPassGhost)) {
             const L2* lp0 = links + link_index<LANES, RECON>((STAGED ? K - 1 : 0) * LANES + lane, 0, 0, P.vh, s.cb);
 #pragma unroll
             for (int e = 0; e < 9; ++e) U0[e] = to_cplx<V2>(widen(ld_stream(lp0 + (int64_t)e * 4 * P.vh, pol_stream)));
@@ -328,6 +340,13 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 #pragma unroll
                 for (int j = 0; j < 2; ++j) {
                     const int hop = j ? 3 : 1;
+                    if (GHOST && P.halo_pass == kPassGhost) {
+                        // ghost pass of the split-by-direction overlap: skip a kind neither of
+                        // whose two hops reaches a ghost face (no link bytes either)
+                        const bool ga = source<V2, GHOST>(P, in, mu, hop, s, 0).ghost;
+                        const bool gb = source<V2, GHOST>(P, in, mu, -hop, s, 0).ghost;
+                        if (!(ga || gb)) continue;
+                    }
                     const float4* lp = links4 + link_index_paired<LANES>(mu, j, 0, P.vh, s.cb);
                     V2 Ua[9], Ub[9];
 #pragma unroll
@@ -342,17 +361,21 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     }
 #pragma unroll
                     for (int sub = 0; sub < 2; ++sub) {
-                        const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0}
+                        const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0, false}
                                                    : source<V2, GHOST>(P, in, mu, sub ? -hop : hop, s, rl * NRHS);
                         const uint32_t sa = stg ? staged_addr<V2>(P, T, sbase, mu, sub ? -hop : hop, s, rl * NRHS) : 0u;
+                        if (GHOST && P.halo_pass == kPassGhost && !src.ghost) continue;
+                        const bool zap = GHOST && P.halo_pass == kPassLocal && src.ghost;
 #pragma unroll
                         for (int r = 0; r < NRHS; ++r) {
                             const int64_t roff = (int64_t)r * 3 * src.stride;
                             V2 v[3];
 #pragma unroll
-                            for (int c = 0; c < 3; ++c)
+                            for (int c = 0; c < 3; ++c) {
                                 v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride,
                                               pol_keep);
+                                if (GHOST) zero_if(v[c], zap);
+                            }
                             if (sub)
                                 matvec_acc<true>(acc[r], Ub, v);
                             else
@@ -364,11 +387,17 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 #pragma unroll
             for (int l = 0; l < 4; ++l) {
                 const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
-                const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0} : source<V2, GHOST>(P, in, mu, h, s, rl * NRHS);
+                const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0, false} : source<V2, GHOST>(P, in, mu, h, s, rl * NRHS);
                 const uint32_t sa = stg ? staged_addr<V2>(P, T, sbase, mu, h, s, rl * NRHS) : 0u;
+                // split-by-direction passes: the ghost pass takes only the ghost hops (the link of
+                // a skipped hop is not read); the local pass stays branch-free, so loads can be
+                // hoisted as in the unsplit kernel: a ghost hop multiplies a zeroed vector (its
+                // link is read in both passes, 144 B per ghost hop)
+                if (GHOST && P.halo_pass == kPassGhost && !src.ghost) continue;
+                const bool zap = GHOST && P.halo_pass == kPassLocal && src.ghost;
                 const L2* lp = links + link_index<LANES, RECON>(mu, l, 0, P.vh, s.cb);
                 V2 U[9];
-                if (kk == 0 && l == 0) {
+                if (kk == 0 && l == 0 && !(GHOST && P.halo_pass == kPassGhost)) {
 #pragma unroll
                     for (int e = 0; e < 9; ++e) U[e] = U0[e];
                 } else {
@@ -382,8 +411,10 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     const int64_t roff = (int64_t)r * 3 * src.stride;  // [rhs][3][vh or face_vh]
                     V2 v[3];
 #pragma unroll
-                    for (int c = 0; c < 3; ++c)
+                    for (int c = 0; c < 3; ++c) {
                         v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride, pol_keep);
+                        if (GHOST) zero_if(v[c], zap);
+                    }
                     if (l & 1)
                         matvec_acc<true>(acc[r], U, v);
                     else
@@ -408,6 +439,23 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
             }
     }
     if (!valid) return;
+    if (GHOST && P.halo_pass == kPassGhost) {
+        // ghost pass: chi = (local pass's partial sum) + (ghost hops), read back per colour this
+        // lane stores below
+#pragma unroll
+        for (int r = 0; r < NRHS; ++r) {
+            const V2* prev = static_cast<const V2*>(P.out) + (int64_t)(rl * NRHS + r) * 3 * P.vh + s.cb;
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                const bool mine = LANES == 1 || (LANES == 2 ? (lane == 0) == (c < 2) : lane == c);
+                if (mine) {
+                    const V2 o = prev[c * P.vh];
+                    acc[r][c].x = o.x + acc[r][c].x;
+                    acc[r][c].y = o.y + acc[r][c].y;
+                }
+            }
+        }
+    }
 #pragma unroll
     for (int r = 0; r < NRHS; ++r) {
         V2* out = static_cast<V2*>(P.out) + (int64_t)(rl * NRHS + r) * 3 * P.vh;
