@@ -63,7 +63,7 @@ def parse():
                     help="bitmask of directions run through the halo path with neighbour = self (1 GPU)")
     ap.add_argument("--parity", type=int, default=0)
     ap.add_argument("--no-overlap", action="store_true")
-    ap.add_argument("--overlap", default="sites", choices=["sites", "dirs"],
+    ap.add_argument("--overlap", default="sites", choices=["sites", "dirs", "fused"],
                     help="with a halo: split by sites (interior box during the exchange, boundary slabs "
                          "after) or by direction (local hops of every site during the exchange, ghost hops "
                          "after)")
@@ -273,9 +273,12 @@ def main():
     args = parse()
     if args.impl == "reference":
         return reference_arm(args)
-    # NCCL writes its log (incl. the "NCCL version" banner rank 0 prints at communicator init) to
-    # stdout by default; the bench's stdout is the one JSON line, so the log goes to stderr
-    os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
+    # The bench's stdout is the one JSON line.  Native code may print to fd 1 (NCCL prints its
+    # "NCCL version" banner with printf at communicator init when NCCL_DEBUG is set), so fd 1
+    # points at stderr for the whole run and is restored only for the JSON line.
+    sys.stdout.flush()
+    real_stdout = os.dup(1)
+    os.dup2(2, 1)
 
     import numpy as np
     import torch
@@ -289,6 +292,7 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if args.gpus != world:
         if world == 1 and args.gpus > 1:
+            os.dup2(real_stdout, 1)
             print(json.dumps({"error": f"--gpus {args.gpus} needs torchrun with {args.gpus} ranks"}))
             return 2
     if args.colocate:
@@ -404,6 +408,8 @@ def main():
     elif overlapped:
         kname = (f"dslash_kernel<lanes={lanes_n}, ghost=true> local pass (all sites) + ghost pass (boundary): "
                  "span per apply" if args.overlap == "dirs" else
+                 f"dslash_fused_kernel<lanes={lanes_n}> one launch, boundary blocks look once at the halo flag "
+                 "(+ clean-up launch): span per apply" if args.overlap == "fused" else
                  f"dslash_kernel<lanes={lanes_n}> interior + boundary (high-priority stream): span per apply")
     elif one_kernel:
         kname = (f"dslash_persistent_kernel<lanes={lanes_n}, ghost={str(any(plan.halo)).lower()}> (all sites)"
@@ -462,6 +468,8 @@ def main():
         cpu, _ = run_oracle_baseline(gdims, parity, args.cpu_seconds)
 
     launches_per_step = (n_all // max(1, args.steps)) if n_all else 1
+    if not n_all and n_span and args.overlap == "fused":
+        launches_per_step = 2   # the fused launch and its clean-up launch (timed together as a span)
     if rank == 0:
         line = {"metric": METRIC, "value": round(gflops, 2), "unit": "GFLOP/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
@@ -491,7 +499,10 @@ def main():
                 "roofline": roof, "clocks": clk.summary(), "e2e": e2e,
                 "gpu_launches": launches_per_step * args.steps,
                 "cpu_baseline": cpu}
+        sys.stdout.flush()
+        os.dup2(real_stdout, 1)
         print(json.dumps(line), flush=True)
+        os.dup2(2, 1)
     D.close()
     if world > 1:
         dist.destroy_process_group()

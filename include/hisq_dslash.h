@@ -122,6 +122,8 @@ enum {
                                    per site read them there; z/t hops stay global loads.  Same link
                                    layout (any time).  fp32 needs Lx/2 even; the persistent path
                                    (DSLASH_OPT_PERSISTENT) does not stage.  0 (default): off        */
+    DSLASH_OPT_FUSED_DEFER = 12,/* testing aid for DSLASH_OVERLAP_FUSED: 1 = every boundary block
+                                   defers to the clean-up launch; any time                         */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */
@@ -133,7 +135,7 @@ enum {
     DSLASH_OVERLAP_SITES = 1,  /* (default) split by sites: the interior box (no ghost source) runs
                                   during the exchange; the boundary slabs run on a high-priority
                                   stream once the faces land                                        */
-    DSLASH_OVERLAP_DIRS = 2    /* split by direction: a local pass over every site during the
+    DSLASH_OVERLAP_DIRS = 2,   /* split by direction: a local pass over every site during the
                                   exchange skips the hops into ghost faces; a ghost pass over the
                                   boundary slabs then adds exactly those hops to the stored partial
                                   sums (+96 B per boundary site).  Hides the exchange even when no
@@ -141,6 +143,13 @@ enum {
                                   sites sum their terms in another order than DSLASH_OVERLAP_NONE:
                                   equal within the fp64 tolerance, not bitwise.  Not for the TMA
                                   kernel                                                             */
+    DSLASH_OVERLAP_FUSED = 3   /* one launch over all sites, interior blocks first; each boundary
+                                  block looks once at the halo flags (set by the exchange with a
+                                  stream memory operation) and either computes its sites or defers
+                                  itself to a stream-ordered clean-up launch.  No block waits, so
+                                  no transport can be starved of SMs.  Bitwise equal to SITES.
+                                  Single-RHS applies of the site / dir2 / dir4 kernels (others
+                                  take SITES)                                                        */
 };
 
 /* Halo transports (DSLASH_OPT_TRANSPORT). */

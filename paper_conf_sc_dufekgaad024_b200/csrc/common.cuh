@@ -49,6 +49,19 @@ __device__ __forceinline__ double2 ld_reuse(const double2* p, uint64_t pol) {
     return r;
 }
 
+// coherent load (L2 only, no L1 / read-only path): for ghost faces that another engine may have
+// written while the reading kernel was already running (DSLASH_OVERLAP_FUSED, persistent kernel)
+__device__ __forceinline__ double2 ld_cg(const double2* p) {
+    double2 r;
+    asm volatile("ld.global.cg.v2.f64 {%0, %1}, [%2];" : "=d"(r.x), "=d"(r.y) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ float2 ld_cg(const float2* p) {
+    float2 r;
+    asm volatile("ld.global.cg.v2.f32 {%0, %1}, [%2];" : "=f"(r.x), "=f"(r.y) : "l"(p));
+    return r;
+}
+
 __device__ __forceinline__ void st_stream(double2* p, double2 v) {
     asm volatile("st.global.cs.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
 }

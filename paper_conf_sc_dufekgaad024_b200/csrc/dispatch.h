@@ -27,6 +27,15 @@ StencilFn pick_f32_r12_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_mixed_r18_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_mixed_r12_stage(bool ghost, int lanes, int nrhs);
 
+// the one-shot fused kernel (stencil.cuh dslash_fused_kernel / _cleanup) of one (precision, recon)
+typedef void (*FusedFn)(StencilParams, FusedArgs);
+FusedFn pick_f64_r18_fused(bool cleanup, int lanes);
+FusedFn pick_f64_r12_fused(bool cleanup, int lanes);
+FusedFn pick_f32_r18_fused(bool cleanup, int lanes);
+FusedFn pick_f32_r12_fused(bool cleanup, int lanes);
+FusedFn pick_mixed_r18_fused(bool cleanup, int lanes);
+FusedFn pick_mixed_r12_fused(bool cleanup, int lanes);
+
 // the persistent fused kernel (stencil.cuh) of one (precision, recon): lanes 1/2/4; mode 0 = no
 // halo, 1 = halo (interior, then boundary tiles if the faces have landed), 2 = boundary clean-up
 PersistFn persist_f64_r18(int mode, int lanes);

@@ -302,6 +302,9 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             h->self_nccl = value != 0;
             return alloc_halo(h, 1);
         }
+        case DSLASH_OPT_FUSED_DEFER:
+            h->fused_defer_all = value != 0;
+            return DSLASH_OK;
         case DSLASH_OPT_STAGE:
             if (value && h->kernel != DSLASH_KERNEL_SITE && h->kernel != DSLASH_KERNEL_DIR2)
                 return fail(h, DSLASH_ERR_UNSUPPORTED, "the neighbour-staged kernel serves the site and dir2 variants");
@@ -310,8 +313,8 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             h->stage = value != 0;
             return DSLASH_OK;
         case DSLASH_OPT_OVERLAP:
-            if (value < 0 || value > DSLASH_OVERLAP_DIRS)
-                return fail(h, DSLASH_ERR_ARG, "overlap mode %lld not in {0, 1, 2}", (long long)value);
+            if (value < 0 || value > DSLASH_OVERLAP_FUSED)
+                return fail(h, DSLASH_ERR_ARG, "overlap mode %lld not in {0, 1, 2, 3}", (long long)value);
             if (value == DSLASH_OVERLAP_DIRS && h->kernel == DSLASH_KERNEL_BULK)
                 return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel has no split-by-direction passes");
             h->overlap = (int)value;
@@ -1189,6 +1192,102 @@ static dslash_status apply_persistent(dslash_t h, StencilParams K, cudaStream_t 
     return DSLASH_OK;
 }
 
+static FusedFn pick_fused_kernel(int precision, int recon, bool cleanup, int lanes) {
+    const bool r12 = recon == 12;
+    switch (precision) {
+        case DSLASH_F32: return r12 ? pick_f32_r12_fused(cleanup, lanes) : pick_f32_r18_fused(cleanup, lanes);
+        case DSLASH_MIXED: return r12 ? pick_mixed_r12_fused(cleanup, lanes) : pick_mixed_r18_fused(cleanup, lanes);
+        default: return r12 ? pick_f64_r12_fused(cleanup, lanes) : pick_f64_r18_fused(cleanup, lanes);
+    }
+}
+
+static cudaError_t launch_fused(bool pdl, FusedFn fn, const StencilParams& K, const FusedArgs& A, unsigned grid,
+                                int bs, cudaStream_t s) {
+    if (!pdl) {
+        fn<<<grid, bs, 0, s>>>(K, A);
+        return cudaGetLastError();
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(bs);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, fn, K, A);
+}
+
+// DSLASH_OVERLAP_FUSED: one launch over all sites, interior blocks first; boundary blocks look
+// once at the halo flags and defer to a stream-ordered clean-up launch if the faces have not
+// landed (stencil.cuh dslash_fused_kernel).  Single right-hand side, site / dir2 / dir4 kernels.
+static dslash_status apply_fused(dslash_t h, StencilParams K, cudaStream_t s) {
+    const dslash_plan_t& p = h->plan;
+    dslash_box_t all[kMaxBoxes];
+    int n = 0;
+    for (int i = 0; i < p.n_interior; ++i) all[n++] = p.interior[i];
+    for (int i = 0; i < p.n_boundary; ++i) all[n++] = p.boundary[i];
+    fill_boxes(K, all, n);
+    const int lanes = lanes_of(h->kernel);
+    const int bs = h->block ? h->block : default_block(lanes);
+    const int64_t sites = K.box_start[K.nbox];
+    const int64_t grid = (sites * lanes + bs - 1) / bs;
+    FusedArgs A{};
+    A.interior_blocks = p.interior_sites * lanes / bs;  // a block straddling into the boundary is a boundary block
+    const int64_t nbnd = grid - A.interior_blocks;
+    if (h->fused_cap < nbnd) {
+        if (h->fused_buf) {
+            CU(h, cudaStreamSynchronize(s));  // a queued clean-up may still read the old list
+            cudaFree(h->fused_buf);
+            h->fused_buf = nullptr;
+        }
+        CU(h, cudaMalloc(&h->fused_buf, (size_t)(2 + nbnd) * sizeof(unsigned int)));
+        CU(h, cudaMemsetAsync(h->fused_buf, 0, 2 * sizeof(unsigned int), s));
+        h->fused_cap = nbnd;
+        h->fused_parity = 0;
+    }
+    A.count = h->fused_buf + h->fused_parity;
+    A.count_next = h->fused_buf + (1 - h->fused_parity);
+    A.deferred = h->fused_buf + 2;
+    A.defer_all = h->fused_defer_all;
+    h->fused_parity ^= 1;
+    if (!h->halo_flag) {
+        CU(h, cudaMalloc(&h->halo_flag, sizeof(unsigned int)));
+        CU(h, cudaMemset(h->halo_flag, 0, sizeof(unsigned int)));
+        h->epoch = 0;
+    }
+    dslash_status st = halo_start_impl(h, K.in, 1, s);
+    if (st != DSLASH_OK) return st;
+    for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
+        K.ghost[d][0] = h->ghost[d][0];
+        K.ghost[d][1] = h->ghost[d][1];
+    }
+    if (h->transport == DSLASH_TRANSPORT_P2P) {
+        for (int d = 3; d >= 2; --d)  // the neighbours raise my ready flags (halo_start_p2p)
+            if (p.halo[d])
+                for (int side = 0; side < 2; ++side) A.flags[A.nflags++] = h->flags + 2 * d + side;
+    } else {
+        ++h->epoch;
+        if (write_value_fn()(h->comm, (unsigned long long)(uintptr_t)h->halo_flag, h->epoch, 0) != 0)
+            return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 failed");
+        A.flags[A.nflags++] = h->halo_flag;
+    }
+    A.epoch = h->epoch;
+    size_t span = (size_t)-1;
+    if (h->timing) {
+        dslash_s::TimedLaunch* tl = nullptr;
+        if ((st = timing_begin(h, DSLASH_TIMING_SPAN, s, &tl)) != DSLASH_OK) return st;
+        span = (size_t)(tl - h->tpool.data());
+    }
+    CU(h, launch_fused(h->pdl, pick_fused_kernel(h->precision, h->recon, false, lanes), K, A, (unsigned)grid, bs, s));
+    if ((st = dslash_halo_wait(h, (dslash_stream_t)s)) != DSLASH_OK) return st;
+    const int64_t g2 = nbnd > 0 ? nbnd : 1;  // one block per boundary block that may have deferred
+    CU(h, launch_fused(h->pdl, pick_fused_kernel(h->precision, h->recon, true, lanes), K, A, (unsigned)g2, bs, s));
+    if (span != (size_t)-1) CU(h, cudaEventRecord(h->tpool[span].b, s));
+    return DSLASH_OK;
+}
+
 static dslash_status check_vectors(dslash_t h, const void* out, const void* in, int nrhs) {
     if (!out || !in) return fail(h, DSLASH_ERR_ARG, "NULL vector pointer");
     if (((uintptr_t)out & 15) || ((uintptr_t)in & 15)) return fail(h, DSLASH_ERR_ARG, "vectors must be 16-byte aligned");
@@ -1235,6 +1334,11 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         write_value_fn())
         return apply_persistent(h, K, s);
     if (!any_halo(p)) return launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
+    // the one-shot fused kernel serves single-RHS applies of the site / dir2 / dir4 kernels; other
+    // applies in this mode take the split by sites
+    if (h->overlap == DSLASH_OVERLAP_FUSED && nrhs == 1 && h->kernel != DSLASH_KERNEL_BULK && !h->stage &&
+        write_value_fn())
+        return apply_fused(h, K, s);
     if ((st = halo_start_impl(h, in, nrhs, s)) != DSLASH_OK) return st;
     for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
         K.ghost[d][0] = h->ghost[d][0];
@@ -1271,7 +1375,7 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         if (span != (size_t)-1) CU(h, cudaEventRecord(h->tpool[span].b, s));
         return DSLASH_OK;
     }
-    if (h->overlap) {
+    if (h->overlap == DSLASH_OVERLAP_SITES || h->overlap == DSLASH_OVERLAP_FUSED) {
         // interior on the caller's stream; boundary on the handle's boundary stream as soon as the
         // halo lands, so it fills the SMs the interior kernel's tail leaves idle; then the caller's
         // stream joins (the two kernels write disjoint sites of out)
@@ -1458,6 +1562,7 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
     if (h->ev_batch) cudaEventDestroy(h->ev_batch);
     if (h->sched) cudaFree(h->sched);
     if (h->halo_flag) cudaFree(h->halo_flag);
+    if (h->fused_buf) cudaFree(h->fused_buf);
     for (void* q : h->ipc_opened) cudaIpcCloseMemHandle(q);
     if (h->flags) cudaFree(h->flags);
     for (void* v : h->cg_vec)

@@ -62,6 +62,11 @@ struct dslash_s {
     // neighbour that fills my ghost[d][side]), [8..15] free_from[d][side] (written by the neighbour
     // whose ghost my bottom (side 0) / top (side 1) face fills, once it consumed it).
     int transport = DSLASH_TRANSPORT_NCCL;
+    // one-shot fused kernel (DSLASH_OVERLAP_FUSED): [0], [1] deferred-block counters (alternate per
+    // apply), then the deferred block list; capacity in entries
+    unsigned int* fused_buf = nullptr;
+    int64_t fused_cap = 0;
+    int fused_parity = 0, fused_defer_all = 0;
     int stage = 0;                      // DSLASH_OPT_STAGE: neighbour-staged kernel (x/y rows in smem by TMA)
     int self_nccl = 0;                  // DSLASH_OPT_SELF_NCCL: self-neighbour faces via NCCL
     unsigned int* flags = nullptr;

@@ -58,6 +58,16 @@ StencilFn pick_stage(bool ghost, int lanes, int nrhs) {
     return ghost ? pick_stage_n<LR, VR, 2, true, RECON>(nrhs) : pick_stage_n<LR, VR, 2, false, RECON>(nrhs);
 }
 
+// the one-shot fused kernel (DSLASH_OVERLAP_FUSED): main launch or clean-up, lanes 1/2/4
+template <typename LR, typename VR, int RECON>
+FusedFn pick_fused(bool cleanup, int lanes) {
+    switch (lanes) {
+        case 1: return cleanup ? dslash_fused_cleanup<LR, VR, 1, RECON> : dslash_fused_kernel<LR, VR, 1, RECON>;
+        case 2: return cleanup ? dslash_fused_cleanup<LR, VR, 2, RECON> : dslash_fused_kernel<LR, VR, 2, RECON>;
+        default: return cleanup ? dslash_fused_cleanup<LR, VR, 4, RECON> : dslash_fused_kernel<LR, VR, 4, RECON>;
+    }
+}
+
 template <typename LR, typename VR, int LANES, int RECON>
 PersistFn pick_persist_l(int mode) {
     switch (mode) {
@@ -85,4 +95,5 @@ PersistFn pick_persist(int mode, int lanes) {
     }                                                                          \
     PersistFn PNAME(int mode, int lanes) { return pick_persist<LR, VR, RECON>(mode, lanes); } \
     StencilFn NAME##_stage(bool ghost, int lanes, int nrhs) { return pick_stage<LR, VR, RECON>(ghost, lanes, nrhs); } \
+    FusedFn NAME##_fused(bool cleanup, int lanes) { return pick_fused<LR, VR, RECON>(cleanup, lanes); } \
     }

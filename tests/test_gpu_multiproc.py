@@ -146,3 +146,13 @@ def test_multirank_p2p_overlap_dirs(gdims, grid):
         fat, lng = fieldgen.workload_links(gdims)
         o = oracle.full_to_cb(oracle.dslash(fat, lng, fieldgen.vector(gdims, SEED), 1), 1)
         assert oracle.normwise_error(got[0], o) <= (1e-12 if tol == 1e-14 else 1e-5)
+
+
+@pytest.mark.parametrize("gdims,grid", [((8, 8, 8, 16), (1, 1, 1, 2)), ((8, 8, 8, 8), (1, 1, 2, 2)),
+                                        ((8, 8, 8, 24), (1, 1, 1, 3))])
+def test_multirank_p2p_overlap_fused(gdims, grid):
+    """The one-shot fused overlap across real ranks (neighbours raise the ready flags the boundary
+    blocks look at): bitwise equal to the 1-rank apply."""
+    world = grid[2] * grid[3]
+    got = _run(world, gdims, grid, {"overlap": "fused"}, 0)
+    assert np.array_equal(got, _single(gdims, {}, 0))

@@ -6,7 +6,7 @@ torch.cuda.set_device(0)
 dims = tuple(int(x) for x in sys.argv[1].split(','))
 mask = int(sys.argv[2])
 fat, lng = fieldgen.workload_links(dims)
-for mode in ("none", "sites", "dirs"):
+for mode in ("none", "sites", "dirs", "fused"):
     for transport in ("nccl", "p2p"):
         with Dslash(dims, parity_mask=0, force_halo=mask, overlap=mode, timing=True, transport=transport) as D:
             D.load_links(fat, lng)
