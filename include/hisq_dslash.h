@@ -313,6 +313,20 @@ DSLASH_API dslash_status dslash_normal_apply(dslash_t h, void* out, const void* 
 DSLASH_API dslash_status dslash_cg(dslash_t h, void* x, const void* b, int32_t parity, double mass, double rel_tol,
                                    int32_t max_iter, int32_t* iters, double* rel_resid, dslash_stream_t stream);
 
+/* Mixed-precision CG by defect correction (QUDA's "mixed precision" solvers):
+ * x = 0, r = b; repeat { solve A_p e = r in fp32 (F32 kernels on fp32 links rounded once from
+ * the handle's fp64 links, fp32 vectors, fp64 dot products) by CG until |r_e| <= inner_tol |r|;
+ * x += e in fp64; r = b - A_p x in fp64 } until |r| <= rel_tol |b| or max_iter inner iterations
+ * in total.  The answer is accurate to rel_tol in fp64 (the TRUE residual is what stops it).
+ * Needs a DSLASH_F64 handle with parity_mask DSLASH_BOTH and a site / dir2 / dir4 kernel; the
+ * fp32 links (half the fp64 link memory) are built on the first call after load_links.
+ * 0 < inner_tol < 1.  iters: inner iterations in total; outer_iters: corrections; rel_resid:
+ * the final true relative residual (each may be NULL).  Synchronous; DSLASH_ERR_NOT_CONVERGED
+ * as dslash_cg. */
+DSLASH_API dslash_status dslash_cg_mixed(dslash_t h, void* x, const void* b, int32_t parity, double mass,
+                                         double rel_tol, double inner_tol, int32_t max_iter, int32_t* iters,
+                                         int32_t* outer_iters, double* rel_resid, dslash_stream_t stream);
+
 /* Halo exchange only: start sending the depth-3 faces of `in` (source parity
  * src_parity) after the work already queued on `stream`; dslash_halo_wait makes
  * `stream` wait for the ghost zones.  No-op when no direction has a halo.  Exposed

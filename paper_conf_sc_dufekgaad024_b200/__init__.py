@@ -233,6 +233,16 @@ class Dslash:
                                      int(max_iter), _stream_handle(stream))
         return st == _abi.DSLASH_OK, it, res
 
+    def cg_mixed(self, x, b, parity, mass, rel_tol=1e-10, inner_tol=1e-4, max_iter=5000, stream=None):
+        """Mixed-precision CG (fp32 inner solves, fp64 defect correction) for the same system as
+        cg(); returns (converged, inner iterations, outer corrections, true rel. residual)."""
+        self._check_vec(x)
+        self._check_vec(b)
+        st, it, outer, res = _abi.dslash_cg_mixed(self.h, x.data_ptr(), b.data_ptr(), int(parity), float(mass),
+                                                  float(rel_tol), float(inner_tol), int(max_iter),
+                                                  _stream_handle(stream))
+        return st == _abi.DSLASH_OK, it, outer, res
+
     def __call__(self, inp, parity, stream=None):
         return self.apply(self.empty_vector(), inp, parity, stream)
 

@@ -99,6 +99,9 @@ _SIGS = {
     "dslash_normal_apply": ([_h, _vp, _vp, ctypes.c_int32, ctypes.c_double, _vp], ctypes.c_int),
     "dslash_cg": ([_h, _vp, _vp, ctypes.c_int32, ctypes.c_double, ctypes.c_double, ctypes.c_int32,
                    ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_double), _vp], ctypes.c_int),
+    "dslash_cg_mixed": ([_h, _vp, _vp, ctypes.c_int32, ctypes.c_double, ctypes.c_double, ctypes.c_double,
+                         ctypes.c_int32, ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_int32),
+                         ctypes.POINTER(ctypes.c_double), _vp], ctypes.c_int),
     "dslash_halo_start": ([_h, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_halo_wait": ([_h, _vp], ctypes.c_int),
     "dslash_sync": ([_h], ctypes.c_int),
@@ -223,6 +226,17 @@ def dslash_cg(h, x_ptr, b_ptr, parity, mass, rel_tol, max_iter, stream=0):
     if st not in (DSLASH_OK, DSLASH_ERR_NOT_CONVERGED):
         check(st, h)
     return st, it.value, res.value
+
+
+def dslash_cg_mixed(h, x_ptr, b_ptr, parity, mass, rel_tol, inner_tol, max_iter, stream=0):
+    """Returns (status, inner iterations, outer corrections, true relative residual)."""
+    it, outer = ctypes.c_int32(), ctypes.c_int32()
+    res = ctypes.c_double()
+    st = lib.dslash_cg_mixed(h, x_ptr, b_ptr, parity, mass, rel_tol, inner_tol, max_iter, ctypes.byref(it),
+                             ctypes.byref(outer), ctypes.byref(res), stream)
+    if st not in (DSLASH_OK, DSLASH_ERR_NOT_CONVERGED):
+        check(st, h)
+    return st, it.value, outer.value, res.value
 
 
 def dslash_halo_start(h, in_ptr, src_parity, stream=0):

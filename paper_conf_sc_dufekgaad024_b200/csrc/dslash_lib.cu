@@ -559,6 +559,11 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
     CUL(cudaStreamSynchronize(s));
     cleanup();
 #undef CUL
+    for (void*& l32 : h->links32)  // the mixed-precision solver's fp32 copies are stale now
+        if (l32) {
+            cudaFree(l32);
+            l32 = nullptr;
+        }
     h->loaded = true;
     return DSLASH_OK;
 }
@@ -566,6 +571,29 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
 extern "C" dslash_status dslash_load_links(dslash_t h, const void* fat, const void* lng, int32_t on_device,
                                            dslash_stream_t stream) {
     return load_links_impl(h, fat, lng, nullptr, nullptr, on_device, stream);
+}
+
+// the mixed-precision solver's fp32 links of `parity` (solver.cu need_sloppy): the fp64 internal
+// links rounded into the fp32 paired layout of the same lane mapping
+dslash_status hisq_convert_links_sloppy(dslash_t h, int parity) {
+    const dslash_plan_t& p = h->plan;
+    LinkConvParams S{};
+    for (int d = 0; d < 4; ++d) S.L[d] = p.local_dims[d];
+    S.lxh = p.local_dims[0] / 2;
+    S.vh = p.vh_local;
+    S.lanes = lanes_of(h->kernel);
+    S.recon = h->recon;
+    S.paired = 0;
+    S.parity = parity;
+    S.links = h->links[parity];
+    LinkConvParams D = S;
+    D.paired = 1;
+    D.links = h->links32[parity];
+    const int64_t n = p.vh_local * 16;
+    convert_internal_kernel<<<(unsigned)((n + 255) / 256), 256>>>(S, D);
+    CU(h, cudaGetLastError());
+    CU(h, cudaDeviceSynchronize());
+    return DSLASH_OK;
 }
 
 extern "C" dslash_status dslash_get_links(dslash_t h, int32_t parity, void* out_host) {
@@ -1565,6 +1593,10 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
     if (h->fused_buf) cudaFree(h->fused_buf);
     for (void* q : h->ipc_opened) cudaIpcCloseMemHandle(q);
     if (h->flags) cudaFree(h->flags);
+    for (void* v : h->cg_vec32)
+        if (v) cudaFree(v);
+    for (void* v : h->links32)
+        if (v) cudaFree(v);
     for (void* v : h->cg_vec)
         if (v) cudaFree(v);
     if (h->cg_partial) cudaFree(h->cg_partial);

@@ -45,6 +45,9 @@ struct dslash_s {
     // conjugate-gradient scratch (solver.cu): r, p, q on the target parity, t on the other one,
     // block partial sums and the reduced scalars
     void* cg_vec[4] = {};
+    // mixed-precision solver (dslash_cg_mixed): fp32 e, r, p, q, t and the fp32 links per parity
+    void* cg_vec32[5] = {};
+    void* links32[2] = {};
     double* cg_partial = nullptr;
     double* cg_scalar = nullptr;
     // tile scheduler of the TMA kernel: ticket counters ([0] interior, [0/1] boundary launches,
@@ -98,6 +101,9 @@ dslash_status hisq_fail(dslash_t h, dslash_status st, const char* fmt, ...);
             return hisq_fail((h), DSLASH_ERR_NCCL, "%s:%d %s: %s", __FILE__, __LINE__, #call,         \
                              ncclGetErrorString(r_));                                                 \
     } while (0)
+
+// round the fp64 internal links of `parity` into h->links32[parity] (fp32 paired layout)
+dslash_status hisq_convert_links_sloppy(dslash_t h, int parity);
 
 // out = D in on target parity `parity` for nrhs back-to-back vectors (dslash_lib.cu)
 dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s);

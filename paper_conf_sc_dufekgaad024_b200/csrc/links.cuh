@@ -108,6 +108,20 @@ __global__ void convert_links_kernel(const LinkConvParams P) {
         }
 }
 
+// fp64 internal layout S -> fp32 layout D (the mixed-precision solver's sloppy links, rounded
+// once): same (mu, l, e) entries, D usually the paired fp32 layout of the same lane mapping.
+__global__ void convert_internal_kernel(const LinkConvParams S, const LinkConvParams D) {
+    const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (gid >= S.vh * 16) return;
+    const int64_t cb = gid >> 4;
+    const int mu = (int)(gid >> 2) & 3;
+    const int l = (int)gid & 3;
+    const int stored = (S.recon == 12 && l >= 2) ? 6 : 9;
+    for (int e = 0; e < stored; ++e)
+        static_cast<float2*>(D.links)[conv_index(D, mu, l, e, cb)] =
+            to_cplx<float2>(static_cast<const double2*>(S.links)[conv_index(S, mu, l, e, cb)]);
+}
+
 // Export (dslash_get_links): internal layout -> out[cb][mu][l][e] (double2), l = Ff, Fb, Nf, Nb.
 // With recon-12 the long matrices' row 2 is not stored: exported as zeros.
 template <typename LR>

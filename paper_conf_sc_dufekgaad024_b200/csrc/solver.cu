@@ -30,29 +30,35 @@ __device__ double block_sum(double v) {
     return s;
 }
 
+// Vector kernels, templated on the complex type (double2: the fp64 solver; float2: the inner
+// solver of dslash_cg_mixed).  Dot products accumulate in fp64 whatever the vector type.
+
 // q = m2 p - q ; partial[block] = sum Re(conj(p) q)
-__global__ void __launch_bounds__(kRedThreads) k_normal_finish(const double2* __restrict__ p, double2* __restrict__ q,
+template <typename V2>
+__global__ void __launch_bounds__(kRedThreads) k_normal_finish(const V2* __restrict__ p, V2* __restrict__ q,
                                                                double m2, int64_t n, double* __restrict__ partial) {
+    using R = decltype(V2{}.x);
     double acc = 0.0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const double2 a = p[i];
-        double2 b = q[i];
-        b.x = m2 * a.x - b.x;
-        b.y = m2 * a.y - b.y;
+        const V2 a = p[i];
+        V2 b = q[i];
+        b.x = (R)m2 * a.x - b.x;
+        b.y = (R)m2 * a.y - b.y;
         q[i] = b;
-        acc += a.x * b.x + a.y * b.y;
+        acc += (double)a.x * b.x + (double)a.y * b.y;
     }
     const double s = block_sum(acc);
     if (partial && threadIdx.x == 0) partial[blockIdx.x] = s;
 }
 
 // partial[block] = sum |v|^2
-__global__ void __launch_bounds__(kRedThreads) k_norm2(const double2* __restrict__ v, int64_t n,
+template <typename V2>
+__global__ void __launch_bounds__(kRedThreads) k_norm2(const V2* __restrict__ v, int64_t n,
                                                        double* __restrict__ partial) {
     double acc = 0.0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const double2 a = v[i];
-        acc += a.x * a.x + a.y * a.y;
+        const V2 a = v[i];
+        acc += (double)a.x * a.x + (double)a.y * a.y;
     }
     const double s = block_sum(acc);
     if (threadIdx.x == 0) partial[blockIdx.x] = s;
@@ -60,37 +66,55 @@ __global__ void __launch_bounds__(kRedThreads) k_norm2(const double2* __restrict
 
 // x += alpha p ; r -= alpha q ; partial[block] = sum |r|^2, alpha = rr / pq read on the device
 // (0 when pq == 0: an exactly converged iterate stays put)
-__global__ void __launch_bounds__(kRedThreads) k_cg_update(double2* __restrict__ x, double2* __restrict__ r,
-                                                           const double2* __restrict__ p, const double2* __restrict__ q,
+template <typename V2>
+__global__ void __launch_bounds__(kRedThreads) k_cg_update(V2* __restrict__ x, V2* __restrict__ r,
+                                                           const V2* __restrict__ p, const V2* __restrict__ q,
                                                            const double* __restrict__ rr, const double* __restrict__ pq,
                                                            int64_t n, double* __restrict__ partial) {
-    const double alpha = (*pq != 0.0) ? *rr / *pq : 0.0;
+    using R = decltype(V2{}.x);
+    const R alpha = (R)((*pq != 0.0) ? *rr / *pq : 0.0);
     double acc = 0.0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        double2 xi = x[i], ri = r[i];
-        const double2 pi = p[i], qi = q[i];
+        V2 xi = x[i], ri = r[i];
+        const V2 pi = p[i], qi = q[i];
         xi.x = fma(alpha, pi.x, xi.x);
         xi.y = fma(alpha, pi.y, xi.y);
         ri.x = fma(-alpha, qi.x, ri.x);
         ri.y = fma(-alpha, qi.y, ri.y);
         x[i] = xi;
         r[i] = ri;
-        acc += ri.x * ri.x + ri.y * ri.y;
+        acc += (double)ri.x * ri.x + (double)ri.y * ri.y;
     }
     const double s = block_sum(acc);
     if (threadIdx.x == 0) partial[blockIdx.x] = s;
 }
 
 // p = r + beta p, beta = rr_new / rr read on the device (0 when rr == 0)
-__global__ void k_cg_direction(double2* __restrict__ p, const double2* __restrict__ r, const double* __restrict__ rr_new,
+template <typename V2>
+__global__ void k_cg_direction(V2* __restrict__ p, const V2* __restrict__ r, const double* __restrict__ rr_new,
                                const double* __restrict__ rr, int64_t n) {
-    const double beta = (*rr != 0.0) ? *rr_new / *rr : 0.0;
+    using R = decltype(V2{}.x);
+    const R beta = (R)((*rr != 0.0) ? *rr_new / *rr : 0.0);
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const double2 ri = r[i];
-        double2 pi = p[i];
+        const V2 ri = r[i];
+        V2 pi = p[i];
         pi.x = fma(beta, pi.x, ri.x);
         pi.y = fma(beta, pi.y, ri.y);
         p[i] = pi;
+    }
+}
+
+// dslash_cg_mixed: r32 = (float) r ; x += (double) e32
+__global__ void k_round_to_f32(float2* __restrict__ o, const double2* __restrict__ v, int64_t n) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        o[i] = make_float2((float)v[i].x, (float)v[i].y);
+}
+__global__ void k_add_f32(double2* __restrict__ x, const float2* __restrict__ e, int64_t n) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        double2 xi = x[i];
+        xi.x += (double)e[i].x;
+        xi.y += (double)e[i].y;
+        x[i] = xi;
     }
 }
 
@@ -163,8 +187,9 @@ static dslash_status check_solver_args(dslash_t h, const void* a, const void* b,
 }
 
 // q = A p, and (if partial) the block partials of Re<p, q>
-static dslash_status normal_apply(dslash_t h, double2* q, const double2* p, int32_t parity, double m2,
-                                  double2* tmp, cudaStream_t s, bool dot) {
+template <typename V2>
+static dslash_status normal_apply(dslash_t h, V2* q, const V2* p, int32_t parity, double m2, V2* tmp, cudaStream_t s,
+                                  bool dot) {
     dslash_status st = hisq_apply(h, tmp, p, 1 - parity, 1, s);  // t = D_{1-p,p} p
     if (st != DSLASH_OK) return st;
     if ((st = hisq_apply(h, q, tmp, parity, 1, s)) != DSLASH_OK) return st;  // q = D_{p,1-p} t
@@ -181,6 +206,85 @@ extern "C" dslash_status dslash_normal_apply(dslash_t h, void* out, const void* 
     if ((st = need_scratch(h)) != DSLASH_OK) return st;
     return normal_apply(h, (double2*)out, (const double2*)in, parity, mass * mass, (double2*)h->cg_vec[3],
                         (cudaStream_t)stream, false);
+}
+
+// CG iterations on A x = b from x = 0, r = p = b (the caller set them up): standard
+// Hestenes-Stiefel recurrences, run until <r, r> <= stop or max_iter.  Device scalars: sc[0], sc[1] =
+// <r,r> of alternate iterations (ping-pong, so no kernel overwrites a value another block may
+// still read), sc[2] = <p, A p>; sc[0] must hold <b, b> on entry.  The host learns <r,r> through
+// pinned memory one iteration late, so the GPU never waits for the host; the solve can run one
+// iteration past convergence, which only refines x.  V2 = double2 (fp64) or float2 (the inner
+// solve of dslash_cg_mixed, on the fp32 links).
+template <typename V2>
+static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int32_t parity, double m2, double stop,
+                             int32_t max_iter, cudaStream_t s, int32_t* iters, double* rr_last, bool* converged) {
+    const int64_t n = 3 * h->plan.vh_local;
+    double* sc = h->cg_scalar;
+    double* host_rr = nullptr;
+    cudaEvent_t ev[2] = {nullptr, nullptr};
+    dslash_status st = DSLASH_OK;
+    auto release = [&]() {
+        for (cudaEvent_t e : ev)
+            if (e) cudaEventDestroy(e);
+        if (host_rr) cudaFreeHost(host_rr);
+    };
+#define CUR(call)                                                                                    \
+    do {                                                                                             \
+        cudaError_t e_ = (call);                                                                     \
+        if (e_ != cudaSuccess) {                                                                     \
+            release();                                                                               \
+            return hisq_fail(h, DSLASH_ERR_CUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call,          \
+                             cudaGetErrorString(e_));                                                \
+        }                                                                                            \
+    } while (0)
+    CUR(cudaMallocHost(&host_rr, 2 * sizeof(double)));
+    CUR(cudaEventCreateWithFlags(&ev[0], cudaEventDisableTiming));
+    CUR(cudaEventCreateWithFlags(&ev[1], cudaEventDisableTiming));
+    *converged = false;
+    int k = 0;
+    for (k = 1; k <= max_iter; ++k) {
+        double* rr_cur = &sc[(k - 1) & 1];
+        double* rr_new = &sc[k & 1];
+        if ((st = normal_apply(h, q, p, parity, m2, t, s, true)) != DSLASH_OK) break;  // q = A p
+        if ((st = reduce_to_slot(h, s, &sc[2])) != DSLASH_OK) break;                 // <p, q>
+        k_cg_update<<<kRedBlocks, kRedThreads, 0, s>>>(x, r, p, q, rr_cur, &sc[2], n, h->cg_partial);
+        CUR(cudaGetLastError());
+        if ((st = reduce_to_slot(h, s, rr_new)) != DSLASH_OK) break;                  // <r, r>
+        k_cg_direction<<<kRedBlocks, kRedThreads, 0, s>>>(p, r, rr_new, rr_cur, n);
+        CUR(cudaGetLastError());
+        CUR(cudaMemcpyAsync(&host_rr[k & 1], rr_new, sizeof(double), cudaMemcpyDeviceToHost, s));
+        CUR(cudaEventRecord(ev[k & 1], s));
+        // check iteration k-1 (already complete or nearly) while iteration k runs
+        if (k >= 2) {
+            CUR(cudaEventSynchronize(ev[(k - 1) & 1]));
+            if (host_rr[(k - 1) & 1] <= stop) {
+                *converged = true;
+                break;
+            }
+        }
+    }
+    if (st == DSLASH_OK) {
+        if (k > max_iter) k = max_iter;
+        CUR(cudaEventSynchronize(ev[k & 1]));
+        *rr_last = host_rr[k & 1];
+        if (*rr_last <= stop) *converged = true;
+    }
+    *iters = k;
+    release();
+#undef CUR
+    return st;
+}
+
+// |b - A x|^2 in fp64 (r receives the residual)
+static dslash_status true_residual(dslash_t h, double2* r, const double2* x, const double2* b, int32_t parity,
+                                   double m2, cudaStream_t s, double* rt) {
+    const int64_t n = 3 * h->plan.vh_local;
+    dslash_status st = normal_apply(h, r, x, parity, m2, (double2*)h->cg_vec[3], s, false);
+    if (st != DSLASH_OK) return st;
+    k_sub_from<<<kRedBlocks, kRedThreads, 0, s>>>(r, b, n);
+    k_norm2<<<kRedBlocks, kRedThreads, 0, s>>>(r, n, h->cg_partial);
+    CU(h, cudaGetLastError());
+    return reduce_to_host(h, s, rt);
 }
 
 extern "C" dslash_status dslash_cg(dslash_t h, void* x_out, const void* b_in, int32_t parity, double mass,
@@ -205,83 +309,133 @@ extern "C" dslash_status dslash_cg(dslash_t h, void* x_out, const void* b_in, in
     CU(h, cudaMemsetAsync(x, 0, bytes, s));
     CU(h, cudaMemcpyAsync(r, b, bytes, cudaMemcpyDeviceToDevice, s));
     CU(h, cudaMemcpyAsync(p, b, bytes, cudaMemcpyDeviceToDevice, s));
-    // Device scalars: sc[0], sc[1] = <r,r> of alternate iterations (ping-pong, so no kernel
-    // overwrites a value another block may still read), sc[2] = <p, A p>, sc[3] = scratch.
-    // The host learns <r,r> through pinned memory one iteration late, so the GPU never waits
-    // for the host; the solve can run one iteration past convergence, which only refines x.
-    double* sc = h->cg_scalar;
-    double bb = 0.0, rr_last = 0.0;
+    double bb = 0.0;
     k_norm2<<<kRedBlocks, kRedThreads, 0, s>>>(b, n, h->cg_partial);
     CU(h, cudaGetLastError());
     if ((st = reduce_to_host(h, s, &bb)) != DSLASH_OK) return st;
-    int k = 0;
+    int32_t k = 0;
     bool converged = !(bb > 0.0);
-    if (bb > 0.0) {
-        CU(h, cudaMemcpyAsync(&sc[0], &bb, sizeof(double), cudaMemcpyHostToDevice, s));
-        const double stop = rel_tol * rel_tol * bb;
-        double* host_rr = nullptr;
-        cudaEvent_t ev[2] = {nullptr, nullptr};
-        CU(h, cudaMallocHost(&host_rr, 2 * sizeof(double)));
-        auto release = [&]() {
-            for (cudaEvent_t e : ev)
-                if (e) cudaEventDestroy(e);
-            cudaFreeHost(host_rr);
-        };
-#define CUR(call)                                                                                    \
-    do {                                                                                             \
-        cudaError_t e_ = (call);                                                                     \
-        if (e_ != cudaSuccess) {                                                                     \
-            release();                                                                               \
-            return hisq_fail(h, DSLASH_ERR_CUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call,          \
-                             cudaGetErrorString(e_));                                                \
-        }                                                                                            \
-    } while (0)
-        CUR(cudaEventCreateWithFlags(&ev[0], cudaEventDisableTiming));
-        CUR(cudaEventCreateWithFlags(&ev[1], cudaEventDisableTiming));
-        for (k = 1; k <= max_iter; ++k) {
-            double* rr_cur = &sc[(k - 1) & 1];
-            double* rr_new = &sc[k & 1];
-            if ((st = normal_apply(h, q, p, parity, m2, t, s, true)) != DSLASH_OK) break;  // q = A p
-            if ((st = reduce_to_slot(h, s, &sc[2])) != DSLASH_OK) break;                 // <p, q>
-            k_cg_update<<<kRedBlocks, kRedThreads, 0, s>>>(x, r, p, q, rr_cur, &sc[2], n, h->cg_partial);
-            CUR(cudaGetLastError());
-            if ((st = reduce_to_slot(h, s, rr_new)) != DSLASH_OK) break;                  // <r, r>
-            k_cg_direction<<<kRedBlocks, kRedThreads, 0, s>>>(p, r, rr_new, rr_cur, n);
-            CUR(cudaGetLastError());
-            CUR(cudaMemcpyAsync(&host_rr[k & 1], rr_new, sizeof(double), cudaMemcpyDeviceToHost, s));
-            CUR(cudaEventRecord(ev[k & 1], s));
-            // check iteration k-1 (already complete or nearly) while iteration k runs
-            if (k >= 2) {
-                CUR(cudaEventSynchronize(ev[(k - 1) & 1]));
-                if (host_rr[(k - 1) & 1] <= stop) {
-                    converged = true;
-                    break;
-                }
-            }
-        }
-        if (st == DSLASH_OK) {
-            if (k > max_iter) k = max_iter;
-            CUR(cudaEventSynchronize(ev[k & 1]));
-            rr_last = host_rr[k & 1];
-            if (rr_last <= stop) converged = true;
-        }
-        release();
-#undef CUR
-        if (st != DSLASH_OK) return st;
-    }
-    // true residual |b - A x| / |b|
     double res = 0.0;
     if (bb > 0.0) {
-        if ((st = normal_apply(h, r, x, parity, m2, t, s, false)) != DSLASH_OK) return st;
-        k_sub_from<<<kRedBlocks, kRedThreads, 0, s>>>(r, b, n);
-        k_norm2<<<kRedBlocks, kRedThreads, 0, s>>>(r, n, h->cg_partial);
-        CU(h, cudaGetLastError());
-        double rt = 0.0;
-        if ((st = reduce_to_host(h, s, &rt)) != DSLASH_OK) return st;
+        CU(h, cudaMemcpyAsync(&h->cg_scalar[0], &bb, sizeof(double), cudaMemcpyHostToDevice, s));
+        double rr_last = 0.0;
+        st = cg_core(h, x, r, p, q, t, parity, m2, rel_tol * rel_tol * bb, max_iter, s, &k, &rr_last, &converged);
+        if (st != DSLASH_OK) return st;
+        double rt = 0.0;  // true residual |b - A x| / |b|
+        if ((st = true_residual(h, r, x, b, parity, m2, s, &rt)) != DSLASH_OK) return st;
         res = std::sqrt(rt / bb);
     }
     if (iters) *iters = k;
     if (rel_resid) *rel_resid = res;
     // not converged: reported, but not a sticky handle error
+    return converged ? DSLASH_OK : DSLASH_ERR_NOT_CONVERGED;
+}
+
+// ---------------------------------------------------------------------------- mixed precision
+// The fp32 ("sloppy") links of both parities, converted once from the handle's fp64 internal
+// links into the fp32 paired layout the F32 kernels read (links.cuh convert_internal_kernel).
+static dslash_status need_sloppy(dslash_t h) {
+    const int64_t n = 3 * h->plan.vh_local;
+    for (void*& v : h->cg_vec32)
+        if (!v) CU(h, cudaMalloc(&v, n * sizeof(float2)));
+    if (h->links32[0]) return DSLASH_OK;
+    for (int par = 0; par < 2; ++par) {
+        CU(h, cudaMalloc(&h->links32[par], h->link_bytes / 2));
+        dslash_status st = hisq_convert_links_sloppy(h, par);
+        if (st != DSLASH_OK) return st;
+    }
+    return DSLASH_OK;
+}
+
+// Run the handle as an fp32 one (F32 kernels on the sloppy links) for the inner solve; every
+// rank does the same, so halo messages keep matching sizes.
+struct SloppyScope {
+    dslash_t h;
+    int precision;
+    void* links[2];
+    explicit SloppyScope(dslash_t hh) : h(hh), precision(hh->precision) {
+        links[0] = h->links[0];
+        links[1] = h->links[1];
+        h->precision = DSLASH_F32;
+        h->links[0] = h->links32[0];
+        h->links[1] = h->links32[1];
+    }
+    ~SloppyScope() {
+        h->precision = precision;
+        h->links[0] = links[0];
+        h->links[1] = links[1];
+    }
+};
+
+extern "C" dslash_status dslash_cg_mixed(dslash_t h, void* x_out, const void* b_in, int32_t parity, double mass,
+                                         double rel_tol, double inner_tol, int32_t max_iter, int32_t* iters,
+                                         int32_t* outer_iters, double* rel_resid, dslash_stream_t stream) {
+    dslash_status st = check_solver_args(h, x_out, b_in, parity);
+    if (st != DSLASH_OK) return st;
+    if (h->precision != DSLASH_F64)
+        return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the mixed-precision solver needs an fp64 handle (DSLASH_F64)");
+    if (h->kernel == DSLASH_KERNEL_BULK)
+        return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the mixed-precision solver needs a register-staged kernel");
+    if (!(rel_tol > 0.0) || max_iter < 1 || !(inner_tol > 0.0) || !(inner_tol < 1.0))
+        return hisq_fail(h, DSLASH_ERR_ARG, "need rel_tol > 0, 0 < inner_tol < 1, max_iter >= 1");
+    if (!(mass != 0.0)) return hisq_fail(h, DSLASH_ERR_ARG, "mass must be nonzero (A is then positive definite)");
+    if ((st = need_scratch(h)) != DSLASH_OK) return st;
+    if ((st = need_sloppy(h)) != DSLASH_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t n = 3 * h->plan.vh_local;
+    const double m2 = mass * mass;
+    double2* x = (double2*)x_out;
+    const double2* b = (const double2*)b_in;
+    double2* r = (double2*)h->cg_vec[0];
+    float2* e = (float2*)h->cg_vec32[0];
+    float2* r32 = (float2*)h->cg_vec32[1];
+    float2* p32 = (float2*)h->cg_vec32[2];
+    float2* q32 = (float2*)h->cg_vec32[3];
+    float2* t32 = (float2*)h->cg_vec32[4];
+    CU(h, cudaMemsetAsync(x, 0, n * sizeof(double2), s));
+    CU(h, cudaMemcpyAsync(r, b, n * sizeof(double2), cudaMemcpyDeviceToDevice, s));
+    double bb = 0.0;
+    k_norm2<<<kRedBlocks, kRedThreads, 0, s>>>(b, n, h->cg_partial);
+    CU(h, cudaGetLastError());
+    if ((st = reduce_to_host(h, s, &bb)) != DSLASH_OK) return st;
+    // Defect correction (iterative refinement): r = b - A x in fp64; solve A e = r in fp32 CG to
+    // relative residual inner_tol; x += e in fp64; repeat until |r| <= rel_tol |b|.
+    double rr = bb;
+    int32_t total = 0, outer = 0;
+    bool converged = !(bb > 0.0);
+    while (!converged && total < max_iter) {
+        if (rr <= rel_tol * rel_tol * bb) {
+            converged = true;
+            break;
+        }
+        k_round_to_f32<<<kRedBlocks, kRedThreads, 0, s>>>(r32, r, n);
+        CU(h, cudaGetLastError());
+        CU(h, cudaMemcpyAsync(p32, r32, n * sizeof(float2), cudaMemcpyDeviceToDevice, s));
+        CU(h, cudaMemsetAsync(e, 0, n * sizeof(float2), s));
+        double rr32 = 0.0;
+        k_norm2<<<kRedBlocks, kRedThreads, 0, s>>>(r32, n, h->cg_partial);
+        CU(h, cudaGetLastError());
+        if ((st = reduce_to_slot(h, s, &h->cg_scalar[0])) != DSLASH_OK) return st;  // sc[0] = <r32, r32>
+        CU(h, cudaMemcpyAsync(&rr32, &h->cg_scalar[0], sizeof(double), cudaMemcpyDeviceToHost, s));
+        CU(h, cudaStreamSynchronize(s));
+        int32_t k = 0;
+        double rr_inner = 0.0;
+        bool inner_conv = false;
+        {
+            SloppyScope scope(h);
+            st = cg_core(h, e, r32, p32, q32, t32, parity, m2, inner_tol * inner_tol * rr32, max_iter - total, s, &k,
+                         &rr_inner, &inner_conv);
+        }
+        if (st != DSLASH_OK) return st;
+        total += k;
+        ++outer;
+        k_add_f32<<<kRedBlocks, kRedThreads, 0, s>>>(x, e, n);
+        CU(h, cudaGetLastError());
+        if ((st = true_residual(h, r, x, b, parity, m2, s, &rr)) != DSLASH_OK) return st;
+    }
+    if (!converged && rr <= rel_tol * rel_tol * bb) converged = true;
+    if (iters) *iters = total;
+    if (outer_iters) *outer_iters = outer;
+    if (rel_resid) *rel_resid = bb > 0.0 ? std::sqrt(rr / bb) : 0.0;
     return converged ? DSLASH_OK : DSLASH_ERR_NOT_CONVERGED;
 }

@@ -126,3 +126,75 @@ def test_cg_not_converged_and_errors(torch_cuda):
         with pytest.raises(_abi.DslashError) as e:
             D.cg(D.empty_vector(), torch.from_numpy(fieldgen.vector_cb(dims, 74, 0)).cuda(), 0, 0.3)
         assert e.value.status == _abi.DSLASH_ERR_ARG
+
+
+@pytest.mark.parametrize("parity", [0, 1])
+@pytest.mark.parametrize("recon", [18, 12])
+def test_cg_mixed_vs_oracle(torch_cuda, parity, recon):
+    """Mixed-precision CG (fp32 inner solves on fp32 links, fp64 defect correction): the answer
+    solves the ORACLE's fp64 system to rel_tol (true residual), and matches the oracle CG's x."""
+    torch = torch_cuda
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 10, 12, 14)
+    fat, lng = fieldgen.workload_links(dims)
+    b = fieldgen.vector(dims, 72)
+    m, tol = 0.25, 1e-10
+    bcb = oracle.full_to_cb(b, parity)
+    with Dslash(dims, recon=recon) as D:
+        D.load_links(fat, lng)
+        x = D.empty_vector()
+        ok, it, outer, res = D.cg_mixed(x, torch.from_numpy(bcb).cuda(), parity, m, rel_tol=tol, inner_tol=1e-4)
+        xg = x.cpu().numpy()
+    assert ok and res <= tol and outer >= 2 and it > outer
+    ax = oracle.full_to_cb(ocg.normal_apply(fat, lng, oracle.cb_to_full(xg, dims, parity), parity, m), parity)
+    assert np.linalg.norm(ax - bcb) / np.linalg.norm(bcb) <= 2 * tol
+    xo, _ = ocg.cg(fat, lng, b, parity, m, rel_tol=tol)
+    assert oracle.normwise_error(xg, oracle.full_to_cb(xo, parity)) < 1e-8
+
+
+def test_cg_mixed_halo_paths_bitwise(torch_cuda):
+    """The same mixed-precision solve through the self-halo paths (device copies, NCCL to self,
+    P2P): bitwise equal, since every fp32 apply, BLAS pass and dot product is deterministic and
+    partition-independent on one rank."""
+    torch = torch_cuda
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 8, 8, 12)
+    fat, lng = fieldgen.workload_links(dims)
+    b = torch.from_numpy(fieldgen.vector_cb(dims, 74, 1)).cuda()
+    sols = []
+    for kw in ({}, {"force_halo": 0xC}, {"force_halo": 0x8, "self_nccl": True}, {"force_halo": 0xC, "transport": "p2p"}):
+        with Dslash(dims, **kw) as D:
+            D.load_links(fat, lng)
+            x = D.empty_vector()
+            ok, it, outer, res = D.cg_mixed(x, b, 1, 0.3, rel_tol=1e-11, inner_tol=1e-3)
+            assert ok and res <= 1e-11
+            sols.append((x.cpu(), it, outer))
+    for k in range(1, len(sols)):
+        assert torch.equal(sols[0][0], sols[k][0]) and sols[0][1:] == sols[k][1:], k
+
+
+def test_cg_mixed_reload_links_and_errors(torch_cuda):
+    """load_links invalidates the fp32 copies: a second solve uses the new links."""
+    torch = torch_cuda
+    from paper_conf_sc_dufekgaad024_b200 import Dslash, DslashError
+    dims = (8, 8, 8, 8)
+    fat, lng = fieldgen.workload_links(dims)
+    fat2 = fieldgen.links(dims, 91)
+    b = fieldgen.vector(dims, 75)
+    bcb = torch.from_numpy(oracle.full_to_cb(b, 0)).cuda()
+    with Dslash(dims) as D:
+        D.load_links(fat, lng)
+        x = D.empty_vector()
+        assert D.cg_mixed(x, bcb, 0, 0.4, rel_tol=1e-10)[0]
+        D.load_links(fat2, lng)
+        ok, it, outer, res = D.cg_mixed(x, bcb, 0, 0.4, rel_tol=1e-10)
+        assert ok
+        xo, _ = ocg.cg(fat2, lng, b, 0, 0.4, rel_tol=1e-10)
+        assert oracle.normwise_error(x.cpu().numpy(), oracle.full_to_cb(xo, 0)) < 1e-8
+        with pytest.raises(DslashError):
+            D.cg_mixed(x, bcb, 0, 0.4, inner_tol=1.5)
+    with Dslash(dims, precision="f32") as D:
+        D.load_links(fat, lng)
+        x = D.empty_vector()
+        with pytest.raises(DslashError):
+            D.cg_mixed(x, torch.zeros_like(x), 0, 0.4)

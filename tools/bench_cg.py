@@ -1,6 +1,8 @@
 """CG solve benchmark: (m^2 - D_eo D_oe) x = b on a 32^4 lattice, fp64.
 
 python tools/bench_cg.py [--dims 32,32,32,32] [--mass 0.05] [--tol 1e-10] [--precision f64|mixed]
+                        [--solver cg|mixed-cg --inner-tol 1e-4]
+(--solver mixed-cg: fp32 inner CG on fp32 links with fp64 defect correction, dslash_cg_mixed)
 Prints one JSON line: iterations, solve time, time per iteration, Dslash GFLOP/s inside the solve
 (2 applies of 1146 flop/site per iteration), true residual.
 """
@@ -23,6 +25,8 @@ ap.add_argument("--mass", type=float, default=0.05)
 ap.add_argument("--tol", type=float, default=1e-10)
 ap.add_argument("--precision", default="f64")
 ap.add_argument("--kernel", default="dir2")
+ap.add_argument("--solver", default="cg", choices=["cg", "mixed-cg"])
+ap.add_argument("--inner-tol", type=float, default=1e-4)
 a = ap.parse_args()
 dims = tuple(int(v) for v in a.dims.split(","))
 fat, lng = fieldgen.workload_links(dims)
@@ -30,14 +34,22 @@ D = Dslash(dims, precision=a.precision, kernel=a.kernel)
 D.load_links(fat, lng)
 b = torch.from_numpy(fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 0)).cuda()
 x = D.empty_vector()
-D.cg(x, b, 0, a.mass, rel_tol=1e-3, max_iter=20)   # warm-up
-torch.cuda.synchronize()
-t0 = time.perf_counter()
-ok, it, res = D.cg(x, b, 0, a.mass, rel_tol=a.tol, max_iter=5000)
+outer = None
+if a.solver == "cg":
+    D.cg(x, b, 0, a.mass, rel_tol=1e-3, max_iter=20)   # warm-up
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    ok, it, res = D.cg(x, b, 0, a.mass, rel_tol=a.tol, max_iter=5000)
+else:
+    D.cg_mixed(x, b, 0, a.mass, rel_tol=1e-3, inner_tol=0.5, max_iter=20)   # warm-up (builds fp32 links)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    ok, it, outer, res = D.cg_mixed(x, b, 0, a.mass, rel_tol=a.tol, inner_tol=a.inner_tol, max_iter=10000)
 torch.cuda.synchronize()
 el = time.perf_counter() - t0
 vh = D.vh
-print(json.dumps({"dims": dims, "precision": a.precision, "mass": a.mass, "tol": a.tol, "converged": ok,
+print(json.dumps({"dims": dims, "precision": a.precision, "solver": a.solver, "outer_corrections": outer,
+                  "inner_tol": a.inner_tol if a.solver != "cg" else None, "mass": a.mass, "tol": a.tol, "converged": ok,
                   "iterations": it, "solve_s": round(el, 4), "ms_per_iteration": round(1e3 * el / max(it, 1), 4),
                   "dslash_gflops_in_solver": round(2 * FLOP_PER_SITE * vh * it / el / 1e9, 1),
                   "true_rel_residual": res}))
