@@ -124,6 +124,10 @@ enum {
                                    (DSLASH_OPT_PERSISTENT) does not stage.  0 (default): off        */
     DSLASH_OPT_FUSED_DEFER = 12,/* testing aid for DSLASH_OVERLAP_FUSED: 1 = every boundary block
                                    defers to the clean-up launch; any time                         */
+    DSLASH_OPT_HALO_DRYRUN = 13,/* timing aid (NCCL / device-copy transport): halo_start keeps its
+                                   events and stream order but moves no bytes, so the ghost faces
+                                   are stale and results WRONG; prices an overlap scheme without the
+                                   exchange itself; any time                                        */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */

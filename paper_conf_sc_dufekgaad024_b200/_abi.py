@@ -24,7 +24,7 @@ PRECISIONS = {"f64": DSLASH_F64, "f32": DSLASH_F32, "mixed": DSLASH_MIXED}
 DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_DIR2, DSLASH_KERNEL_BULK = 0, 1, 2, 3
 DSLASH_OPT_KERNEL, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_OVERLAP, DSLASH_OPT_TIMING, \
     DSLASH_OPT_MIN_BLOCKS, DSLASH_OPT_LONG_RECON, DSLASH_OPT_PERSISTENT, DSLASH_OPT_TRANSPORT, \
-    DSLASH_OPT_PDL, DSLASH_OPT_SELF_NCCL, DSLASH_OPT_STAGE, DSLASH_OPT_FUSED_DEFER = range(13)
+    DSLASH_OPT_PDL, DSLASH_OPT_SELF_NCCL, DSLASH_OPT_STAGE, DSLASH_OPT_FUSED_DEFER, DSLASH_OPT_HALO_DRYRUN = range(14)
 DSLASH_TRANSPORT_NCCL, DSLASH_TRANSPORT_P2P = 0, 1
 DSLASH_OVERLAP_NONE, DSLASH_OVERLAP_SITES, DSLASH_OVERLAP_DIRS, DSLASH_OVERLAP_FUSED = 0, 1, 2, 3
 OVERLAPS = {"none": DSLASH_OVERLAP_NONE, "sites": DSLASH_OVERLAP_SITES, "dirs": DSLASH_OVERLAP_DIRS,

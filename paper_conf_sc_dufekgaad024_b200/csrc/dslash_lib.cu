@@ -302,6 +302,11 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             h->self_nccl = value != 0;
             return alloc_halo(h, 1);
         }
+        case DSLASH_OPT_HALO_DRYRUN:
+            if (value && h->transport != DSLASH_TRANSPORT_NCCL)
+                return fail(h, DSLASH_ERR_UNSUPPORTED, "HALO_DRYRUN serves the NCCL / device-copy transport");
+            h->halo_dryrun = value != 0;
+            return DSLASH_OK;
         case DSLASH_OPT_FUSED_DEFER:
             h->fused_defer_all = value != 0;
             return DSLASH_OK;
@@ -835,6 +840,11 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
     const size_t rows = (size_t)3 * nrhs;  // (rhs, colour) rows of length vh
     CU(h, cudaEventRecord(h->ev_start, s));
     CU(h, cudaStreamWaitEvent(h->comm, h->ev_start, 0));
+    if (h->halo_dryrun) {  // testing aid: the stream structure of the exchange without its bytes
+        CU(h, cudaEventRecord(h->ev_halo, h->comm));
+        h->halo_pending = true;
+        return DSLASH_OK;
+    }
     bool nccl_work = false;
     const size_t tslab = 3 * lxh * L1 * L2;  // sites in 3 t-slices of one parity
     if (p.halo[3]) {

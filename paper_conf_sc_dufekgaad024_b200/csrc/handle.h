@@ -70,6 +70,7 @@ struct dslash_s {
     unsigned int* fused_buf = nullptr;
     int64_t fused_cap = 0;
     int fused_parity = 0, fused_defer_all = 0;
+    int halo_dryrun = 0;                // DSLASH_OPT_HALO_DRYRUN (timing aid: exchange moves no bytes)
     int stage = 0;                      // DSLASH_OPT_STAGE: neighbour-staged kernel (x/y rows in smem by TMA)
     int self_nccl = 0;                  // DSLASH_OPT_SELF_NCCL: self-neighbour faces via NCCL
     unsigned int* flags = nullptr;

@@ -115,3 +115,27 @@ def test_fused_chained_cg(torch_cuda):
             assert ok
             res.append((x.cpu(), it))
     assert torch.equal(res[0][0], res[1][0]) and res[0][1] == res[1][1]
+
+
+def test_halo_dryrun_timing_aid(torch_cuda):
+    """DSLASH_OPT_HALO_DRYRUN keeps the exchange's stream structure but moves no bytes: interior
+    sites are still right (they read no ghost), and the P2P transport refuses it."""
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash, DslashError, _abi
+    dims = (8, 8, 8, 12)
+    fat, lng = fieldgen.workload_links(dims)
+    src = torch.from_numpy(fieldgen.vector_cb(dims, 60, 1)).cuda()
+    with Dslash(dims) as D:
+        D.load_links(fat, lng)
+        base = D(src, 0).cpu().numpy()
+    with Dslash(dims, force_halo=0x8) as D:
+        D.load_links(fat, lng)
+        _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_HALO_DRYRUN, 1)
+        got = D(src, 0).cpu().numpy()
+    lex = oracle.lex_sites_of_parity(dims, 0)
+    t = lex // (dims[0] * dims[1] * dims[2])
+    inside = (t >= 3) & (t < dims[3] - 3)
+    assert np.array_equal(got[:, inside], base[:, inside])
+    with Dslash(dims, force_halo=0x8, transport="p2p") as D:
+        with pytest.raises(DslashError):
+            _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_HALO_DRYRUN, 1)

@@ -6,10 +6,14 @@ torch.cuda.set_device(0)
 dims = tuple(int(x) for x in sys.argv[1].split(','))
 mask = int(sys.argv[2])
 fat, lng = fieldgen.workload_links(dims)
+from paper_conf_sc_dufekgaad024_b200 import _abi
 for mode in ("none", "sites", "dirs", "fused"):
-    for transport in ("nccl", "p2p"):
-        with Dslash(dims, parity_mask=0, force_halo=mask, overlap=mode, timing=True, transport=transport) as D:
+    for transport in ("nccl", "p2p", "dryrun"):
+        tr = "nccl" if transport == "dryrun" else transport
+        with Dslash(dims, parity_mask=0, force_halo=mask, overlap=mode, timing=True, transport=tr) as D:
             D.load_links(fat, lng)
+            if transport == "dryrun":   # same stream structure, no bytes moved (timing only)
+                _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_HALO_DRYRUN, 1)
             srcs = [torch.from_numpy(fieldgen.vector_cb(dims, 3 + r, 1)).cuda() for r in range(4)]
             outs = [D.empty_vector() for _ in range(4)]
             for i in range(20): D.apply(outs[i % 4], srcs[i % 4], 0)

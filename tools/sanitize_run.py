@@ -19,10 +19,26 @@ ref = None
 cases = [dict(kernel=k) for k in ("site", "dir2", "dir4", "bulk")]
 cases += [dict(force_halo=m, persistent=pers) for m in (0x8, 0xC) for pers in (False, True)]
 cases += [dict(force_halo=0xC, transport="p2p"), dict(recon=12), dict(precision="mixed"), dict(pdl=False)]
+# later additions: the neighbour-staged kernel (TMA bulk copies + mbarrier into shared memory), the
+# split-by-direction and one-shot fused overlaps (with and without forced deferral), NCCL to self,
+# and the mixed-precision CG (fp32 links converted from the fp64 ones)
+cases += [dict(stage=True), dict(stage=True, kernel="site", force_halo=0xC), dict(stage=True, precision="f32"),
+          dict(force_halo=0xC, overlap="dirs"), dict(force_halo=0xC, overlap="dirs", precision="f32"),
+          dict(force_halo=0xC, overlap="fused"), dict(force_halo=0x8, overlap="fused", defer=True),
+          dict(force_halo=0xC, self_nccl=True), dict(cg_mixed=True)]
 n = 0
 for kw in cases:
+    kw = dict(kw)
+    defer = kw.pop("defer", False)
+    mixed_cg = kw.pop("cg_mixed", False)
     with Dslash(dims, **kw) as D:
         D.load_links(fat, lng)
+        if defer:
+            from paper_conf_sc_dufekgaad024_b200 import _abi
+            _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_FUSED_DEFER, 1)
+        if mixed_cg:
+            x = D.empty_vector()
+            D.cg_mixed(x, src[0], 0, 0.5, rel_tol=1e-8, inner_tol=1e-2, max_iter=100)
         out = D(src[1].to(D.dtype), 0)
         o2 = D.empty_vector()
         D.apply(o2, out.to(D.dtype), 1)
@@ -36,7 +52,7 @@ for kw in cases:
         r = out.cpu().numpy().astype(np.complex128)
         if ref is None:
             ref = r
-        tol = 1e-5 if kw.get("precision") == "mixed" else 1e-12
+        tol = 1e-5 if kw.get("precision") in ("mixed", "f32") else 1e-12
         err = np.abs(r - ref).max() / np.abs(ref).max()
         assert err <= tol, (kw, err)
         assert torch.equal(mo[0], mo[1])
