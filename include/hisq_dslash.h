@@ -128,6 +128,14 @@ enum {
                                    events and stream order but moves no bytes, so the ghost faces
                                    are stale and results WRONG; prices an overlap scheme without the
                                    exchange itself; any time                                        */
+    DSLASH_OPT_PUSH = 14,       /* 1: producer push (P2P transport only; before load_links and the IPC
+                                   setup).  The ghosts get two banks (epoch e reads bank e & 1) and
+                                   dslash_apply_push / the normal operator / CG store the depth-3
+                                   faces of an apply's OUTPUT straight into the neighbours' ghosts
+                                   from the stencil kernel's epilogue (peer memory over NVLink), so
+                                   the next apply, whose source that output is, moves no bytes.
+                                   Not with the persistent or one-shot fused kernels (the split
+                                   by sites runs instead) nor the TMA kernel; 0 (default): off  */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */
@@ -297,13 +305,25 @@ DSLASH_API dslash_status dslash_apply_host_batch(dslash_t h, int32_t n, void* co
                                                  const void* const* in_host, int32_t parity,
                                                  dslash_stream_t stream);
 
+/* dslash_apply that also hands its output to the next apply (DSLASH_OPT_PUSH; the
+ * "compute step followed by an exchange" of D_{p,1-p} D_{1-p,p}).  Every target site within 3
+ * slices of a partitioned face stores its result into the neighbour's ghost face as well as
+ * into out; the neighbours' ready flags are raised behind the kernel.  The NEXT apply (or
+ * halo_start) on this handle, on every rank, must take `out` as its source: it then exchanges
+ * no bytes; any other source returns DSLASH_ERR_STATE.  Without a halo it equals dslash_apply.
+ * Errors as dslash_apply, plus DSLASH_ERR_STATE without DSLASH_OPT_PUSH and
+ * DSLASH_ERR_UNSUPPORTED for the TMA kernel. */
+DSLASH_API dslash_status dslash_apply_push(dslash_t h, void* out, const void* in, int32_t parity,
+                                           dslash_stream_t stream);
+
 /* The even-odd normal operator (the conjugate-gradient step of MILC's
  * su3_rhmd_hisq):  out = A_p in,  A_p = m^2 - D_{p,1-p} D_{1-p,p}, where D_{a,b}
  * is the Dslash from parity b to target parity a.  D is anti-Hermitian, so A_p = m^2 +
  * D_{1-p,p}^dag D_{1-p,p} is Hermitian positive definite for m != 0.  in, out: fp64 [3][Vh]
  * vectors on parity p.  Needs parity_mask DSLASH_BOTH and fp64 vectors (DSLASH_F64 or
  * DSLASH_MIXED; DSLASH_F32 returns DSLASH_ERR_UNSUPPORTED).  Two applies + one fused
- * m^2-subtraction kernel, stream-ordered. */
+ * m^2-subtraction kernel, stream-ordered.  With DSLASH_OPT_PUSH the first apply pushes its
+ * output's faces (dslash_apply_push), so the second exchanges no bytes (also inside CG). */
 DSLASH_API dslash_status dslash_normal_apply(dslash_t h, void* out, const void* in, int32_t parity, double mass,
                                              dslash_stream_t stream);
 

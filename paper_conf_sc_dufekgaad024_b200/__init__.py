@@ -55,7 +55,8 @@ class Dslash:
 
     def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="dir2", block=0,
                  force_halo=0, overlap=True, timing=False, rank=0, world_size=1, min_blocks=0, precision="f64",
-                 recon=18, persistent=False, transport="nccl", pdl=True, self_nccl=False, stage=False):
+                 recon=18, persistent=False, transport="nccl", pdl=True, self_nccl=False, stage=False,
+                 push=False):
         import torch
         self.global_dims = tuple(int(d) for d in global_dims)
         self.precision = precision
@@ -95,6 +96,8 @@ class Dslash:
             _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_PDL, int(bool(pdl)))
             if transport == "p2p" and (world_size == 1 or use_nccl):
                 _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_TRANSPORT, _abi.DSLASH_TRANSPORT_P2P)
+            if push:  # producer push: two ghost banks, allocated before they are IPC-exported
+                _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_PUSH, 1)
             if transport == "p2p":
                 if world_size > 1:      # exchange CUDA IPC handles through torch.distributed
                     import torch.distributed as dist
@@ -203,6 +206,14 @@ class Dslash:
         self._check_vec(out)
         self._check_vec(inp)
         _abi.dslash_apply(self.h, out.data_ptr(), inp.data_ptr(), int(parity), _stream_handle(stream))
+        return out
+
+    def apply_push(self, out, inp, parity, stream=None):
+        """out = D inp, and the faces of out go straight into the neighbours' ghosts (push=True):
+        the next apply on every rank must take ``out`` as its source."""
+        self._check_vec(out)
+        self._check_vec(inp)
+        _abi.dslash_apply_push(self.h, out.data_ptr(), inp.data_ptr(), int(parity), _stream_handle(stream))
         return out
 
     def apply_multi(self, out, inp, parity, stream=None):

@@ -24,7 +24,8 @@ PRECISIONS = {"f64": DSLASH_F64, "f32": DSLASH_F32, "mixed": DSLASH_MIXED}
 DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_DIR2, DSLASH_KERNEL_BULK = 0, 1, 2, 3
 DSLASH_OPT_KERNEL, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_OVERLAP, DSLASH_OPT_TIMING, \
     DSLASH_OPT_MIN_BLOCKS, DSLASH_OPT_LONG_RECON, DSLASH_OPT_PERSISTENT, DSLASH_OPT_TRANSPORT, \
-    DSLASH_OPT_PDL, DSLASH_OPT_SELF_NCCL, DSLASH_OPT_STAGE, DSLASH_OPT_FUSED_DEFER, DSLASH_OPT_HALO_DRYRUN = range(14)
+    DSLASH_OPT_PDL, DSLASH_OPT_SELF_NCCL, DSLASH_OPT_STAGE, DSLASH_OPT_FUSED_DEFER, DSLASH_OPT_HALO_DRYRUN, \
+    DSLASH_OPT_PUSH = range(15)
 DSLASH_TRANSPORT_NCCL, DSLASH_TRANSPORT_P2P = 0, 1
 DSLASH_OVERLAP_NONE, DSLASH_OVERLAP_SITES, DSLASH_OVERLAP_DIRS, DSLASH_OVERLAP_FUSED = 0, 1, 2, 3
 OVERLAPS = {"none": DSLASH_OVERLAP_NONE, "sites": DSLASH_OVERLAP_SITES, "dirs": DSLASH_OVERLAP_DIRS,
@@ -92,6 +93,7 @@ _SIGS = {
     "dslash_set_option": ([_h, ctypes.c_int32, ctypes.c_int64], ctypes.c_int),
     "dslash_load_links": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
+    "dslash_apply_push": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply_multi": ([_h, ctypes.c_int32, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply_host": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply_host_batch": ([_h, ctypes.c_int32, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.c_int32,
@@ -194,6 +196,10 @@ def dslash_load_links(h, fat_ptr, lng_ptr, on_device, stream=0):
 
 def dslash_apply(h, out_ptr, in_ptr, parity, stream=0):
     return check(lib.dslash_apply(h, out_ptr, in_ptr, parity, stream), h)
+
+
+def dslash_apply_push(h, out_ptr, in_ptr, parity, stream=0):
+    return check(lib.dslash_apply_push(h, out_ptr, in_ptr, parity, stream), h)
 
 
 def dslash_apply_multi(h, nrhs, out_ptr, in_ptr, parity, stream=0):

@@ -205,6 +205,11 @@ struct StencilParams {
     FastDiv div_xh[kMaxBoxes], div_y[kMaxBoxes], div_z[kMaxBoxes];
     int stage_ty;              // rows per tile of the neighbour-staged kernel (DSLASH_OPT_STAGE)
     int halo_pass;             // GHOST kernels: kPassAll, or one pass of the split-by-direction overlap
+    // producer push (DSLASH_OPT_PUSH; GHOST kernels only): a target site within 3 slices of the
+    // bottom (top) of a direction mu in push_mask also stores its output into push[mu][0] ([mu][1]):
+    // the minus (plus) neighbour's plus (minus) ghost face, [3][face_vh[mu]], peer memory over NVLink
+    void* push[4][2];
+    int push_mask;
 };
 
 // Passes of a GHOST kernel (StencilParams::halo_pass).  kPassAll reads local sources and ghost

@@ -185,8 +185,13 @@ static dslash_status alloc_halo(dslash_t h, int nrhs) {
     const dslash_plan_t& p = h->plan;
     const size_t es = h->precision == DSLASH_F32 ? 8 : 16;
     for (int d = 2; d < 4; ++d) {
+        h->ghost_bank[d] = 0;
         if (!p.halo[d]) continue;
-        for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->ghost[d][s], (size_t)nrhs * 3 * p.face_vh[d] * es));
+        // producer push: two banks, so an apply can push the next apply's faces into one while
+        // its own boundary kernel (and the neighbours') still read the other
+        const size_t bank = (size_t)nrhs * 3 * p.face_vh[d] * es;
+        if (h->push) h->ghost_bank[d] = bank;
+        for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->ghost[d][s], h->push ? 2 * bank : bank));
     }
     if (p.halo[2] && exch_remote(h, 2))
         for (int s = 0; s < 2; ++s) CU(h, cudaMalloc(&h->zsend[s], (size_t)nrhs * 3 * p.face_vh[2] * es));
@@ -335,6 +340,7 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             if (value == DSLASH_TRANSPORT_NCCL && h->plan.nranks > 1 && !h->nccl)
                 return fail(h, DSLASH_ERR_STATE, "NCCL transport needs dslash_create with an NCCL unique id");
             h->transport = (int)value;
+            if (value != DSLASH_TRANSPORT_P2P) h->push = 0;
             dslash_status st = alloc_halo(h, value == DSLASH_TRANSPORT_P2P ? kP2PMaxRhs : 1);
             if (st == DSLASH_OK && value == DSLASH_TRANSPORT_P2P) st = alloc_flags(h);
             return st;
@@ -352,6 +358,16 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
                 return fail(h, DSLASH_ERR_STATE, "long-link recon fixes the link layout: set it before load_links");
             h->recon = (int)value;
             return DSLASH_OK;
+        case DSLASH_OPT_PUSH: {
+            if (h->loaded || h->p2p_ready)
+                return fail(h, DSLASH_ERR_STATE, "PUSH must be set before load_links and the IPC setup");
+            if (value && h->transport != DSLASH_TRANSPORT_P2P)
+                return fail(h, DSLASH_ERR_UNSUPPORTED, "the producer push needs the P2P transport (peer-mapped ghosts)");
+            h->push = value != 0;
+            h->pushed_epoch = 0;
+            h->pushed_src = nullptr;
+            return alloc_halo(h, kP2PMaxRhs);
+        }
         case DSLASH_OPT_MIN_BLOCKS:
             if (value != 0 && (value < 2 || value > 4))
                 return fail(h, DSLASH_ERR_ARG, "min_blocks %lld must be 0, 2, 3 or 4", (long long)value);
@@ -761,6 +777,47 @@ static dslash_status p2p_prepare(dslash_t h) {
 // ============================================================================ halo exchange
 static bool any_halo(const dslash_plan_t& p) { return p.halo[2] || p.halo[3]; }
 
+// byte offset of the ghost bank that holds epoch e's faces of direction d (producer push: e & 1;
+// otherwise the single bank)
+static size_t bank_off(const dslash_s* h, int d, unsigned int e) { return (size_t)(e & 1u) * h->ghost_bank[d]; }
+
+// Producer push (apply_push of epoch e = h->epoch).  Its kernels store the faces of their output
+// into the neighbours' ghost bank (e + 1) & 1, which the neighbours last read at epoch e - 1 and
+// release at their halo_start of epoch e: stream x (the one the pushing kernels run on) first
+// waits for those releases, then the kernels run with K.push set, then x raises the neighbours'
+// ready flags to e + 1 (stream memory operations: the write is fenced behind the kernels' stores).
+static dslash_status push_wait_free(dslash_t h, cudaStream_t x) {
+    WaitValue32Fn wt = wait_value_fn();
+    for (int d = 3; d >= 2; --d)
+        if (h->plan.halo[d])
+            for (int side = 0; side < 2; ++side)
+                if (wt(x, (unsigned long long)(uintptr_t)(h->flags + 8 + 2 * d + side), h->epoch - 1, 0) != 0)
+                    return fail(h, DSLASH_ERR_CUDA, "cuStreamWaitValue32 (push free) failed");
+    return DSLASH_OK;
+}
+
+static void push_params(const dslash_s* h, StencilParams& K) {
+    for (int d = 2; d < 4; ++d)
+        if (h->plan.halo[d]) {
+            K.push_mask |= 1 << d;
+            for (int side = 0; side < 2; ++side) K.push[d][side] = h->peer_ghost[d][side] + bank_off(h, d, h->epoch + 1);
+        }
+}
+
+static dslash_status push_signal(dslash_t h, cudaStream_t x, const void* out, int nrhs) {
+    WriteValue32Fn wr = write_value_fn();
+    const unsigned int e1 = h->epoch + 1;
+    for (int d = 3; d >= 2; --d)
+        if (h->plan.halo[d])
+            for (int side = 0; side < 2; ++side)
+                if (wr(x, (unsigned long long)(uintptr_t)h->peer_ready[d][side], e1, 0) != 0)
+                    return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 (push ready) failed");
+    h->pushed_epoch = e1;
+    h->pushed_src = out;
+    h->pushed_rhs = nrhs;
+    return DSLASH_OK;
+}
+
 // P2P exchange of epoch e on the communication stream (copy engines + stream memory operations):
 //   1. release my ghosts of epoch e-1 to the ranks that filled them (every kernel that read them
 //      precedes ev_start),
@@ -778,7 +835,13 @@ static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaSt
     WriteValue32Fn wr = write_value_fn();
     WaitValue32Fn wt = wait_value_fn();
     if (!wr || !wt) return fail(h, DSLASH_ERR_UNSUPPORTED, "stream memory operations unavailable");
-    const unsigned int e = ++h->epoch;
+    const unsigned int e = h->epoch + 1;
+    // producer push: the previous apply already stored this source's faces in our ghosts
+    const bool pushed = h->push && h->pushed_epoch == e;
+    if (pushed && (in != h->pushed_src || nrhs != h->pushed_rhs))
+        return fail(h, DSLASH_ERR_STATE, "the apply after apply_push must take the pushed output as its source");
+    h->epoch = e;
+    h->pushed_epoch = 0;
     const size_t es = vec_elem(h);
     const char* src = static_cast<const char*>(in);
     const size_t vh = (size_t)p.vh_local;
@@ -792,6 +855,11 @@ static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaSt
             for (int side = 0; side < 2; ++side)
                 if (wr(h->comm, (unsigned long long)(uintptr_t)h->peer_free[d][side], e - 1, 0) != 0)
                     return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 (release) failed");
+    if (pushed) {  // no bytes to move: the neighbours raise our ready flags after their push
+        CU(h, cudaEventRecord(h->ev_halo, h->comm));
+        h->halo_pending = true;
+        return DSLASH_OK;
+    }
     for (int d = 3; d >= 2; --d)
         if (p.halo[d])
             for (int side = 0; side < 2; ++side)
@@ -799,16 +867,18 @@ static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaSt
                     return fail(h, DSLASH_ERR_CUDA, "cuStreamWaitValue32 (free) failed");
     if (p.halo[3]) {
         const size_t tslab = 3 * lxh * L1 * L2;
-        CU(h, cudaMemcpy2DAsync(h->peer_ghost[3][0], tslab * es, src, vh * es, tslab * es, rows,
+        const size_t b = bank_off(h, 3, e);
+        CU(h, cudaMemcpy2DAsync(h->peer_ghost[3][0] + b, tslab * es, src, vh * es, tslab * es, rows,
                                 cudaMemcpyDeviceToDevice, h->comm));
-        CU(h, cudaMemcpy2DAsync(h->peer_ghost[3][1], tslab * es, src + (vh - tslab) * es, vh * es, tslab * es, rows,
+        CU(h, cudaMemcpy2DAsync(h->peer_ghost[3][1] + b, tslab * es, src + (vh - tslab) * es, vh * es, tslab * es, rows,
                                 cudaMemcpyDeviceToDevice, h->comm));
     }
     if (p.halo[2]) {
         const size_t zrow = lxh * L1;
-        CU(h, cudaMemcpy2DAsync(h->peer_ghost[2][0], 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
+        const size_t b = bank_off(h, 2, e);
+        CU(h, cudaMemcpy2DAsync(h->peer_ghost[2][0] + b, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
                                 cudaMemcpyDeviceToDevice, h->comm));
-        CU(h, cudaMemcpy2DAsync(h->peer_ghost[2][1], 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es,
+        CU(h, cudaMemcpy2DAsync(h->peer_ghost[2][1] + b, 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es,
                                 3 * zrow * es, rows * L3, cudaMemcpyDeviceToDevice, h->comm));
     }
     for (int d = 3; d >= 2; --d)
@@ -1107,6 +1177,8 @@ static dslash_status launch_rhs(dslash_t h, StencilParams K, const dslash_box_t*
     char* out0 = static_cast<char*>(K.out);
     const void* g0[4][2];
     memcpy(g0, K.ghost, sizeof g0);
+    void* p0[4][2];
+    memcpy(p0, K.push, sizeof p0);
     for (int r0 = 0; r0 < nrhs;) {
         const int left = nrhs - r0;
         int nr = left >= 8 ? 8 : left >= 4 ? 4 : left >= 2 ? 2 : 1;
@@ -1114,9 +1186,12 @@ static dslash_status launch_rhs(dslash_t h, StencilParams K, const dslash_box_t*
         K.in = in0 + (size_t)r0 * 3 * K.vh * es;
         K.out = out0 + (size_t)r0 * 3 * K.vh * es;
         for (int d = 0; d < 4; ++d)
-            for (int side = 0; side < 2; ++side)
+            for (int side = 0; side < 2; ++side) {
                 K.ghost[d][side] = g0[d][side] ? static_cast<const char*>(g0[d][side]) + (size_t)r0 * 3 * K.face_vh[d] * es
                                                : nullptr;
+                K.push[d][side] = p0[d][side] ? static_cast<char*>(p0[d][side]) + (size_t)r0 * 3 * K.face_vh[d] * es
+                                              : nullptr;
+            }
         dslash_status st = launch(h, K, ghost, kind, s, nr);
         if (st != DSLASH_OK) return st;
         r0 += nr;
@@ -1336,14 +1411,15 @@ static dslash_status check_vectors(dslash_t h, const void* out, const void* in, 
 }
 
 static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs,
-                                dslash_stream_t stream);
+                                dslash_stream_t stream, bool push_out = false);
 
-dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s) {
-    return apply_impl(h, out, in, parity, nrhs, (dslash_stream_t)s);
+dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s,
+                         bool push) {
+    return apply_impl(h, out, in, parity, nrhs, (dslash_stream_t)s, push);
 }
 
 static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs,
-                                dslash_stream_t stream) {
+                                dslash_stream_t stream, bool push_out) {
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (parity & ~1) return fail(h, DSLASH_ERR_ARG, "parity %d not in {0,1}", parity);
     if (nrhs < 1) return fail(h, DSLASH_ERR_ARG, "nrhs %d < 1", nrhs);
@@ -1367,21 +1443,33 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         K.face_vh[d] = p.face_vh[d];
         if (p.halo[d]) K.halo_mask |= 1 << d;
     }
-    // persistent: 1 = when a halo is exchanged (default), 2 = always
+    // producer push: only with a halo (without one the next apply needs no faces) and only from
+    // the stencil kernels' epilogue (not the TMA kernel's)
+    push_out = push_out && any_halo(p);
+    if (push_out) {
+        if (!h->push) return fail(h, DSLASH_ERR_STATE, "apply_push needs DSLASH_OPT_PUSH");
+        if (h->kernel == DSLASH_KERNEL_BULK)
+            return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel does not push faces");
+    }
+    // persistent: 1 = when a halo is exchanged (default), 2 = always (not with the producer push,
+    // whose two ghost banks only the split launches address)
     if (h->persistent && (h->persistent == 2 || any_halo(p)) && nrhs == 1 && h->kernel != DSLASH_KERNEL_BULK &&
-        write_value_fn())
+        !h->push && write_value_fn())
         return apply_persistent(h, K, s);
     if (!any_halo(p)) return launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
     // the one-shot fused kernel serves single-RHS applies of the site / dir2 / dir4 kernels; other
     // applies in this mode take the split by sites
     if (h->overlap == DSLASH_OVERLAP_FUSED && nrhs == 1 && h->kernel != DSLASH_KERNEL_BULK && !h->stage &&
-        write_value_fn())
+        !h->push && write_value_fn())
         return apply_fused(h, K, s);
     if ((st = halo_start_impl(h, in, nrhs, s)) != DSLASH_OK) return st;
     for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
-        K.ghost[d][0] = h->ghost[d][0];
-        K.ghost[d][1] = h->ghost[d][1];
+        K.ghost[d][0] = h->ghost[d][0] ? h->ghost[d][0] + bank_off(h, d, h->epoch) : nullptr;
+        K.ghost[d][1] = h->ghost[d][1] ? h->ghost[d][1] + bank_off(h, d, h->epoch) : nullptr;
     }
+    // the interior launches never push (no interior site lies within 3 slices of a face)
+    StencilParams Kp = K;
+    if (push_out) push_params(h, Kp);
     if (h->overlap == DSLASH_OVERLAP_DIRS) {
         // split by direction: the local pass runs over EVERY site while the faces are in flight,
         // skipping the hops into ghost faces; once they landed, the ghost pass adds exactly those
@@ -1407,9 +1495,11 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         }
         if (st != DSLASH_OK) return st;
         if ((st = dslash_halo_wait(h, stream)) != DSLASH_OK) return st;
-        K.halo_pass = kPassGhost;
-        if ((st = launch_rhs(h, K, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, s, nrhs)) != DSLASH_OK)
+        if (push_out && (st = push_wait_free(h, s)) != DSLASH_OK) return st;
+        Kp.halo_pass = kPassGhost;
+        if ((st = launch_rhs(h, Kp, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, s, nrhs)) != DSLASH_OK)
             return st;
+        if (push_out && (st = push_signal(h, s, out, nrhs)) != DSLASH_OK) return st;
         if (span != (size_t)-1) CU(h, cudaEventRecord(h->tpool[span].b, s));
         return DSLASH_OK;
     }
@@ -1434,29 +1524,39 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         st = launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
         if (st != DSLASH_OK) return st;
         if ((st = dslash_halo_wait(h, (dslash_stream_t)h->bstream)) != DSLASH_OK) return st;
-        st = launch_rhs(h, K, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, h->bstream, nrhs);
+        if (push_out && (st = push_wait_free(h, h->bstream)) != DSLASH_OK) return st;
+        st = launch_rhs(h, Kp, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, h->bstream, nrhs);
         if (st != DSLASH_OK) return st;
+        if (push_out && (st = push_signal(h, h->bstream, out, nrhs)) != DSLASH_OK) return st;
         CU(h, cudaEventRecord(h->ev_bdone, h->bstream));
         CU(h, cudaStreamWaitEvent(s, h->ev_bdone, 0));
         if (span != (size_t)-1) CU(h, cudaEventRecord(h->tpool[span].b, s));
         return DSLASH_OK;
     }
     if ((st = dslash_halo_wait(h, stream)) != DSLASH_OK) return st;
+    if (push_out && (st = push_wait_free(h, s)) != DSLASH_OK) return st;
     if (p.n_interior + p.n_boundary > kMaxBoxes) {
         // 5 boxes (t and z halo): launch the interior part first, then the boundary boxes
         st = launch_rhs(h, K, p.interior, p.n_interior, true, DSLASH_TIMING_INTERIOR, s, nrhs);
-        if (st != DSLASH_OK) return st;
-        return launch_rhs(h, K, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, s, nrhs);
+        if (st == DSLASH_OK) st = launch_rhs(h, Kp, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, s, nrhs);
+    } else {
+        dslash_box_t all[kMaxBoxes];
+        int n = 0;
+        for (int i = 0; i < p.n_interior; ++i) all[n++] = p.interior[i];
+        for (int i = 0; i < p.n_boundary; ++i) all[n++] = p.boundary[i];
+        st = launch_rhs(h, Kp, all, n, true, DSLASH_TIMING_ALL, s, nrhs);
     }
-    dslash_box_t all[kMaxBoxes];
-    int n = 0;
-    for (int i = 0; i < p.n_interior; ++i) all[n++] = p.interior[i];
-    for (int i = 0; i < p.n_boundary; ++i) all[n++] = p.boundary[i];
-    return launch_rhs(h, K, all, n, true, DSLASH_TIMING_ALL, s, nrhs);
+    if (st == DSLASH_OK && push_out) st = push_signal(h, s, out, nrhs);
+    return st;
 }
 
 extern "C" dslash_status dslash_apply(dslash_t h, void* out, const void* in, int32_t parity, dslash_stream_t stream) {
     return apply_impl(h, out, in, parity, 1, stream);
+}
+
+extern "C" dslash_status dslash_apply_push(dslash_t h, void* out, const void* in, int32_t parity,
+                                           dslash_stream_t stream) {
+    return apply_impl(h, out, in, parity, 1, stream, true);
 }
 
 extern "C" dslash_status dslash_apply_multi(dslash_t h, int32_t nrhs, void* out, const void* in, int32_t parity,

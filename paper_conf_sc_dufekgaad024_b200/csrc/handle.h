@@ -79,6 +79,15 @@ struct dslash_s {
     unsigned int* peer_free[4][2] = {};   // [d][0]: minus nbr's free_from[d][1]; [d][1]: plus nbr's free_from[d][0]
     std::vector<void*> ipc_opened;
     bool p2p_ready = false;
+    // producer push (DSLASH_OPT_PUSH, P2P transport): the ghosts hold two banks (epoch e reads bank
+    // e & 1); an apply_push of epoch e stores the faces of its output straight into the neighbours'
+    // bank (e + 1) & 1 from the stencil kernel's epilogue, so the next apply (epoch e + 1, source =
+    // that output) exchanges no bytes
+    int push = 0;
+    size_t ghost_bank[4] = {};          // bytes from bank 0 to bank 1 of ghost[d][side]
+    const void* pushed_src = nullptr;   // the vector whose faces were pushed for epoch pushed_epoch
+    unsigned int pushed_epoch = 0;      // 0: none pending
+    int pushed_rhs = 0;
     dslash_status err = DSLASH_OK;
     std::string msg;
 };
@@ -106,5 +115,7 @@ dslash_status hisq_fail(dslash_t h, dslash_status st, const char* fmt, ...);
 // round the fp64 internal links of `parity` into h->links32[parity] (fp32 paired layout)
 dslash_status hisq_convert_links_sloppy(dslash_t h, int parity);
 
-// out = D in on target parity `parity` for nrhs back-to-back vectors (dslash_lib.cu)
-dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s);
+// out = D in on target parity `parity` for nrhs back-to-back vectors (dslash_lib.cu); push: also
+// push the faces of out into the neighbours' ghosts for the next apply (DSLASH_OPT_PUSH)
+dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s,
+                         bool push = false);

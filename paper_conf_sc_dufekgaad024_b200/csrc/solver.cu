@@ -168,7 +168,8 @@ static dslash_status reduce_to_host(dslash_t h, cudaStream_t s, double* value) {
     return DSLASH_OK;
 }
 
-static dslash_status check_solver_args(dslash_t h, const void* a, const void* b, int32_t parity) {
+static dslash_status check_solver_args(dslash_t h, const void* a, const void* b, int32_t parity,
+                                       bool reduces = true) {
     if (!h) return hisq_fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (parity & ~1) return hisq_fail(h, DSLASH_ERR_ARG, "parity %d not in {0,1}", parity);
     if (h->parity_mask != DSLASH_BOTH)
@@ -176,7 +177,7 @@ static dslash_status check_solver_args(dslash_t h, const void* a, const void* b,
     if (h->precision == DSLASH_F32)
         return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the solver works on fp64 vectors (DSLASH_F64 or DSLASH_MIXED)");
     if (!h->loaded) return hisq_fail(h, DSLASH_ERR_STATE, "solver before load_links");
-    if (h->plan.nranks > 1 && !h->nccl)
+    if (reduces && h->plan.nranks > 1 && !h->nccl)
         return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "dot products across ranks need an NCCL communicator");
     if (!a || !b || ((uintptr_t)a & 15) || ((uintptr_t)b & 15))
         return hisq_fail(h, DSLASH_ERR_ARG, "NULL or misaligned vector");
@@ -190,7 +191,8 @@ static dslash_status check_solver_args(dslash_t h, const void* a, const void* b,
 template <typename V2>
 static dslash_status normal_apply(dslash_t h, V2* q, const V2* p, int32_t parity, double m2, V2* tmp, cudaStream_t s,
                                   bool dot) {
-    dslash_status st = hisq_apply(h, tmp, p, 1 - parity, 1, s);  // t = D_{1-p,p} p
+    // t = D_{1-p,p} p; with the producer push its faces go straight to the neighbours' ghosts
+    dslash_status st = hisq_apply(h, tmp, p, 1 - parity, 1, s, h->push != 0);
     if (st != DSLASH_OK) return st;
     if ((st = hisq_apply(h, q, tmp, parity, 1, s)) != DSLASH_OK) return st;  // q = D_{p,1-p} t
     const int64_t n = 3 * h->plan.vh_local;
@@ -201,7 +203,7 @@ static dslash_status normal_apply(dslash_t h, V2* q, const V2* p, int32_t parity
 
 extern "C" dslash_status dslash_normal_apply(dslash_t h, void* out, const void* in, int32_t parity, double mass,
                                              dslash_stream_t stream) {
-    dslash_status st = check_solver_args(h, out, in, parity);
+    dslash_status st = check_solver_args(h, out, in, parity, false);  // no dot product
     if (st != DSLASH_OK) return st;
     if ((st = need_scratch(h)) != DSLASH_OK) return st;
     return normal_apply(h, (double2*)out, (const double2*)in, parity, mass * mass, (double2*)h->cg_vec[3],

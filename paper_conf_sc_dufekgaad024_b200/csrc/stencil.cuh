@@ -477,6 +477,40 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
             if (lane < 3) st_stream(out + lane * P.vh + s.cb, lane == 0 ? acc[r][0] : lane == 1 ? acc[r][1] : acc[r][2]);
         }
     }
+    if constexpr (GHOST) {
+        // producer push (DSLASH_OPT_PUSH): a site in the 3 bottom (top) slices of a pushed
+        // direction is a source of the minus (plus) neighbour's next apply; store its output
+        // straight into that neighbour's ghost face (peer memory), in the face order
+        // halo_start's copies use, so the next apply exchanges no bytes.  The local pass of the
+        // split by direction holds partial sums only and never pushes.
+        if (P.push_mask && P.halo_pass != kPassLocal) {
+#pragma unroll
+            for (int mu = 2; mu < 4; ++mu) {
+                if (!((P.push_mask >> mu) & 1)) continue;
+                const int c = mu == 2 ? s.z : s.t;
+                const int L = P.L[mu];
+                const int64_t fv = P.face_vh[mu];
+#pragma unroll
+                for (int side = 0; side < 2; ++side) {
+                    // (with L = 4 a slice can be both a bottom and a top slice)
+                    if (side == 0 ? c >= 3 : c < L - 3) continue;
+                    const int d = side ? c - (L - 3) : c;
+                    const int64_t f = (mu == 3)
+                                          ? s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (s.z + (int64_t)P.L[2] * d))
+                                          : s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (d + 3 * (int64_t)s.t));
+#pragma unroll
+                    for (int r = 0; r < NRHS; ++r) {
+                        V2* g = static_cast<V2*>(P.push[mu][side]) + (int64_t)(rl * NRHS + r) * 3 * fv + f;
+#pragma unroll
+                        for (int cc = 0; cc < 3; ++cc) {
+                            const bool mine = LANES == 1 || (LANES == 2 ? (lane == 0) == (cc < 2) : lane == cc);
+                            if (mine) g[cc * fv] = acc[r][cc];
+                        }
+                    }
+                }
+            }
+        }
+    }
 }
 
 template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1, int RHSL = 1>
