@@ -891,6 +891,48 @@ static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaSt
     return DSLASH_OK;
 }
 
+dslash_status hisq_push_begin(dslash_t h, cudaStream_t s, FacePush* fp) {
+    memset(fp, 0, sizeof *fp);
+    const dslash_plan_t& p = h->plan;
+    if (!h->push || !any_halo(p)) return DSLASH_OK;
+    dslash_status st = p2p_prepare(h);
+    if (st != DSLASH_OK) return st;
+    if ((st = push_wait_free(h, s)) != DSLASH_OK) return st;
+    StencilParams K{};
+    push_params(h, K);
+    memcpy(fp->dst, K.push, sizeof fp->dst);
+    fp->mask = K.push_mask;
+    fp->vh = p.vh_local;
+    for (int d = 0; d < 4; ++d) fp->face_vh[d] = p.face_vh[d];
+    fp->lxh = p.local_dims[0] / 2;
+    fp->L1 = p.local_dims[1];
+    fp->L2 = p.local_dims[2];
+    fp->L3 = p.local_dims[3];
+    return DSLASH_OK;
+}
+
+dslash_status hisq_push_end(dslash_t h, cudaStream_t s, const void* out) {
+    if (!h->push || !any_halo(h->plan)) return DSLASH_OK;
+    return push_signal(h, s, out, 1);
+}
+
+dslash_status hisq_push_discard(dslash_t h, cudaStream_t s) {
+    if (!h->pushed_epoch) return DSLASH_OK;
+    WriteValue32Fn wr = write_value_fn();
+    const dslash_plan_t& p = h->plan;
+    const unsigned int e = h->pushed_epoch;
+    h->epoch = e;
+    h->pushed_epoch = 0;
+    CU(h, cudaEventRecord(h->ev_start, s));
+    CU(h, cudaStreamWaitEvent(h->comm, h->ev_start, 0));
+    for (int d = 3; d >= 2; --d)
+        if (p.halo[d])
+            for (int side = 0; side < 2; ++side)
+                if (wr(h->comm, (unsigned long long)(uintptr_t)h->peer_free[d][side], e - 1, 0) != 0)
+                    return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 (release) failed");
+    return DSLASH_OK;
+}
+
 // Exchange the depth-3 faces of nrhs source vectors stored back to back ([nrhs][3][vh]).
 static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaStream_t s) {
     const dslash_plan_t& p = h->plan;
@@ -1711,6 +1753,9 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
         if (v) cudaFree(v);
     if (h->cg_partial) cudaFree(h->cg_partial);
     if (h->cg_scalar) cudaFree(h->cg_scalar);
+    if (h->cg_host_rr) cudaFreeHost(h->cg_host_rr);
+    for (cudaEvent_t e : h->cg_ev)
+        if (e) cudaEventDestroy(e);
     if (h->h2d) cudaStreamDestroy(h->h2d);
     if (h->d2h) cudaStreamDestroy(h->d2h);
     for (auto& t : h->tpool) {

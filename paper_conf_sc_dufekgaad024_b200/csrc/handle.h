@@ -50,6 +50,11 @@ struct dslash_s {
     void* links32[2] = {};
     double* cg_partial = nullptr;
     double* cg_scalar = nullptr;
+    // CG host side, kept across solves (pinned allocation and event creation cost more than a
+    // short solve): <r,r> per iteration, pinned; events of the lagged convergence check
+    double* cg_host_rr = nullptr;
+    int cg_host_cap = 0;
+    cudaEvent_t cg_ev[4] = {};
     // tile scheduler of the TMA kernel: ticket counters ([0] interior, [0/1] boundary launches,
     // which may overlap) and the first ticket of each counter's next launch
     unsigned long long* sched = nullptr;   // [0] TMA interior, [1] TMA boundary, [2] persistent
@@ -111,6 +116,23 @@ dslash_status hisq_fail(dslash_t h, dslash_status st, const char* fmt, ...);
             return hisq_fail((h), DSLASH_ERR_NCCL, "%s:%d %s: %s", __FILE__, __LINE__, #call,         \
                              ncclGetErrorString(r_));                                                 \
     } while (0)
+
+// Producer push from a vector kernel (the CG direction update p = r + beta p): the element of
+// colour c at cb of a site within 3 slices of a pushed face is also stored into the neighbour's
+// ghost bank, in the face order of the stencil kernel's push (stencil.cuh).
+struct FacePush {
+    void* dst[4][2];      // [mu][side] peer ghost banks, [3][face_vh[mu]] (only where mask has mu)
+    int mask;             // bit mu: push direction mu (2 = z, 3 = t)
+    int64_t vh, face_vh[4];
+    int lxh, L1, L2, L3;  // local extents (lxh = Lx / 2)
+};
+// before the pushing kernel on stream s: wait for the neighbours' releases, fill *fp (mask 0 when
+// the handle does not push or has no halo); after it: raise the neighbours' ready flags
+dslash_status hisq_push_begin(dslash_t h, cudaStream_t s, FacePush* fp);
+dslash_status hisq_push_end(dslash_t h, cudaStream_t s, const void* out);
+// drop pushed faces no apply will consume (the CG's last direction update): the pushed epoch is
+// retired as if an apply had consumed it, on every rank alike
+dslash_status hisq_push_discard(dslash_t h, cudaStream_t s);
 
 // round the fp64 internal links of `parity` into h->links32[parity] (fp32 paired layout)
 dslash_status hisq_convert_links_sloppy(dslash_t h, int parity);

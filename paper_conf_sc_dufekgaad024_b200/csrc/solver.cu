@@ -7,7 +7,10 @@
 // is Hermitian positive definite on parity p for m != 0, and CG solves A_p x = b.
 // Dot products are reduced deterministically (fixed block partition, fixed final order) and,
 // with several ranks, summed with ncclAllReduce: the solver's one true collective.
+#include <chrono>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "handle.h"
@@ -65,14 +68,15 @@ __global__ void __launch_bounds__(kRedThreads) k_norm2(const V2* __restrict__ v,
 }
 
 // x += alpha p ; r -= alpha q ; partial[block] = sum |r|^2, alpha = rr / pq read on the device
-// (0 when pq == 0: an exactly converged iterate stays put)
+// (0 when pq == 0, or once rr <= stop: an iterate that converged stays put through the iterations
+// the host queued before it saw the convergence)
 template <typename V2>
 __global__ void __launch_bounds__(kRedThreads) k_cg_update(V2* __restrict__ x, V2* __restrict__ r,
                                                            const V2* __restrict__ p, const V2* __restrict__ q,
                                                            const double* __restrict__ rr, const double* __restrict__ pq,
-                                                           int64_t n, double* __restrict__ partial) {
+                                                           double stop, int64_t n, double* __restrict__ partial) {
     using R = decltype(V2{}.x);
-    const R alpha = (R)((*pq != 0.0) ? *rr / *pq : 0.0);
+    const R alpha = (R)((*pq != 0.0 && *rr > stop) ? *rr / *pq : 0.0);
     double acc = 0.0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         V2 xi = x[i], ri = r[i];
@@ -89,10 +93,33 @@ __global__ void __launch_bounds__(kRedThreads) k_cg_update(V2* __restrict__ x, V
     if (threadIdx.x == 0) partial[blockIdx.x] = s;
 }
 
-// p = r + beta p, beta = rr_new / rr read on the device (0 when rr == 0)
+// element i = c * vh + cb of a [3][vh] vector: also store it into the pushed ghost faces its site
+// belongs to (F.mask != 0; the face order of the stencil kernel's push, stencil.cuh)
+template <typename V2>
+__device__ __forceinline__ void push_element(const FacePush& F, int64_t i, V2 v) {
+    const int64_t c = i / F.vh, cb = i - c * F.vh;
+    const int64_t zrow = (int64_t)F.lxh * F.L1, tslab = zrow * F.L2;
+    const int t = (int)(cb / tslab);
+    if (F.mask & 8) {
+        const int64_t fv = F.face_vh[3];
+        if (t < 3) static_cast<V2*>(F.dst[3][0])[c * fv + cb] = v;
+        if (t >= F.L3 - 3) static_cast<V2*>(F.dst[3][1])[c * fv + cb - (int64_t)(F.L3 - 3) * tslab] = v;
+    }
+    if (F.mask & 4) {
+        const int64_t fv = F.face_vh[2];
+        const int64_t in_row = cb % zrow;
+        const int z = (int)((cb / zrow) % F.L2);
+        if (z < 3) static_cast<V2*>(F.dst[2][0])[c * fv + in_row + zrow * (z + 3 * (int64_t)t)] = v;
+        if (z >= F.L2 - 3)
+            static_cast<V2*>(F.dst[2][1])[c * fv + in_row + zrow * (z - (F.L2 - 3) + 3 * (int64_t)t)] = v;
+    }
+}
+
+// p = r + beta p, beta = rr_new / rr read on the device (0 when rr == 0); with the producer push the
+// faces of the new p go straight to the neighbours' ghosts for the next iteration's first apply
 template <typename V2>
 __global__ void k_cg_direction(V2* __restrict__ p, const V2* __restrict__ r, const double* __restrict__ rr_new,
-                               const double* __restrict__ rr, int64_t n) {
+                               const double* __restrict__ rr, int64_t n, const FacePush F) {
     using R = decltype(V2{}.x);
     const R beta = (R)((*rr != 0.0) ? *rr_new / *rr : 0.0);
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
@@ -101,6 +128,7 @@ __global__ void k_cg_direction(V2* __restrict__ p, const V2* __restrict__ r, con
         pi.x = fma(beta, pi.x, ri.x);
         pi.y = fma(beta, pi.y, ri.y);
         p[i] = pi;
+        if (F.mask) push_element(F, i, pi);
     }
 }
 
@@ -214,22 +242,22 @@ extern "C" dslash_status dslash_normal_apply(dslash_t h, void* out, const void* 
 // Hestenes-Stiefel recurrences, run until <r, r> <= stop or max_iter.  Device scalars: sc[0], sc[1] =
 // <r,r> of alternate iterations (ping-pong, so no kernel overwrites a value another block may
 // still read), sc[2] = <p, A p>; sc[0] must hold <b, b> on entry.  The host learns <r,r> through
-// pinned memory one iteration late, so the GPU never waits for the host; the solve can run one
-// iteration past convergence, which only refines x.  V2 = double2 (fp64) or float2 (the inner
-// solve of dslash_cg_mixed, on the fp32 links).
+// pinned memory kCgLag iterations late, so the GPU never waits for the host and the host's
+// enqueue jitter is absorbed by a queue several iterations deep.  The iterations queued past
+// convergence are frozen on the device (k_cg_update takes alpha = 0 once <r,r> <= stop), so x is
+// exactly the first converged iterate and *iters its index.  V2 = double2 (fp64) or float2 (the
+// inner solve of dslash_cg_mixed, on the fp32 links).
+constexpr int kCgLag = 3;
+
 template <typename V2>
 static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int32_t parity, double m2, double stop,
                              int32_t max_iter, cudaStream_t s, int32_t* iters, double* rr_last, bool* converged) {
     const int64_t n = 3 * h->plan.vh_local;
     double* sc = h->cg_scalar;
-    double* host_rr = nullptr;
-    cudaEvent_t ev[2] = {nullptr, nullptr};
+    static_assert(kCgLag + 1 <= (int)(sizeof(dslash_s::cg_ev) / sizeof(cudaEvent_t)), "event ring");
+    cudaEvent_t* ev = h->cg_ev;
     dslash_status st = DSLASH_OK;
-    auto release = [&]() {
-        for (cudaEvent_t e : ev)
-            if (e) cudaEventDestroy(e);
-        if (host_rr) cudaFreeHost(host_rr);
-    };
+    auto release = [&]() {};
 #define CUR(call)                                                                                    \
     do {                                                                                             \
         cudaError_t e_ = (call);                                                                     \
@@ -239,37 +267,75 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
                              cudaGetErrorString(e_));                                                \
         }                                                                                            \
     } while (0)
-    CUR(cudaMallocHost(&host_rr, 2 * sizeof(double)));
-    CUR(cudaEventCreateWithFlags(&ev[0], cudaEventDisableTiming));
-    CUR(cudaEventCreateWithFlags(&ev[1], cudaEventDisableTiming));
+    int need = (max_iter < 1 ? 1 : max_iter) + 1;
+    if (h->cg_host_cap < need) {
+        need = need < 2 * h->cg_host_cap ? 2 * h->cg_host_cap : need < 8192 ? 8192 : need;
+        if (h->cg_host_rr) CUR(cudaFreeHost(h->cg_host_rr));
+        h->cg_host_rr = nullptr;
+        h->cg_host_cap = 0;
+        CUR(cudaMallocHost(&h->cg_host_rr, (size_t)need * sizeof(double)));
+        h->cg_host_cap = need;
+    }
+    double* host_rr = h->cg_host_rr;  // host_rr[k] = <r,r> after iteration k
+    host_rr[0] = HUGE_VAL;            // (max_iter < 1: no iteration, not converged)
+    for (int i = 0; i <= kCgLag; ++i)
+        if (!ev[i]) CUR(cudaEventCreateWithFlags(&ev[i], cudaEventDisableTiming));
     *converged = false;
-    int k = 0;
+    int k = 0, kstar = 0;  // last enqueued iteration; first converged one (0: none seen yet)
+    // HISQ_CG_PROFILE=1: host time per iteration spent enqueueing vs waiting, to stderr
+    static const bool prof = getenv("HISQ_CG_PROFILE") != nullptr;
+    using clk = std::chrono::steady_clock;
+    double enq_us = 0.0, enq_max = 0.0, wait_us = 0.0;
     for (k = 1; k <= max_iter; ++k) {
+        const auto t0 = prof ? clk::now() : clk::time_point{};
         double* rr_cur = &sc[(k - 1) & 1];
         double* rr_new = &sc[k & 1];
         if ((st = normal_apply(h, q, p, parity, m2, t, s, true)) != DSLASH_OK) break;  // q = A p
         if ((st = reduce_to_slot(h, s, &sc[2])) != DSLASH_OK) break;                 // <p, q>
-        k_cg_update<<<kRedBlocks, kRedThreads, 0, s>>>(x, r, p, q, rr_cur, &sc[2], n, h->cg_partial);
+        k_cg_update<<<kRedBlocks, kRedThreads, 0, s>>>(x, r, p, q, rr_cur, &sc[2], stop, n, h->cg_partial);
         CUR(cudaGetLastError());
         if ((st = reduce_to_slot(h, s, rr_new)) != DSLASH_OK) break;                  // <r, r>
-        k_cg_direction<<<kRedBlocks, kRedThreads, 0, s>>>(p, r, rr_new, rr_cur, n);
+        FacePush fp;
+        if ((st = hisq_push_begin(h, s, &fp)) != DSLASH_OK) break;
+        k_cg_direction<<<kRedBlocks, kRedThreads, 0, s>>>(p, r, rr_new, rr_cur, n, fp);
         CUR(cudaGetLastError());
-        CUR(cudaMemcpyAsync(&host_rr[k & 1], rr_new, sizeof(double), cudaMemcpyDeviceToHost, s));
-        CUR(cudaEventRecord(ev[k & 1], s));
-        // check iteration k-1 (already complete or nearly) while iteration k runs
-        if (k >= 2) {
-            CUR(cudaEventSynchronize(ev[(k - 1) & 1]));
-            if (host_rr[(k - 1) & 1] <= stop) {
-                *converged = true;
+        if ((st = hisq_push_end(h, s, p)) != DSLASH_OK) break;
+        CUR(cudaMemcpyAsync(&host_rr[k], rr_new, sizeof(double), cudaMemcpyDeviceToHost, s));
+        CUR(cudaEventRecord(ev[k % (kCgLag + 1)], s));
+        // check iteration k - kCgLag (complete or nearly) while the later ones run
+        const int j = k - kCgLag;
+        if (prof) {
+            const double e = std::chrono::duration<double, std::micro>(clk::now() - t0).count();
+            enq_us += e;
+            enq_max = e > enq_max ? e : enq_max;
+        }
+        if (j >= 1) {
+            const auto t1 = prof ? clk::now() : clk::time_point{};
+            CUR(cudaEventSynchronize(ev[j % (kCgLag + 1)]));
+            if (prof) wait_us += std::chrono::duration<double, std::micro>(clk::now() - t1).count();
+            if (host_rr[j] <= stop) {
+                kstar = j;
                 break;
             }
         }
     }
+    if (prof && k > 0)
+        fprintf(stderr, "[hisq cg] %d iterations: enqueue %.1f us/iter (max %.1f), wait %.1f us/iter\n", k,
+                enq_us / k, enq_max, wait_us / k);
+    // the last direction update pushed faces of a p no apply will read
+    if (st == DSLASH_OK) st = hisq_push_discard(h, s);
     if (st == DSLASH_OK) {
         if (k > max_iter) k = max_iter;
-        CUR(cudaEventSynchronize(ev[k & 1]));
-        *rr_last = host_rr[k & 1];
-        if (*rr_last <= stop) *converged = true;
+        CUR(cudaStreamSynchronize(s));
+        if (!kstar)  // the last kCgLag iterations were not checked yet
+            for (int j = k - kCgLag + 1 < 1 ? 1 : k - kCgLag + 1; j <= k; ++j)
+                if (host_rr[j] <= stop) {
+                    kstar = j;
+                    break;
+                }
+        *converged = kstar > 0;
+        if (kstar) k = kstar;
+        *rr_last = host_rr[k];
     }
     *iters = k;
     release();
