@@ -47,8 +47,9 @@ def parse():
     ap.add_argument("--min-blocks", type=int, default=0)
     ap.add_argument("--nrhs", type=int, default=1, choices=[1, 2, 3, 4, 5, 6, 7, 8],
                     help="right-hand sides per apply, one link pass (SURVEY §8(f)-4)")
-    ap.add_argument("--recon", type=int, default=18, choices=[18, 12],
-                    help="12: long links stored as 2 rows (SURVEY §8(f)-2, QUDA recon-12, PAPER.md L325)")
+    ap.add_argument("--recon", type=int, default=18, choices=[18, 12, 9],
+                    help="12: long links stored as 2 rows (SURVEY §8(f)-2, QUDA recon-12, PAPER.md L325); "
+                         "9: 8 SU(3) parameters + a phase (fp64)")
     ap.add_argument("--precision", default="f64", choices=["f64", "f32", "mixed"],
                     help="f64 is the paper's (L278) and the headline; f32/mixed are SURVEY §8(f)-1")
     ap.add_argument("--block", type=int, default=0)

@@ -93,6 +93,15 @@ enum {
                                    (QUDA "recon-12").  Requires every long link
                                    (and the link halo) to be s*W with W in SU(3) and one real s;
                                    load_links verifies it and returns DSLASH_ERR_ARG otherwise.
+                                   9: each long matrix M = s e^{i psi} W (W in SU(3), one real s
+                                   per handle) stored as the 8 parameters of W (arg a1, arg c1, a2,
+                                   a3, b1) + psi, rebuilt in registers (QUDA "recon-9"; accepts
+                                   folded staggered signs and U(1) phases).  fp64 register kernels
+                                   only (DSLASH_ERR_UNSUPPORTED for F32 / MIXED / the TMA kernel
+                                   and dslash_cg_mixed); load_links verifies that every long link
+                                   is rebuilt within 1e-12 s, which also rejects links near the
+                                   parameterisation's singular set |a2|^2 + |a3|^2 -> 0 (e.g.
+                                   multiples of the identity): DSLASH_ERR_ARG.
                                    Before load_links                                                  */
     DSLASH_OPT_PERSISTENT = 7,  /* 0 (default): separate interior / boundary launches (measured faster
                                    on B200, profiles/README.md).  1: when a halo is exchanged, one
@@ -269,7 +278,8 @@ DSLASH_API dslash_status dslash_load_links_halo(dslash_t h, const void* fat, con
  * load_links): out_host[cb][mu][l][3][3] complex fp64, Vh_local x 144 complex, with
  * l = 0 F(x,mu), 1 F(x-mu,mu)^dag, 2 N(x,mu), 3 N(x-3mu,mu)^dag (PAPER.md L51's |l| = 4 arrays)
  * for the target site x of checkerboard index cb.  Values as stored (fp32 widened); with
- * recon-12 row 2 of the long matrices is not stored and reads as 0.  Synchronous. */
+ * recon-12 row 2 of the long matrices is not stored and reads as 0; with recon-9 the long
+ * matrices are returned rebuilt from their stored parameters.  Synchronous. */
 DSLASH_API dslash_status dslash_get_links(dslash_t h, int32_t parity, void* out_host);
 
 /* chi = D psi on target parity `parity`.  out: device [3][Vh_local] complex on parity

@@ -24,11 +24,12 @@ ALGO_BYTES = {"f64": 2304 + 48 + 48, "f32": 1152 + 24 + 24, "mixed": 1152 + 48 +
 
 def algo_bytes(precision="f64", recon=18, nrhs=1):
     """Algorithmic bytes per target site for one launch over nrhs right-hand sides: links
-    (recon-12 stores 6 of 9 entries of the 8 long matrices) + nrhs x (source with ideal reuse +
+    (recon-12 stores 6 of 9 entries of the 8 long matrices, recon-9 4 + a shared phase entry) + nrhs x (source with ideal reuse +
     output)."""
     lb = 16 if precision == "f64" else 8
     vb = 8 if precision == "f32" else 16
-    link_entries = 8 * 9 + 8 * (6 if recon == 12 else 9)
+    # recon-9: 4 entries per long matrix + one (psi_f, psi_b) entry per direction
+    link_entries = 8 * 9 + (8 * 6 if recon == 12 else 8 * 4 + 4 if recon == 9 else 8 * 9)
     return link_entries * lb + nrhs * 2 * 3 * vb
 
 __all__ = ["Dslash", "DslashError", "dslash_plan", "FLOP_PER_SITE", "ALGO_BYTES_PER_SITE"]

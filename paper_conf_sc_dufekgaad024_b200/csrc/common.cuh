@@ -195,6 +195,7 @@ struct StencilParams {
     int64_t vh;
     int64_t face_vh[4];
     double long_inv_scale;     // 1/s of the long links N = s W (recon-12 only)
+    double long_scale;         // s of the long links N = s e^{i psi} W (recon-9 only)
     int L[4];                  // local extents
     int lxh;                   // L[0] / 2
     int parity;                // (target parity + origin sum) & 1, origin sum is even -> target parity

@@ -353,7 +353,8 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             h->persistent = (int)value;
             return DSLASH_OK;
         case DSLASH_OPT_LONG_RECON:
-            if (value != 18 && value != 12) return fail(h, DSLASH_ERR_ARG, "long-link recon %lld must be 18 or 12", (long long)value);
+            if (value != 18 && value != 12 && value != 9)
+                return fail(h, DSLASH_ERR_ARG, "long-link recon %lld must be 18, 12 or 9", (long long)value);
             if (h->loaded && value != h->recon)
                 return fail(h, DSLASH_ERR_STATE, "long-link recon fixes the link layout: set it before load_links");
             h->recon = (int)value;
@@ -393,6 +394,8 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
                                      const void* const* slab_lng_in, int32_t on_device, dslash_stream_t stream) {
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!fat || !lng) return fail(h, DSLASH_ERR_ARG, "NULL link pointer");
+    if (h->recon == 9 && (h->precision != DSLASH_F64 || h->kernel == DSLASH_KERNEL_BULK))
+        return fail(h, DSLASH_ERR_UNSUPPORTED, "recon-9 serves fp64 links and the register kernels (site/dir2/dir4)");
     cudaStream_t s = (cudaStream_t)stream;
     const dslash_plan_t& p = h->plan;
     const int64_t V = 2 * p.vh_local;
@@ -516,6 +519,48 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
         C.slab_fat[d] = slab[d][0];
         C.slab_lng[d] = slab[d][1];
     }
+    if (h->recon == 9) {
+        // s from the first local long link: |det(s e^{i psi} W)| = s^3
+        double2 A[9];
+        CUL(cudaMemcpyAsync(A, dlng, sizeof A, cudaMemcpyDeviceToHost, s));
+        CUL(cudaStreamSynchronize(s));
+        auto cm = [](double2 a, double2 b) { return make_double2(a.x * b.x - a.y * b.y, a.x * b.y + a.y * b.x); };
+        auto sub = [](double2 a, double2 b) { return make_double2(a.x - b.x, a.y - b.y); };
+        const double2 m0 = sub(cm(A[4], A[8]), cm(A[5], A[7]));
+        const double2 m1 = sub(cm(A[3], A[8]), cm(A[5], A[6]));
+        const double2 m2 = sub(cm(A[3], A[7]), cm(A[4], A[6]));
+        const double2 d0 = cm(A[0], m0), d1 = cm(A[1], m1), d2 = cm(A[2], m2);
+        const double sc = std::cbrt(std::hypot(d0.x - d1.x + d2.x, d0.y - d1.y + d2.y));
+        if (!(sc > 0.0) || !std::isfinite(sc)) {
+            cleanup();
+            return fail(h, DSLASH_ERR_ARG, "recon-9: first long link has zero determinant");
+        }
+        unsigned long long* dmax;
+        CUL(cudaMalloc(&dmax, sizeof *dmax));
+        tmp.push_back(dmax);
+        CUL(cudaMemsetAsync(dmax, 0, sizeof *dmax, s));
+        auto check = [&](const double2* arr, int64_t nmat) {
+            if (nmat > 0) recon9_check_kernel<<<(unsigned)((nmat + 255) / 256), 256, 0, s>>>(arr, nmat, sc, dmax);
+        };
+        check(dlng, V * 4);
+        for (int d = 2; d < 4; ++d)
+            if (slab[d][1]) check(slab[d][1], 3 * (V / p.local_dims[d]) * 4);
+        CUL(cudaGetLastError());
+        unsigned long long bits = 0;
+        CUL(cudaMemcpyAsync(&bits, dmax, sizeof bits, cudaMemcpyDeviceToHost, s));
+        CUL(cudaStreamSynchronize(s));
+        double err;
+        memcpy(&err, &bits, sizeof err);
+        if (!(err <= 1e-12 * sc)) {
+            cleanup();
+            return fail(h, DSLASH_ERR_ARG,
+                        "recon-9: long links are not s*e^{i psi}*SU(3) with one real s = %.17g, or lie near the "
+                        "parameterisation's singular set (max deviation %.3e)", sc, err);
+        }
+        h->long_scale = sc;
+        h->long_inv_scale = 1.0 / sc;
+        C.s9 = sc;
+    }
     if (h->recon == 12) {
         // s from the first local long link: det(s W) = s^3
         double2 A[9];
@@ -556,7 +601,7 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
         }
         h->long_inv_scale = 1.0 / sc;
     }
-    const size_t link_bytes = (size_t)p.vh_local * (h->recon == 12 ? 120 : 144) * link_elem(h);
+    const size_t link_bytes = (size_t)p.vh_local * (h->recon == 12 ? 120 : h->recon == 9 ? 108 : 144) * link_elem(h);
     for (int par = 0; par < 2; ++par)  // a recon change alters the size: reallocate
         if (h->links[par] && h->link_bytes != link_bytes) {
             cudaFree(h->links[par]);
@@ -627,6 +672,7 @@ extern "C" dslash_status dslash_get_links(dslash_t h, int32_t parity, void* out_
     C.vh = p.vh_local;
     C.lanes = h->kernel == DSLASH_KERNEL_BULK ? 0 : lanes_of(h->kernel);
     C.recon = h->recon;
+    C.s9 = h->long_scale;
     C.paired = h->precision != DSLASH_F64 && h->kernel != DSLASH_KERNEL_BULK;
     const size_t bytes = (size_t)p.vh_local * 144 * sizeof(double2);
     void* tmp = nullptr;
@@ -1060,6 +1106,7 @@ static void fill_boxes(StencilParams& K, const dslash_box_t* boxes, int n) {
 template <bool GHOST>
 static StencilFn pick_kernel(int precision, int recon, int lanes, int minb, int nrhs) {
     const bool r12 = recon == 12;
+    if (recon == 9) return pick_f64_r9(GHOST, lanes, minb, nrhs);  // fp64 only (load_links checks)
     switch (precision) {
         case DSLASH_F32: return r12 ? pick_f32_r12(GHOST, lanes, minb, nrhs) : pick_f32_r18(GHOST, lanes, minb, nrhs);
         case DSLASH_MIXED: return r12 ? pick_mixed_r12(GHOST, lanes, minb, nrhs) : pick_mixed_r18(GHOST, lanes, minb, nrhs);
@@ -1074,6 +1121,7 @@ static int default_minb(int lanes) { return lanes == 4 ? 2 : 2; }
 
 static StencilFn pick_stage_kernel(int precision, int recon, bool ghost, int lanes, int nrhs) {
     const bool r12 = recon == 12;
+    if (recon == 9) return pick_f64_r9_stage(ghost, lanes, nrhs);
     switch (precision) {
         case DSLASH_F32:
             return r12 ? pick_f32_r12_stage(ghost, lanes, nrhs) : pick_f32_r18_stage(ghost, lanes, nrhs);
@@ -1258,6 +1306,7 @@ static int persist_occupancy(dslash_t h, PersistFn fn, int bs) {
 
 static PersistFn pick_persist(int precision, int recon, int mode, int lanes) {
     const bool r12 = recon == 12;
+    if (recon == 9) return persist_f64_r9(mode, lanes);
     switch (precision) {
         case DSLASH_F32: return r12 ? persist_f32_r12(mode, lanes) : persist_f32_r18(mode, lanes);
         case DSLASH_MIXED: return r12 ? persist_mixed_r12(mode, lanes) : persist_mixed_r18(mode, lanes);
@@ -1349,6 +1398,7 @@ static dslash_status apply_persistent(dslash_t h, StencilParams K, cudaStream_t 
 
 static FusedFn pick_fused_kernel(int precision, int recon, bool cleanup, int lanes) {
     const bool r12 = recon == 12;
+    if (recon == 9) return pick_f64_r9_fused(cleanup, lanes);
     switch (precision) {
         case DSLASH_F32: return r12 ? pick_f32_r12_fused(cleanup, lanes) : pick_f32_r18_fused(cleanup, lanes);
         case DSLASH_MIXED: return r12 ? pick_mixed_r12_fused(cleanup, lanes) : pick_mixed_r18_fused(cleanup, lanes);
@@ -1480,6 +1530,7 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
     K.lxh = p.local_dims[0] / 2;
     K.parity = parity;
     K.long_inv_scale = h->long_inv_scale;
+    K.long_scale = h->long_scale;
     for (int d = 0; d < 4; ++d) {
         K.L[d] = p.local_dims[d];
         K.face_vh[d] = p.face_vh[d];

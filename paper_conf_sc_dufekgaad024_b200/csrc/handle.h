@@ -17,6 +17,7 @@ struct dslash_s {
     int kernel = DSLASH_KERNEL_DIR2, block = 0, force_halo = 0, overlap = 1, timing = 0, min_blocks = 0;
     int recon = 18;
     double long_inv_scale = 1.0;
+    double long_scale = 1.0;        // recon-9: s of N = s e^{i psi} W
     size_t link_bytes = 0;
     bool loaded = false;
     void* links[2] = {nullptr, nullptr};

@@ -30,7 +30,9 @@ struct LinkConvParams {
     int halo_mask;
     int lanes;                    // layout of the kernel that will read the links: 1, 2 or 4,
                                   // or 0 = tiled (the TMA kernel, bulk.cuh)
-    int recon;                    // 18 = full matrices, 12 = long links keep rows 0 and 1 only
+    int recon;                    // 18 = full matrices, 12 = long links keep rows 0 and 1 only,
+                                  // 9 = long links as 8 SU(3) parameters + a phase (stencil.cuh)
+    double s9;                    // recon-9: the long links' real scale s
     int paired;                   // 1: fp32 paired layout (link_index_paired), register kernels only
 };
 
@@ -48,6 +50,10 @@ __host__ __device__ __forceinline__ int64_t conv_index(const LinkConvParams& P, 
         return P.lanes == 1 ? link_index<1, 12>(mu, l, e, P.vh, cb)
              : P.lanes == 2 ? link_index<2, 12>(mu, l, e, P.vh, cb)
                             : link_index<4, 12>(mu, l, e, P.vh, cb);
+    if (P.recon == 9)
+        return P.lanes == 1 ? link_index<1, 9>(mu, l, e, P.vh, cb)
+             : P.lanes == 2 ? link_index<2, 9>(mu, l, e, P.vh, cb)
+                            : link_index<4, 9>(mu, l, e, P.vh, cb);
     return P.lanes == 1 ? link_index<1>(mu, l, e, P.vh, cb)
          : P.lanes == 2 ? link_index<2>(mu, l, e, P.vh, cb)
                         : link_index<4>(mu, l, e, P.vh, cb);
@@ -73,6 +79,29 @@ __device__ __forceinline__ const double2* canon_link(const LinkConvParams& P, bo
     return (is_long ? P.lng : P.fat) + (lex * 4 + mu) * 9;
 }
 
+// recon-9 compression of M = s e^{i psi} W (stencil.cuh reconstruct_9): psi = arg(det M) / 3,
+// W = e^{-i psi} M / s; P[0] = (arg W00, arg W20) / pi, P[1] = W01, P[2] = W02, P[3] = W10; the
+// returned psi is in units of pi too
+__device__ __forceinline__ void compress_9(const double2 M[9], double s, double2 P[4], double& psi) {
+    const double2 m0 = make_double2(M[4].x * M[8].x - M[4].y * M[8].y - (M[5].x * M[7].x - M[5].y * M[7].y),
+                                    M[4].x * M[8].y + M[4].y * M[8].x - (M[5].x * M[7].y + M[5].y * M[7].x));
+    const double2 m1 = make_double2(M[3].x * M[8].x - M[3].y * M[8].y - (M[5].x * M[6].x - M[5].y * M[6].y),
+                                    M[3].x * M[8].y + M[3].y * M[8].x - (M[5].x * M[6].y + M[5].y * M[6].x));
+    const double2 m2 = make_double2(M[3].x * M[7].x - M[3].y * M[7].y - (M[4].x * M[6].x - M[4].y * M[6].y),
+                                    M[3].x * M[7].y + M[3].y * M[7].x - (M[4].x * M[6].y + M[4].y * M[6].x));
+    const double2 d0 = cmul(M[0], m0), d1 = cmul(M[1], m1), d2 = cmul(M[2], m2);
+    const double dx = d0.x - d1.x + d2.x, dy = d0.y - d1.y + d2.y;
+    psi = atan2(dy, dx) / (3.0 * M_PI);  // in units of pi
+    double sp, cp;
+    sincospi(psi, &sp, &cp);
+    const double2 z = make_double2(cp / s, -sp / s);  // e^{-i pi psi} / s
+    const double2 w00 = cmul(z, M[0]), w20 = cmul(z, M[6]);
+    P[0] = make_double2(atan2(w00.y, w00.x) / M_PI, atan2(w20.y, w20.x) / M_PI);
+    P[1] = cmul(z, M[1]);
+    P[2] = cmul(z, M[2]);
+    P[3] = cmul(z, M[3]);
+}
+
 // one thread per (target site, mu, l); LR = stored real type (fp64 input rounded to LR)
 template <typename LR>
 __global__ void convert_links_kernel(const LinkConvParams P) {
@@ -93,6 +122,21 @@ __global__ void convert_links_kernel(const LinkConvParams P) {
     const bool is_long = l >= 2;
     const int back = (l == 1) ? 1 : (l == 3) ? 3 : 0;
     const double2* A = canon_link(P, is_long, mu, x, y, z, t, back);
+    if (P.recon == 9 && is_long) {
+        double2 M[9], Q[4];
+        for (int i = 0; i < 3; ++i)
+            for (int j = 0; j < 3; ++j) {
+                double2 v = back ? A[3 * j + i] : A[3 * i + j];
+                if (back) v.y = -v.y;
+                M[3 * i + j] = v;
+            }
+        double psi;
+        compress_9(M, P.s9, Q, psi);
+        for (int e = 0; e < 4; ++e) static_cast<L2*>(P.links)[conv_index(P, mu, l, e, cb)] = to_cplx<L2>(Q[e]);
+        // the psi pair: Nf's in .x, Nb's in .y
+        reinterpret_cast<LR*>(static_cast<L2*>(P.links) + conv_index(P, mu, 2, kRecon9PhaseElem, cb))[l - 2] = (LR)psi;
+        return;
+    }
     const int rows = (P.recon == 12 && is_long) ? 2 : 3;
     for (int i = 0; i < rows; ++i)
         for (int j = 0; j < 3; ++j) {
@@ -123,7 +167,8 @@ __global__ void convert_internal_kernel(const LinkConvParams S, const LinkConvPa
 }
 
 // Export (dslash_get_links): internal layout -> out[cb][mu][l][e] (double2), l = Ff, Fb, Nf, Nb.
-// With recon-12 the long matrices' row 2 is not stored: exported as zeros.
+// With recon-12 the long matrices' row 2 is not stored: exported as zeros.  With recon-9 the long
+// matrices are exported reconstructed.
 template <typename LR>
 __global__ void export_links_kernel(const LinkConvParams P, double2* out) {
     using L2 = cplx_t<LR>;
@@ -133,6 +178,14 @@ __global__ void export_links_kernel(const LinkConvParams P, double2* out) {
     const int mu = (int)(gid >> 2) & 3;
     const int l = (int)gid & 3;
     const L2* links = static_cast<const L2*>(P.links);
+    if (P.recon == 9 && l >= 2) {  // recon-9: exported reconstructed
+        double2 U[9];
+        for (int e = 0; e < 4; ++e) U[e] = widen(links[conv_index(P, mu, l, e, cb)]);
+        const double2 ph = widen(links[conv_index(P, mu, 2, kRecon9PhaseElem, cb)]);
+        reconstruct_9(U, P.s9, l == 2 ? ph.x : ph.y);
+        for (int e = 0; e < 9; ++e) out[((cb * 4 + mu) * 4 + l) * 9 + e] = U[e];
+        return;
+    }
     const int stored = (P.recon == 12 && l >= 2) ? 6 : 9;
     for (int e = 0; e < 9; ++e) {
         double2 v = make_double2(0.0, 0.0);
@@ -157,6 +210,36 @@ __global__ void recon_check_kernel(const double2* lng, int64_t nmat, double inv_
         for (int j = 0; j < 3; ++j) err = fmax(err, fmax(fabs(R[6 + j].x - U[6 + j].x), fabs(R[6 + j].y - U[6 + j].y)));
     }
     // warp max, then one atomic per warp
+    for (int off = 16; off; off >>= 1) err = fmax(err, __shfl_xor_sync(0xffffffffu, err, off));
+    if ((threadIdx.x & 31) == 0) atomicMax(max_bits, (unsigned long long)__double_as_longlong(err));
+}
+
+// recon-9 admissibility: for every canonical long link N (fp64 input) and its adjoint (the
+// back-link form), the largest entry deviation of reconstruct_9(compress_9(M)) from M; atomicMax
+// on the bits as in recon_check_kernel.  Fails where a link is not s e^{i psi} SU(3) with the
+// handle's s, or lies too near the parameterisation's singular set (|a2|^2 + |a3|^2 -> 0).
+__global__ void recon9_check_kernel(const double2* lng, int64_t nmat, double s, unsigned long long* max_bits) {
+    const int64_t m = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    double err = 0.0;
+    if (m < nmat) {
+        const double2* A = lng + m * 9;
+        for (int adj = 0; adj < 2; ++adj) {
+            double2 M[9], U[9];
+            for (int i = 0; i < 3; ++i)
+                for (int j = 0; j < 3; ++j) {
+                    double2 v = adj ? A[3 * j + i] : A[3 * i + j];
+                    if (adj) v.y = -v.y;
+                    M[3 * i + j] = v;
+                }
+            double psi;
+            compress_9(M, s, U, psi);
+            reconstruct_9(U, s, psi);
+            for (int e = 0; e < 9; ++e) {
+                const double dx = fabs(U[e].x - M[e].x), dy = fabs(U[e].y - M[e].y);
+                err = (dx == dx && dy == dy) ? fmax(err, fmax(dx, dy)) : HUGE_VAL;  // NaN (singular): reject
+            }
+        }
+    }
     for (int off = 16; off; off >>= 1) err = fmax(err, __shfl_xor_sync(0xffffffffu, err, off));
     if ((threadIdx.x & 31) == 0) atomicMax(max_bits, (unsigned long long)__double_as_longlong(err));
 }

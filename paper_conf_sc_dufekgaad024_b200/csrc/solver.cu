@@ -403,6 +403,8 @@ extern "C" dslash_status dslash_cg(dslash_t h, void* x_out, const void* b_in, in
 // The fp32 ("sloppy") links of both parities, converted once from the handle's fp64 internal
 // links into the fp32 paired layout the F32 kernels read (links.cuh convert_internal_kernel).
 static dslash_status need_sloppy(dslash_t h) {
+    if (h->recon == 9)
+        return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the mixed-precision solver's fp32 links take recon 18 or 12");
     const int64_t n = 3 * h->plan.vh_local;
     for (void*& v : h->cg_vec32)
         if (!v) CU(h, cudaMalloc(&v, n * sizeof(float2)));

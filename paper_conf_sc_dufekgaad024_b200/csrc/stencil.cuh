@@ -29,16 +29,19 @@ namespace hisq {
 // 3 = Nb (-3)) of direction mu at target site cb stores its elements e (row-major 3*i + j) at
 //   links[(((base(l) + e) * K + k) * vh + cb) * LANES + j],   K = 4 / LANES,
 // base(l) = 9 l without compression; with RECON = 12 the long matrices keep only rows 0 and 1
-// (e < 6), base(2) = 18, base(3) = 24.  At every load instruction the lanes of a warp read one
-// contiguous span, and consecutive elements of a matrix are 4*vh complex apart.
+// (e < 6), base(2) = 18, base(3) = 24; with RECON = 9 they keep 4 entries (e < 4: (arg a1,
+// arg c1), a2, a3, b1), base(2) = 18, base(3) = 22, and the pair (psi of Nf, psi of Nb) is
+// element 26 (= base(2) + 8).  At every load instruction the lanes of a warp read one contiguous
+// span, and consecutive elements of a matrix are 4*vh complex apart.
 template <int RECON>
 __host__ __device__ __forceinline__ int elem_base(int l) {
-    return (RECON == 12 && l >= 2) ? 18 + (l - 2) * 6 : l * 9;
+    return (RECON == 12 && l >= 2) ? 18 + (l - 2) * 6 : (RECON == 9 && l >= 2) ? 18 + (l - 2) * 4 : l * 9;
 }
 template <int RECON>
 __host__ __device__ __forceinline__ int elems_of(int l) {
-    return (RECON == 12 && l >= 2) ? 6 : 9;
+    return (RECON == 12 && l >= 2) ? 6 : (RECON == 9 && l >= 2) ? 4 : 9;
 }
+constexpr int kRecon9PhaseElem = 8;  // link_index<LANES, 9>(mu, 2, 8, ...) = the psi pair
 template <int LANES, int RECON = 18>
 __host__ __device__ __forceinline__ int64_t link_index(int mu, int l, int e, int64_t vh, int64_t cb) {
     constexpr int K = 4 / LANES;
@@ -70,6 +73,67 @@ __device__ __forceinline__ void reconstruct_row2(V2 U[9], R inv_s) {
         U[6 + j].x = xr * inv_s;
         U[6 + j].y = -xi * inv_s;
     }
+}
+
+// recon-9 (QUDA's 8 SU(3) parameters + one phase for the long links with folded staggered
+// phases): M = s e^{i psi} W with W in SU(3), s > 0 one real scale per handle, psi = arg(det M)/3.
+// Stored: U[0] = (arg a1, arg c1) / pi, U[1] = a2, U[2] = a3, U[3] = b1, with rows a, b, c of W,
+// and psi / pi (in the direction's psi pair).
+// Unitarity and det W = 1 give |a1|^2 = 1 - |a2|^2 - |a3|^2, |c1|^2 = |a2|^2 + |a3|^2 - |b1|^2, and
+// (rows orthogonal to a, b = conj(c x a), c = conj(a x b)), with n = |a2|^2 + |a3|^2:
+//   b2 = -(a1* b1 a2 + a3* c1*) / n,   b3 = (a2* c1* - a1* b1 a3) / n,
+//   c2 = (a3* b1* - a1* c1 a2) / n,    c3 = -(a2* b1* + a1* c1 a3) / n.
+template <typename V2>
+__device__ __forceinline__ V2 cmul(V2 a, V2 b) {
+    return V2{a.x * b.x - a.y * b.y, a.x * b.y + a.y * b.x};
+}
+template <typename V2>
+__device__ __forceinline__ V2 cconj(V2 a) {
+    return V2{a.x, -a.y};
+}
+// SCALE = false leaves U = W and only returns z = s e^{i pi psi} (the stencil multiplies the
+// 3-vector W v by z instead of the 9 entries of W)
+template <bool SCALE = true, typename V2, typename R>
+__device__ __forceinline__ V2 reconstruct_9(V2 U[9], R s, R psi) {
+    const V2 a2 = U[1], a3 = U[2], b1 = U[3];
+    const R n = a2.x * a2.x + a2.y * a2.y + a3.x * a3.x + a3.y * a3.y;
+    const R a1m = sqrt(fmax(R(1) - n, R(0)));
+    const R c1m = sqrt(fmax(n - (b1.x * b1.x + b1.y * b1.y), R(0)));
+    R sa, ca, sc, cc, sp, cp;
+    sincospi(U[0].x, &sa, &ca);  // angles are stored in units of pi: no large-argument reduction
+    sincospi(U[0].y, &sc, &cc);
+    sincospi(psi, &sp, &cp);
+    const V2 a1{a1m * ca, a1m * sa}, c1{c1m * cc, c1m * sc};
+    const R inv = R(1) / n;
+    const V2 a1b1 = cmul(cconj(a1), b1), a1c1 = cmul(cconj(a1), c1);
+    const V2 t0 = cmul(a1b1, a2), t1 = cmul(cconj(a3), cconj(c1));
+    const V2 t2 = cmul(cconj(a2), cconj(c1)), t3 = cmul(a1b1, a3);
+    const V2 t4 = cmul(cconj(a3), cconj(b1)), t5 = cmul(a1c1, a2);
+    const V2 t6 = cmul(cconj(a2), cconj(b1)), t7 = cmul(a1c1, a3);
+    const V2 b2{-(t0.x + t1.x) * inv, -(t0.y + t1.y) * inv};
+    const V2 b3{(t2.x - t3.x) * inv, (t2.y - t3.y) * inv};
+    const V2 c2{(t4.x - t5.x) * inv, (t4.y - t5.y) * inv};
+    const V2 c3{-(t6.x + t7.x) * inv, -(t6.y + t7.y) * inv};
+    const V2 z{s * cp, s * sp};
+    if (SCALE) {
+        U[0] = cmul(z, a1);
+        U[1] = cmul(z, a2);
+        U[2] = cmul(z, a3);
+        U[3] = cmul(z, b1);
+        U[4] = cmul(z, b2);
+        U[5] = cmul(z, b3);
+        U[6] = cmul(z, c1);
+        U[7] = cmul(z, c2);
+        U[8] = cmul(z, c3);
+    } else {
+        U[0] = a1;
+        U[4] = b2;
+        U[5] = b3;
+        U[6] = c1;
+        U[7] = c2;
+        U[8] = c3;
+    }
+    return z;
 }
 
 struct Site {
@@ -387,9 +451,15 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     }
                 }
             } else {
+            V2 ph9;  // recon-9: (psi of Nf, psi of Nb) of direction mu
 #pragma unroll
             for (int l = 0; l < 4; ++l) {
                 const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
+                if constexpr (RECON == 9) {
+                    if (l == 2)
+                        ph9 = to_cplx<V2>(widen(
+                            ld_stream(links + link_index<LANES, 9>(mu, 2, kRecon9PhaseElem, P.vh, s.cb), pol_stream)));
+                }
                 const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0, false} : source<V2, GHOST>(P, in, mu, h, s, rl * NRHS);
                 const uint32_t sa = stg ? staged_addr<V2>(P, T, sbase, mu, h, s, rl * NRHS) : 0u;
                 // split-by-direction passes: the ghost pass takes only the ghost hops (the link of
@@ -409,6 +479,10 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                         U[e] = to_cplx<V2>(widen(ld_stream(lp + (int64_t)e * 4 * P.vh, pol_stream)));
                 }
                 if (elems_of<RECON>(l) == 6) reconstruct_row2(U, (VR)P.long_inv_scale);
+                V2 z9;  // recon-9: N = z9 W
+                if constexpr (RECON == 9) {
+                    if (l >= 2) z9 = reconstruct_9<false>(U, (VR)P.long_scale, l == 2 ? ph9.x : ph9.y);
+                }
 #pragma unroll
                 for (int r = 0; r < NRHS; ++r) {
                     const int64_t roff = (int64_t)r * 3 * src.stride;  // [rhs][3][vh or face_vh]
@@ -419,10 +493,23 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                                       COH && src.ghost);
                         if (GHOST) zero_if(v[c], zap);
                     }
-                    if (l & 1)
+                    if (RECON == 9 && l >= 2) {
+                        V2 w[3];
+#pragma unroll
+                        for (int i = 0; i < 3; ++i) w[i].x = w[i].y = VR(0);
+                        matvec_acc<false>(w, U, v);
+#pragma unroll
+                        for (int i = 0; i < 3; ++i) {
+                            if (l & 1)
+                                cmsub(acc[r][i], z9, w[i]);
+                            else
+                                cmadd(acc[r][i], z9, w[i]);
+                        }
+                    } else if (l & 1) {
                         matvec_acc<true>(acc[r], U, v);
-                    else
+                    } else {
                         matvec_acc<false>(acc[r], U, v);
+                    }
                 }
             }
             }  // unpaired links
