@@ -451,14 +451,25 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     }
                 }
             } else {
-            V2 ph9;  // recon-9: (psi of Nf, psi of Nb) of direction mu
+            V2 ph9;       // recon-9: (psi of Nf, psi of Nb) of direction mu
+            V2 L9[2][4];  // recon-9: the stored parameters of Nf, Nb
 #pragma unroll
             for (int l = 0; l < 4; ++l) {
                 const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
                 if constexpr (RECON == 9) {
-                    if (l == 2)
+                    // the direction's long-link parameters are fetched with its first (fat) matrix,
+                    // so their latency overlaps the fat matvecs rather than the reconstruction
+                    if (l == 0) {
                         ph9 = to_cplx<V2>(widen(
                             ld_stream(links + link_index<LANES, 9>(mu, 2, kRecon9PhaseElem, P.vh, s.cb), pol_stream)));
+#pragma unroll
+                        for (int q = 0; q < 2; ++q)
+#pragma unroll
+                            for (int e = 0; e < 4; ++e)
+                                L9[q][e] = to_cplx<V2>(widen(ld_stream(
+                                    links + link_index<LANES, 9>(mu, 2 + q, 0, P.vh, s.cb) + (int64_t)e * 4 * P.vh,
+                                    pol_stream)));
+                    }
                 }
                 const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0, false} : source<V2, GHOST>(P, in, mu, h, s, rl * NRHS);
                 const uint32_t sa = stg ? staged_addr<V2>(P, T, sbase, mu, h, s, rl * NRHS) : 0u;
@@ -473,6 +484,9 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                 if (kk == 0 && l == 0 && !(GHOST && P.halo_pass == kPassGhost)) {
 #pragma unroll
                     for (int e = 0; e < 9; ++e) U[e] = U0[e];
+                } else if (RECON == 9 && l >= 2) {
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) U[e] = L9[l - 2][e];
                 } else {
 #pragma unroll
                     for (int e = 0; e < elems_of<RECON>(l); ++e)
