@@ -26,6 +26,10 @@ cases += [dict(stage=True), dict(stage=True, kernel="site", force_halo=0xC), dic
           dict(force_halo=0xC, overlap="dirs"), dict(force_halo=0xC, overlap="dirs", precision="f32"),
           dict(force_halo=0xC, overlap="fused"), dict(force_halo=0x8, overlap="fused", defer=True),
           dict(force_halo=0xC, self_nccl=True), dict(cg_mixed=True)]
+# third session: the producer push (stencil epilogue and CG direction update store into the
+# peer-mapped ghost bank; flag waits/writes on the streams) and recon-9 long links
+cases += [dict(force_halo=0xC, transport="p2p", push=True), dict(force_halo=0x8, transport="p2p", push=True, overlap="dirs"),
+          dict(recon=9), dict(recon=9, kernel="site", force_halo=0xC), dict(recon=9, stage=True)]
 n = 0
 for kw in cases:
     kw = dict(kw)
@@ -39,7 +43,8 @@ for kw in cases:
         if mixed_cg:
             x = D.empty_vector()
             D.cg_mixed(x, src[0], 0, 0.5, rel_tol=1e-8, inner_tol=1e-2, max_iter=100)
-        out = D(src[1].to(D.dtype), 0)
+        out = D.empty_vector()
+        (D.apply_push if kw.get("push") else D.apply)(out, src[1].to(D.dtype), 0)
         o2 = D.empty_vector()
         D.apply(o2, out.to(D.dtype), 1)
         multi = torch.stack([src[1], src[1]]).to(D.dtype)
