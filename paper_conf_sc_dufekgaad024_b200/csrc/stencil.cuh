@@ -186,12 +186,11 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, const void*
     if (cw >= L) cw -= L;
     if (cw >= L) cw -= L;
     int64_t idx;
+    int64_t st = 1;
     if (mu == 0) {
         idx = s.cb - s.xh + (cw >> 1);
     } else {
-        const int64_t st = mu == 1 ? (int64_t)P.lxh
-                         : mu == 2 ? (int64_t)P.lxh * P.L[1]
-                                   : (int64_t)P.lxh * P.L[1] * P.L[2];
+        st = mu == 1 ? (int64_t)P.lxh : mu == 2 ? (int64_t)P.lxh * P.L[1] : (int64_t)P.lxh * P.L[1] * P.L[2];
         idx = s.cb + (int64_t)(cw - c) * st;
     }
     const V2* local = static_cast<const V2*>(in) + (int64_t)rhs * 3 * P.vh + idx;
@@ -200,9 +199,9 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, const void*
     // different directions, so a branch here would diverge within the warp
     const bool ghost = ((P.halo_mask >> mu) & 1) && (cn < 0 || cn >= L);
     const int side = cn >= L;
-    const int d = side ? cn - L : cn + 3;
-    const int64_t f = (mu == 3) ? s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (s.z + (int64_t)P.L[2] * d))
-                                : s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (d + 3 * (int64_t)s.t));
+    // face index f of depth d = (side ? cn - L : cn + 3): t face [d][z][y][xh] = cb + st (d - t),
+    // z face [t][d][y][xh] = cb + st (d - z) + st (3 - Lz) t (st = the direction's cb stride)
+    const int64_t f = s.cb + st * (h + (side ? -L : 3)) + (mu == 2 ? st * (3 - P.L[2]) * (int64_t)s.t : 0);
     const int64_t fv = P.face_vh[mu];
     const V2* gp = static_cast<const V2*>(P.ghost[mu][side]) + (int64_t)rhs * 3 * fv + f;
     // local pass of the split-by-direction overlap: the face is still in flight, so a ghost hop
