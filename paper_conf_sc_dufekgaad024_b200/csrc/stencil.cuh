@@ -353,8 +353,15 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
     constexpr int K = 4 / LANES;
     constexpr int kFirstStaged = LANES == 1 ? 2 : 1;  // first loop step that reads the tile
     const int lane = (LANES == 1) ? 0 : (int)(gid & (LANES - 1));
-    const int rl = (RHSL == 1) ? 0 : (int)((gid / LANES) % RHSL);
-    const int64_t site = gid / (LANES * RHSL);
+    // thread -> (site, right-hand-side group).  LANES 1 x RHSL 2 in a one-dimensional grid of
+    // whole warps (not the staged kernel): each quarter-warp (8 lanes) takes 8 consecutive sites of
+    // ONE group, so a 16-byte load of a quarter-warp touches one 128-byte line (one L1 wavefront)
+    // instead of two; the warp still covers the same 16 sites
+    constexpr bool kQuarterRuns = LANES == 1 && RHSL == 2 && !STAGED;
+    const int rl = (RHSL == 1)    ? 0
+                   : kQuarterRuns ? (int)((gid >> 3) & 1)
+                                  : (int)((gid / LANES) % RHSL);
+    const int64_t site = kQuarterRuns ? ((gid >> 5) << 4) + (((gid >> 4) & 1) << 3) + (gid & 7) : gid / (LANES * RHSL);
     const bool valid = site < site_end;
     if (LANES == 1 && !valid) return;
     V2 acc[NRHS][3];
