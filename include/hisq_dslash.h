@@ -188,8 +188,11 @@ enum {
 
 /* Kernel classes for dslash_kernel_timing.  SPAN: with a halo and the classic split, the time
  * from the interior kernel's start to the join after the (overlapping, higher-priority) boundary
- * kernel, i.e. the duration of the apply's stencil work; ALL sums the kernel launches only. */
-enum { DSLASH_TIMING_INTERIOR = 0, DSLASH_TIMING_BOUNDARY = 1, DSLASH_TIMING_ALL = 2, DSLASH_TIMING_SPAN = 3 };
+ * kernel, i.e. the duration of the apply's stencil work; EXCHANGE: the halo exchange on the
+ * communication stream (NCCL send/recv, device copies or P2P copies, from the comm stream's
+ * start of the exchange to its end); ALL sums the kernel launches only. */
+enum { DSLASH_TIMING_INTERIOR = 0, DSLASH_TIMING_BOUNDARY = 1, DSLASH_TIMING_ALL = 2, DSLASH_TIMING_SPAN = 3,
+       DSLASH_TIMING_EXCHANGE = 4 };
 
 /* Host-only decomposition of the local lattice (no CUDA calls).  A "box" is
  * [lo[d], hi[d]) per dimension in local coordinates; the target-parity sites of a
@@ -377,6 +380,15 @@ DSLASH_API dslash_status dslash_sync(dslash_t h);
  * one event pair until the next reset. */
 DSLASH_API dslash_status dslash_kernel_timing(dslash_t h, int32_t which, double* total_ms, int64_t* launches);
 DSLASH_API dslash_status dslash_kernel_timing_reset(dslash_t h);
+
+/* The recorded intervals themselves, in record order (DSLASH_OPT_TIMING = 1): a timeline of
+ * kernels and exchanges across the handle's streams (the overlap of the exchange with the
+ * interior kernel, without a system profiler).  Writes up to max_entries
+ * entries: kinds[i] (DSLASH_TIMING_*), start_ms[i] and end_ms[i] relative to the start of the
+ * first recorded interval since the last reset; *n receives the number of entries recorded
+ * (may exceed max_entries).  Synchronises on the recorded events.  Host arrays, caller-owned. */
+DSLASH_API dslash_status dslash_timeline(dslash_t h, int64_t max_entries, int32_t* kinds, double* start_ms,
+                                         double* end_ms, int64_t* n);
 
 /* Copy the plan the handle uses. */
 DSLASH_API dslash_status dslash_get_plan(dslash_t h, dslash_plan_t* plan);

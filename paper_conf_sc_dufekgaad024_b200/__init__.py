@@ -277,6 +277,11 @@ class Dslash:
         """(total ms, launches) of the kernels of class `which` recorded since the last reset."""
         return _abi.dslash_kernel_timing(self.h, which)
 
+    def timeline(self, max_entries=4096):
+        """Recorded intervals in record order: [(kind name, start_ms, end_ms)] relative to the
+        first one since the last reset (timing=True): kernels, spans and halo exchanges."""
+        return [(_abi.TIMING_KINDS.get(k, k), a, b) for k, a, b in _abi.dslash_timeline(self.h, max_entries)]
+
     def kernel_timing_reset(self):
         _abi.dslash_kernel_timing_reset(self.h)
 

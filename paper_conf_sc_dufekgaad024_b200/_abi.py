@@ -31,7 +31,8 @@ DSLASH_OVERLAP_NONE, DSLASH_OVERLAP_SITES, DSLASH_OVERLAP_DIRS, DSLASH_OVERLAP_F
 OVERLAPS = {"none": DSLASH_OVERLAP_NONE, "sites": DSLASH_OVERLAP_SITES, "dirs": DSLASH_OVERLAP_DIRS,
             "fused": DSLASH_OVERLAP_FUSED}
 TRANSPORTS = {"nccl": DSLASH_TRANSPORT_NCCL, "p2p": DSLASH_TRANSPORT_P2P}
-DSLASH_TIMING_INTERIOR, DSLASH_TIMING_BOUNDARY, DSLASH_TIMING_ALL, DSLASH_TIMING_SPAN = range(4)
+DSLASH_TIMING_INTERIOR, DSLASH_TIMING_BOUNDARY, DSLASH_TIMING_ALL, DSLASH_TIMING_SPAN, DSLASH_TIMING_EXCHANGE = range(5)
+TIMING_KINDS = {0: "interior", 1: "boundary", 2: "all", 3: "span", 4: "exchange"}
 KERNELS = {"site": DSLASH_KERNEL_SITE, "dir4": DSLASH_KERNEL_DIR4, "dir2": DSLASH_KERNEL_DIR2,
            "bulk": DSLASH_KERNEL_BULK}
 
@@ -110,6 +111,8 @@ _SIGS = {
     "dslash_kernel_timing": ([_h, ctypes.c_int32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64)],
                              ctypes.c_int),
     "dslash_kernel_timing_reset": ([_h], ctypes.c_int),
+    "dslash_timeline": ([_h, ctypes.c_int64, ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_double),
+                         ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64)], ctypes.c_int),
     "dslash_get_plan": ([_h, ctypes.POINTER(dslash_plan_t)], ctypes.c_int),
     "dslash_local_half_volume": ([_h], ctypes.c_int64),
     "dslash_destroy": ([_h], ctypes.c_int),
@@ -266,6 +269,16 @@ def dslash_kernel_timing(h, which=DSLASH_TIMING_ALL):
 
 def dslash_kernel_timing_reset(h):
     return check(lib.dslash_kernel_timing_reset(h), h)
+
+
+def dslash_timeline(h, max_entries=4096):
+    """[(kind, start_ms, end_ms)] of the recorded intervals (kernels, spans, exchanges)."""
+    n = ctypes.c_int64(0)
+    kinds = (ctypes.c_int32 * max_entries)()
+    a = (ctypes.c_double * max_entries)()
+    b = (ctypes.c_double * max_entries)()
+    check(lib.dslash_timeline(h, max_entries, kinds, a, b, ctypes.byref(n)), h)
+    return [(kinds[i], a[i], b[i]) for i in range(min(n.value, max_entries))]
 
 
 def dslash_get_plan(h) -> dslash_plan_t:

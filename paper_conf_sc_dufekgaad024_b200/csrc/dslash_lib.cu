@@ -823,6 +823,10 @@ static dslash_status p2p_prepare(dslash_t h) {
 // ============================================================================ halo exchange
 static bool any_halo(const dslash_plan_t& p) { return p.halo[2] || p.halo[3]; }
 
+// an interval of class `kind` whose start is recorded on stream s now (DSLASH_OPT_TIMING; *out =
+// nullptr when timing is off); the caller records (*out)->b at its end
+static dslash_status timing_begin(dslash_t h, int kind, cudaStream_t s, dslash_s::TimedLaunch** out);
+
 // byte offset of the ghost bank that holds epoch e's faces of direction d (producer push: e & 1;
 // otherwise the single bank)
 static size_t bank_off(const dslash_s* h, int d, unsigned int e) { return (size_t)(e & 1u) * h->ghost_bank[d]; }
@@ -896,12 +900,16 @@ static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaSt
     const size_t rows = (size_t)3 * nrhs;
     CU(h, cudaEventRecord(h->ev_start, s));
     CU(h, cudaStreamWaitEvent(h->comm, h->ev_start, 0));
+    dslash_s::TimedLaunch* xt = nullptr;  // DSLASH_TIMING_EXCHANGE interval on the comm stream
+    dslash_status tst = timing_begin(h, DSLASH_TIMING_EXCHANGE, h->comm, &xt);
+    if (tst != DSLASH_OK) return tst;
     for (int d = 3; d >= 2; --d)
         if (p.halo[d])
             for (int side = 0; side < 2; ++side)
                 if (wr(h->comm, (unsigned long long)(uintptr_t)h->peer_free[d][side], e - 1, 0) != 0)
                     return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 (release) failed");
-    if (pushed) {  // no bytes to move: the neighbours raise our ready flags after their push
+    if (pushed) {
+        if (xt) CU(h, cudaEventRecord(xt->b, h->comm));  // no bytes to move: the neighbours raise our ready flags after their push
         CU(h, cudaEventRecord(h->ev_halo, h->comm));
         h->halo_pending = true;
         return DSLASH_OK;
@@ -932,6 +940,7 @@ static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaSt
             for (int side = 0; side < 2; ++side)
                 if (wr(h->comm, (unsigned long long)(uintptr_t)h->peer_ready[d][side], e, 0) != 0)
                     return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 (ready) failed");
+    if (xt) CU(h, cudaEventRecord(xt->b, h->comm));
     CU(h, cudaEventRecord(h->ev_halo, h->comm));
     h->halo_pending = true;
     return DSLASH_OK;
@@ -998,7 +1007,11 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
     const size_t rows = (size_t)3 * nrhs;  // (rhs, colour) rows of length vh
     CU(h, cudaEventRecord(h->ev_start, s));
     CU(h, cudaStreamWaitEvent(h->comm, h->ev_start, 0));
+    dslash_s::TimedLaunch* xt = nullptr;  // DSLASH_TIMING_EXCHANGE interval on the comm stream
+    dslash_status tst = timing_begin(h, DSLASH_TIMING_EXCHANGE, h->comm, &xt);
+    if (tst != DSLASH_OK) return tst;
     if (h->halo_dryrun) {  // testing aid: the stream structure of the exchange without its bytes
+        if (xt) CU(h, cudaEventRecord(xt->b, h->comm));
         CU(h, cudaEventRecord(h->ev_halo, h->comm));
         h->halo_pending = true;
         return DSLASH_OK;
@@ -1055,6 +1068,7 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
         }
         NC(h, ncclGroupEnd());
     }
+    if (xt) CU(h, cudaEventRecord(xt->b, h->comm));
     CU(h, cudaEventRecord(h->ev_halo, h->comm));
     h->halo_pending = true;
     return DSLASH_OK;
@@ -1746,8 +1760,11 @@ extern "C" dslash_status dslash_kernel_timing(dslash_t h, int32_t which, double*
     int64_t n = 0;
     for (size_t i = 0; i < h->tused; ++i) {
         const auto& t = h->tpool[i];
-        // ALL = every kernel launch (spans excluded: they cover launches already counted)
-        if (which == DSLASH_TIMING_ALL ? t.kind == DSLASH_TIMING_SPAN : t.kind != which) continue;
+        // ALL = every kernel launch (spans excluded: they cover launches already counted; exchanges
+        // are not kernels of this library)
+        if (which == DSLASH_TIMING_ALL ? (t.kind == DSLASH_TIMING_SPAN || t.kind == DSLASH_TIMING_EXCHANGE)
+                                       : t.kind != which)
+            continue;
         CU(h, cudaEventSynchronize(t.b));
         float ms = 0.f;
         CU(h, cudaEventElapsedTime(&ms, t.a, t.b));
@@ -1756,6 +1773,24 @@ extern "C" dslash_status dslash_kernel_timing(dslash_t h, int32_t which, double*
     }
     *total_ms = tot;
     *launches = n;
+    return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_timeline(dslash_t h, int64_t max_entries, int32_t* kinds, double* start_ms,
+                                         double* end_ms, int64_t* n) {
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (!n || (max_entries > 0 && (!kinds || !start_ms || !end_ms))) return fail(h, DSLASH_ERR_ARG, "NULL output");
+    *n = (int64_t)h->tused;
+    for (size_t i = 0; i < h->tused && (int64_t)i < max_entries; ++i) {
+        const auto& t = h->tpool[i];
+        CU(h, cudaEventSynchronize(t.b));
+        float a = 0.f, b = 0.f;
+        CU(h, cudaEventElapsedTime(&a, h->tpool[0].a, t.a));
+        CU(h, cudaEventElapsedTime(&b, h->tpool[0].a, t.b));
+        kinds[i] = t.kind;
+        start_ms[i] = a;
+        end_ms[i] = b;
+    }
     return DSLASH_OK;
 }
 
