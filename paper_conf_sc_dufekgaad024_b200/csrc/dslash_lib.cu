@@ -1353,7 +1353,8 @@ static dslash_status apply_persistent(dslash_t h, StencilParams K, cudaStream_t 
     A.interior_sites = isites;
     A.ntiles_int = (isites * lanes + bs - 1) / bs;
     A.ntiles_bnd = ((sites - isites) * lanes + bs - 1) / bs;
-    dslash_s::TimedLaunch* tl = nullptr;
+    // an index, not a pointer: halo_start below may grow tpool (its exchange interval)
+    size_t tl = (size_t)-1;
     if (h->timing) {
         if (h->tused == h->tpool.size()) {
             dslash_s::TimedLaunch t{};
@@ -1361,8 +1362,8 @@ static dslash_status apply_persistent(dslash_t h, StencilParams K, cudaStream_t 
             CU(h, cudaEventCreate(&t.b));
             h->tpool.push_back(t);
         }
-        tl = &h->tpool[h->tused++];
-        tl->kind = DSLASH_TIMING_ALL;
+        tl = h->tused++;
+        h->tpool[tl].kind = DSLASH_TIMING_ALL;
     }
     if (halo) {
         if (!h->halo_flag) {
@@ -1394,7 +1395,7 @@ static dslash_status apply_persistent(dslash_t h, StencilParams K, cudaStream_t 
     const int64_t cap = (int64_t)persist_occupancy(h, fn, bs) * num_sms(h);
     const int64_t want = A.ntiles_int + (halo ? A.ntiles_bnd : 0);
     const unsigned grid = (unsigned)(want < cap ? (want > 0 ? want : 1) : cap);
-    if (tl) CU(h, cudaEventRecord(tl->a, s));
+    if (tl != (size_t)-1) CU(h, cudaEventRecord(h->tpool[tl].a, s));
     fn<<<grid, bs, 0, s>>>(K, A);
     CU(h, cudaGetLastError());
     h->sched_next[2] += (unsigned long long)A.ntiles_int + 2ull * grid;
@@ -1406,7 +1407,7 @@ static dslash_status apply_persistent(dslash_t h, StencilParams K, cudaStream_t 
         clean<<<g2, bs, 0, s>>>(K, A);
         CU(h, cudaGetLastError());
     }
-    if (tl) CU(h, cudaEventRecord(tl->b, s));
+    if (tl != (size_t)-1) CU(h, cudaEventRecord(h->tpool[tl].b, s));
     return DSLASH_OK;
 }
 
