@@ -1840,6 +1840,8 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
         if (v) cudaFree(v);
     if (h->cg_partial) cudaFree(h->cg_partial);
     if (h->cg_scalar) cudaFree(h->cg_scalar);
+    if (h->cg_partial2) cudaFree(h->cg_partial2);
+    if (h->cg_bar) cudaFree(h->cg_bar);
     if (h->cg_host_rr) cudaFreeHost(h->cg_host_rr);
     for (cudaEvent_t e : h->cg_ev)
         if (e) cudaEventDestroy(e);

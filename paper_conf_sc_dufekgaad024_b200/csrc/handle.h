@@ -51,6 +51,12 @@ struct dslash_s {
     void* links32[2] = {};
     double* cg_partial = nullptr;
     double* cg_scalar = nullptr;
+    // fused CG step (one rank): the |r|^2 block partials and the grid-barrier counter with the
+    // arrivals expected by the end of the next launch's barrier
+    double* cg_partial2 = nullptr;
+    unsigned long long* cg_bar = nullptr;
+    unsigned long long cg_bar_next = 0;
+    int cg_fused = -1;  // -1: not probed yet; 0: cooperative launch unavailable; 1: fused step
     // CG host side, kept across solves (pinned allocation and event creation cost more than a
     // short solve): <r,r> per iteration, pinned; events of the lagged convergence check
     double* cg_host_rr = nullptr;

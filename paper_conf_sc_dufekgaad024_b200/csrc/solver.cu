@@ -93,6 +93,14 @@ __global__ void __launch_bounds__(kRedThreads) k_cg_update(V2* __restrict__ x, V
     if (threadIdx.x == 0) partial[blockIdx.x] = s;
 }
 
+// sum of the kRedBlocks block partials in k_finalize's order (every block of kRedThreads threads
+// gets the same bits); result valid in thread 0
+__device__ __forceinline__ double sum_partials(const double* __restrict__ partial, int n) {
+    double acc = 0.0;
+    for (int k = threadIdx.x; k < n; k += kRedThreads) acc += partial[k];
+    return block_sum(acc);
+}
+
 // element i = c * vh + cb of a [3][vh] vector: also store it into the pushed ghost faces its site
 // belongs to (F.mask != 0; the face order of the stencil kernel's push, stencil.cuh)
 template <typename V2>
@@ -122,6 +130,70 @@ __global__ void k_cg_direction(V2* __restrict__ p, const V2* __restrict__ r, con
                                const double* __restrict__ rr, int64_t n, const FacePush F) {
     using R = decltype(V2{}.x);
     const R beta = (R)((*rr != 0.0) ? *rr_new / *rr : 0.0);
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const V2 ri = r[i];
+        V2 pi = p[i];
+        pi.x = fma(beta, pi.x, ri.x);
+        pi.y = fma(beta, pi.y, ri.y);
+        p[i] = pi;
+        if (F.mask) push_element(F, i, pi);
+    }
+}
+
+// One CG step after q = A p (one rank, cooperative launch of kRedBlocks co-resident blocks):
+//   pq = sum(partial)                       (k_finalize)
+//   x += alpha p ; r -= alpha q ; |r|^2 partials -> partial2           (k_cg_update)
+//   grid barrier
+//   rr_new = sum(partial2) ; p = r + beta p (+ face push)              (k_finalize, k_cg_direction)
+// with the same per-element arithmetic, grid and reduction order as those four kernels, so the
+// iterates are bitwise the unfused ones; three launches and their gaps fewer, and r, p are
+// re-read from L2.  The barrier counter is monotonic: this launch's blocks wait for `target`.
+template <typename V2>
+__global__ void __launch_bounds__(kRedThreads) k_cg_step(V2* __restrict__ x, V2* __restrict__ r, V2* __restrict__ p,
+                                                         const V2* __restrict__ q, const double* __restrict__ rr,
+                                                         double* __restrict__ pq_out, double* __restrict__ rr_new_out,
+                                                         double stop, int64_t n, const double* __restrict__ partial,
+                                                         double* __restrict__ partial2, unsigned long long* bar,
+                                                         unsigned long long target, const FacePush F) {
+    using R = decltype(V2{}.x);
+    __shared__ double s_val;
+    double s0 = sum_partials(partial, kRedBlocks);
+    if (threadIdx.x == 0) s_val = s0;
+    __syncthreads();
+    const double pq = s_val;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *pq_out = pq;
+    const double rrv = *rr;
+    const R alpha = (R)((pq != 0.0 && rrv > stop) ? rrv / pq : 0.0);
+    double acc = 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        V2 xi = x[i], ri = r[i];
+        const V2 pi = p[i], qi = q[i];
+        xi.x = fma(alpha, pi.x, xi.x);
+        xi.y = fma(alpha, pi.y, xi.y);
+        ri.x = fma(-alpha, qi.x, ri.x);
+        ri.y = fma(-alpha, qi.y, ri.y);
+        x[i] = xi;
+        r[i] = ri;
+        acc += (double)ri.x * ri.x + (double)ri.y * ri.y;
+    }
+    const double s1 = block_sum(acc);
+    if (threadIdx.x == 0) {
+        partial2[blockIdx.x] = s1;
+        __threadfence();
+        atomicAdd(bar, 1ull);
+        unsigned long long v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(bar) : "memory");
+        } while (v < target);
+    }
+    __syncthreads();
+    const double s2 = sum_partials(partial2, kRedBlocks);
+    __syncthreads();  // s_val is reused
+    if (threadIdx.x == 0) s_val = s2;
+    __syncthreads();
+    const double rr_new = s_val;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *rr_new_out = rr_new;
+    const R beta = (R)((rrv != 0.0) ? rr_new / rrv : 0.0);
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const V2 ri = r[i];
         V2 pi = p[i];
@@ -170,11 +242,26 @@ __global__ void __launch_bounds__(kRedThreads) k_finalize(const double* __restri
 }  // namespace
 
 // ---------------------------------------------------------------------------- host helpers
+static int num_sms_solver() {
+    static int n = 0;
+    int dev = 0;
+    if (!n && (cudaGetDevice(&dev) != cudaSuccess ||
+               cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess))
+        n = 148;
+    return n;
+}
+
 static dslash_status need_scratch(dslash_t h) {
     const size_t bytes = 3 * (size_t)h->plan.vh_local * sizeof(double2);
     for (void*& v : h->cg_vec)
         if (!v) CU(h, cudaMalloc(&v, bytes));
     if (!h->cg_partial) CU(h, cudaMalloc(&h->cg_partial, kRedBlocks * sizeof(double)));
+    if (!h->cg_partial2) CU(h, cudaMalloc(&h->cg_partial2, kRedBlocks * sizeof(double)));
+    if (!h->cg_bar) {
+        CU(h, cudaMalloc(&h->cg_bar, sizeof(unsigned long long)));
+        CU(h, cudaMemset(h->cg_bar, 0, sizeof(unsigned long long)));
+        h->cg_bar_next = 0;
+    }
     if (!h->cg_scalar) CU(h, cudaMalloc(&h->cg_scalar, 4 * sizeof(double)));
     return DSLASH_OK;
 }
@@ -282,6 +369,25 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
         if (!ev[i]) CUR(cudaEventCreateWithFlags(&ev[i], cudaEventDisableTiming));
     *converged = false;
     int k = 0, kstar = 0;  // last enqueued iteration; first converged one (0: none seen yet)
+    // fused CG step: one rank (no cross-rank sum between the update and the direction), and all
+    // kRedBlocks blocks co-resident (probed once per handle); HISQ_CG_UNFUSED=1 forces the
+    // four-kernel path
+    if (h->cg_fused < 0) {
+        int occ = 0, dev = 0, coop = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev);
+        const bool ok = coop &&
+                        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_cg_step<double2>, kRedThreads, 0) ==
+                            cudaSuccess &&
+                        occ * num_sms_solver() >= kRedBlocks;
+        int occ32 = 0;
+        const bool ok32 = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ32, k_cg_step<float2>, kRedThreads, 0) ==
+                              cudaSuccess &&
+                          occ32 * num_sms_solver() >= kRedBlocks;
+        cudaGetLastError();
+        h->cg_fused = (ok && ok32 && !getenv("HISQ_CG_UNFUSED")) ? 1 : 0;
+    }
+    const bool fused = h->cg_fused == 1 && !h->nccl;
     // HISQ_CG_PROFILE=1: host time per iteration spent enqueueing vs waiting, to stderr
     static const bool prof = getenv("HISQ_CG_PROFILE") != nullptr;
     using clk = std::chrono::steady_clock;
@@ -291,6 +397,22 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
         double* rr_cur = &sc[(k - 1) & 1];
         double* rr_new = &sc[k & 1];
         if ((st = normal_apply(h, q, p, parity, m2, t, s, true)) != DSLASH_OK) break;  // q = A p
+        if (fused) {  // one rank: the rest of the step in one cooperative launch
+            FacePush fp;
+            if ((st = hisq_push_begin(h, s, &fp)) != DSLASH_OK) break;
+            h->cg_bar_next += kRedBlocks;
+            unsigned long long target = h->cg_bar_next;
+            double stop_v = stop;
+            int64_t n_v = n;
+            double* pq_slot = &sc[2];
+            const double* rr_c = rr_cur;
+            double* part = h->cg_partial;
+            double* part2 = h->cg_partial2;
+            unsigned long long* bar = h->cg_bar;
+            void* args[] = {&x, &r, &p, &q, &rr_c, &pq_slot, &rr_new, &stop_v, &n_v, &part, &part2, &bar, &target, &fp};
+            CUR(cudaLaunchCooperativeKernel((const void*)k_cg_step<V2>, kRedBlocks, kRedThreads, args, 0, s));
+            if ((st = hisq_push_end(h, s, p)) != DSLASH_OK) break;
+        } else {
         if ((st = reduce_to_slot(h, s, &sc[2])) != DSLASH_OK) break;                 // <p, q>
         k_cg_update<<<kRedBlocks, kRedThreads, 0, s>>>(x, r, p, q, rr_cur, &sc[2], stop, n, h->cg_partial);
         CUR(cudaGetLastError());
@@ -300,6 +422,7 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
         k_cg_direction<<<kRedBlocks, kRedThreads, 0, s>>>(p, r, rr_new, rr_cur, n, fp);
         CUR(cudaGetLastError());
         if ((st = hisq_push_end(h, s, p)) != DSLASH_OK) break;
+        }
         CUR(cudaMemcpyAsync(&host_rr[k], rr_new, sizeof(double), cudaMemcpyDeviceToHost, s));
         CUR(cudaEventRecord(ev[k % (kCgLag + 1)], s));
         // check iteration k - kCgLag (complete or nearly) while the later ones run
