@@ -1175,6 +1175,18 @@ static dslash_status timing_begin(dslash_t h, int kind, cudaStream_t s, dslash_s
 // touching psi or chi, stencil.cuh) or as an ordinary launch
 static cudaError_t launch_pdl(bool pdl, StencilFn fn, const StencilParams& K, unsigned grid, int bs, size_t smem,
                               cudaStream_t s) {
+    // HISQ_L1_CARVEOUT=<percent>: shared-memory carveout preference of the stencil kernels
+    // (0 = largest L1), set once per kernel; a measurement aid
+    static const char* cv = getenv("HISQ_L1_CARVEOUT");
+    if (cv) {
+        static std::vector<StencilFn> done;
+        bool seen = false;
+        for (StencilFn f : done) seen = seen || f == fn;
+        if (!seen) {
+            done.push_back(fn);
+            cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, atoi(cv));
+        }
+    }
     if (!pdl) {
         fn<<<grid, bs, smem, s>>>(K);
         return cudaGetLastError();
