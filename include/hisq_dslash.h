@@ -147,8 +147,7 @@ enum {
                                    by sites runs instead) nor the TMA kernel; 0 (default): off  */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
-                                   4 (<= 64); 1 (<= 255) for 4 right-hand sides per launch (other
-                                   launches take 2); 0 = default; any time                          */
+                                   4 (<= 64); 0 = default; any time                                    */
 };
 
 /* Overlap modes (DSLASH_OPT_OVERLAP) of an apply that exchanges a halo. */

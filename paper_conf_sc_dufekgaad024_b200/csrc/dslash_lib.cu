@@ -370,8 +370,8 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             return alloc_halo(h, kP2PMaxRhs);
         }
         case DSLASH_OPT_MIN_BLOCKS:
-            if (value != 0 && (value < 1 || value > 4))
-                return fail(h, DSLASH_ERR_ARG, "min_blocks %lld must be 0 .. 4", (long long)value);
+            if (value != 0 && (value < 2 || value > 4))
+                return fail(h, DSLASH_ERR_ARG, "min_blocks %lld must be 0, 2, 3 or 4", (long long)value);
             h->min_blocks = (int)value;
             return DSLASH_OK;
         default:

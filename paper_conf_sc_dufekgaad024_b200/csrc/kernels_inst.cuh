@@ -15,13 +15,11 @@ template <typename LR, typename VR, int LANES, bool GHOST, int RECON>
 StencilFn pick_minb(int minb, int nrhs) {
     switch (nrhs) {
         case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 2>;
-        case 4:  // MINB 1: up to 255 registers (a second link matrix in flight), half the occupancy
-            return minb == 1 ? dslash_kernel<LR, VR, LANES, GHOST, 1, RECON, 4> : dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4>;
+        case 4: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4>;
         case 8: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2>;  // 2 thread groups x 4 RHS each
         default: break;
     }
     switch (minb) {
-        case 1:  // (MINB 1 is instantiated for 4 right-hand sides only)
         case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON>;
         case 3: return dslash_kernel<LR, VR, LANES, GHOST, 3, RECON>;
         default: return dslash_kernel<LR, VR, LANES, GHOST, 4, RECON>;
