@@ -91,6 +91,8 @@ def parse():
                     help="the persistent kernel also without a halo")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-read-calibration", action="store_true",
+                    help="skip the same-run HBM read-stream calibration (2 GiB torch.sum)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="oracle CPU-baseline budget")
     return ap.parse_args()
 
@@ -463,6 +465,28 @@ def main():
                "steps": ke, "ms_per_step": float(te.item()) / ke,
                "path": "dslash_apply_host_batch (C ABI): per step pinned host psi -> device, apply, "
                        "device -> pinned host chi; copies of neighbouring steps overlap the compute"}
+
+    # calibration in the same run: the achievable HBM READ bandwidth of this GPU now,
+    # a plain reduction over a 2 GiB fp64 tensor (torch's kernel: a calibration, not the product),
+    # after the timed region; the stencil streams 98% reads, so this is its tighter ceiling
+    if roof is not None and not args.no_read_calibration:
+        try:
+            cal = torch.empty(2 ** 28, dtype=torch.float64, device="cuda").fill_(1.0)
+            for _ in range(3):
+                cal.sum()
+            torch.cuda.synchronize()
+            ca, cb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            ca.record()
+            for _ in range(10):
+                cal.sum()
+            cb.record()
+            torch.cuda.synchronize()
+            rgbs = cal.numel() * 8 * 10 / (ca.elapsed_time(cb) * 1e-3) / 1e9
+            roof["read_stream_gbs_same_run"] = round(rgbs, 1)
+            roof["frac_of_read_stream"] = round(roof["achieved"] / rgbs, 4)
+            del cal
+        except Exception as exc:  # pragma: no cover - calibration is optional
+            roof["read_stream_gbs_same_run"] = f"unavailable: {exc}"
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.global_dims:
