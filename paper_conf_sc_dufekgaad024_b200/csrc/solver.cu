@@ -400,8 +400,9 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
         if (fused) {  // one rank: the rest of the step in one cooperative launch
             FacePush fp;
             if ((st = hisq_push_begin(h, s, &fp)) != DSLASH_OK) break;
-            h->cg_bar_next += kRedBlocks;
-            unsigned long long target = h->cg_bar_next;
+            // the counter only advances once the launch is accepted (a refused launch must not
+            // leave the next one waiting for arrivals that never come)
+            unsigned long long target = h->cg_bar_next + kRedBlocks;
             double stop_v = stop;
             int64_t n_v = n;
             double* pq_slot = &sc[2];
@@ -411,6 +412,7 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
             unsigned long long* bar = h->cg_bar;
             void* args[] = {&x, &r, &p, &q, &rr_c, &pq_slot, &rr_new, &stop_v, &n_v, &part, &part2, &bar, &target, &fp};
             CUR(cudaLaunchCooperativeKernel((const void*)k_cg_step<V2>, kRedBlocks, kRedThreads, args, 0, s));
+            h->cg_bar_next = target;
             if ((st = hisq_push_end(h, s, p)) != DSLASH_OK) break;
         } else {
         if ((st = reduce_to_slot(h, s, &sc[2])) != DSLASH_OK) break;                 // <p, q>
