@@ -154,7 +154,8 @@ __global__ void __launch_bounds__(kRedThreads) k_cg_step(V2* __restrict__ x, V2*
                                                          double* __restrict__ pq_out, double* __restrict__ rr_new_out,
                                                          double stop, int64_t n, const double* __restrict__ partial,
                                                          double* __restrict__ partial2, unsigned long long* bar,
-                                                         unsigned long long target, const FacePush F) {
+                                                         unsigned long long target, double* rr_host,
+                                                         const FacePush F) {
     using R = decltype(V2{}.x);
     __shared__ double s_val;
     double s0 = sum_partials(partial, kRedBlocks);
@@ -192,7 +193,13 @@ __global__ void __launch_bounds__(kRedThreads) k_cg_step(V2* __restrict__ x, V2*
     if (threadIdx.x == 0) s_val = s2;
     __syncthreads();
     const double rr_new = s_val;
-    if (blockIdx.x == 0 && threadIdx.x == 0) *rr_new_out = rr_new;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        *rr_new_out = rr_new;
+        if (rr_host) {  // the host's copy, through the mapped pinned buffer (no copy in the stream)
+            *(volatile double*)rr_host = rr_new;
+            __threadfence_system();
+        }
+    }
     const R beta = (R)((rrv != 0.0) ? rr_new / rrv : 0.0);
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const V2 ri = r[i];
@@ -364,6 +371,8 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
         h->cg_host_cap = need;
     }
     double* host_rr = h->cg_host_rr;  // host_rr[k] = <r,r> after iteration k
+    double* host_rr_dev = nullptr;     // its device alias (pinned host memory is mapped under UVA)
+    CUR(cudaHostGetDevicePointer((void**)&host_rr_dev, host_rr, 0));
     host_rr[0] = HUGE_VAL;            // (max_iter < 1: no iteration, not converged)
     for (int i = 0; i <= kCgLag; ++i)
         if (!ev[i]) CUR(cudaEventCreateWithFlags(&ev[i], cudaEventDisableTiming));
@@ -410,7 +419,9 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
             double* part = h->cg_partial;
             double* part2 = h->cg_partial2;
             unsigned long long* bar = h->cg_bar;
-            void* args[] = {&x, &r, &p, &q, &rr_c, &pq_slot, &rr_new, &stop_v, &n_v, &part, &part2, &bar, &target, &fp};
+            double* rr_host = host_rr_dev + k;  // host_rr[k], written by the kernel
+            void* args[] = {&x,    &r,     &p,   &q,      &rr_c,    &pq_slot, &rr_new, &stop_v,
+                            &n_v,  &part,  &part2, &bar,  &target,  &rr_host, &fp};
             CUR(cudaLaunchCooperativeKernel((const void*)k_cg_step<V2>, kRedBlocks, kRedThreads, args, 0, s));
             h->cg_bar_next = target;
             if ((st = hisq_push_end(h, s, p)) != DSLASH_OK) break;
@@ -425,7 +436,7 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
         CUR(cudaGetLastError());
         if ((st = hisq_push_end(h, s, p)) != DSLASH_OK) break;
         }
-        CUR(cudaMemcpyAsync(&host_rr[k], rr_new, sizeof(double), cudaMemcpyDeviceToHost, s));
+        if (!fused) CUR(cudaMemcpyAsync(&host_rr[k], rr_new, sizeof(double), cudaMemcpyDeviceToHost, s));
         CUR(cudaEventRecord(ev[k % (kCgLag + 1)], s));
         // check iteration k - kCgLag (complete or nearly) while the later ones run
         const int j = k - kCgLag;
