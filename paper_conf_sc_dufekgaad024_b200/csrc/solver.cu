@@ -95,9 +95,10 @@ __global__ void __launch_bounds__(kRedThreads) k_cg_update(V2* __restrict__ x, V
 
 // sum of the kRedBlocks block partials in k_finalize's order (every block of kRedThreads threads
 // gets the same bits); result valid in thread 0
-__device__ __forceinline__ double sum_partials(const double* __restrict__ partial, int n) {
+// (coherent L2 loads: in the fused CG step other blocks wrote the partials during this launch)
+__device__ __forceinline__ double sum_partials(const double* partial, int n) {
     double acc = 0.0;
-    for (int k = threadIdx.x; k < n; k += kRedThreads) acc += partial[k];
+    for (int k = threadIdx.x; k < n; k += kRedThreads) acc += __ldcg(partial + k);
     return block_sum(acc);
 }
 
@@ -140,7 +141,19 @@ __global__ void k_cg_direction(V2* __restrict__ p, const V2* __restrict__ r, con
     }
 }
 
+// grid barrier of a cooperative launch (thread 0 of every block): publish this block's writes,
+// arrive, wait until the monotonic counter reaches `target`
+__device__ __forceinline__ void grid_arrive_wait(unsigned long long* bar, unsigned long long target) {
+    __threadfence();
+    atomicAdd(bar, 1ull);
+    unsigned long long v;
+    do {
+        asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(bar) : "memory");
+    } while (v < target);
+}
+
 // One CG step after q = A p (one rank, cooperative launch of kRedBlocks co-resident blocks):
+//   q = m2 p - q ; <p, q> partials -> partial ; grid barrier          (k_normal_finish)
 //   pq = sum(partial)                       (k_finalize)
 //   x += alpha p ; r -= alpha q ; |r|^2 partials -> partial2           (k_cg_update)
 //   grid barrier
@@ -150,14 +163,31 @@ __global__ void k_cg_direction(V2* __restrict__ p, const V2* __restrict__ r, con
 // re-read from L2.  The barrier counter is monotonic: this launch's blocks wait for `target`.
 template <typename V2>
 __global__ void __launch_bounds__(kRedThreads) k_cg_step(V2* __restrict__ x, V2* __restrict__ r, V2* __restrict__ p,
-                                                         const V2* __restrict__ q, const double* __restrict__ rr,
+                                                         V2* __restrict__ q, double m2, const double* __restrict__ rr,
                                                          double* __restrict__ pq_out, double* __restrict__ rr_new_out,
-                                                         double stop, int64_t n, const double* __restrict__ partial,
-                                                         double* __restrict__ partial2, unsigned long long* bar,
+                                                         double stop, int64_t n, double* partial,
+                                                         double* partial2, unsigned long long* bar,
                                                          unsigned long long target, double* rr_host,
                                                          const FacePush F) {
     using R = decltype(V2{}.x);
     __shared__ double s_val;
+    {  // q = m2 p - q and the <p, q> block partials (k_normal_finish), then a grid barrier
+        double acc0 = 0.0;
+        for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+            const V2 a = p[i];
+            V2 b = q[i];
+            b.x = (R)m2 * a.x - b.x;
+            b.y = (R)m2 * a.y - b.y;
+            q[i] = b;
+            acc0 += (double)a.x * b.x + (double)a.y * b.y;
+        }
+        const double s = block_sum(acc0);
+        if (threadIdx.x == 0) {
+            partial[blockIdx.x] = s;
+            grid_arrive_wait(bar, target - kRedBlocks);
+        }
+        __syncthreads();
+    }
     double s0 = sum_partials(partial, kRedBlocks);
     if (threadIdx.x == 0) s_val = s0;
     __syncthreads();
@@ -180,12 +210,7 @@ __global__ void __launch_bounds__(kRedThreads) k_cg_step(V2* __restrict__ x, V2*
     const double s1 = block_sum(acc);
     if (threadIdx.x == 0) {
         partial2[blockIdx.x] = s1;
-        __threadfence();
-        atomicAdd(bar, 1ull);
-        unsigned long long v;
-        do {
-            asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(bar) : "memory");
-        } while (v < target);
+        grid_arrive_wait(bar, target);
     }
     __syncthreads();
     const double s2 = sum_partials(partial2, kRedBlocks);
@@ -312,11 +337,12 @@ static dslash_status check_solver_args(dslash_t h, const void* a, const void* b,
 // q = A p, and (if partial) the block partials of Re<p, q>
 template <typename V2>
 static dslash_status normal_apply(dslash_t h, V2* q, const V2* p, int32_t parity, double m2, V2* tmp, cudaStream_t s,
-                                  bool dot) {
+                                  bool dot, bool finish = true) {
     // t = D_{1-p,p} p; with the producer push its faces go straight to the neighbours' ghosts
     dslash_status st = hisq_apply(h, tmp, p, 1 - parity, 1, s, h->push != 0);
     if (st != DSLASH_OK) return st;
     if ((st = hisq_apply(h, q, tmp, parity, 1, s)) != DSLASH_OK) return st;  // q = D_{p,1-p} t
+    if (!finish) return DSLASH_OK;  // the caller's kernel applies q = m^2 p - q (fused CG step)
     const int64_t n = 3 * h->plan.vh_local;
     k_normal_finish<<<kRedBlocks, kRedThreads, 0, s>>>(p, q, m2, n, dot ? h->cg_partial : nullptr);
     CU(h, cudaGetLastError());
@@ -405,13 +431,15 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
         const auto t0 = prof ? clk::now() : clk::time_point{};
         double* rr_cur = &sc[(k - 1) & 1];
         double* rr_new = &sc[k & 1];
-        if ((st = normal_apply(h, q, p, parity, m2, t, s, true)) != DSLASH_OK) break;  // q = A p
+        // q = A p (with the fused step, q = D D p here and m^2 p - q inside the step kernel)
+        if ((st = normal_apply(h, q, p, parity, m2, t, s, true, !fused)) != DSLASH_OK) break;
         if (fused) {  // one rank: the rest of the step in one cooperative launch
             FacePush fp;
             if ((st = hisq_push_begin(h, s, &fp)) != DSLASH_OK) break;
             // the counter only advances once the launch is accepted (a refused launch must not
             // leave the next one waiting for arrivals that never come)
-            unsigned long long target = h->cg_bar_next + kRedBlocks;
+            unsigned long long target = h->cg_bar_next + 2 * kRedBlocks;  // two barriers per launch
+            double m2_v = m2;
             double stop_v = stop;
             int64_t n_v = n;
             double* pq_slot = &sc[2];
@@ -420,8 +448,8 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
             double* part2 = h->cg_partial2;
             unsigned long long* bar = h->cg_bar;
             double* rr_host = host_rr_dev + k;  // host_rr[k], written by the kernel
-            void* args[] = {&x,    &r,     &p,   &q,      &rr_c,    &pq_slot, &rr_new, &stop_v,
-                            &n_v,  &part,  &part2, &bar,  &target,  &rr_host, &fp};
+            void* args[] = {&x,    &r,    &p,     &q,   &m2_v,   &rr_c,    &pq_slot, &rr_new,
+                            &stop_v, &n_v, &part, &part2, &bar, &target, &rr_host, &fp};
             CUR(cudaLaunchCooperativeKernel((const void*)k_cg_step<V2>, kRedBlocks, kRedThreads, args, 0, s));
             h->cg_bar_next = target;
             if ((st = hisq_push_end(h, s, p)) != DSLASH_OK) break;
