@@ -342,7 +342,9 @@ DSLASH_API dslash_status dslash_normal_apply(dslash_t h, void* out, const void* 
 
 /* Conjugate gradient for A_p x = b (A_p as above), starting from x = 0, stopping when
  * |r_k| <= rel_tol |b| or after max_iter iterations.  Dot products are reduced
- * deterministically on each GPU and summed over ranks with ncclAllReduce.  Synchronous:
+ * deterministically on each GPU and summed over ranks with ncclAllReduce.  With one rank the
+ * vector work of an iteration (m^2 p - q, both dot products, the x / r / p updates) runs as one
+ * cooperative kernel with the same arithmetic and reduction order (bitwise the same iterates).  Synchronous:
  * returns after the solve (it reads each dot product on the host).  iters (may be NULL)
  * receives the iteration count, rel_resid (may be NULL) the TRUE relative residual
  * |b - A x| / |b| recomputed at the end.  Returns DSLASH_ERR_NOT_CONVERGED (not sticky) if the
