@@ -89,7 +89,7 @@ def _single(gdims, kw, parity, nrhs=1):
     import torch
     from paper_conf_sc_dufekgaad024_b200 import Dslash
     fat, lng = fieldgen.workload_links(gdims)
-    with Dslash(gdims, **(kw or {})) as D:
+    with Dslash(gdims, **{k: v for k, v in (kw or {}).items() if k != "push"}) as D:   # push: a P2P option
         D.load_links(fat, lng)
         outs = [D(torch.from_numpy(fieldgen.vector_cb(gdims, SEED + r, 1 - parity)).cuda(), parity).cpu().numpy()
                 for r in range(nrhs)]
@@ -111,7 +111,8 @@ def test_multirank_p2p_bitwise(gdims, grid, persistent):   # True = persistent k
         assert oracle.normwise_error(got[0], o) <= 1e-12
 
 
-@pytest.mark.parametrize("kw", [{"kernel": "site"}, {"kernel": "dir4", "recon": 12}, {"precision": "mixed"}])
+@pytest.mark.parametrize("kw", [{"kernel": "site"}, {"kernel": "dir4", "recon": 12}, {"precision": "mixed"},
+                                {"kernel": "site", "recon": 9}, {"recon": 9, "push": True}])
 def test_multirank_p2p_variants(kw):
     gdims, grid = (8, 8, 8, 16), (1, 1, 1, 2)
     got = _run(2, gdims, grid, kw, 1)
