@@ -43,7 +43,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=2000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--kernel", default="dir2", choices=["site", "dir2", "dir4", "bulk"])
+    ap.add_argument("--kernel", default=None, choices=["site", "dir2", "dir4", "bulk"],
+                    help="default: dir2 (site with --recon 9, measured best for it)")
     ap.add_argument("--min-blocks", type=int, default=0)
     ap.add_argument("--nrhs", type=int, default=1, choices=[1, 2, 3, 4, 5, 6, 7, 8],
                     help="right-hand sides per apply, one link pass (SURVEY §8(f)-4)")
@@ -94,7 +95,10 @@ def parse():
     ap.add_argument("--no-read-calibration", action="store_true",
                     help="skip the same-run HBM read-stream calibration (2 GiB torch.sum)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="oracle CPU-baseline budget")
-    return ap.parse_args()
+    args = ap.parse_args()
+    if args.kernel is None:
+        args.kernel = "site" if args.recon == 9 else "dir2"
+    return args
 
 
 def workload(args, world):
