@@ -97,8 +97,9 @@ enum {
                                    per handle) stored as the 8 parameters of W (arg a1, arg c1, a2,
                                    a3, b1) + psi, rebuilt in registers (QUDA "recon-9"; accepts
                                    folded staggered signs and U(1) phases).  fp64 register kernels
-                                   only (DSLASH_ERR_UNSUPPORTED for F32 / MIXED / the TMA kernel
-                                   and dslash_cg_mixed); load_links verifies that every long link
+                                   only (DSLASH_ERR_UNSUPPORTED for F32 / MIXED / the TMA kernel;
+                                   dslash_cg_mixed's fp32 copies are rebuilt in full); load_links
+                                   verifies that every long link
                                    is rebuilt within 1e-12 s, which also rejects links near the
                                    parameterisation's singular set |a2|^2 + |a3|^2 -> 0 (e.g.
                                    multiples of the identity): DSLASH_ERR_ARG.

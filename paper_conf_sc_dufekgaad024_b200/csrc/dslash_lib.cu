@@ -649,11 +649,13 @@ dslash_status hisq_convert_links_sloppy(dslash_t h, int parity) {
     S.vh = p.vh_local;
     S.lanes = lanes_of(h->kernel);
     S.recon = h->recon;
+    S.s9 = h->long_scale;
     S.paired = 0;
     S.parity = parity;
     S.links = h->links[parity];
     LinkConvParams D = S;
     D.paired = 1;
+    if (h->recon == 9) D.recon = 18;  // the fp32 kernels take recon-9 links rebuilt in full
     D.links = h->links32[parity];
     const int64_t n = p.vh_local * 16;
     convert_internal_kernel<<<(unsigned)((n + 255) / 256), 256>>>(S, D);

@@ -153,13 +153,23 @@ __global__ void convert_links_kernel(const LinkConvParams P) {
 }
 
 // fp64 internal layout S -> fp32 layout D (the mixed-precision solver's sloppy links, rounded
-// once): same (mu, l, e) entries, D usually the paired fp32 layout of the same lane mapping.
+// once): same (mu, l, e) entries, D usually the paired fp32 layout of the same lane mapping; a
+// recon-9 source is rebuilt and stored in full (D.recon = 18).
 __global__ void convert_internal_kernel(const LinkConvParams S, const LinkConvParams D) {
     const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (gid >= S.vh * 16) return;
     const int64_t cb = gid >> 4;
     const int mu = (int)(gid >> 2) & 3;
     const int l = (int)gid & 3;
+    if (S.recon == 9 && l >= 2) {  // recon-9 source: rebuilt in fp64, stored in full (D.recon 18)
+        const double2* src = static_cast<const double2*>(S.links);
+        double2 U[9];
+        for (int e = 0; e < 4; ++e) U[e] = src[conv_index(S, mu, l, e, cb)];
+        const double2 ph = src[conv_index(S, mu, 2, kRecon9PhaseElem, cb)];
+        reconstruct_9(U, S.s9, l == 2 ? ph.x : ph.y);
+        for (int e = 0; e < 9; ++e) static_cast<float2*>(D.links)[conv_index(D, mu, l, e, cb)] = to_cplx<float2>(U[e]);
+        return;
+    }
     const int stored = (S.recon == 12 && l >= 2) ? 6 : 9;
     for (int e = 0; e < stored; ++e)
         static_cast<float2*>(D.links)[conv_index(D, mu, l, e, cb)] =

@@ -567,14 +567,14 @@ extern "C" dslash_status dslash_cg(dslash_t h, void* x_out, const void* b_in, in
 // The fp32 ("sloppy") links of both parities, converted once from the handle's fp64 internal
 // links into the fp32 paired layout the F32 kernels read (links.cuh convert_internal_kernel).
 static dslash_status need_sloppy(dslash_t h) {
-    if (h->recon == 9)
-        return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the mixed-precision solver's fp32 links take recon 18 or 12");
     const int64_t n = 3 * h->plan.vh_local;
     for (void*& v : h->cg_vec32)
         if (!v) CU(h, cudaMalloc(&v, n * sizeof(float2)));
     if (h->links32[0]) return DSLASH_OK;
     for (int par = 0; par < 2; ++par) {
-        CU(h, cudaMalloc(&h->links32[par], h->link_bytes / 2));
+        // fp32 paired links of the same recon (recon-9 links are stored in full: 144 entries)
+        const size_t bytes32 = h->recon == 9 ? (size_t)h->plan.vh_local * 144 * sizeof(float2) : h->link_bytes / 2;
+        CU(h, cudaMalloc(&h->links32[par], bytes32));
         dslash_status st = hisq_convert_links_sloppy(h, par);
         if (st != DSLASH_OK) return st;
     }
@@ -585,17 +585,19 @@ static dslash_status need_sloppy(dslash_t h) {
 // rank does the same, so halo messages keep matching sizes.
 struct SloppyScope {
     dslash_t h;
-    int precision;
+    int precision, recon;
     void* links[2];
-    explicit SloppyScope(dslash_t hh) : h(hh), precision(hh->precision) {
+    explicit SloppyScope(dslash_t hh) : h(hh), precision(hh->precision), recon(hh->recon) {
         links[0] = h->links[0];
         links[1] = h->links[1];
         h->precision = DSLASH_F32;
+        if (h->recon == 9) h->recon = 18;  // the fp32 copies of recon-9 links are stored in full
         h->links[0] = h->links32[0];
         h->links[1] = h->links32[1];
     }
     ~SloppyScope() {
         h->precision = precision;
+        h->recon = recon;
         h->links[0] = links[0];
         h->links[1] = links[1];
     }

@@ -143,7 +143,7 @@ def test_recon9_rejections(torch_cuda):
             with pytest.raises(_abi.DslashError) as e:
                 D.load_links(fat, bad)
             assert e.value.status == _abi.DSLASH_ERR_ARG
-    for kw in ({"precision": "f32"}, {"precision": "mixed"}, {"kernel": "bulk"}):
+    for kw in ({"precision": "f32"}, {"precision": "mixed"}, {"kernel": "bulk"}):   # fp64 register kernels only
         d16 = (16, 8, 8, 8)   # the TMA kernel needs Lx / 2 to be a multiple of 8
         with Dslash(d16, recon=9, **kw) as D:
             fat, lng = fieldgen.links(d16, 1), fieldgen.links(d16, 2, scale=fieldgen.LONG_SCALE)
@@ -156,8 +156,29 @@ def test_recon9_rejections(torch_cuda):
     with Dslash(dims, recon=9) as D:
         D.load_links(fat, lng)
         b = torch.from_numpy(fieldgen.vector_cb(dims, 4, 0)).cuda()
-        with pytest.raises(_abi.DslashError) as e:
-            D.cg_mixed(D.empty_vector(), b, 0, 0.3)
-        assert e.value.status == _abi.DSLASH_ERR_UNSUPPORTED
         ok, it, res = D.cg(D.empty_vector(), b, 0, 0.3, rel_tol=1e-10)   # the fp64 solver runs
         assert ok and res <= 2e-10
+
+
+@pytest.mark.gpu
+def test_recon9_mixed_cg(torch_cuda):
+    """Mixed-precision CG on a recon-9 handle: the fp32 sloppy links are the recon-9 links rebuilt
+    in fp64 and rounded once, stored in full; the answer solves the fp64 system like recon 18's."""
+    torch = torch_cuda
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 8, 8, 12)
+    fat = fieldgen.links(dims, 1)
+    lng = _phased_long_links(dims, 6)
+    b = torch.from_numpy(fieldgen.vector_cb(dims, 7, 1)).cuda()
+    sols = {}
+    for recon in (18, 9):
+        with Dslash(dims, recon=recon) as D:
+            D.load_links(fat, lng)
+            x = D.empty_vector()
+            ok, it, outer, res = D.cg_mixed(x, b, 1, 0.3, rel_tol=1e-11, inner_tol=1e-3)
+            assert ok and res <= 1e-11, (recon, res)
+            x2 = D.empty_vector()
+            D.cg(x2, b, 1, 0.3, rel_tol=1e-12)
+            sols[recon] = (x.cpu().numpy(), x2.cpu().numpy())
+    assert oracle.normwise_error(sols[9][0], sols[18][1]) <= 1e-9
+    assert oracle.normwise_error(sols[9][1], sols[18][1]) <= 1e-10
