@@ -96,8 +96,8 @@ enum {
                                    9: each long matrix M = s e^{i psi} W (W in SU(3), one real s
                                    per handle) stored as the 8 parameters of W (arg a1, arg c1, a2,
                                    a3, b1) + psi, rebuilt in registers (QUDA "recon-9"; accepts
-                                   folded staggered signs and U(1) phases).  fp64 register kernels
-                                   only (DSLASH_ERR_UNSUPPORTED for F32 / MIXED / the TMA kernel;
+                                   folded staggered signs and U(1) phases).  Register kernels, all
+                                   precisions (DSLASH_ERR_UNSUPPORTED for the TMA kernel;
                                    dslash_cg_mixed's fp32 copies are rebuilt in full); load_links
                                    verifies that every long link
                                    is rebuilt within 1e-12 s, which also rejects links near the

@@ -28,8 +28,10 @@ def algo_bytes(precision="f64", recon=18, nrhs=1):
     output)."""
     lb = 16 if precision == "f64" else 8
     vb = 8 if precision == "f32" else 16
-    # recon-9: 4 entries per long matrix + one (psi_f, psi_b) entry per direction
-    link_entries = 8 * 9 + (8 * 6 if recon == 12 else 8 * 4 + 4 if recon == 9 else 8 * 9)
+    # recon-9: 4 entries per long matrix + the (psi_f, psi_b) pair per direction (one complex
+    # entry in fp64, a whole float4 = two complex entries in the fp32 paired layout)
+    r9 = 8 * 4 + (4 if precision == "f64" else 8)
+    link_entries = 8 * 9 + (8 * 6 if recon == 12 else r9 if recon == 9 else 8 * 9)
     return link_entries * lb + nrhs * 2 * 3 * vb
 
 __all__ = ["Dslash", "DslashError", "dslash_plan", "FLOP_PER_SITE", "ALGO_BYTES_PER_SITE"]

@@ -18,7 +18,9 @@ StencilFn pick_f32_r18(bool ghost, int lanes, int minb, int nrhs);
 StencilFn pick_f32_r12(bool ghost, int lanes, int minb, int nrhs);
 StencilFn pick_mixed_r18(bool ghost, int lanes, int minb, int nrhs);
 StencilFn pick_mixed_r12(bool ghost, int lanes, int minb, int nrhs);
-StencilFn pick_f64_r9(bool ghost, int lanes, int minb, int nrhs);  // recon-9: fp64 only
+StencilFn pick_f64_r9(bool ghost, int lanes, int minb, int nrhs);
+StencilFn pick_f32_r9(bool ghost, int lanes, int minb, int nrhs);
+StencilFn pick_mixed_r9(bool ghost, int lanes, int minb, int nrhs);
 
 // the neighbour-staged kernel (stencil.cuh dslash_stage_kernel) of one (precision, recon): lanes 1/2
 StencilFn pick_f64_r18_stage(bool ghost, int lanes, int nrhs);
@@ -28,6 +30,8 @@ StencilFn pick_f32_r12_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_mixed_r18_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_mixed_r12_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_f64_r9_stage(bool ghost, int lanes, int nrhs);
+StencilFn pick_f32_r9_stage(bool ghost, int lanes, int nrhs);
+StencilFn pick_mixed_r9_stage(bool ghost, int lanes, int nrhs);
 
 // the one-shot fused kernel (stencil.cuh dslash_fused_kernel / _cleanup) of one (precision, recon)
 typedef void (*FusedFn)(StencilParams, FusedArgs);
@@ -38,6 +42,8 @@ FusedFn pick_f32_r12_fused(bool cleanup, int lanes);
 FusedFn pick_mixed_r18_fused(bool cleanup, int lanes);
 FusedFn pick_mixed_r12_fused(bool cleanup, int lanes);
 FusedFn pick_f64_r9_fused(bool cleanup, int lanes);
+FusedFn pick_f32_r9_fused(bool cleanup, int lanes);
+FusedFn pick_mixed_r9_fused(bool cleanup, int lanes);
 
 // the persistent fused kernel (stencil.cuh) of one (precision, recon): lanes 1/2/4; mode 0 = no
 // halo, 1 = halo (interior, then boundary tiles if the faces have landed), 2 = boundary clean-up
@@ -48,6 +54,8 @@ PersistFn persist_f32_r12(int mode, int lanes);
 PersistFn persist_mixed_r18(int mode, int lanes);
 PersistFn persist_mixed_r12(int mode, int lanes);
 PersistFn persist_f64_r9(int mode, int lanes);
+PersistFn persist_f32_r9(int mode, int lanes);
+PersistFn persist_mixed_r9(int mode, int lanes);
 
 // The TMA-staged persistent kernel (bulk.cuh): function, dynamic shared memory, threads per CTA,
 // sites per tile.  precision: 0 fp64, 1 fp32, 2 mixed (DSLASH_F64/F32/MIXED).

@@ -394,8 +394,8 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
                                      const void* const* slab_lng_in, int32_t on_device, dslash_stream_t stream) {
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!fat || !lng) return fail(h, DSLASH_ERR_ARG, "NULL link pointer");
-    if (h->recon == 9 && (h->precision != DSLASH_F64 || h->kernel == DSLASH_KERNEL_BULK))
-        return fail(h, DSLASH_ERR_UNSUPPORTED, "recon-9 serves fp64 links and the register kernels (site/dir2/dir4)");
+    if (h->recon == 9 && h->kernel == DSLASH_KERNEL_BULK)
+        return fail(h, DSLASH_ERR_UNSUPPORTED, "recon-9 serves the register kernels (site/dir2/dir4)");
     cudaStream_t s = (cudaStream_t)stream;
     const dslash_plan_t& p = h->plan;
     const int64_t V = 2 * p.vh_local;
@@ -601,7 +601,11 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
         }
         h->long_inv_scale = 1.0 / sc;
     }
-    const size_t link_bytes = (size_t)p.vh_local * (h->recon == 12 ? 120 : h->recon == 9 ? 108 : 144) * link_elem(h);
+    // complex entries per target site: 4 mu x (18 fat + long: 18 / 12 / recon-9 8 + the psi entry;
+    // the fp32 paired layout gives the psi pair a whole float4)
+    const int r9_entries = h->precision == DSLASH_F64 ? 108 : 112;
+    const size_t link_bytes =
+        (size_t)p.vh_local * (h->recon == 12 ? 120 : h->recon == 9 ? r9_entries : 144) * link_elem(h);
     for (int par = 0; par < 2; ++par)  // a recon change alters the size: reallocate
         if (h->links[par] && h->link_bytes != link_bytes) {
             cudaFree(h->links[par]);
@@ -1122,7 +1126,10 @@ static void fill_boxes(StencilParams& K, const dslash_box_t* boxes, int n) {
 template <bool GHOST>
 static StencilFn pick_kernel(int precision, int recon, int lanes, int minb, int nrhs) {
     const bool r12 = recon == 12;
-    if (recon == 9) return pick_f64_r9(GHOST, lanes, minb, nrhs);  // fp64 only (load_links checks)
+    if (recon == 9)
+        return precision == DSLASH_F32     ? pick_f32_r9(GHOST, lanes, minb, nrhs)
+               : precision == DSLASH_MIXED ? pick_mixed_r9(GHOST, lanes, minb, nrhs)
+                                           : pick_f64_r9(GHOST, lanes, minb, nrhs);
     switch (precision) {
         case DSLASH_F32: return r12 ? pick_f32_r12(GHOST, lanes, minb, nrhs) : pick_f32_r18(GHOST, lanes, minb, nrhs);
         case DSLASH_MIXED: return r12 ? pick_mixed_r12(GHOST, lanes, minb, nrhs) : pick_mixed_r18(GHOST, lanes, minb, nrhs);
@@ -1137,7 +1144,10 @@ static int default_minb(int lanes) { return lanes == 4 ? 2 : 2; }
 
 static StencilFn pick_stage_kernel(int precision, int recon, bool ghost, int lanes, int nrhs) {
     const bool r12 = recon == 12;
-    if (recon == 9) return pick_f64_r9_stage(ghost, lanes, nrhs);
+    if (recon == 9)
+        return precision == DSLASH_F32     ? pick_f32_r9_stage(ghost, lanes, nrhs)
+               : precision == DSLASH_MIXED ? pick_mixed_r9_stage(ghost, lanes, nrhs)
+                                           : pick_f64_r9_stage(ghost, lanes, nrhs);
     switch (precision) {
         case DSLASH_F32:
             return r12 ? pick_f32_r12_stage(ghost, lanes, nrhs) : pick_f32_r18_stage(ghost, lanes, nrhs);
@@ -1334,7 +1344,10 @@ static int persist_occupancy(dslash_t h, PersistFn fn, int bs) {
 
 static PersistFn pick_persist(int precision, int recon, int mode, int lanes) {
     const bool r12 = recon == 12;
-    if (recon == 9) return persist_f64_r9(mode, lanes);
+    if (recon == 9)
+        return precision == DSLASH_F32     ? persist_f32_r9(mode, lanes)
+               : precision == DSLASH_MIXED ? persist_mixed_r9(mode, lanes)
+                                           : persist_f64_r9(mode, lanes);
     switch (precision) {
         case DSLASH_F32: return r12 ? persist_f32_r12(mode, lanes) : persist_f32_r18(mode, lanes);
         case DSLASH_MIXED: return r12 ? persist_mixed_r12(mode, lanes) : persist_mixed_r18(mode, lanes);
@@ -1427,7 +1440,10 @@ static dslash_status apply_persistent(dslash_t h, StencilParams K, cudaStream_t 
 
 static FusedFn pick_fused_kernel(int precision, int recon, bool cleanup, int lanes) {
     const bool r12 = recon == 12;
-    if (recon == 9) return pick_f64_r9_fused(cleanup, lanes);
+    if (recon == 9)
+        return precision == DSLASH_F32     ? pick_f32_r9_fused(cleanup, lanes)
+               : precision == DSLASH_MIXED ? pick_mixed_r9_fused(cleanup, lanes)
+                                           : pick_f64_r9_fused(cleanup, lanes);
     switch (precision) {
         case DSLASH_F32: return r12 ? pick_f32_r12_fused(cleanup, lanes) : pick_f32_r18_fused(cleanup, lanes);
         case DSLASH_MIXED: return r12 ? pick_mixed_r12_fused(cleanup, lanes) : pick_mixed_r18_fused(cleanup, lanes);

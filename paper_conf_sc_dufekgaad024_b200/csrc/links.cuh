@@ -133,8 +133,10 @@ __global__ void convert_links_kernel(const LinkConvParams P) {
         double psi;
         compress_9(M, P.s9, Q, psi);
         for (int e = 0; e < 4; ++e) static_cast<L2*>(P.links)[conv_index(P, mu, l, e, cb)] = to_cplx<L2>(Q[e]);
-        // the psi pair: Nf's in .x, Nb's in .y
-        reinterpret_cast<LR*>(static_cast<L2*>(P.links) + conv_index(P, mu, 2, kRecon9PhaseElem, cb))[l - 2] = (LR)psi;
+        if (P.paired)  // fp32 paired: entry 4 of the pair holds (psi_f, 0, psi_b, 0)
+            static_cast<L2*>(P.links)[conv_index(P, mu, l, 4, cb)] = to_cplx<L2>(make_double2(psi, 0.0));
+        else  // the psi pair: Nf's in .x, Nb's in .y
+            reinterpret_cast<LR*>(static_cast<L2*>(P.links) + conv_index(P, mu, 2, kRecon9PhaseElem, cb))[l - 2] = (LR)psi;
         return;
     }
     const int rows = (P.recon == 12 && is_long) ? 2 : 3;
@@ -191,8 +193,14 @@ __global__ void export_links_kernel(const LinkConvParams P, double2* out) {
     if (P.recon == 9 && l >= 2) {  // recon-9: exported reconstructed
         double2 U[9];
         for (int e = 0; e < 4; ++e) U[e] = widen(links[conv_index(P, mu, l, e, cb)]);
-        const double2 ph = widen(links[conv_index(P, mu, 2, kRecon9PhaseElem, cb)]);
-        reconstruct_9(U, P.s9, l == 2 ? ph.x : ph.y);
+        double psi;
+        if (P.paired) {
+            psi = widen(links[conv_index(P, mu, l, 4, cb)]).x;
+        } else {
+            const double2 ph = widen(links[conv_index(P, mu, 2, kRecon9PhaseElem, cb)]);
+            psi = l == 2 ? ph.x : ph.y;
+        }
+        reconstruct_9(U, P.s9, psi);
         for (int e = 0; e < 9; ++e) out[((cb * 4 + mu) * 4 + l) * 9 + e] = U[e];
         return;
     }

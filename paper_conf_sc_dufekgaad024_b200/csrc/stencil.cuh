@@ -410,6 +410,12 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                 // fp32 links, paired layout: one 16-byte load feeds the forward and the backward
                 // matrix of a kind; the FMA order is that of the unpaired loop (l = 0, 1, 2, 3)
                 const float4* links4 = static_cast<const float4*>(P.links);
+                float4 L9w[5];  // recon-9: the long pair's entries, fetched with the fat pair (latency)
+                if constexpr (RECON == 9) {
+                    const float4* lq = links4 + link_index_paired<LANES>(mu, 1, 0, P.vh, s.cb);
+#pragma unroll
+                    for (int e = 0; e < 5; ++e) L9w[e] = ld_stream(lq + (int64_t)e * 4 * P.vh, pol_stream);
+                }
 #pragma unroll
                 for (int j = 0; j < 2; ++j) {
                     const int hop = j ? 3 : 1;
@@ -424,13 +430,21 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     V2 Ua[9], Ub[9];
 #pragma unroll
                     for (int e = 0; e < elems_of<RECON>(2 * j); ++e) {
-                        const float4 w = ld_stream(lp + (int64_t)e * 4 * P.vh, pol_stream);
+                        const float4 w = (RECON == 9 && j == 1) ? L9w[e] : ld_stream(lp + (int64_t)e * 4 * P.vh, pol_stream);
                         Ua[e] = to_cplx<V2>(widen(make_float2(w.x, w.y)));
                         Ub[e] = to_cplx<V2>(widen(make_float2(w.z, w.w)));
                     }
                     if (elems_of<RECON>(2 * j) == 6) {
                         reconstruct_row2(Ua, (VR)P.long_inv_scale);
                         reconstruct_row2(Ub, (VR)P.long_inv_scale);
+                    }
+                    V2 za, zb;  // recon-9: Nf = za Wa, Nb = zb Wb (the psi pair is entry 4: (psi_f, 0, psi_b, 0))
+                    if constexpr (RECON == 9) {
+                        if (j == 1) {
+                            const float4 w = L9w[4];
+                            za = reconstruct_9<false>(Ua, (VR)P.long_scale, (VR)w.x);
+                            zb = reconstruct_9<false>(Ub, (VR)P.long_scale, (VR)w.z);
+                        }
                     }
 #pragma unroll
                     for (int sub = 0; sub < 2; ++sub) {
@@ -449,10 +463,23 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                                               pol_keep, COH && src.ghost);
                                 if (GHOST) zero_if(v[c], zap);
                             }
-                            if (sub)
+                            if (RECON == 9 && j == 1) {
+                                V2 w3[3];
+#pragma unroll
+                                for (int i = 0; i < 3; ++i) w3[i].x = w3[i].y = VR(0);
+                                matvec_acc<false>(w3, sub ? Ub : Ua, v);
+#pragma unroll
+                                for (int i = 0; i < 3; ++i) {
+                                    if (sub)
+                                        cmsub(acc[r][i], zb, w3[i]);
+                                    else
+                                        cmadd(acc[r][i], za, w3[i]);
+                                }
+                            } else if (sub) {
                                 matvec_acc<true>(acc[r], Ub, v);
-                            else
+                            } else {
                                 matvec_acc<false>(acc[r], Ua, v);
+                            }
                         }
                     }
                 }

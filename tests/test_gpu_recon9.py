@@ -23,6 +23,7 @@ def test_recon9_algorithmic_bytes():
     from paper_conf_sc_dufekgaad024_b200 import algo_bytes
     assert algo_bytes("f64", 9) == 1824 and algo_bytes("f64", 12) == 2016 and algo_bytes("f64", 18) == 2400
     assert algo_bytes("f64", 9, nrhs=4) == 1728 + 4 * 96
+    assert algo_bytes("f32", 9) == 896 + 48 and algo_bytes("mixed", 9) == 896 + 96
 
 
 def _phased_long_links(dims, seed=2):
@@ -55,6 +56,29 @@ def test_recon9_vs_oracle(torch_cuda, kernel, dims):
             src = torch.from_numpy(fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 1 - parity)).cuda()
             got = D(src, parity).cpu().numpy()
             assert oracle.normwise_error(got, ref) <= 1e-12
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("kernel", KERNELS)
+@pytest.mark.parametrize("precision", ["f32", "mixed"])
+def test_recon9_reduced_precision_vs_oracle(torch_cuda, kernel, precision):
+    """fp32 paired layout: the recon-9 parameters rounded to fp32, (psi_f, 0, psi_b, 0) in one
+    float4; rebuilt in fp32 (f32) or fp64 (mixed); 1e-5 against the fp64 oracle, and the error is
+    above fp64 rounding (reduced precision really ran)."""
+    torch = torch_cuda
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 10, 12, 14)
+    fat = fieldgen.links(dims, 1)
+    lng = _phased_long_links(dims, 8)
+    psi = fieldgen.vector(dims, 9)
+    with Dslash(dims, kernel=kernel, recon=9, precision=precision) as D:
+        D.load_links(fat, lng)
+        for parity in (0, 1):
+            ref = oracle.full_to_cb(oracle.dslash(fat, lng, psi, parity), parity)
+            src = torch.from_numpy(fieldgen.vector_cb(dims, 9, 1 - parity)).to(D.dtype).cuda()
+            got = D(src, parity).cpu().numpy().astype(np.complex128)
+            err = oracle.normwise_error(got, ref)
+            assert 1e-12 < err <= 1e-5, err
 
 
 @pytest.mark.gpu
@@ -143,7 +167,7 @@ def test_recon9_rejections(torch_cuda):
             with pytest.raises(_abi.DslashError) as e:
                 D.load_links(fat, bad)
             assert e.value.status == _abi.DSLASH_ERR_ARG
-    for kw in ({"precision": "f32"}, {"precision": "mixed"}, {"kernel": "bulk"}):   # fp64 register kernels only
+    for kw in ({"kernel": "bulk"}, {"kernel": "bulk", "precision": "f32"}):   # the register kernels only
         d16 = (16, 8, 8, 8)   # the TMA kernel needs Lx / 2 to be a multiple of 8
         with Dslash(d16, recon=9, **kw) as D:
             fat, lng = fieldgen.links(d16, 1), fieldgen.links(d16, 2, scale=fieldgen.LONG_SCALE)
