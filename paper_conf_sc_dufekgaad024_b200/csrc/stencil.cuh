@@ -441,9 +441,23 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     V2 za, zb;  // recon-9: Nf = za Wa, Nb = zb Wb (the psi pair is entry 4: (psi_f, 0, psi_b, 0))
                     if constexpr (RECON == 9) {
                         if (j == 1) {
-                            const float4 w = L9w[4];
-                            za = reconstruct_9<false>(Ua, (VR)P.long_scale, (VR)w.x);
-                            zb = reconstruct_9<false>(Ub, (VR)P.long_scale, (VR)w.z);
+                            // rebuilt in fp32, the precision the parameters are stored in (mixed
+                            // widens the result: an fp64 rebuild of fp32 data adds no accuracy)
+                            float2 fa[9], fb[9];
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) {
+                                fa[e] = make_float2(L9w[e].x, L9w[e].y);
+                                fb[e] = make_float2(L9w[e].z, L9w[e].w);
+                            }
+                            const float2 zfa = reconstruct_9<false>(fa, (float)P.long_scale, L9w[4].x);
+                            const float2 zfb = reconstruct_9<false>(fb, (float)P.long_scale, L9w[4].z);
+#pragma unroll
+                            for (int e = 0; e < 9; ++e) {
+                                Ua[e] = to_cplx<V2>(widen(fa[e]));
+                                Ub[e] = to_cplx<V2>(widen(fb[e]));
+                            }
+                            za = to_cplx<V2>(widen(zfa));
+                            zb = to_cplx<V2>(widen(zfb));
                         }
                     }
 #pragma unroll
