@@ -91,20 +91,30 @@ template <typename V2>
 __device__ __forceinline__ V2 cconj(V2 a) {
     return V2{a.x, -a.y};
 }
+// fp32 reconstruction (recon-9 is rebuilt in the precision its parameters are stored in) takes the
+// hardware approximations: MUFU sin/cos of pi*a for |a| <= 1 (abs. error ~4e-7) and rsqrt; fp64
+// keeps the libdevice routines
+__device__ __forceinline__ void sincospi_r(double a, double* s, double* c) { sincospi(a, s, c); }
+__device__ __forceinline__ void sincospi_r(float a, float* s, float* c) { __sincosf(a * 3.14159265358979f, s, c); }
+__device__ __forceinline__ double sqrt0_r(double x) { return sqrt(fmax(x, 0.0)); }
+__device__ __forceinline__ float sqrt0_r(float x) { return x > 0.f ? x * rsqrtf(x) : 0.f; }
+__device__ __forceinline__ double rcp_r(double x) { return 1.0 / x; }
+__device__ __forceinline__ float rcp_r(float x) { return __frcp_rn(x); }
+
 // SCALE = false leaves U = W and only returns z = s e^{i pi psi} (the stencil multiplies the
 // 3-vector W v by z instead of the 9 entries of W)
 template <bool SCALE = true, typename V2, typename R>
 __device__ __forceinline__ V2 reconstruct_9(V2 U[9], R s, R psi) {
     const V2 a2 = U[1], a3 = U[2], b1 = U[3];
     const R n = a2.x * a2.x + a2.y * a2.y + a3.x * a3.x + a3.y * a3.y;
-    const R a1m = sqrt(fmax(R(1) - n, R(0)));
-    const R c1m = sqrt(fmax(n - (b1.x * b1.x + b1.y * b1.y), R(0)));
+    const R a1m = sqrt0_r(R(1) - n);
+    const R c1m = sqrt0_r(n - (b1.x * b1.x + b1.y * b1.y));
     R sa, ca, sc, cc, sp, cp;
-    sincospi(U[0].x, &sa, &ca);  // angles are stored in units of pi: no large-argument reduction
-    sincospi(U[0].y, &sc, &cc);
-    sincospi(psi, &sp, &cp);
+    sincospi_r(U[0].x, &sa, &ca);  // angles are stored in units of pi: no large-argument reduction
+    sincospi_r(U[0].y, &sc, &cc);
+    sincospi_r(psi, &sp, &cp);
     const V2 a1{a1m * ca, a1m * sa}, c1{c1m * cc, c1m * sc};
-    const R inv = R(1) / n;
+    const R inv = rcp_r(n);
     const V2 a1b1 = cmul(cconj(a1), b1), a1c1 = cmul(cconj(a1), c1);
     const V2 t0 = cmul(a1b1, a2), t1 = cmul(cconj(a3), cconj(c1));
     const V2 t2 = cmul(cconj(a2), cconj(c1)), t3 = cmul(a1b1, a3);
