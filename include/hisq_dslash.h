@@ -72,10 +72,7 @@ enum { DSLASH_F64 = 0, DSLASH_F32 = 1, DSLASH_MIXED = 2 };
 enum {
     DSLASH_KERNEL_SITE = 0, /* one thread per target site, 16 link matrices streamed per thread   */
     DSLASH_KERNEL_DIR4 = 1, /* four lanes per site (one per mu), 2-step shuffle reduction ("3LP") */
-    DSLASH_KERNEL_DIR2 = 2, /* two lanes per site (two directions each), 1-step shuffle reduction  */
-    DSLASH_KERNEL_BULK = 3  /* persistent TMA pipeline: cp.async.bulk link tiles into shared memory,
-                               one producer thread, 8 consumer warps (DIR4 mapping); needs Lx/2 to
-                               be a multiple of 8; one right-hand side per launch                  */
+    DSLASH_KERNEL_DIR2 = 2  /* two lanes per site (two directions each), 1-step shuffle reduction  */
 };
 
 /* Options (dslash_set_option). */
@@ -97,22 +94,13 @@ enum {
                                    per handle) stored as the 8 parameters of W (arg a1, arg c1, a2,
                                    a3, b1) + psi, rebuilt in registers (QUDA "recon-9"; accepts
                                    folded staggered signs and U(1) phases).  Register kernels, all
-                                   precisions (DSLASH_ERR_UNSUPPORTED for the TMA kernel;
-                                   dslash_cg_mixed's fp32 copies are rebuilt in full); load_links
+                                   precisions (dslash_cg_mixed's fp32 copies are rebuilt in full);
+                                   load_links
                                    verifies that every long link
                                    is rebuilt within 1e-12 s, which also rejects links near the
                                    parameterisation's singular set |a2|^2 + |a3|^2 -> 0 (e.g.
                                    multiples of the identity): DSLASH_ERR_ARG.
                                    Before load_links                                                  */
-    DSLASH_OPT_PERSISTENT = 7,  /* 0 (default): separate interior / boundary launches (measured faster
-                                   on B200, profiles/README.md).  1: when a halo is exchanged, one
-                                   persistent launch per
-                                   apply; blocks draw tiles from ticket counters, interior first; a
-                                   block out of interior tiles looks once at the halo flag and takes
-                                   boundary tiles only if the faces have landed (never waits, so it
-                                   cannot starve the exchange); a stream-ordered clean-up launch takes
-                                   the rest.  2: persistent also without a halo.  Single-RHS applies
-                                   only; any time                                                     */
     DSLASH_OPT_TRANSPORT = 8,   /* DSLASH_TRANSPORT_NCCL / _P2P; before load_links                    */
     DSLASH_OPT_PDL = 9,         /* 1 (default): launch the stencil kernels with programmatic stream
                                    serialization, so an apply's blocks start (and prefetch their
@@ -130,10 +118,10 @@ enum {
                                    (z, t); the TMA engine copies the source rows y0-3 .. y0+TY+2 into
                                    shared memory once (cp.async.bulk + mbarrier) and the 8 x/y hops
                                    per site read them there; z/t hops stay global loads.  Same link
-                                   layout (any time).  fp32 needs Lx/2 even; the persistent path
-                                   (DSLASH_OPT_PERSISTENT) does not stage.  0 (default): off        */
-    DSLASH_OPT_FUSED_DEFER = 12,/* testing aid for DSLASH_OVERLAP_FUSED: 1 = every boundary block
-                                   defers to the clean-up launch; any time                         */
+                                   layout (any time).  An x-row must be a multiple of 16 bytes
+                                   (fp32 vectors: Lx/2 even), else DSLASH_ERR_UNSUPPORTED, also at
+                                   apply time when dslash_cg_mixed runs the handle in fp32.
+                                   0 (default): off                                                 */
     DSLASH_OPT_HALO_DRYRUN = 13,/* timing aid (NCCL / device-copy transport): halo_start keeps its
                                    events and stream order but moves no bytes, so the ghost faces
                                    are stale and results WRONG; prices an overlap scheme without the
@@ -144,8 +132,7 @@ enum {
                                    faces of an apply's OUTPUT straight into the neighbours' ghosts
                                    from the stencil kernel's epilogue (peer memory over NVLink), so
                                    the next apply, whose source that output is, moves no bytes.
-                                   Not with the persistent or one-shot fused kernels (the split
-                                   by sites runs instead) nor the TMA kernel; 0 (default): off  */
+                                   0 (default): off                                                 */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */
@@ -157,21 +144,13 @@ enum {
     DSLASH_OVERLAP_SITES = 1,  /* (default) split by sites: the interior box (no ghost source) runs
                                   during the exchange; the boundary slabs run on a high-priority
                                   stream once the faces land                                        */
-    DSLASH_OVERLAP_DIRS = 2,   /* split by direction: a local pass over every site during the
+    DSLASH_OVERLAP_DIRS = 2    /* split by direction: a local pass over every site during the
                                   exchange skips the hops into ghost faces; a ghost pass over the
                                   boundary slabs then adds exactly those hops to the stored partial
                                   sums (+96 B per boundary site).  Hides the exchange even when no
                                   site is interior (local extent 6 with a depth-3 halo).  Boundary
                                   sites sum their terms in another order than DSLASH_OVERLAP_NONE:
-                                  equal within the fp64 tolerance, not bitwise.  Not for the TMA
-                                  kernel                                                             */
-    DSLASH_OVERLAP_FUSED = 3   /* one launch over all sites, interior blocks first; each boundary
-                                  block looks once at the halo flags (set by the exchange with a
-                                  stream memory operation) and either computes its sites or defers
-                                  itself to a stream-ordered clean-up launch.  No block waits, so
-                                  no transport can be starved of SMs.  Bitwise equal to SITES.
-                                  Single-RHS applies of the site / dir2 / dir4 kernels (others
-                                  take SITES)                                                        */
+                                  equal within the fp64 tolerance, not bitwise                      */
 };
 
 /* Halo transports (DSLASH_OPT_TRANSPORT). */
@@ -325,8 +304,7 @@ DSLASH_API dslash_status dslash_apply_host_batch(dslash_t h, int32_t n, void* co
  * into out; the neighbours' ready flags are raised behind the kernel.  The NEXT apply (or
  * halo_start) on this handle, on every rank, must take `out` as its source: it then exchanges
  * no bytes; any other source returns DSLASH_ERR_STATE.  Without a halo it equals dslash_apply.
- * Errors as dslash_apply, plus DSLASH_ERR_STATE without DSLASH_OPT_PUSH and
- * DSLASH_ERR_UNSUPPORTED for the TMA kernel. */
+ * Errors as dslash_apply, plus DSLASH_ERR_STATE without DSLASH_OPT_PUSH. */
 DSLASH_API dslash_status dslash_apply_push(dslash_t h, void* out, const void* in, int32_t parity,
                                            dslash_stream_t stream);
 

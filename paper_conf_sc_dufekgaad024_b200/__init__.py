@@ -58,8 +58,7 @@ class Dslash:
 
     def __init__(self, global_dims, proc_grid=(1, 1, 1, 1), parity_mask=DSLASH_BOTH, kernel="dir2", block=0,
                  force_halo=0, overlap=True, timing=False, rank=0, world_size=1, min_blocks=0, precision="f64",
-                 recon=18, persistent=False, transport="nccl", pdl=True, self_nccl=False, stage=False,
-                 push=False):
+                 recon=18, transport="nccl", pdl=True, self_nccl=False, stage=False, push=False):
         import torch
         self.global_dims = tuple(int(d) for d in global_dims)
         self.precision = precision
@@ -107,9 +106,6 @@ class Dslash:
                     blobs = [None] * world_size
                     dist.all_gather_object(blobs, _abi.dslash_get_ipc_blob(self.h))
                     _abi.dslash_open_ipc_blobs(self.h, b"".join(blobs))
-            # True -> 1 (persistent when a halo is exchanged), "always" -> 2, False -> 0
-            _abi.dslash_set_option(self.h, _abi.DSLASH_OPT_PERSISTENT,
-                                   2 if persistent == "always" else int(bool(persistent)))
             if force_halo:
                 _abi.dslash_set_option(self.h, DSLASH_OPT_FORCE_HALO, force_halo)
             if self_nccl:

@@ -21,20 +21,19 @@ STATUS_NAMES = {0: "DSLASH_OK", 1: "DSLASH_ERR_ARG", 2: "DSLASH_ERR_STATE", 3: "
 DSLASH_EVEN, DSLASH_ODD, DSLASH_BOTH = 0, 1, 2
 DSLASH_F64, DSLASH_F32, DSLASH_MIXED = 0, 1, 2
 PRECISIONS = {"f64": DSLASH_F64, "f32": DSLASH_F32, "mixed": DSLASH_MIXED}
-DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_DIR2, DSLASH_KERNEL_BULK = 0, 1, 2, 3
+DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_DIR2 = 0, 1, 2
+# option keys (the values 7 and 12 belonged to options that were removed)
 DSLASH_OPT_KERNEL, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_OVERLAP, DSLASH_OPT_TIMING, \
-    DSLASH_OPT_MIN_BLOCKS, DSLASH_OPT_LONG_RECON, DSLASH_OPT_PERSISTENT, DSLASH_OPT_TRANSPORT, \
-    DSLASH_OPT_PDL, DSLASH_OPT_SELF_NCCL, DSLASH_OPT_STAGE, DSLASH_OPT_FUSED_DEFER, DSLASH_OPT_HALO_DRYRUN, \
-    DSLASH_OPT_PUSH = range(15)
+    DSLASH_OPT_MIN_BLOCKS, DSLASH_OPT_LONG_RECON = range(7)
+DSLASH_OPT_TRANSPORT, DSLASH_OPT_PDL, DSLASH_OPT_SELF_NCCL, DSLASH_OPT_STAGE = range(8, 12)
+DSLASH_OPT_HALO_DRYRUN, DSLASH_OPT_PUSH = 13, 14
 DSLASH_TRANSPORT_NCCL, DSLASH_TRANSPORT_P2P = 0, 1
-DSLASH_OVERLAP_NONE, DSLASH_OVERLAP_SITES, DSLASH_OVERLAP_DIRS, DSLASH_OVERLAP_FUSED = 0, 1, 2, 3
-OVERLAPS = {"none": DSLASH_OVERLAP_NONE, "sites": DSLASH_OVERLAP_SITES, "dirs": DSLASH_OVERLAP_DIRS,
-            "fused": DSLASH_OVERLAP_FUSED}
+DSLASH_OVERLAP_NONE, DSLASH_OVERLAP_SITES, DSLASH_OVERLAP_DIRS = 0, 1, 2
+OVERLAPS = {"none": DSLASH_OVERLAP_NONE, "sites": DSLASH_OVERLAP_SITES, "dirs": DSLASH_OVERLAP_DIRS}
 TRANSPORTS = {"nccl": DSLASH_TRANSPORT_NCCL, "p2p": DSLASH_TRANSPORT_P2P}
 DSLASH_TIMING_INTERIOR, DSLASH_TIMING_BOUNDARY, DSLASH_TIMING_ALL, DSLASH_TIMING_SPAN, DSLASH_TIMING_EXCHANGE = range(5)
 TIMING_KINDS = {0: "interior", 1: "boundary", 2: "all", 3: "span", 4: "exchange"}
-KERNELS = {"site": DSLASH_KERNEL_SITE, "dir4": DSLASH_KERNEL_DIR4, "dir2": DSLASH_KERNEL_DIR2,
-           "bulk": DSLASH_KERNEL_BULK}
+KERNELS = {"site": DSLASH_KERNEL_SITE, "dir4": DSLASH_KERNEL_DIR4, "dir2": DSLASH_KERNEL_DIR2}
 
 
 class dslash_box_t(ctypes.Structure):

@@ -7,7 +7,9 @@
 namespace hisq {
 
 // ---------------------------------------------------------------- fast unsigned division
-// q = n / d for 0 <= n < 2^31 and d >= 1 via one mul.hi (round-up multiplier method).
+// q = n / d for 0 <= n < 2^31 and d >= 1 via one mul.hi: the round-up magic-number division of
+// Granlund & Montgomery, "Division by invariant integers using multiplication" (PLDI 1994, §4),
+// m = 2^32 (2^s - d) / d + 1, q = (umulhi(n, m) + n) >> s with s = ceil(log2 d).
 struct FastDiv {
     uint32_t d, m, s;
     __host__ void init(uint32_t div) {
@@ -46,19 +48,6 @@ __device__ __forceinline__ double2 ld_stream(const double2* p, uint64_t pol) {
 __device__ __forceinline__ double2 ld_reuse(const double2* p, uint64_t pol) {
     double2 r;
     asm("ld.global.nc.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(r.x), "=d"(r.y) : "l"(p), "l"(pol));
-    return r;
-}
-
-// coherent load (L2 only, no L1 / read-only path): for ghost faces that another engine may have
-// written while the reading kernel was already running (DSLASH_OVERLAP_FUSED, persistent kernel)
-__device__ __forceinline__ double2 ld_cg(const double2* p) {
-    double2 r;
-    asm volatile("ld.global.cg.v2.f64 {%0, %1}, [%2];" : "=d"(r.x), "=d"(r.y) : "l"(p));
-    return r;
-}
-__device__ __forceinline__ float2 ld_cg(const float2* p) {
-    float2 r;
-    asm volatile("ld.global.cg.v2.f32 {%0, %1}, [%2];" : "=f"(r.x), "=f"(r.y) : "l"(p));
     return r;
 }
 

@@ -17,7 +17,6 @@
 #include "common.cuh"
 #include "links.cuh"
 #include "stencil.cuh"
-#include "bulk.cuh"
 #include "dispatch.h"
 
 using namespace hisq;
@@ -269,13 +268,8 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     switch (key) {
         case DSLASH_OPT_KERNEL:
-            if (value != DSLASH_KERNEL_SITE && value != DSLASH_KERNEL_DIR4 && value != DSLASH_KERNEL_DIR2 &&
-                value != DSLASH_KERNEL_BULK)
+            if (value != DSLASH_KERNEL_SITE && value != DSLASH_KERNEL_DIR4 && value != DSLASH_KERNEL_DIR2)
                 return fail(h, DSLASH_ERR_ARG, "unknown kernel variant %lld", (long long)value);
-            if (value == DSLASH_KERNEL_BULK && h->overlap == DSLASH_OVERLAP_DIRS)
-                return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel has no split-by-direction passes");
-            if (value == DSLASH_KERNEL_BULK && (h->plan.local_dims[0] / 2) % kBulkTile)
-                return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel needs Lx/2 to be a multiple of %d", kBulkTile);
             if (h->loaded && value != h->kernel)
                 return fail(h, DSLASH_ERR_STATE, "kernel variant fixes the link layout: set it before load_links");
             if (h->stage && value != DSLASH_KERNEL_SITE && value != DSLASH_KERNEL_DIR2)
@@ -312,9 +306,6 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
                 return fail(h, DSLASH_ERR_UNSUPPORTED, "HALO_DRYRUN serves the NCCL / device-copy transport");
             h->halo_dryrun = value != 0;
             return DSLASH_OK;
-        case DSLASH_OPT_FUSED_DEFER:
-            h->fused_defer_all = value != 0;
-            return DSLASH_OK;
         case DSLASH_OPT_STAGE:
             if (value && h->kernel != DSLASH_KERNEL_SITE && h->kernel != DSLASH_KERNEL_DIR2)
                 return fail(h, DSLASH_ERR_UNSUPPORTED, "the neighbour-staged kernel serves the site and dir2 variants");
@@ -323,10 +314,8 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             h->stage = value != 0;
             return DSLASH_OK;
         case DSLASH_OPT_OVERLAP:
-            if (value < 0 || value > DSLASH_OVERLAP_FUSED)
-                return fail(h, DSLASH_ERR_ARG, "overlap mode %lld not in {0, 1, 2, 3}", (long long)value);
-            if (value == DSLASH_OVERLAP_DIRS && h->kernel == DSLASH_KERNEL_BULK)
-                return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel has no split-by-direction passes");
+            if (value < 0 || value > DSLASH_OVERLAP_DIRS)
+                return fail(h, DSLASH_ERR_ARG, "overlap mode %lld not in {0, 1, 2}", (long long)value);
             h->overlap = (int)value;
             return DSLASH_OK;
         case DSLASH_OPT_TIMING:
@@ -347,10 +336,6 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
         }
         case DSLASH_OPT_PDL:
             h->pdl = value != 0;
-            return DSLASH_OK;
-        case DSLASH_OPT_PERSISTENT:
-            if (value < 0 || value > 2) return fail(h, DSLASH_ERR_ARG, "persistent mode %lld not in {0,1,2}", (long long)value);
-            h->persistent = (int)value;
             return DSLASH_OK;
         case DSLASH_OPT_LONG_RECON:
             if (value != 18 && value != 12 && value != 9)
@@ -384,7 +369,7 @@ static size_t vec_elem(const dslash_s* h) { return h->precision == DSLASH_F32 ? 
 static size_t link_elem(const dslash_s* h) { return h->precision == DSLASH_F64 ? 16 : 8; }
 
 static int lanes_of(int kernel) {
-    return (kernel == DSLASH_KERNEL_DIR4 || kernel == DSLASH_KERNEL_BULK) ? 4 : kernel == DSLASH_KERNEL_DIR2 ? 2 : 1;
+    return kernel == DSLASH_KERNEL_DIR4 ? 4 : kernel == DSLASH_KERNEL_DIR2 ? 2 : 1;
 }
 
 // ============================================================================ link loading
@@ -394,8 +379,6 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
                                      const void* const* slab_lng_in, int32_t on_device, dslash_stream_t stream) {
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!fat || !lng) return fail(h, DSLASH_ERR_ARG, "NULL link pointer");
-    if (h->recon == 9 && h->kernel == DSLASH_KERNEL_BULK)
-        return fail(h, DSLASH_ERR_UNSUPPORTED, "recon-9 serves the register kernels (site/dir2/dir4)");
     cudaStream_t s = (cudaStream_t)stream;
     const dslash_plan_t& p = h->plan;
     const int64_t V = 2 * p.vh_local;
@@ -434,9 +417,9 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
     for (int d = 0; d < 4; ++d) C.L[d] = p.local_dims[d];
     C.lxh = p.local_dims[0] / 2;
     C.vh = p.vh_local;
-    C.lanes = h->kernel == DSLASH_KERNEL_BULK ? 0 : lanes_of(h->kernel);
+    C.lanes = lanes_of(h->kernel);
     C.recon = h->recon;
-    C.paired = h->precision != DSLASH_F64 && h->kernel != DSLASH_KERNEL_BULK;
+    C.paired = h->precision != DSLASH_F64;
     int halo_mask = 0;
     for (int d = 2; d < 4; ++d)
         if (p.halo[d]) halo_mask |= 1 << d;
@@ -676,10 +659,10 @@ extern "C" dslash_status dslash_get_links(dslash_t h, int32_t parity, void* out_
     LinkConvParams C{};
     C.links = h->links[parity];
     C.vh = p.vh_local;
-    C.lanes = h->kernel == DSLASH_KERNEL_BULK ? 0 : lanes_of(h->kernel);
+    C.lanes = lanes_of(h->kernel);
     C.recon = h->recon;
     C.s9 = h->long_scale;
-    C.paired = h->precision != DSLASH_F64 && h->kernel != DSLASH_KERNEL_BULK;
+    C.paired = h->precision != DSLASH_F64;
     const size_t bytes = (size_t)p.vh_local * 144 * sizeof(double2);
     void* tmp = nullptr;
     CU(h, cudaMalloc(&tmp, bytes));
@@ -706,8 +689,8 @@ extern "C" dslash_status dslash_load_links_halo(dslash_t h, const void* fat, con
     return load_links_impl(h, fat, lng, slab_fat, slab_lng, on_device, stream);
 }
 
-// cuStreamWriteValue32 through the runtime's driver entry point (no link-time libcuda): the halo
-// stream's front end writes the epoch flag the persistent kernel waits on, without an SM.
+// cuStreamWriteValue32 through the runtime's driver entry point (no link-time libcuda): a stream's
+// front end writes the P2P epoch flags (ready / free), without an SM.
 typedef int (*WriteValue32Fn)(cudaStream_t, unsigned long long, unsigned int, unsigned int);
 static WriteValue32Fn write_value_fn() {
     static WriteValue32Fn fn = nullptr;
@@ -1139,8 +1122,7 @@ static StencilFn pick_kernel(int precision, int recon, int lanes, int minb, int 
 
 // defaults chosen by measurement on B200 (tools/sweep.py; profiles/README.md): at 32^4 and 48^4
 // every mapping is best at <= 128 registers (min 2 blocks of 256), LANES 1/2 at 64-128 threads
-static int default_block(int lanes) { return lanes == 4 ? 64 : 64; }
-static int default_minb(int lanes) { return lanes == 4 ? 2 : 2; }
+static constexpr int kDefaultBlock = 64, kDefaultMinBlocks = 2;
 
 static StencilFn pick_stage_kernel(int precision, int recon, bool ghost, int lanes, int nrhs) {
     const bool r12 = recon == 12;
@@ -1220,6 +1202,12 @@ static cudaError_t launch_pdl(bool pdl, StencilFn fn, const StencilParams& K, un
 static dslash_status launch_stage(dslash_t h, StencilParams K, bool ghost, int kind, cudaStream_t s, int nrhs,
                                   int lanes) {
     const int64_t sites = K.box_start[K.nbox];
+    // cp.async.bulk copies whole x-rows: sizes and shared-memory offsets must be 16-byte
+    // multiples (checked here, not only in set_option: dslash_cg_mixed runs an F64 handle's
+    // staged kernels as F32 ones)
+    if ((K.lxh * vec_elem(h)) % 16)
+        return fail(h, DSLASH_ERR_UNSUPPORTED, "staged kernel: an x-row of %d sites x %zu B is not a 16-byte multiple",
+                    K.lxh, vec_elem(h));
     const int rhsl = nrhs == 8 ? 2 : 1;
     const int ty = stage_rows(h, lanes * rhsl);
     if (!ty)
@@ -1259,29 +1247,10 @@ static int num_sms(dslash_t h) {
 static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int kind, cudaStream_t s, int nrhs) {
     const int64_t sites = K.box_start[K.nbox];
     if (sites == 0) return DSLASH_OK;
-    if (h->kernel == DSLASH_KERNEL_BULK) {
-        const BulkKernel bk = pick_bulk(h->precision, h->recon, ghost);
-        const int64_t ntiles = sites / bk.tile;
-        const unsigned grid = (unsigned)(ntiles < num_sms(h) ? ntiles : num_sms(h));
-        dslash_s::TimedLaunch* tl = nullptr;
-        dslash_status st = timing_begin(h, kind, s, &tl);
-        if (st != DSLASH_OK) return st;
-        // one ticket counter per kernel class: interior and boundary launches may run concurrently
-        if (!h->sched) {
-            CU(h, cudaMalloc(&h->sched, 4 * sizeof(unsigned long long)));
-            CU(h, cudaMemset(h->sched, 0, 4 * sizeof(unsigned long long)));
-        }
-        const int slot = ghost ? 1 : 0;
-        CU(h, cudaMemsetAsync(h->sched + slot, 0, sizeof(unsigned long long), s));  // fresh tickets
-        bk.fn<<<grid, bk.threads, bk.smem, s>>>(K, h->sched + slot, 0ull);
-        CU(h, cudaGetLastError());
-        if (tl) CU(h, cudaEventRecord(tl->b, s));
-        return DSLASH_OK;
-    }
     const int lanes = lanes_of(h->kernel);
     if (h->stage) return launch_stage(h, K, ghost, kind, s, nrhs, lanes);
-    const int bs = h->block ? h->block : default_block(lanes);
-    const int minb = h->min_blocks ? h->min_blocks : default_minb(lanes);
+    const int bs = h->block ? h->block : kDefaultBlock;
+    const int minb = h->min_blocks ? h->min_blocks : kDefaultMinBlocks;
     // right-hand sides are register-blocked per thread; 8 of them use 2 thread groups of 4
     const int64_t threads = sites * lanes * (nrhs == 8 ? 2 : 1);
     const unsigned grid = (unsigned)((threads + bs - 1) / bs);
@@ -1310,7 +1279,6 @@ static dslash_status launch_rhs(dslash_t h, StencilParams K, const dslash_box_t*
     for (int r0 = 0; r0 < nrhs;) {
         const int left = nrhs - r0;
         int nr = left >= 8 ? 8 : left >= 4 ? 4 : left >= 2 ? 2 : 1;
-        if (h->kernel == DSLASH_KERNEL_BULK) nr = 1;  // the TMA kernel streams one right-hand side
         K.in = in0 + (size_t)r0 * 3 * K.vh * es;
         K.out = out0 + (size_t)r0 * 3 * K.vh * es;
         for (int d = 0; d < 4; ++d)
@@ -1324,217 +1292,6 @@ static dslash_status launch_rhs(dslash_t h, StencilParams K, const dslash_box_t*
         if (st != DSLASH_OK) return st;
         r0 += nr;
     }
-    return DSLASH_OK;
-}
-
-// ---------------------------------------------------------------------------- persistent path
-static int persist_occupancy(dslash_t h, PersistFn fn, int bs) {
-    static PersistFn last_fn = nullptr;
-    static int last_bs = 0, last_occ = 1;
-    if (fn != last_fn || bs != last_bs) {
-        int occ = 1;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, bs, 0) != cudaSuccess || occ < 1) occ = 1;
-        last_fn = fn;
-        last_bs = bs;
-        last_occ = occ;
-    }
-    (void)h;
-    return last_occ;
-}
-
-static PersistFn pick_persist(int precision, int recon, int mode, int lanes) {
-    const bool r12 = recon == 12;
-    if (recon == 9)
-        return precision == DSLASH_F32     ? persist_f32_r9(mode, lanes)
-               : precision == DSLASH_MIXED ? persist_mixed_r9(mode, lanes)
-                                           : persist_f64_r9(mode, lanes);
-    switch (precision) {
-        case DSLASH_F32: return r12 ? persist_f32_r12(mode, lanes) : persist_f32_r18(mode, lanes);
-        case DSLASH_MIXED: return r12 ? persist_mixed_r12(mode, lanes) : persist_mixed_r18(mode, lanes);
-        default: return r12 ? persist_f64_r12(mode, lanes) : persist_f64_r18(mode, lanes);
-    }
-}
-
-// One persistent launch per apply (stencil.cuh, dslash_persistent_kernel): interior boxes
-// first; with a halo, blocks continue with boundary tiles if the faces have landed, and a
-// stream-ordered clean-up launch after the halo event takes the boundary tiles left over.
-static dslash_status apply_persistent(dslash_t h, StencilParams K, cudaStream_t s) {
-    const dslash_plan_t& p = h->plan;
-    const bool halo = any_halo(p);
-    dslash_box_t all[kMaxBoxes];
-    int n = 0;
-    for (int i = 0; i < p.n_interior; ++i) all[n++] = p.interior[i];
-    for (int i = 0; i < p.n_boundary; ++i) all[n++] = p.boundary[i];
-    fill_boxes(K, all, n);
-    if (!h->sched) {
-        CU(h, cudaMalloc(&h->sched, 4 * sizeof(unsigned long long)));
-        CU(h, cudaMemset(h->sched, 0, 4 * sizeof(unsigned long long)));
-    }
-    const int lanes = lanes_of(h->kernel);
-    const int bs = h->block ? h->block : default_block(lanes);
-    const int64_t sites = K.box_start[K.nbox];
-    const int64_t isites = halo ? p.interior_sites : sites;
-    PersistArgs A{};
-    A.sched = h->sched + 2;
-    A.base = h->sched_next[2];
-    A.interior_sites = isites;
-    A.ntiles_int = (isites * lanes + bs - 1) / bs;
-    A.ntiles_bnd = ((sites - isites) * lanes + bs - 1) / bs;
-    // an index, not a pointer: halo_start below may grow tpool (its exchange interval)
-    size_t tl = (size_t)-1;
-    if (h->timing) {
-        if (h->tused == h->tpool.size()) {
-            dslash_s::TimedLaunch t{};
-            CU(h, cudaEventCreate(&t.a));
-            CU(h, cudaEventCreate(&t.b));
-            h->tpool.push_back(t);
-        }
-        tl = h->tused++;
-        h->tpool[tl].kind = DSLASH_TIMING_ALL;
-    }
-    if (halo) {
-        if (!h->halo_flag) {
-            CU(h, cudaMalloc(&h->halo_flag, sizeof(unsigned int)));
-            CU(h, cudaMemset(h->halo_flag, 0, sizeof(unsigned int)));
-            h->epoch = 0;
-        }
-        CU(h, cudaMemsetAsync(A.sched + 1, 0, sizeof(unsigned long long), s));  // boundary tickets
-        dslash_status st = halo_start_impl(h, K.in, 1, s);
-        if (st != DSLASH_OK) return st;
-        for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
-            K.ghost[d][0] = h->ghost[d][0];
-            K.ghost[d][1] = h->ghost[d][1];
-        }
-        if (h->transport == DSLASH_TRANSPORT_P2P) {
-            // the faces have landed when the neighbours raised my ready flags (halo_start_p2p)
-            for (int d = 3; d >= 2; --d)
-                if (p.halo[d])
-                    for (int side = 0; side < 2; ++side) A.flags[A.nflags++] = h->flags + 2 * d + side;
-        } else {
-            ++h->epoch;
-            if (write_value_fn()(h->comm, (unsigned long long)(uintptr_t)h->halo_flag, h->epoch, 0) != 0)
-                return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 failed");
-            A.flags[A.nflags++] = h->halo_flag;
-        }
-        A.epoch = h->epoch;
-    }
-    const PersistFn fn = pick_persist(h->precision, h->recon, halo ? 1 : 0, lanes);
-    const int64_t cap = (int64_t)persist_occupancy(h, fn, bs) * num_sms(h);
-    const int64_t want = A.ntiles_int + (halo ? A.ntiles_bnd : 0);
-    const unsigned grid = (unsigned)(want < cap ? (want > 0 ? want : 1) : cap);
-    if (tl != (size_t)-1) CU(h, cudaEventRecord(h->tpool[tl].a, s));
-    fn<<<grid, bs, 0, s>>>(K, A);
-    CU(h, cudaGetLastError());
-    h->sched_next[2] += (unsigned long long)A.ntiles_int + 2ull * grid;
-    if (halo) {
-        dslash_status st = dslash_halo_wait(h, (dslash_stream_t)s);  // the faces are in the ghosts
-        if (st != DSLASH_OK) return st;
-        const PersistFn clean = pick_persist(h->precision, h->recon, 2, lanes);
-        const unsigned g2 = (unsigned)(A.ntiles_bnd < cap ? (A.ntiles_bnd > 0 ? A.ntiles_bnd : 1) : cap);
-        clean<<<g2, bs, 0, s>>>(K, A);
-        CU(h, cudaGetLastError());
-    }
-    if (tl != (size_t)-1) CU(h, cudaEventRecord(h->tpool[tl].b, s));
-    return DSLASH_OK;
-}
-
-static FusedFn pick_fused_kernel(int precision, int recon, bool cleanup, int lanes) {
-    const bool r12 = recon == 12;
-    if (recon == 9)
-        return precision == DSLASH_F32     ? pick_f32_r9_fused(cleanup, lanes)
-               : precision == DSLASH_MIXED ? pick_mixed_r9_fused(cleanup, lanes)
-                                           : pick_f64_r9_fused(cleanup, lanes);
-    switch (precision) {
-        case DSLASH_F32: return r12 ? pick_f32_r12_fused(cleanup, lanes) : pick_f32_r18_fused(cleanup, lanes);
-        case DSLASH_MIXED: return r12 ? pick_mixed_r12_fused(cleanup, lanes) : pick_mixed_r18_fused(cleanup, lanes);
-        default: return r12 ? pick_f64_r12_fused(cleanup, lanes) : pick_f64_r18_fused(cleanup, lanes);
-    }
-}
-
-static cudaError_t launch_fused(bool pdl, FusedFn fn, const StencilParams& K, const FusedArgs& A, unsigned grid,
-                                int bs, cudaStream_t s) {
-    if (!pdl) {
-        fn<<<grid, bs, 0, s>>>(K, A);
-        return cudaGetLastError();
-    }
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(grid);
-    cfg.blockDim = dim3(bs);
-    cfg.stream = s;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[0].val.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, fn, K, A);
-}
-
-// DSLASH_OVERLAP_FUSED: one launch over all sites, interior blocks first; boundary blocks look
-// once at the halo flags and defer to a stream-ordered clean-up launch if the faces have not
-// landed (stencil.cuh dslash_fused_kernel).  Single right-hand side, site / dir2 / dir4 kernels.
-static dslash_status apply_fused(dslash_t h, StencilParams K, cudaStream_t s) {
-    const dslash_plan_t& p = h->plan;
-    dslash_box_t all[kMaxBoxes];
-    int n = 0;
-    for (int i = 0; i < p.n_interior; ++i) all[n++] = p.interior[i];
-    for (int i = 0; i < p.n_boundary; ++i) all[n++] = p.boundary[i];
-    fill_boxes(K, all, n);
-    const int lanes = lanes_of(h->kernel);
-    const int bs = h->block ? h->block : default_block(lanes);
-    const int64_t sites = K.box_start[K.nbox];
-    const int64_t grid = (sites * lanes + bs - 1) / bs;
-    FusedArgs A{};
-    A.interior_blocks = p.interior_sites * lanes / bs;  // a block straddling into the boundary is a boundary block
-    const int64_t nbnd = grid - A.interior_blocks;
-    if (h->fused_cap < nbnd) {
-        if (h->fused_buf) {
-            CU(h, cudaStreamSynchronize(s));  // a queued clean-up may still read the old list
-            cudaFree(h->fused_buf);
-            h->fused_buf = nullptr;
-        }
-        CU(h, cudaMalloc(&h->fused_buf, (size_t)(2 + nbnd) * sizeof(unsigned int)));
-        CU(h, cudaMemsetAsync(h->fused_buf, 0, 2 * sizeof(unsigned int), s));
-        h->fused_cap = nbnd;
-        h->fused_parity = 0;
-    }
-    A.count = h->fused_buf + h->fused_parity;
-    A.count_next = h->fused_buf + (1 - h->fused_parity);
-    A.deferred = h->fused_buf + 2;
-    A.defer_all = h->fused_defer_all;
-    h->fused_parity ^= 1;
-    if (!h->halo_flag) {
-        CU(h, cudaMalloc(&h->halo_flag, sizeof(unsigned int)));
-        CU(h, cudaMemset(h->halo_flag, 0, sizeof(unsigned int)));
-        h->epoch = 0;
-    }
-    dslash_status st = halo_start_impl(h, K.in, 1, s);
-    if (st != DSLASH_OK) return st;
-    for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
-        K.ghost[d][0] = h->ghost[d][0];
-        K.ghost[d][1] = h->ghost[d][1];
-    }
-    if (h->transport == DSLASH_TRANSPORT_P2P) {
-        for (int d = 3; d >= 2; --d)  // the neighbours raise my ready flags (halo_start_p2p)
-            if (p.halo[d])
-                for (int side = 0; side < 2; ++side) A.flags[A.nflags++] = h->flags + 2 * d + side;
-    } else {
-        ++h->epoch;
-        if (write_value_fn()(h->comm, (unsigned long long)(uintptr_t)h->halo_flag, h->epoch, 0) != 0)
-            return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 failed");
-        A.flags[A.nflags++] = h->halo_flag;
-    }
-    A.epoch = h->epoch;
-    size_t span = (size_t)-1;
-    if (h->timing) {
-        dslash_s::TimedLaunch* tl = nullptr;
-        if ((st = timing_begin(h, DSLASH_TIMING_SPAN, s, &tl)) != DSLASH_OK) return st;
-        span = (size_t)(tl - h->tpool.data());
-    }
-    CU(h, launch_fused(h->pdl, pick_fused_kernel(h->precision, h->recon, false, lanes), K, A, (unsigned)grid, bs, s));
-    if ((st = dslash_halo_wait(h, (dslash_stream_t)s)) != DSLASH_OK) return st;
-    const int64_t g2 = nbnd > 0 ? nbnd : 1;  // one block per boundary block that may have deferred
-    CU(h, launch_fused(h->pdl, pick_fused_kernel(h->precision, h->recon, true, lanes), K, A, (unsigned)g2, bs, s));
-    if (span != (size_t)-1) CU(h, cudaEventRecord(h->tpool[span].b, s));
     return DSLASH_OK;
 }
 
@@ -1581,25 +1338,10 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         K.face_vh[d] = p.face_vh[d];
         if (p.halo[d]) K.halo_mask |= 1 << d;
     }
-    // producer push: only with a halo (without one the next apply needs no faces) and only from
-    // the stencil kernels' epilogue (not the TMA kernel's)
+    // producer push: only with a halo (without one the next apply needs no faces)
     push_out = push_out && any_halo(p);
-    if (push_out) {
-        if (!h->push) return fail(h, DSLASH_ERR_STATE, "apply_push needs DSLASH_OPT_PUSH");
-        if (h->kernel == DSLASH_KERNEL_BULK)
-            return fail(h, DSLASH_ERR_UNSUPPORTED, "the TMA kernel does not push faces");
-    }
-    // persistent: 1 = when a halo is exchanged (default), 2 = always (not with the producer push,
-    // whose two ghost banks only the split launches address)
-    if (h->persistent && (h->persistent == 2 || any_halo(p)) && nrhs == 1 && h->kernel != DSLASH_KERNEL_BULK &&
-        !h->push && write_value_fn())
-        return apply_persistent(h, K, s);
+    if (push_out && !h->push) return fail(h, DSLASH_ERR_STATE, "apply_push needs DSLASH_OPT_PUSH");
     if (!any_halo(p)) return launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
-    // the one-shot fused kernel serves single-RHS applies of the site / dir2 / dir4 kernels; other
-    // applies in this mode take the split by sites
-    if (h->overlap == DSLASH_OVERLAP_FUSED && nrhs == 1 && h->kernel != DSLASH_KERNEL_BULK && !h->stage &&
-        !h->push && write_value_fn())
-        return apply_fused(h, K, s);
     if ((st = halo_start_impl(h, in, nrhs, s)) != DSLASH_OK) return st;
     for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
         K.ghost[d][0] = h->ghost[d][0] ? h->ghost[d][0] + bank_off(h, d, h->epoch) : nullptr;
@@ -1644,7 +1386,7 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
     // without interior sites (e.g. 48^4 on 8 GPUs, local Lt = 6) nothing can overlap the exchange:
     // one launch on the caller's stream after it, no boundary stream and join (measured equal,
     // 153.7 vs 153.8 us per apply at 48^3 x 6 with a t self-halo)
-    if ((h->overlap == DSLASH_OVERLAP_SITES || h->overlap == DSLASH_OVERLAP_FUSED) && p.interior_sites > 0) {
+    if (h->overlap == DSLASH_OVERLAP_SITES && p.interior_sites > 0) {
         // interior on the caller's stream; boundary on the handle's boundary stream as soon as the
         // halo lands, so it fills the SMs the interior kernel's tail leaves idle; then the caller's
         // stream joins (the two kernels write disjoint sites of out)
@@ -1860,9 +1602,6 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
             if (e) cudaEventDestroy(e);
     }
     if (h->ev_batch) cudaEventDestroy(h->ev_batch);
-    if (h->sched) cudaFree(h->sched);
-    if (h->halo_flag) cudaFree(h->halo_flag);
-    if (h->fused_buf) cudaFree(h->fused_buf);
     for (void* q : h->ipc_opened) cudaIpcCloseMemHandle(q);
     if (h->flags) cudaFree(h->flags);
     for (void* v : h->cg_vec32)

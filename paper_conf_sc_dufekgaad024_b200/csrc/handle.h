@@ -62,26 +62,13 @@ struct dslash_s {
     double* cg_host_rr = nullptr;
     int cg_host_cap = 0;
     cudaEvent_t cg_ev[4] = {};
-    // tile scheduler of the TMA kernel: ticket counters ([0] interior, [0/1] boundary launches,
-    // which may overlap) and the first ticket of each counter's next launch
-    unsigned long long* sched = nullptr;   // [0] TMA interior, [1] TMA boundary, [2] persistent
-                                           // interior (monotonic), [3] persistent boundary (reset)
-    unsigned long long sched_next[3] = {0, 0, 0};
-    // persistent fused kernel (DSLASH_OPT_PERSISTENT): the halo epoch flag it looks at
-    int persistent = 0;
     int pdl = 1;                        // programmatic dependent launch of the stencil kernels
-    unsigned int* halo_flag = nullptr;
-    unsigned int epoch = 0;             // halo exchanges started so far
+    unsigned int epoch = 0;             // halo exchanges started so far (P2P epoch flags)
     // P2P transport (DSLASH_TRANSPORT_P2P): CUDA-IPC-mapped neighbour buffers, copy engines and
     // stream memory operations.  flags (device, IPC-exported): [0..7] ready[d][side] (written by the
     // neighbour that fills my ghost[d][side]), [8..15] free_from[d][side] (written by the neighbour
     // whose ghost my bottom (side 0) / top (side 1) face fills, once it consumed it).
     int transport = DSLASH_TRANSPORT_NCCL;
-    // one-shot fused kernel (DSLASH_OVERLAP_FUSED): [0], [1] deferred-block counters (alternate per
-    // apply), then the deferred block list; capacity in entries
-    unsigned int* fused_buf = nullptr;
-    int64_t fused_cap = 0;
-    int fused_parity = 0, fused_defer_all = 0;
     int halo_dryrun = 0;                // DSLASH_OPT_HALO_DRYRUN (timing aid: exchange moves no bytes)
     int stage = 0;                      // DSLASH_OPT_STAGE: neighbour-staged kernel (x/y rows in smem by TMA)
     int self_nccl = 0;                  // DSLASH_OPT_SELF_NCCL: self-neighbour faces via NCCL

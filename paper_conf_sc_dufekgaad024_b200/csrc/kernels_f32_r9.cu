@@ -1,4 +1,4 @@
 // kernels_f32_r9.cu -- dslash_kernel instantiations: links float, vectors float, long-link recon 9.
 #include "kernels_inst.cuh"
 
-HISQ_DEFINE_PICK(pick_f32_r9, persist_f32_r9, float, float, 9)
+HISQ_DEFINE_PICK(pick_f32_r9, float, float, 9)

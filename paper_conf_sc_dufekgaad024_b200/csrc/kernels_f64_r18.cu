@@ -1,4 +1,4 @@
 // kernels_f64_r18.cu -- dslash_kernel instantiations: links double, vectors double, long-link recon 18.
 #include "kernels_inst.cuh"
 
-HISQ_DEFINE_PICK(pick_f64_r18, persist_f64_r18, double, double, 18)
+HISQ_DEFINE_PICK(pick_f64_r18, double, double, 18)

@@ -58,42 +58,12 @@ StencilFn pick_stage(bool ghost, int lanes, int nrhs) {
     return ghost ? pick_stage_n<LR, VR, 2, true, RECON>(nrhs) : pick_stage_n<LR, VR, 2, false, RECON>(nrhs);
 }
 
-// the one-shot fused kernel (DSLASH_OVERLAP_FUSED): main launch or clean-up, lanes 1/2/4
-template <typename LR, typename VR, int RECON>
-FusedFn pick_fused(bool cleanup, int lanes) {
-    switch (lanes) {
-        case 1: return cleanup ? dslash_fused_cleanup<LR, VR, 1, RECON> : dslash_fused_kernel<LR, VR, 1, RECON>;
-        case 2: return cleanup ? dslash_fused_cleanup<LR, VR, 2, RECON> : dslash_fused_kernel<LR, VR, 2, RECON>;
-        default: return cleanup ? dslash_fused_cleanup<LR, VR, 4, RECON> : dslash_fused_kernel<LR, VR, 4, RECON>;
-    }
-}
-
-template <typename LR, typename VR, int LANES, int RECON>
-PersistFn pick_persist_l(int mode) {
-    switch (mode) {
-        case 0: return dslash_persistent_kernel<LR, VR, LANES, false, RECON, false>;  // no halo
-        case 1: return dslash_persistent_kernel<LR, VR, LANES, true, RECON, false>;   // halo, main
-        default: return dslash_persistent_kernel<LR, VR, LANES, true, RECON, true>;   // halo, clean-up
-    }
-}
-
-template <typename LR, typename VR, int RECON>
-PersistFn pick_persist(int mode, int lanes) {
-    switch (lanes) {
-        case 1: return pick_persist_l<LR, VR, 1, RECON>(mode);
-        case 2: return pick_persist_l<LR, VR, 2, RECON>(mode);
-        default: return pick_persist_l<LR, VR, 4, RECON>(mode);
-    }
-}
-
 }  // namespace hisq
 
-#define HISQ_DEFINE_PICK(NAME, PNAME, LR, VR, RECON)                           \
-    namespace hisq {                                                           \
-    StencilFn NAME(bool ghost, int lanes, int minb, int nrhs) {                \
-        return pick_any<LR, VR, RECON>(ghost, lanes, minb, nrhs);              \
-    }                                                                          \
-    PersistFn PNAME(int mode, int lanes) { return pick_persist<LR, VR, RECON>(mode, lanes); } \
+#define HISQ_DEFINE_PICK(NAME, LR, VR, RECON)                                                                  \
+    namespace hisq {                                                                                          \
+    StencilFn NAME(bool ghost, int lanes, int minb, int nrhs) {                                               \
+        return pick_any<LR, VR, RECON>(ghost, lanes, minb, nrhs);                                             \
+    }                                                                                                         \
     StencilFn NAME##_stage(bool ghost, int lanes, int nrhs) { return pick_stage<LR, VR, RECON>(ghost, lanes, nrhs); } \
-    FusedFn NAME##_fused(bool cleanup, int lanes) { return pick_fused<LR, VR, RECON>(cleanup, lanes); } \
     }

@@ -1,4 +1,4 @@
 // kernels_mixed_r18.cu -- dslash_kernel instantiations: links float, vectors double, long-link recon 18.
 #include "kernels_inst.cuh"
 
-HISQ_DEFINE_PICK(pick_mixed_r18, persist_mixed_r18, float, double, 18)
+HISQ_DEFINE_PICK(pick_mixed_r18, float, double, 18)

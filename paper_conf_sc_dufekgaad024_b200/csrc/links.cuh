@@ -13,7 +13,6 @@
 
 #include "common.cuh"
 #include "stencil.cuh"
-#include "bulk.cuh"
 
 namespace hisq {
 
@@ -28,8 +27,7 @@ struct LinkConvParams {
     int lxh;
     int parity;
     int halo_mask;
-    int lanes;                    // layout of the kernel that will read the links: 1, 2 or 4,
-                                  // or 0 = tiled (the TMA kernel, bulk.cuh)
+    int lanes;                    // layout of the kernel that will read the links: 1, 2 or 4
     int recon;                    // 18 = full matrices, 12 = long links keep rows 0 and 1 only,
                                   // 9 = long links as 8 SU(3) parameters + a phase (stencil.cuh)
     double s9;                    // recon-9: the long links' real scale s
@@ -38,8 +36,6 @@ struct LinkConvParams {
 
 // float2 offset of entry (mu, l, e) of site cb in the layout selected by P
 __host__ __device__ __forceinline__ int64_t conv_index(const LinkConvParams& P, int mu, int l, int e, int64_t cb) {
-    if (P.lanes == 0)
-        return P.recon == 12 ? link_index_tiled<12>(mu, l, e, cb) : link_index_tiled<18>(mu, l, e, cb);
     if (P.paired) {
         const int64_t o4 = P.lanes == 1   ? link_index_paired<1>(mu, l >> 1, e, P.vh, cb)
                            : P.lanes == 2 ? link_index_paired<2>(mu, l >> 1, e, P.vh, cb)

@@ -610,8 +610,6 @@ extern "C" dslash_status dslash_cg_mixed(dslash_t h, void* x_out, const void* b_
     if (st != DSLASH_OK) return st;
     if (h->precision != DSLASH_F64)
         return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the mixed-precision solver needs an fp64 handle (DSLASH_F64)");
-    if (h->kernel == DSLASH_KERNEL_BULK)
-        return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the mixed-precision solver needs a register-staged kernel");
     if (!(rel_tol > 0.0) || max_iter < 1 || !(inner_tol > 0.0) || !(inner_tol < 1.0))
         return hisq_fail(h, DSLASH_ERR_ARG, "need rel_tol > 0, 0 < inner_tol < 1, max_iter >= 1");
     if (!(mass != 0.0)) return hisq_fail(h, DSLASH_ERR_ARG, "mass must be nonzero (A is then positive definite)");

@@ -304,9 +304,8 @@ __device__ __forceinline__ float2 lds_at(uint32_t a, float2*) {
 
 // one neighbour colour component: from the staged tile (shared address sa + off_b) or from global
 template <typename V2>
-__device__ __forceinline__ V2 ld_src(bool staged, uint32_t sa, uint32_t off_b, const V2* p, uint64_t pol,
-                                     bool coherent = false) {
-    return staged ? lds_at(sa + off_b, (V2*)nullptr) : coherent ? ld_cg(p) : ld_reuse(p, pol);
+__device__ __forceinline__ V2 ld_src(bool staged, uint32_t sa, uint32_t off_b, const V2* p, uint64_t pol) {
+    return staged ? lds_at(sa + off_b, (V2*)nullptr) : ld_reuse(p, pol);
 }
 
 // v = 0 when z (a select, so acc + U * 0 leaves acc's value unchanged without a branch)
@@ -351,9 +350,7 @@ __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[
 // staged kernel visits the global (z, t) directions first and the tile's (x, y) ones last, so
 // the tile's bulk copies land while the z/t links and neighbours stream (a different summation
 // order from the unstaged kernel: equal within the fp64 tolerance, not bitwise).
-// COH: ghost faces are read with coherent loads (kernels that may start before the faces land)
-template <typename LR, typename VR, int LANES, bool GHOST, int RECON, int NRHS, int RHSL = 1, bool STAGED = false,
-          bool COH = false>
+template <typename LR, typename VR, int LANES, bool GHOST, int RECON, int NRHS, int RHSL = 1, bool STAGED = false>
 __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_t gid, const int64_t site_end,
                                             const StageTile<cplx_t<VR>> T = {}) {
     static_assert(LANES == 1 || LANES == 2 || LANES == 4, "LANES must divide 4");
@@ -484,7 +481,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 #pragma unroll
                             for (int c = 0; c < 3; ++c) {
                                 v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride,
-                                              pol_keep, COH && src.ghost);
+                                              pol_keep);
                                 if (GHOST) zero_if(v[c], zap);
                             }
                             if (RECON == 9 && j == 1) {
@@ -560,8 +557,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     V2 v[3];
 #pragma unroll
                     for (int c = 0; c < 3; ++c) {
-                        v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride, pol_keep,
-                                      COH && src.ghost);
+                        v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride, pol_keep);
                         if (GHOST) zero_if(v[c], zap);
                     }
                     if (RECON == 9 && l >= 2) {
@@ -705,132 +701,6 @@ __global__ void __launch_bounds__(256, 2) dslash_stage_kernel(const StencilParam
     T.sbase = smem_addr(stage_smem);
     dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL, true>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
                                                                P.box_start[P.nbox], T);
-}
-
-// ---------------------------------------------------------------- one-shot fused kernel
-// DSLASH_OVERLAP_FUSED: ONE launch over all sites per apply, interior blocks first (blockIdx order
-// is dispatch order), so by the time the boundary blocks are dispatched the exchange has long
-// finished.  A boundary block looks ONCE at the halo flags: if the faces have landed it computes
-// its sites (reading the ghosts with coherent loads), otherwise it appends its index to a
-// deferred list and exits.  A stream-ordered clean-up launch after the halo event computes the
-// deferred blocks.  No block ever waits, so no transport (NCCL kernels included) can be starved
-// of SMs; every site runs the same per-site arithmetic as the split by sites (bitwise equal).
-struct FusedArgs {
-    const unsigned int* flags[4];  // halo epoch flags that must all reach `epoch`
-    int nflags;
-    unsigned int epoch;
-    int64_t interior_blocks;       // blocks [0, interior_blocks) hold interior sites only
-    unsigned int* deferred;        // block indices deferred to the clean-up launch
-    unsigned int* count;           // entries in `deferred` (this apply)
-    unsigned int* count_next;      // the next apply's counter, zeroed by the clean-up launch
-    int defer_all;                 // testing aid: every boundary block defers
-};
-
-template <typename LR, typename VR, int LANES, int RECON>
-__global__ void __launch_bounds__(256, 2) dslash_fused_kernel(const StencilParams P, const FusedArgs A) {
-    asm volatile("griddepcontrol.launch_dependents;");
-    const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if ((int64_t)blockIdx.x < A.interior_blocks) {
-        dslash_body<LR, VR, LANES, false, RECON, 1>(P, gid, P.box_start[P.nbox]);
-        return;
-    }
-    __shared__ int ready;
-    // after the previous grid on the stream completed: it may be the previous apply's clean-up,
-    // which reads the deferred list and zeroes this apply's counter
-    asm volatile("griddepcontrol.wait;" ::: "memory");
-    if (threadIdx.x == 0) {
-        int ok = !A.defer_all;
-        for (int f = 0; f < A.nflags; ++f) {
-            unsigned int v;
-            asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(A.flags[f]) : "memory");
-            if ((int)(v - A.epoch) < 0) ok = 0;
-        }
-        if (!ok) A.deferred[atomicAdd(A.count, 1u)] = blockIdx.x;
-        ready = ok;
-    }
-    __syncthreads();
-    if (!ready) return;
-    dslash_body<LR, VR, LANES, true, RECON, 1, 1, false, true>(P, gid, P.box_start[P.nbox]);
-}
-
-template <typename LR, typename VR, int LANES, int RECON>
-__global__ void __launch_bounds__(256, 2) dslash_fused_cleanup(const StencilParams P, const FusedArgs A) {
-    asm volatile("griddepcontrol.wait;" ::: "memory");  // the main launch has decided every block
-    const unsigned int n = *(volatile unsigned int*)A.count;
-    if (blockIdx.x == 0 && threadIdx.x == 0) *A.count_next = 0u;
-    // one block per potential deferral: all deferred blocks run at once, the others exit
-    if (blockIdx.x >= n) return;
-    const int64_t b = A.deferred[blockIdx.x];
-    dslash_body<LR, VR, LANES, true, RECON, 1, 1, false, true>(P, b * blockDim.x + threadIdx.x, P.box_start[P.nbox]);
-}
-
-// ---------------------------------------------------------------- persistent fused kernel
-// One launch per apply (DSLASH_OPT_PERSISTENT): blocks stay resident and draw tiles of
-// blockDim.x threads from ticket counters.  Interior sites (the first `interior_sites` of the
-// box enumeration) come from counter sched[0]: a launch consumes exactly ntiles_int + 2
-// gridDim.x tickets from `base` (each block draws one ahead, so the atomic's latency overlaps a
-// tile).  With a halo, a block that runs out of interior tiles looks ONCE at the halo epoch
-// flag, which the halo stream sets after the exchange (cuStreamWriteValue32, no SM involved):
-// if the faces have landed it goes on with boundary tiles from counter sched[1] (reset to 0
-// before the launch), otherwise it exits.  No block ever waits, so the kernel cannot starve the
-// exchange of SMs (NCCL's send/recv kernels, or a copy kernel); a stream-ordered clean-up launch
-// after the halo event (BOUNDARY_ONLY) takes whatever boundary tiles are left.  Interior work
-// and the exchange thus overlap inside one kernel, and dynamic tiles end every SM together.
-struct PersistArgs {
-    unsigned long long* sched;  // [0] interior tickets (monotonic), [1] boundary tickets (reset per apply)
-    unsigned long long base;    // first interior ticket of this launch
-    int64_t interior_sites;     // sites [0, interior_sites) are interior
-    int64_t ntiles_int;         // ceil(interior_sites * LANES / blockDim.x)
-    int64_t ntiles_bnd;         // ceil(boundary sites * LANES / blockDim.x)
-    const unsigned int* flags[4];  // halo epoch flags that must all reach `epoch` (none: no halo)
-    int nflags;
-    unsigned int epoch;
-};
-
-template <typename LR, typename VR, int LANES, bool GHOST, int RECON, bool BOUNDARY_ONLY>
-__global__ void __launch_bounds__(256, 2) dslash_persistent_kernel(const StencilParams P, const PersistArgs A) {
-    __shared__ long long s_tile;
-    const int64_t total = P.box_start[P.nbox];
-    if (!BOUNDARY_ONLY) {
-        long long next = 0;
-        if (threadIdx.x == 0) next = (long long)(atomicAdd(A.sched, 1ull) - A.base);
-        for (;;) {
-            if (threadIdx.x == 0) {
-                s_tile = next;
-                next = (long long)(atomicAdd(A.sched, 1ull) - A.base);  // in flight while this tile runs
-            }
-            __syncthreads();
-            const long long t = s_tile;
-            __syncthreads();  // all threads hold t before thread 0 publishes the next tile
-            if (t >= A.ntiles_int) break;
-            // interior sites never reach a ghost face: the ghost-free addressing suffices
-            dslash_body<LR, VR, LANES, false, RECON, 1>(P, t * blockDim.x + threadIdx.x, A.interior_sites);
-        }
-        if (!GHOST) return;
-        // boundary tiles only if the halo has already landed: one look, never a wait
-        if (threadIdx.x == 0) {
-            long long ok = 1;
-            for (int f = 0; f < A.nflags; ++f) {
-                unsigned int v;
-                asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(A.flags[f]) : "memory");
-                if ((int)(v - A.epoch) < 0) ok = 0;
-            }
-            s_tile = ok;
-        }
-        __syncthreads();
-        const bool ready = s_tile != 0;
-        __syncthreads();
-        if (!ready) return;
-    }
-    const int64_t bnd0 = A.interior_sites * LANES;  // first boundary thread index
-    for (;;) {
-        if (threadIdx.x == 0) s_tile = (long long)atomicAdd(A.sched + 1, 1ull);
-        __syncthreads();
-        const long long t = s_tile;
-        __syncthreads();
-        if (t >= A.ntiles_bnd) break;
-        dslash_body<LR, VR, LANES, GHOST, RECON, 1, 1, false, true>(P, bnd0 + t * blockDim.x + threadIdx.x, total);
-    }
 }
 
 }  // namespace hisq

@@ -1,8 +1,8 @@
 """Real multi-rank runs on ONE GPU: several processes, each a rank with its own library handle,
 exchanging depth-3 halos through the P2P transport (CUDA IPC-mapped ghost buffers, copy
 engines, stream-memory epoch flags).  NCCL cannot put two ranks on one device, so this is how
-the multi-rank data path (plan, ghost addressing, link halo, epoch protocol, persistent kernel
-and clean-up launch) is exercised end to end on a single B200.
+the multi-rank data path (plan, ghost addressing, link halo, epoch protocol, interior and
+boundary launches) is exercised end to end on a single B200.
 
 The gathered N-rank result must equal the 1-rank result BITWISE (same per-site device function,
 SURVEY §8(c) P11) and match the oracle."""
@@ -98,10 +98,10 @@ def _single(gdims, kw, parity, nrhs=1):
 
 @pytest.mark.parametrize("gdims,grid", [((8, 8, 8, 16), (1, 1, 1, 2)), ((8, 8, 16, 8), (1, 1, 2, 1)),
                                         ((8, 8, 8, 8), (1, 1, 2, 2)), ((8, 8, 8, 24), (1, 1, 1, 3))])
-@pytest.mark.parametrize("persistent", [True, False])
-def test_multirank_p2p_bitwise(gdims, grid, persistent):   # True = persistent kernel when a halo exists
+@pytest.mark.parametrize("overlap", [True, False])
+def test_multirank_p2p_bitwise(gdims, grid, overlap):   # split by sites, or one launch after the exchange
     world = grid[2] * grid[3]
-    kw = {"persistent": persistent}
+    kw = {"overlap": overlap}
     for parity in (0, 1):
         got = _run(world, gdims, grid, kw, parity)
         ref = _single(gdims, kw, parity)
@@ -147,13 +147,3 @@ def test_multirank_p2p_overlap_dirs(gdims, grid):
         fat, lng = fieldgen.workload_links(gdims)
         o = oracle.full_to_cb(oracle.dslash(fat, lng, fieldgen.vector(gdims, SEED), 1), 1)
         assert oracle.normwise_error(got[0], o) <= (1e-12 if tol == 1e-14 else 1e-5)
-
-
-@pytest.mark.parametrize("gdims,grid", [((8, 8, 8, 16), (1, 1, 1, 2)), ((8, 8, 8, 8), (1, 1, 2, 2)),
-                                        ((8, 8, 8, 24), (1, 1, 1, 3))])
-def test_multirank_p2p_overlap_fused(gdims, grid):
-    """The one-shot fused overlap across real ranks (neighbours raise the ready flags the boundary
-    blocks look at): bitwise equal to the 1-rank apply."""
-    world = grid[2] * grid[3]
-    got = _run(world, gdims, grid, {"overlap": "fused"}, 0)
-    assert np.array_equal(got, _single(gdims, {}, 0))

@@ -162,6 +162,4 @@ def test_dirs_option_errors(torch_cuda):
     from paper_conf_sc_dufekgaad024_b200 import Dslash, DslashError, _abi
     with Dslash((16, 8, 8, 8)) as D:
         with pytest.raises(DslashError):
-            _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_OVERLAP, 4)
-    with pytest.raises(DslashError):
-        Dslash((16, 8, 8, 8), kernel="bulk", overlap="dirs")
+            _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_OVERLAP, 3)   # the removed one-shot fused mode

@@ -106,7 +106,7 @@ def test_recon9_folded_phases(torch_cuda, kernel):
 
 @pytest.mark.gpu
 def test_recon9_halo_paths_and_rhs_bitwise(torch_cuda):
-    """Self-halo (t, z, t+z), split by direction, one-shot fused, persistent, staged and multi-RHS
+    """Self-halo (t, z, t+z), split by direction, producer push, staged and multi-RHS
     recon-9 applies against the unpartitioned recon-9 apply: bitwise where the per-site
     arithmetic is the same, within 1e-13 where the summation order differs."""
     torch = torch_cuda
@@ -123,8 +123,6 @@ def test_recon9_halo_paths_and_rhs_bitwise(torch_cuda):
     ref = oracle.full_to_cb(oracle.dslash(fat, lng, fieldgen.vector(dims, 10), 1), 1)
     assert oracle.normwise_error(base[0].numpy(), ref) <= 1e-12
     for kw, exact in (({"force_halo": 0x8}, True), ({"force_halo": 0xC}, True),
-                      ({"force_halo": 0xC, "overlap": "fused"}, True),
-                      ({"force_halo": 0xC, "persistent": True}, True),
                       ({"force_halo": 0xC, "transport": "p2p", "push": True}, True),
                       ({"force_halo": 0xC, "overlap": "dirs"}, False),
                       ({"stage": True}, False)):
@@ -167,13 +165,6 @@ def test_recon9_rejections(torch_cuda):
             with pytest.raises(_abi.DslashError) as e:
                 D.load_links(fat, bad)
             assert e.value.status == _abi.DSLASH_ERR_ARG
-    for kw in ({"kernel": "bulk"}, {"kernel": "bulk", "precision": "f32"}):   # the register kernels only
-        d16 = (16, 8, 8, 8)   # the TMA kernel needs Lx / 2 to be a multiple of 8
-        with Dslash(d16, recon=9, **kw) as D:
-            fat, lng = fieldgen.links(d16, 1), fieldgen.links(d16, 2, scale=fieldgen.LONG_SCALE)
-            with pytest.raises(_abi.DslashError) as e:
-                D.load_links(fat, lng)
-            assert e.value.status == _abi.DSLASH_ERR_UNSUPPORTED
     import torch
     fat = fieldgen.links(dims, 1)
     lng = fieldgen.links(dims, 2, scale=fieldgen.LONG_SCALE)

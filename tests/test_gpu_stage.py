@@ -163,3 +163,24 @@ def test_stage_option_errors(torch_cuda):
     with Dslash((8, 8, 8, 8), stage=True) as D:
         with pytest.raises(DslashError):
             _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_KERNEL, _abi.DSLASH_KERNEL_DIR4)
+
+
+def test_stage_cg_mixed_odd_half_row_refused(torch_cuda):
+    """dslash_cg_mixed runs an F64 handle's kernels as F32 ones (SloppyScope).  With the staged
+    kernel and Lx/2 odd the fp32 rows are not 16-byte multiples, so cp.async.bulk would fault:
+    the launch refuses with DSLASH_ERR_UNSUPPORTED before any copy is issued, and the context
+    stays usable (an unstaged solve on a fresh handle still converges)."""
+    from paper_conf_sc_dufekgaad024_b200 import Dslash, DslashError, _abi
+    torch = torch_cuda
+    dims = (6, 8, 8, 8)                                          # Lx/2 = 3
+    fat, lng = fieldgen.workload_links(dims)
+    b = torch.from_numpy(fieldgen.vector_cb(dims, 4, 0)).cuda()
+    with Dslash(dims, stage=True) as D:                          # fp64 rows (48 B): allowed
+        D.load_links(fat, lng)
+        with pytest.raises(DslashError) as e:
+            D.cg_mixed(D.empty_vector(), b, 0, 0.5, rel_tol=1e-10)
+        assert e.value.status == _abi.DSLASH_ERR_UNSUPPORTED
+    with Dslash(dims) as D:
+        D.load_links(fat, lng)
+        ok, it, outer, res = D.cg_mixed(D.empty_vector(), b, 0, 0.5, rel_tol=1e-10)
+        assert ok and res <= 2e-10

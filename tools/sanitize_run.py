@@ -16,15 +16,14 @@ dims = (16, 8, 8, 8)
 fat, lng = fieldgen.workload_links(dims)
 src = {p: torch.from_numpy(fieldgen.vector_cb(dims, 3, p)).cuda() for p in (0, 1)}
 ref = None
-cases = [dict(kernel=k) for k in ("site", "dir2", "dir4", "bulk")]
-cases += [dict(force_halo=m, persistent=pers) for m in (0x8, 0xC) for pers in (False, True)]
+cases = [dict(kernel=k) for k in ("site", "dir2", "dir4")]
+cases += [dict(force_halo=m, overlap=ov) for m in (0x8, 0xC) for ov in (True, False)]
 cases += [dict(force_halo=0xC, transport="p2p"), dict(recon=12), dict(precision="mixed"), dict(pdl=False)]
 # later additions: the neighbour-staged kernel (TMA bulk copies + mbarrier into shared memory), the
-# split-by-direction and one-shot fused overlaps (with and without forced deferral), NCCL to self,
+# split-by-direction overlap, NCCL to self,
 # and the mixed-precision CG (fp32 links converted from the fp64 ones)
 cases += [dict(stage=True), dict(stage=True, kernel="site", force_halo=0xC), dict(stage=True, precision="f32"),
           dict(force_halo=0xC, overlap="dirs"), dict(force_halo=0xC, overlap="dirs", precision="f32"),
-          dict(force_halo=0xC, overlap="fused"), dict(force_halo=0x8, overlap="fused", defer=True),
           dict(force_halo=0xC, self_nccl=True), dict(cg_mixed=True)]
 # third session: the producer push (stencil epilogue and CG direction update store into the
 # peer-mapped ghost bank; flag waits/writes on the streams) and recon-9 long links
@@ -33,13 +32,9 @@ cases += [dict(force_halo=0xC, transport="p2p", push=True), dict(force_halo=0x8,
 n = 0
 for kw in cases:
     kw = dict(kw)
-    defer = kw.pop("defer", False)
     mixed_cg = kw.pop("cg_mixed", False)
     with Dslash(dims, **kw) as D:
         D.load_links(fat, lng)
-        if defer:
-            from paper_conf_sc_dufekgaad024_b200 import _abi
-            _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_FUSED_DEFER, 1)
         if mixed_cg:
             x = D.empty_vector()
             D.cg_mixed(x, src[0], 0, 0.5, rel_tol=1e-8, inner_tol=1e-2, max_iter=100)
@@ -50,7 +45,7 @@ for kw in cases:
         multi = torch.stack([src[1], src[1]]).to(D.dtype)
         mo = torch.empty_like(multi)
         D.apply_multi(mo, multi, 0)
-        if D.precision != "f32" and kw.get("kernel") != "bulk":
+        if D.precision != "f32":
             x = D.empty_vector()
             D.cg(x, src[0], 0, 0.5, rel_tol=1e-8, max_iter=50)
         torch.cuda.synchronize()
