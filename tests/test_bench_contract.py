@@ -47,3 +47,28 @@ def test_product_arm_fails_loudly_without_gpu():
     r = _run(["--steps", "3", "--warmup", "3", "--no-cpu-baseline"])
     assert r.returncode != 0
     assert '"value"' not in r.stdout          # no number from a CPU fallback
+
+
+def test_self_launch_without_torchrun():
+    """`bench.py --gpus N` outside torchrun launches N ranks itself (torch.distributed.run,
+    127.0.0.1 rendezvous); rank 0 alone prints one JSON line holding the max over ranks.  The
+    CPU variant of the same launch path (--selftest-launch: gloo, no CUDA)."""
+    r = _run(["--gpus", "2", "--selftest-launch"], timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.strip()]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["world_size"] == 2 and d["n_gpus"] == 2 and d["max_over_ranks"] == 2.0
+
+
+def test_strong_scaling_grid_rule():
+    """The documented strong-scaling process-grid rule (bench.choose_grid): maximise
+    the interior fraction, then the fewest face bytes, then the larger Pt."""
+    sys.path.insert(0, ROOT)
+    import bench
+    assert bench.choose_grid((48, 48, 48, 48), 1) == (1, 1, 1, 1)
+    assert bench.choose_grid((48, 48, 48, 48), 2) == (1, 1, 1, 2)
+    assert bench.choose_grid((48, 48, 48, 48), 4) == (1, 1, 1, 4)      # Lt = 12: 50% interior
+    assert bench.choose_grid((48, 48, 48, 48), 8) == (1, 1, 2, 4)      # t8 (Lt = 6) has no interior site
+    assert bench.interior_fraction((48, 48, 24, 12), (2, 3)) == 0.375
+    assert bench.interior_fraction((48, 48, 48, 6), (3,)) == 0.0
