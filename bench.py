@@ -203,17 +203,21 @@ def ncu_traffic(kernel_name, local_dims):
 
 class ClockSampler:
     """Samples SM clock and throttle reasons with NVML from the start of the warm-up to the end of
-    the timed region (every ~0.25 ms, so even a 20-step run of ~5 ms gets >= 10 samples)."""
+    the timed region.  The polling thread starts (and makes its first, slow NVML calls) before
+    the window opens; inside the window it records a sample every ~0.1 ms and the interpreter
+    switches threads every 50 us, so even a 20-step run (~5 ms of GPU work) gets >= 10 samples."""
 
     REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
                0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
                0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
-    PERIOD_S = 0.00025
+    PERIOD_S = 0.0001
 
     def __init__(self, device_index):
         self.samples, self.reasons, self.max_mhz = [], 0, None
         self._stop = threading.Event()
+        self._active = threading.Event()
         self.t_start = self.t_stop = None
+        self._switch = sys.getswitchinterval()
         try:
             import pynvml
             pynvml.nvmlInit()
@@ -222,26 +226,46 @@ class ClockSampler:
             self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.hdl, pynvml.NVML_CLOCK_SM)
         except Exception:
             self.nv = None
+        if self.nv:
+            self._ready = threading.Event()
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+            self._ready.wait(5.0)
+
+    def _sample(self):
+        c = self.nv.nvmlDeviceGetClockInfo(self.hdl, self.nv.NVML_CLOCK_SM)
+        r = int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.hdl))
+        return c, r
 
     def _run(self):
+        try:
+            self._sample()          # first calls (lazy NVML setup) outside the window
+        except Exception:
+            pass
+        self._ready.set()
         while not self._stop.is_set():
+            if not self._active.wait(0.001):
+                continue
             try:
-                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.hdl, self.nv.NVML_CLOCK_SM))
-                self.reasons |= int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.hdl))
+                c, r = self._sample()
+                if self._active.is_set():
+                    self.samples.append(c)
+                    self.reasons |= r
             except Exception:
                 pass
             time.sleep(self.PERIOD_S)
 
     def start(self):
+        sys.setswitchinterval(5e-5)
         self.t_start = time.perf_counter()
-        if self.nv:
-            self.t = threading.Thread(target=self._run, daemon=True)
-            self.t.start()
+        self._active.set()
         return self
 
     def stop(self):
-        self._stop.set()
+        self._active.clear()
         self.t_stop = time.perf_counter()
+        sys.setswitchinterval(self._switch)
+        self._stop.set()
         if self.nv:
             self.t.join()
 

@@ -13,10 +13,10 @@ i=0
 for cmd in "$@"; do
   i=$((i+1)); f=$(printf "%s/%02d.txt" "$out" $i)
   echo "\$ $cmd" > "$f"
-  t0=$(date +%s.%N)
+  t0=$(date +%s%N)
   bash -c "$cmd" >> "$f" 2>&1
   rc=$?
-  t1=$(date +%s.%N)
-  printf "%02d rc=%d %.1fs %s\n" $i $rc $(echo "$t1 - $t0" | bc) "$cmd" | tee -a "$out/summary.txt"
+  t1=$(date +%s%N)
+  printf "%02d rc=%d %ds %s\n" $i $rc $(( (t1 - t0) / 1000000000 )) "$cmd" | tee -a "$out/summary.txt"
   tail -3 "$f"
 done
