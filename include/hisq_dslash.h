@@ -160,10 +160,13 @@ enum {
     DSLASH_TRANSPORT_P2P = 1   /* SM-free: faces are copied by the copy engines straight into the
                                   neighbours' CUDA-IPC-mapped ghost buffers (NVLink within a node),
                                   and cuStreamWriteValue32/WaitValue32 epoch flags order producers and
-                                  consumers.  Needs dslash_get_ipc_blob / dslash_open_ipc_blobs, and
-                                  dslash_load_links_halo when neighbours are other ranks.  Also works
-                                  for several ranks on ONE GPU (NCCL refuses that).  At most 8
-                                  right-hand sides per apply                                         */
+                                  consumers.  Needs dslash_get_ipc_blob / dslash_open_ipc_blobs before
+                                  load_links when neighbours are other ranks; load_links then copies
+                                  its top link slices into the plus neighbours' IPC-mapped slab
+                                  buffers itself, and the solver's dot products are summed through
+                                  the ranks' IPC-mapped control blocks.  Also works for several ranks
+                                  on ONE GPU (NCCL refuses that).  At most 8 right-hand sides per
+                                  apply                                                              */
 };
 
 /* Kernel classes for dslash_kernel_timing.  SPAN: with a halo and the classic split, the time
@@ -221,11 +224,15 @@ DSLASH_API dslash_status dslash_create(const int32_t global_dims[4], const int32
                             int32_t precision, const void* nccl_unique_id, int32_t nranks, int32_t rank,
                             dslash_t* out);
 
-/* P2P transport setup.  dslash_ipc_blob_size() bytes describe one rank's halo buffers (CUDA IPC
- * handles of its ghost buffers and epoch flags).  Every rank writes its blob with
- * dslash_get_ipc_blob, the caller all-gathers them (blobs of rank r at r * size) and every rank
- * calls dslash_open_ipc_blobs.  Both need DSLASH_OPT_TRANSPORT = P2P first.  Ranks must be on
- * GPUs of one node (or the same GPU). */
+/* P2P transport setup.  dslash_ipc_blob_size() bytes describe one rank's buffers (CUDA IPC
+ * handles of its ghost buffers, its link-slab receive buffers and its control block of epoch
+ * flags and reduction slots; the library allocates them, library-owned like the ghosts).  Every
+ * rank writes its blob with dslash_get_ipc_blob, the caller all-gathers them (blobs of rank r at
+ * r * size) and every rank calls dslash_open_ipc_blobs once, which maps every rank's control
+ * block and the neighbours' buffers.  Both need DSLASH_OPT_TRANSPORT = P2P (and DSLASH_OPT_PUSH,
+ * if wanted) first.  Ranks must be on GPUs of one node (or the same GPU).  Errors:
+ * DSLASH_ERR_ARG for a malformed or misordered blob (e.g. from another library version),
+ * DSLASH_ERR_STATE for a second dslash_open_ipc_blobs. */
 DSLASH_API int64_t dslash_ipc_blob_size(void);
 DSLASH_API dslash_status dslash_get_ipc_blob(dslash_t h, void* blob);
 DSLASH_API dslash_status dslash_open_ipc_blobs(dslash_t h, const void* blobs);
@@ -241,9 +248,13 @@ DSLASH_API dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
  * building the back-links F(x-mu,mu)^dag and N(x-3mu,mu)^dag (|l| = 4
  * link arrays; Z2).  fat, lng: canonical layout over the local volume,
  * fp64 complex; on_device = 1 if they are device pointers, 0 for host memory.  When
- * partitioned, one NCCL exchange fetches the 3 link slices below each halo face.
+ * partitioned, every rank sends its top 3 link slices of each halo direction to its plus
+ * neighbour and receives the 3 slices below its origin from its minus neighbour: NCCL
+ * send/recv, or, with DSLASH_TRANSPORT_P2P, copy-engine copies straight into the plus
+ * neighbour's IPC-mapped slab buffer ordered by epoch flags (every rank of the partition must
+ * call load_links; DSLASH_ERR_STATE if the IPC blobs were not opened).
  * Synchronous: on return the caller may free fat and lng.  Callable again to replace
- * the links. */
+ * the links (collectively). */
 DSLASH_API dslash_status dslash_load_links(dslash_t h, const void* fat, const void* lng, int32_t on_device,
                                 dslash_stream_t stream);
 
@@ -251,8 +262,8 @@ DSLASH_API dslash_status dslash_load_links(dslash_t h, const void* fat, const vo
  * another rank, slab_fat[d] / slab_lng[d] hold the 3 coordinate slices just below the local
  * origin, taken from the minus neighbour's canonical links (its top 3 slices): layout
  * [d][z][y][x][mu][3][3] for d = t (3), [t][d][y][x][mu][3][3] for d = z (2).  Entries of other
- * directions are ignored (may be NULL).  Same device-ness as fat and lng (on_device).  This is
- * how the P2P transport (no NCCL communicator) loads links. */
+ * directions are ignored (may be NULL).  Same device-ness as fat and lng (on_device).  For
+ * callers that already hold the neighbours' slices (no exchange happens). */
 DSLASH_API dslash_status dslash_load_links_halo(dslash_t h, const void* fat, const void* lng,
                                                 const void* const slab_fat[4], const void* const slab_lng[4],
                                                 int32_t on_device, dslash_stream_t stream);
@@ -320,8 +331,12 @@ DSLASH_API dslash_status dslash_normal_apply(dslash_t h, void* out, const void* 
                                              dslash_stream_t stream);
 
 /* Conjugate gradient for A_p x = b (A_p as above), starting from x = 0, stopping when
- * |r_k| <= rel_tol |b| or after max_iter iterations.  Dot products are reduced
- * deterministically on each GPU and summed over ranks with ncclAllReduce.  With one rank the
+ * |r_k| <= rel_tol |b| or after max_iter iterations.  Dot products are accumulated as
+ * double-double sums (per thread, block, GPU and over the ranks in rank order: the per-rank
+ * sums are all-gathered with ncclAllGather, or through the P2P transport's IPC-mapped slots when
+ * the handle has no communicator) and rounded once, so every rank gets the same bits and a
+ * P-rank solve runs the 1-rank iterates bit for bit (unless a sum lies within ~1e-26 relative of
+ * a rounding boundary; DESIGN.md §12 f-3).  With one rank the
  * vector work of an iteration (m^2 p - q, both dot products, the x / r / p updates) runs as one
  * cooperative kernel with the same arithmetic and reduction order (bitwise the same iterates).  Synchronous:
  * returns after the solve (it reads each dot product on the host).  iters (may be NULL)

@@ -128,8 +128,6 @@ class Dslash:
     # -- links
     def load_links(self, fat, lng, stream=None):
         import numpy as np
-        if self.transport == "p2p" and self.world_size > 1:
-            return self._load_links_p2p(np.asarray(fat), np.asarray(lng), stream)
         if isinstance(fat, np.ndarray):
             fat = np.ascontiguousarray(fat, dtype=np.complex128)
             lng = np.ascontiguousarray(lng, dtype=np.complex128)
@@ -149,40 +147,6 @@ class Dslash:
         out = np.empty((self.vh, 4, 4, 3, 3), np.complex128)
         _abi.dslash_get_links(self.h, int(parity), out.ctypes.data)
         return out
-
-    def _load_links_p2p(self, fat, lng, stream):
-        """Link halo through torch.distributed: send my top 3 slices (t, then z) to the plus
-        neighbour, receive the 3 slices below my origin from the minus neighbour."""
-        import numpy as np
-        import torch
-        import torch.distributed as dist
-        fat = np.ascontiguousarray(fat, dtype=np.complex128)
-        lng = np.ascontiguousarray(lng, dtype=np.complex128)
-        self._check_links(fat.shape, lng.shape)
-        dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
-        slabs = {2: [None, None], 3: [None, None]}
-        keep = []
-        for d, axis in ((3, 0), (2, 1)):
-            if not self.plan.halo[d]:
-                continue
-            plus, minus = self.plan.nbr_rank[d][1], self.plan.nbr_rank[d][0]
-            for k, arr in enumerate((fat, lng)):
-                top = np.ascontiguousarray(np.take(arr, range(arr.shape[axis] - 3, arr.shape[axis]), axis=axis))
-                if plus == self.rank:
-                    slabs[d][k] = top
-                    continue
-                send = torch.from_numpy(top.view(np.float64)).to(dev)
-                recv = torch.empty_like(send)
-                reqs = [dist.isend(send, plus), dist.irecv(recv, minus)]
-                for r in reqs:
-                    r.wait()
-                slabs[d][k] = np.ascontiguousarray(recv.cpu().numpy()).view(np.complex128)
-        for d in (2, 3):
-            keep += [s for s in slabs[d] if s is not None]
-        sf = [slabs[d][0].ctypes.data if d in slabs and slabs[d][0] is not None else 0 for d in range(4)]
-        sl = [slabs[d][1].ctypes.data if d in slabs and slabs[d][1] is not None else 0 for d in range(4)]
-        _abi.dslash_load_links_halo(self.h, fat.ctypes.data, lng.ctypes.data, sf, sl, 0, _stream_handle(stream))
-        del keep
 
     def _check_links(self, a, b):
         lx, ly, lz, lt = self.local_dims

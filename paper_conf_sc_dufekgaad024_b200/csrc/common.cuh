@@ -166,6 +166,39 @@ __device__ __forceinline__ void cmsub(float2& acc, float2 a, float2 b) {
     acc.y = fmaf(-a.y, b.x, acc.y);
 }
 
+// ---------------------------------------------------------------- double-double sums
+// The solver's dot products are accumulated as unevaluated sums hi + lo (Dekker / Knuth TwoSum,
+// "double-double"), at every level: per thread, per block, over the blocks and over the ranks.
+// The rounded result hi is then the correctly rounded sum of the (bitwise identical, element-wise)
+// terms unless that exact sum lies within ~n u^2 |sum| of a rounding boundary, so it no longer
+// depends on how the lattice is split over ranks (DESIGN.md §12 f-3): a P-rank CG runs the
+// 1-rank iterates bit for bit.  Operands are combined with explicit __dadd_rn / __dsub_rn, which
+// the compiler never contracts or reassociates.
+__device__ __forceinline__ double2 two_sum(double a, double b) {
+    const double s = __dadd_rn(a, b);
+    const double bb = __dsub_rn(s, a);
+    const double e = __dadd_rn(__dsub_rn(a, __dsub_rn(s, bb)), __dsub_rn(b, bb));
+    return make_double2(s, e);
+}
+// x + t (t a double); renormalised with TwoSum (no |a| >= |b| precondition, so cancellation is safe)
+__device__ __forceinline__ double2 dd_add(double2 x, double t) {
+    const double2 s = two_sum(x.x, t);
+    return two_sum(s.x, __dadd_rn(s.y, x.y));
+}
+// x + y (both double-double; the low parts are added with TwoSum too).  Symmetric in x and y
+// (TwoSum's error term is exact), so a shuffle butterfly gives every lane the same bits.
+__device__ __forceinline__ double2 dd_add(double2 x, double2 y) {
+    const double2 s = two_sum(x.x, y.x);
+    const double2 t = two_sum(x.y, y.y);
+    const double2 u = two_sum(s.x, __dadd_rn(s.y, t.x));
+    return two_sum(u.x, __dadd_rn(u.y, t.y));
+}
+// Re(conj(a) b) of one complex element, in one fixed expression (the same bits in every kernel)
+__device__ __forceinline__ double dot_term(double2 a, double2 b) { return __fma_rn(a.x, b.x, __dmul_rn(a.y, b.y)); }
+__device__ __forceinline__ double dot_term(float2 a, float2 b) {
+    return __fma_rn((double)a.x, (double)b.x, __dmul_rn((double)a.y, (double)b.y));
+}
+
 // ---------------------------------------------------------------- kernel parameters
 constexpr int kMaxBoxes = 5;  // interior + up to 4 boundary slabs (t and z halo)
 

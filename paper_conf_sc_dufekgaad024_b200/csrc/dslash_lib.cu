@@ -200,10 +200,31 @@ static dslash_status alloc_halo(dslash_t h, int nrhs) {
 
 static constexpr int kP2PMaxRhs = 8;  // ghost capacity with the P2P transport (IPC-exported once)
 
+// the P2P control block (epoch flags, reduction slots; handle.h P2PControl)
 static dslash_status alloc_flags(dslash_t h) {
-    if (!h->flags) {
-        CU(h, cudaMalloc(&h->flags, 16 * sizeof(unsigned int)));
-        CU(h, cudaMemset(h->flags, 0, 16 * sizeof(unsigned int)));
+    if (!h->ctl) {
+        CU(h, cudaMalloc(&h->ctl, sizeof(P2PControl)));
+        CU(h, cudaMemset(h->ctl, 0, sizeof(P2PControl)));
+        h->flags = h->ctl->flags;
+    }
+    return DSLASH_OK;
+}
+
+// bytes of ONE kind (fat or long) of the 3 canonical link slices below the local origin in
+// direction d (the link halo of load_links)
+static size_t link_slab_bytes(const dslash_plan_t& p, int d) {
+    const int64_t V = 2 * p.vh_local;
+    return (size_t)3 * (V / p.local_dims[d]) * 36 * sizeof(double2);
+}
+
+// P2P: the link-slab receive buffers ([fat | long]) of the halo directions whose minus neighbour
+// is another rank; IPC-exported with the ghosts, so they exist before dslash_get_ipc_blob
+static dslash_status alloc_lslab(dslash_t h) {
+    const dslash_plan_t& p = h->plan;
+    for (int d = 2; d < 4; ++d) {
+        if (!p.halo[d] || p.nbr_rank[d][0] == p.rank || h->lslab[d]) continue;
+        h->lslab_bytes[d] = link_slab_bytes(p, d);
+        CU(h, cudaMalloc(&h->lslab[d], 2 * h->lslab_bytes[d]));
     }
     return DSLASH_OK;
 }
@@ -372,6 +393,12 @@ static int lanes_of(int kernel) {
     return kernel == DSLASH_KERNEL_DIR4 ? 4 : kernel == DSLASH_KERNEL_DIR2 ? 2 : 1;
 }
 
+typedef int (*WriteValue32Fn)(cudaStream_t, unsigned long long, unsigned int, unsigned int);
+typedef int (*WaitValue32Fn)(cudaStream_t, unsigned long long, unsigned int, unsigned int);
+static WriteValue32Fn write_value_fn();
+static WaitValue32Fn wait_value_fn();
+static dslash_status p2p_prepare(dslash_t h);
+
 // ============================================================================ link loading
 // slab_fat / slab_lng (may be NULL): caller-provided lower link slabs per direction (same device-ness
 // as fat / lng); where absent for a halo direction with another rank as neighbour, NCCL fetches them
@@ -384,7 +411,25 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
     const int64_t V = 2 * p.vh_local;
     const size_t canon_bytes = (size_t)V * 36 * sizeof(double2);
     std::vector<void*> tmp;
+    // P2P link halo (below): directions whose slab arrives in h->lslab, and the epoch of this load
+    bool p2p_link[4] = {false, false, false, false};
+    unsigned int le = 0;
+    bool p2p_released = false;
+    // my slab buffers are consumed (or this load failed after the exchange): release them to my
+    // minus neighbours, so their next load_links does not wait forever
+    auto release_p2p = [&]() -> bool {
+        if (!le || p2p_released) return true;
+        p2p_released = true;
+        WriteValue32Fn wr = write_value_fn();
+        for (int d = 3; d >= 2; --d)
+            if (p2p_link[d] && wr((cudaStream_t)stream,
+                                  (unsigned long long)(uintptr_t)(h->peer_ctl[h->plan.nbr_rank[d][0]]->flags + 20 + d),
+                                  le, 0) != 0)
+                return false;
+        return true;
+    };
     auto cleanup = [&]() {
+        release_p2p();
         for (void* q : tmp) cudaFree(q);
     };
 #define CUL(call)                                                                                     \
@@ -426,22 +471,37 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
     C.halo_mask = halo_mask;
     double2* slab[4][2] = {};   // [mu][fat/long] received
     double2* send[4][2] = {};   // packed top slabs (z, NCCL only)
-    for (int d = 2; d < 4; ++d) {
-        if (!p.halo[d]) continue;
-        const int64_t slab_elems = 3 * (V / p.local_dims[d]) * 36;
-        for (int k = 0; k < 2; ++k) {
-            CUL(cudaMalloc(&slab[d][k], slab_elems * sizeof(double2)));
-            tmp.push_back(slab[d][k]);
-        }
-    }
     // Exchange: rank sends its top 3 slices to its plus neighbour, receives into its lower
     // slab from its minus neighbour.  All ranks issue t then z, fat then long (same order).
+    // NCCL transport: ncclSend / ncclRecv.  P2P transport: the slices are copied straight into
+    // the plus neighbour's IPC-mapped slab buffer (p2p_link), ordered by epoch flags.
     bool need_nccl = false;
     bool given[4] = {false, false, false, false};
     for (int d = 3; d >= 2; --d) {
         if (!p.halo[d]) continue;
         given[d] = slab_fat_in && slab_lng_in && slab_fat_in[d] && slab_lng_in[d];
-        if (!given[d] && exch_remote(h, d)) need_nccl = true;
+        if (given[d] || !exch_remote(h, d)) continue;
+        if (h->transport == DSLASH_TRANSPORT_P2P)
+            p2p_link[d] = true;
+        else
+            need_nccl = true;
+    }
+    for (int d = 2; d < 4; ++d) {
+        if (!p.halo[d]) continue;
+        if (p2p_link[d]) {   // received in place, in the library-owned IPC-exported buffer
+            if (!h->lslab[d]) {
+                cleanup();
+                return fail(h, DSLASH_ERR_STATE, "P2P link halo: call dslash_get_ipc_blob / dslash_open_ipc_blobs first");
+            }
+            slab[d][0] = (double2*)h->lslab[d];
+            slab[d][1] = (double2*)(h->lslab[d] + h->lslab_bytes[d]);
+            continue;
+        }
+        const int64_t slab_elems = 3 * (V / p.local_dims[d]) * 36;
+        for (int k = 0; k < 2; ++k) {
+            CUL(cudaMalloc(&slab[d][k], slab_elems * sizeof(double2)));
+            tmp.push_back(slab[d][k]);
+        }
     }
     if (need_nccl && !h->nccl) {
         cleanup();
@@ -459,6 +519,7 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
             CUL(cudaMemcpyAsync(slab[d][1], slab_lng_in[d], bytes, kind, s));
             continue;
         }
+        if (p2p_link[d]) continue;   // below
         for (int k = 0; k < 2; ++k) {
             const double2* src = k ? dlng : dfat;
             if (d == 3) {
@@ -497,6 +558,49 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
             cleanup();
             return fail(h, DSLASH_ERR_NCCL, "link halo exchange: %s", ncclGetErrorString(r));
         }
+    }
+    // P2P link halo of epoch e: wait until my plus neighbour converted what I sent at e - 1,
+    // copy my top slices into its buffer, raise its lslab_ready; then wait for my minus
+    // neighbour's (all ranks send before they wait: no cycle of waits).  Released after the
+    // conversion below.
+    const bool any_p2p = p2p_link[2] || p2p_link[3];
+    if (any_p2p) {
+        dslash_status pst = p2p_prepare(h);
+        WriteValue32Fn wr = write_value_fn();
+        WaitValue32Fn wt = wait_value_fn();
+        if (pst == DSLASH_OK && (!wr || !wt)) pst = fail(h, DSLASH_ERR_UNSUPPORTED, "stream memory operations unavailable");
+        if (pst != DSLASH_OK) {
+            cleanup();
+            return pst;
+        }
+        le = ++h->link_epoch;
+        for (int d = 3; d >= 2; --d) {
+            if (!p2p_link[d]) continue;
+            const int plus = p.nbr_rank[d][1];
+            if (wt(s, (unsigned long long)(uintptr_t)(h->flags + 20 + d), le - 1, 0) != 0) {
+                cleanup();
+                return fail(h, DSLASH_ERR_CUDA, "cuStreamWaitValue32 (link slab free) failed");
+            }
+            for (int k = 0; k < 2; ++k) {
+                const double2* src = k ? dlng : dfat;
+                char* dst = h->peer_lslab[d] + k * h->lslab_bytes[d];
+                if (d == 3)
+                    CUL(cudaMemcpyAsync(dst, src + (size_t)(L3 - 3) * L2 * L1 * L0 * 36, 3 * (size_t)L2 * row,
+                                        cudaMemcpyDeviceToDevice, s));
+                else  // [t][z in L2-3..L2-1][y][x] -> [t][d][y][x]
+                    CUL(cudaMemcpy2DAsync(dst, 3 * row, src + (size_t)(L2 - 3) * L1 * L0 * 36, (size_t)L2 * row,
+                                          3 * row, L3, cudaMemcpyDeviceToDevice, s));
+            }
+            if (wr(s, (unsigned long long)(uintptr_t)(h->peer_ctl[plus]->flags + 16 + d), le, 0) != 0) {
+                cleanup();
+                return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 (link slab ready) failed");
+            }
+        }
+        for (int d = 3; d >= 2; --d)
+            if (p2p_link[d] && wt(s, (unsigned long long)(uintptr_t)(h->flags + 16 + d), le, 0) != 0) {
+                cleanup();
+                return fail(h, DSLASH_ERR_CUDA, "cuStreamWaitValue32 (link slab ready) failed");
+            }
     }
     for (int d = 0; d < 4; ++d) {
         C.slab_fat[d] = slab[d][0];
@@ -609,6 +713,10 @@ static dslash_status load_links_impl(dslash_t h, const void* fat, const void* ln
             convert_links_kernel<float><<<(unsigned)((n + bs - 1) / bs), bs, 0, s>>>(C);
         CUL(cudaGetLastError());
     }
+    if (!release_p2p()) {
+        cleanup();
+        return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 (link slab free) failed");
+    }
     CUL(cudaStreamSynchronize(s));
     cleanup();
 #undef CUL
@@ -691,7 +799,6 @@ extern "C" dslash_status dslash_load_links_halo(dslash_t h, const void* fat, con
 
 // cuStreamWriteValue32 through the runtime's driver entry point (no link-time libcuda): a stream's
 // front end writes the P2P epoch flags (ready / free), without an SM.
-typedef int (*WriteValue32Fn)(cudaStream_t, unsigned long long, unsigned int, unsigned int);
 static WriteValue32Fn write_value_fn() {
     static WriteValue32Fn fn = nullptr;
     static bool tried = false;
@@ -709,7 +816,6 @@ static WriteValue32Fn write_value_fn() {
 }
 
 // cuStreamWaitValue32 (flags 0 = CU_STREAM_WAIT_VALUE_GEQ: wait until (int32)(*addr - value) >= 0)
-typedef int (*WaitValue32Fn)(cudaStream_t, unsigned long long, unsigned int, unsigned int);
 static WaitValue32Fn wait_value_fn() {
     static WaitValue32Fn fn = nullptr;
     static bool tried = false;
@@ -729,26 +835,32 @@ static WaitValue32Fn wait_value_fn() {
 
 // ---------------------------------------------------------------------------- P2P transport
 struct IpcBlob {
-    int32_t magic, rank, device, reserved;
+    int32_t magic, rank, device, nranks;
     cudaIpcMemHandle_t ghost[4][2];
-    cudaIpcMemHandle_t flags;
+    cudaIpcMemHandle_t ctl;        // P2PControl: epoch flags, reduction slots
+    cudaIpcMemHandle_t lslab[4];   // link-slab receive buffers (halo directions, remote minus neighbour)
 };
-static constexpr int32_t kIpcMagic = 0x48495351;  // "HISQ"
+static constexpr int32_t kIpcMagic = 0x48495352;  // "HISR" (layout 2: control block + link slabs)
 
 extern "C" int64_t dslash_ipc_blob_size(void) { return (int64_t)sizeof(IpcBlob); }
 
 extern "C" dslash_status dslash_get_ipc_blob(dslash_t h, void* blob) {
     if (!h || !blob) return fail(h, DSLASH_ERR_ARG, "NULL argument");
     if (h->transport != DSLASH_TRANSPORT_P2P) return fail(h, DSLASH_ERR_STATE, "set DSLASH_TRANSPORT_P2P first");
+    dslash_status st = alloc_lslab(h);
+    if (st != DSLASH_OK) return st;
     IpcBlob b;
     memset(&b, 0, sizeof b);
     b.magic = kIpcMagic;
     b.rank = h->plan.rank;
     b.device = h->device;
-    for (int d = 2; d < 4; ++d)
+    b.nranks = h->plan.nranks;
+    for (int d = 2; d < 4; ++d) {
         for (int side = 0; side < 2; ++side)
             if (h->ghost[d][side]) CU(h, cudaIpcGetMemHandle(&b.ghost[d][side], h->ghost[d][side]));
-    CU(h, cudaIpcGetMemHandle(&b.flags, h->flags));
+        if (h->lslab[d]) CU(h, cudaIpcGetMemHandle(&b.lslab[d], h->lslab[d]));
+    }
+    CU(h, cudaIpcGetMemHandle(&b.ctl, h->ctl));
     memcpy(blob, &b, sizeof b);
     return DSLASH_OK;
 }
@@ -762,12 +874,35 @@ static void set_peer(dslash_t h, int d, int side, char* nbr_ghost_other_side, un
     h->peer_free[d][side] = nbr_flags + 8 + 2 * d + other;
 }
 
+static dslash_status ipc_open(dslash_t h, void** p, cudaIpcMemHandle_t handle) {
+    CU(h, cudaIpcOpenMemHandle(p, handle, cudaIpcMemLazyEnablePeerAccess));
+    h->ipc_opened.push_back(*p);
+    return DSLASH_OK;
+}
+
+// Every rank's control block (reduction slots, flags); the neighbours' ghosts and the plus
+// neighbours' link-slab buffers.
 extern "C" dslash_status dslash_open_ipc_blobs(dslash_t h, const void* blobs) {
     if (!h || !blobs) return fail(h, DSLASH_ERR_ARG, "NULL argument");
     if (h->transport != DSLASH_TRANSPORT_P2P) return fail(h, DSLASH_ERR_STATE, "set DSLASH_TRANSPORT_P2P first");
+    if (h->p2p_ready) return fail(h, DSLASH_ERR_STATE, "IPC blobs already opened");
     const dslash_plan_t& p = h->plan;
     const IpcBlob* all = static_cast<const IpcBlob*>(blobs);
-    std::vector<unsigned int*> flags_of(p.nranks, nullptr);
+    for (int r = 0; r < p.nranks; ++r)
+        if (all[r].magic != kIpcMagic || all[r].rank != r || all[r].nranks != p.nranks)
+            return fail(h, DSLASH_ERR_ARG, "IPC blob of rank %d is malformed or out of order", r);
+    dslash_status st = alloc_lslab(h);
+    if (st != DSLASH_OK) return st;
+    h->peer_ctl.assign(p.nranks, nullptr);
+    for (int r = 0; r < p.nranks; ++r) {
+        if (r == p.rank) {
+            h->peer_ctl[r] = h->ctl;
+            continue;
+        }
+        void* cp = nullptr;
+        if ((st = ipc_open(h, &cp, all[r].ctl)) != DSLASH_OK) return st;
+        h->peer_ctl[r] = static_cast<P2PControl*>(cp);
+    }
     for (int d = 2; d < 4; ++d) {
         if (!p.halo[d]) continue;
         for (int side = 0; side < 2; ++side) {
@@ -776,19 +911,15 @@ extern "C" dslash_status dslash_open_ipc_blobs(dslash_t h, const void* blobs) {
                 set_peer(h, d, side, h->ghost[d][1 - side], h->flags);
                 continue;
             }
-            const IpcBlob& b = all[nbr];
-            if (b.magic != kIpcMagic || b.rank != nbr)
-                return fail(h, DSLASH_ERR_ARG, "IPC blob of rank %d is malformed or out of order", nbr);
-            if (!flags_of[nbr]) {
-                void* fp = nullptr;
-                CU(h, cudaIpcOpenMemHandle(&fp, b.flags, cudaIpcMemLazyEnablePeerAccess));
-                h->ipc_opened.push_back(fp);
-                flags_of[nbr] = static_cast<unsigned int*>(fp);
-            }
             void* gp = nullptr;
-            CU(h, cudaIpcOpenMemHandle(&gp, b.ghost[d][1 - side], cudaIpcMemLazyEnablePeerAccess));
-            h->ipc_opened.push_back(gp);
-            set_peer(h, d, side, static_cast<char*>(gp), flags_of[nbr]);
+            if ((st = ipc_open(h, &gp, all[nbr].ghost[d][1 - side])) != DSLASH_OK) return st;
+            set_peer(h, d, side, static_cast<char*>(gp), h->peer_ctl[nbr]->flags);
+        }
+        const int plus = p.nbr_rank[d][1];
+        if (plus != p.rank) {
+            void* lp = nullptr;
+            if ((st = ipc_open(h, &lp, all[plus].lslab[d])) != DSLASH_OK) return st;
+            h->peer_lslab[d] = static_cast<char*>(lp);
         }
     }
     h->p2p_ready = true;
@@ -799,13 +930,41 @@ extern "C" dslash_status dslash_open_ipc_blobs(dslash_t h, const void* blobs) {
 static dslash_status p2p_prepare(dslash_t h) {
     if (h->p2p_ready) return DSLASH_OK;
     const dslash_plan_t& p = h->plan;
-    for (int d = 2; d < 4; ++d)
-        if (p.halo[d] && (p.nbr_rank[d][0] != p.rank || p.nbr_rank[d][1] != p.rank))
-            return fail(h, DSLASH_ERR_STATE, "P2P transport: call dslash_open_ipc_blobs first");
+    if (p.nranks > 1) return fail(h, DSLASH_ERR_STATE, "P2P transport: call dslash_open_ipc_blobs first");
+    dslash_status st = alloc_flags(h);
+    if (st != DSLASH_OK) return st;
+    h->peer_ctl.assign(1, h->ctl);
     for (int d = 2; d < 4; ++d)
         if (p.halo[d])
             for (int side = 0; side < 2; ++side) set_peer(h, d, side, h->ghost[d][1 - side], h->flags);
     h->p2p_ready = true;
+    return DSLASH_OK;
+}
+
+// Cross-rank gather of one double-double per rank for the solver's dot products (solver.cu
+// reduce_to_slot), without NCCL: copy `mine` into slot [rank] of bank e & 1 of every rank's
+// control block (copy engine; my own block too), raise red_flag[rank] = e there, and make s wait
+// until every rank's flag in MY block reached e.  Bank e & 1 can be rewritten only at e + 2, and a
+// rank starts e + 2 only after every rank contributed to e + 1, i.e. after every rank's stream
+// finished reading e's values (the rank sum precedes its next contribution in stream order).
+dslash_status hisq_p2p_gather(dslash_t h, cudaStream_t s, const double2* mine, const double2** all) {
+    const dslash_plan_t& p = h->plan;
+    dslash_status st = p2p_prepare(h);
+    if (st != DSLASH_OK) return st;
+    WriteValue32Fn wr = write_value_fn();
+    WaitValue32Fn wt = wait_value_fn();
+    if (!wr || !wt) return fail(h, DSLASH_ERR_UNSUPPORTED, "stream memory operations unavailable");
+    const unsigned int e = ++h->red_epoch;
+    const int bank = (int)(e & 1u);
+    for (int r = 0; r < p.nranks; ++r)
+        CU(h, cudaMemcpyAsync(&h->peer_ctl[r]->red_val[bank][p.rank], mine, sizeof(double2), cudaMemcpyDeviceToDevice, s));
+    for (int r = 0; r < p.nranks; ++r)
+        if (wr(s, (unsigned long long)(uintptr_t)&h->peer_ctl[r]->red_flag[p.rank], e, 0) != 0)
+            return fail(h, DSLASH_ERR_CUDA, "cuStreamWriteValue32 (reduction) failed");
+    for (int r = 0; r < p.nranks; ++r)
+        if (wt(s, (unsigned long long)(uintptr_t)&h->ctl->red_flag[r], e, 0) != 0)
+            return fail(h, DSLASH_ERR_CUDA, "cuStreamWaitValue32 (reduction) failed");
+    *all = &h->ctl->red_val[bank][0];
     return DSLASH_OK;
 }
 
@@ -1603,7 +1762,10 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
     }
     if (h->ev_batch) cudaEventDestroy(h->ev_batch);
     for (void* q : h->ipc_opened) cudaIpcCloseMemHandle(q);
-    if (h->flags) cudaFree(h->flags);
+    if (h->ctl) cudaFree(h->ctl);
+    for (char* q : h->lslab)
+        if (q) cudaFree(q);
+    if (h->cg_dd) cudaFree(h->cg_dd);
     for (void* v : h->cg_vec32)
         if (v) cudaFree(v);
     for (void* v : h->links32)

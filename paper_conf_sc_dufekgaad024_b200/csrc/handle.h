@@ -10,6 +10,23 @@
 #include "hisq_dslash.h"
 #include "dispatch.h"
 
+// P2P transport control block (device memory, CUDA-IPC-exported; every rank maps every other
+// rank's block).  Flags are epoch counters written by stream memory operations
+// (cuStreamWriteValue32) and waited on with cuStreamWaitValue32 (GEQ).
+constexpr int kMaxRanks = 64;
+struct P2PControl {
+    // [0..7] ready[d][side]: written by the neighbour that fills my ghost[d][side];
+    // [8..15] free_from[d][side]: written by the neighbour whose ghost my bottom (side 0) / top
+    //         (side 1) face fills, once it consumed it;
+    // [16..19] lslab_ready[d]: my minus neighbour filled my link-slab buffer of direction d;
+    // [20..23] lslab_free[d]: my plus neighbour converted the link slab I sent it
+    unsigned int flags[32];
+    // cross-rank reduction (dslash_cg without NCCL): rank r's double-double partial of reduction
+    // e lands in red_val[e & 1][r] and then red_flag[r] = e
+    unsigned int red_flag[kMaxRanks];
+    double2 red_val[2][kMaxRanks];
+};
+
 struct dslash_s {
     dslash_plan_t plan{};
     int32_t global_dims[4]{}, proc_grid[4]{};
@@ -49,11 +66,12 @@ struct dslash_s {
     // mixed-precision solver (dslash_cg_mixed): fp32 e, r, p, q, t and the fp32 links per parity
     void* cg_vec32[5] = {};
     void* links32[2] = {};
-    double* cg_partial = nullptr;
+    double2* cg_partial = nullptr;      // block partials, double-double
     double* cg_scalar = nullptr;
+    double2* cg_dd = nullptr;           // [0] this rank's sum, [1 + r] rank r's (ncclAllGather)
     // fused CG step (one rank): the |r|^2 block partials and the grid-barrier counter with the
     // arrivals expected by the end of the next launch's barrier
-    double* cg_partial2 = nullptr;
+    double2* cg_partial2 = nullptr;
     unsigned long long* cg_bar = nullptr;
     unsigned long long cg_bar_next = 0;
     int cg_fused = -1;  // -1: not probed yet; 0: cooperative launch unavailable; 1: fused step
@@ -72,7 +90,17 @@ struct dslash_s {
     int halo_dryrun = 0;                // DSLASH_OPT_HALO_DRYRUN (timing aid: exchange moves no bytes)
     int stage = 0;                      // DSLASH_OPT_STAGE: neighbour-staged kernel (x/y rows in smem by TMA)
     int self_nccl = 0;                  // DSLASH_OPT_SELF_NCCL: self-neighbour faces via NCCL
-    unsigned int* flags = nullptr;
+    P2PControl* ctl = nullptr;          // my control block (IPC-exported)
+    unsigned int* flags = nullptr;      // = ctl->flags
+    std::vector<P2PControl*> peer_ctl;  // every rank's control block (mine at [rank])
+    // link halo under P2P (dslash_load_links): the minus neighbour copies its top 3 link slices
+    // straight into lslab[d] ([fat | long], canonical slab layout), then raises my
+    // lslab_ready[d]; load_links_count numbers those exchanges
+    char* lslab[4] = {};
+    size_t lslab_bytes[4] = {};         // bytes of ONE kind (fat or long) in lslab[d]
+    char* peer_lslab[4] = {};           // my plus neighbour's lslab[d]
+    unsigned int link_epoch = 0;
+    unsigned int red_epoch = 0;         // cross-rank reductions so far
     char* peer_ghost[4][2] = {};        // [d][0]: minus nbr's plus ghost; [d][1]: plus nbr's minus ghost
     unsigned int* peer_ready[4][2] = {};  // the ready flag of that ghost
     unsigned int* peer_free[4][2] = {};   // [d][0]: minus nbr's free_from[d][1]; [d][1]: plus nbr's free_from[d][0]
@@ -127,6 +155,11 @@ dslash_status hisq_push_end(dslash_t h, cudaStream_t s, const void* out);
 // drop pushed faces no apply will consume (the CG's last direction update): the pushed epoch is
 // retired as if an apply had consumed it, on every rank alike
 dslash_status hisq_push_discard(dslash_t h, cudaStream_t s);
+
+// P2P transport, several ranks: copy this rank's double-double `mine` (device) into slot
+// [rank] of every rank's control block, raise their flags, and make stream s wait until every
+// rank's value has arrived in mine; *all = my control block's slots (nranks values, rank order)
+dslash_status hisq_p2p_gather(dslash_t h, cudaStream_t s, const double2* mine, const double2** all);
 
 // round the fp64 internal links of `parity` into h->links32[parity] (fp32 paired layout)
 dslash_status hisq_convert_links_sloppy(dslash_t h, int parity);

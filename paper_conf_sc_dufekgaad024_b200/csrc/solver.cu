@@ -5,8 +5,10 @@
 // With D anti-Hermitian (D_{p,1-p} = -D_{1-p,p}^dag, pin P3), the operator
 //     A_p = m^2 - D_{p,1-p} D_{1-p,p} = m^2 + D_{1-p,p}^dag D_{1-p,p}
 // is Hermitian positive definite on parity p for m != 0, and CG solves A_p x = b.
-// Dot products are reduced deterministically (fixed block partition, fixed final order) and,
-// with several ranks, summed with ncclAllReduce: the solver's one true collective.
+// Dot products are accumulated as double-double sums at every level (thread, block, grid, ranks;
+// common.cuh) and rounded once, so they do not depend on the decomposition: with several ranks
+// the per-rank sums are all-gathered (ncclAllGather, or the P2P transport's IPC-mapped slots)
+// and every rank adds them in rank order, the solver's one true collective.
 #include <chrono>
 #include <cmath>
 #include <cstdio>
@@ -17,19 +19,23 @@
 
 namespace {
 
+using hisq::dd_add;
+using hisq::dot_term;
+
 constexpr int kRedThreads = 256;
 constexpr int kRedBlocks = 592;  // 4 x 148 SMs; fixed, so the summation order never changes
 
-// block-level sum of v (all threads call); result valid in thread 0
-__device__ double block_sum(double v) {
-    __shared__ double warp_part[kRedThreads / 32];
+// block-level double-double sum of v (all threads call); result valid in thread 0
+__device__ double2 block_sum(double2 v) {
+    __shared__ double2 warp_part[kRedThreads / 32];
 #pragma unroll
-    for (int off = 16; off; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+    for (int off = 16; off; off >>= 1)
+        v = dd_add(v, make_double2(__shfl_xor_sync(0xffffffffu, v.x, off), __shfl_xor_sync(0xffffffffu, v.y, off)));
     if ((threadIdx.x & 31) == 0) warp_part[threadIdx.x >> 5] = v;
     __syncthreads();
-    double s = 0.0;
+    double2 s = make_double2(0.0, 0.0);
     if (threadIdx.x == 0)
-        for (int w = 0; w < kRedThreads / 32; ++w) s += warp_part[w];
+        for (int w = 0; w < kRedThreads / 32; ++w) s = dd_add(s, warp_part[w]);
     return s;
 }
 
@@ -39,31 +45,31 @@ __device__ double block_sum(double v) {
 // q = m2 p - q ; partial[block] = sum Re(conj(p) q)
 template <typename V2>
 __global__ void __launch_bounds__(kRedThreads) k_normal_finish(const V2* __restrict__ p, V2* __restrict__ q,
-                                                               double m2, int64_t n, double* __restrict__ partial) {
+                                                               double m2, int64_t n, double2* __restrict__ partial) {
     using R = decltype(V2{}.x);
-    double acc = 0.0;
+    double2 acc = make_double2(0.0, 0.0);
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const V2 a = p[i];
         V2 b = q[i];
         b.x = (R)m2 * a.x - b.x;
         b.y = (R)m2 * a.y - b.y;
         q[i] = b;
-        acc += (double)a.x * b.x + (double)a.y * b.y;
+        acc = dd_add(acc, dot_term(a, b));
     }
-    const double s = block_sum(acc);
+    const double2 s = block_sum(acc);
     if (partial && threadIdx.x == 0) partial[blockIdx.x] = s;
 }
 
 // partial[block] = sum |v|^2
 template <typename V2>
 __global__ void __launch_bounds__(kRedThreads) k_norm2(const V2* __restrict__ v, int64_t n,
-                                                       double* __restrict__ partial) {
-    double acc = 0.0;
+                                                       double2* __restrict__ partial) {
+    double2 acc = make_double2(0.0, 0.0);
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const V2 a = v[i];
-        acc += (double)a.x * a.x + (double)a.y * a.y;
+        acc = dd_add(acc, dot_term(a, a));
     }
-    const double s = block_sum(acc);
+    const double2 s = block_sum(acc);
     if (threadIdx.x == 0) partial[blockIdx.x] = s;
 }
 
@@ -74,10 +80,10 @@ template <typename V2>
 __global__ void __launch_bounds__(kRedThreads) k_cg_update(V2* __restrict__ x, V2* __restrict__ r,
                                                            const V2* __restrict__ p, const V2* __restrict__ q,
                                                            const double* __restrict__ rr, const double* __restrict__ pq,
-                                                           double stop, int64_t n, double* __restrict__ partial) {
+                                                           double stop, int64_t n, double2* __restrict__ partial) {
     using R = decltype(V2{}.x);
     const R alpha = (R)((*pq != 0.0 && *rr > stop) ? *rr / *pq : 0.0);
-    double acc = 0.0;
+    double2 acc = make_double2(0.0, 0.0);
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         V2 xi = x[i], ri = r[i];
         const V2 pi = p[i], qi = q[i];
@@ -87,18 +93,18 @@ __global__ void __launch_bounds__(kRedThreads) k_cg_update(V2* __restrict__ x, V
         ri.y = fma(-alpha, qi.y, ri.y);
         x[i] = xi;
         r[i] = ri;
-        acc += (double)ri.x * ri.x + (double)ri.y * ri.y;
+        acc = dd_add(acc, dot_term(ri, ri));
     }
-    const double s = block_sum(acc);
+    const double2 s = block_sum(acc);
     if (threadIdx.x == 0) partial[blockIdx.x] = s;
 }
 
 // sum of the kRedBlocks block partials in k_finalize's order (every block of kRedThreads threads
 // gets the same bits); result valid in thread 0
 // (coherent L2 loads: in the fused CG step other blocks wrote the partials during this launch)
-__device__ __forceinline__ double sum_partials(const double* partial, int n) {
-    double acc = 0.0;
-    for (int k = threadIdx.x; k < n; k += kRedThreads) acc += __ldcg(partial + k);
+__device__ __forceinline__ double2 sum_partials(const double2* partial, int n) {
+    double2 acc = make_double2(0.0, 0.0);
+    for (int k = threadIdx.x; k < n; k += kRedThreads) acc = dd_add(acc, __ldcg(partial + k));
     return block_sum(acc);
 }
 
@@ -165,37 +171,37 @@ template <typename V2>
 __global__ void __launch_bounds__(kRedThreads) k_cg_step(V2* __restrict__ x, V2* __restrict__ r, V2* __restrict__ p,
                                                          V2* __restrict__ q, double m2, const double* __restrict__ rr,
                                                          double* __restrict__ pq_out, double* __restrict__ rr_new_out,
-                                                         double stop, int64_t n, double* partial,
-                                                         double* partial2, unsigned long long* bar,
+                                                         double stop, int64_t n, double2* partial,
+                                                         double2* partial2, unsigned long long* bar,
                                                          unsigned long long target, double* rr_host,
                                                          const FacePush F) {
     using R = decltype(V2{}.x);
     __shared__ double s_val;
     {  // q = m2 p - q and the <p, q> block partials (k_normal_finish), then a grid barrier
-        double acc0 = 0.0;
+        double2 acc0 = make_double2(0.0, 0.0);
         for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
             const V2 a = p[i];
             V2 b = q[i];
             b.x = (R)m2 * a.x - b.x;
             b.y = (R)m2 * a.y - b.y;
             q[i] = b;
-            acc0 += (double)a.x * b.x + (double)a.y * b.y;
+            acc0 = dd_add(acc0, dot_term(a, b));
         }
-        const double s = block_sum(acc0);
+        const double2 s = block_sum(acc0);
         if (threadIdx.x == 0) {
             partial[blockIdx.x] = s;
             grid_arrive_wait(bar, target - kRedBlocks);
         }
         __syncthreads();
     }
-    double s0 = sum_partials(partial, kRedBlocks);
+    const double s0 = sum_partials(partial, kRedBlocks).x;   // one rank: the rounded sum is hi
     if (threadIdx.x == 0) s_val = s0;
     __syncthreads();
     const double pq = s_val;
     if (blockIdx.x == 0 && threadIdx.x == 0) *pq_out = pq;
     const double rrv = *rr;
     const R alpha = (R)((pq != 0.0 && rrv > stop) ? rrv / pq : 0.0);
-    double acc = 0.0;
+    double2 acc = make_double2(0.0, 0.0);
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         V2 xi = x[i], ri = r[i];
         const V2 pi = p[i], qi = q[i];
@@ -205,15 +211,15 @@ __global__ void __launch_bounds__(kRedThreads) k_cg_step(V2* __restrict__ x, V2*
         ri.y = fma(-alpha, qi.y, ri.y);
         x[i] = xi;
         r[i] = ri;
-        acc += (double)ri.x * ri.x + (double)ri.y * ri.y;
+        acc = dd_add(acc, dot_term(ri, ri));
     }
-    const double s1 = block_sum(acc);
+    const double2 s1 = block_sum(acc);
     if (threadIdx.x == 0) {
         partial2[blockIdx.x] = s1;
         grid_arrive_wait(bar, target);
     }
     __syncthreads();
-    const double s2 = sum_partials(partial2, kRedBlocks);
+    const double s2 = sum_partials(partial2, kRedBlocks).x;
     __syncthreads();  // s_val is reused
     if (threadIdx.x == 0) s_val = s2;
     __syncthreads();
@@ -261,14 +267,26 @@ __global__ void k_sub_from(double2* __restrict__ r, const double2* __restrict__ 
     }
 }
 
-// out[0] = sum_{k < n} partial[k]: thread t sums k = t, t + 256, ... in order, then the fixed
-// shuffle tree of block_sum (one block: deterministic)
-__global__ void __launch_bounds__(kRedThreads) k_finalize(const double* __restrict__ partial, int n,
-                                                          double* __restrict__ out) {
-    double acc = 0.0;
-    for (int k = threadIdx.x; k < n; k += kRedThreads) acc += partial[k];
-    const double s = block_sum(acc);
-    if (threadIdx.x == 0) out[0] = s;
+// The rank's double-double sum of the n block partials (thread t adds k = t, t + 256, ... in order,
+// then the fixed shuffle tree of block_sum): *dd_out (for the cross-rank sum) and, with one rank,
+// the rounded result *out = hi (out may be NULL)
+__global__ void __launch_bounds__(kRedThreads) k_finalize(const double2* __restrict__ partial, int n,
+                                                          double2* __restrict__ dd_out, double* __restrict__ out) {
+    double2 acc = make_double2(0.0, 0.0);
+    for (int k = threadIdx.x; k < n; k += kRedThreads) acc = dd_add(acc, partial[k]);
+    const double2 s = block_sum(acc);
+    if (threadIdx.x == 0) {
+        *dd_out = s;
+        if (out) *out = s.x;
+    }
+}
+
+// *out = the rounded sum of the ranks' double-double sums v[0..n), added in rank order (every rank
+// runs this on the same gathered values: the same bits everywhere)
+__global__ void k_rank_sum(const double2* __restrict__ v, int n, double* __restrict__ out) {
+    double2 acc = make_double2(0.0, 0.0);
+    for (int r = 0; r < n; ++r) acc = dd_add(acc, v[r]);
+    *out = acc.x;
 }
 
 }  // namespace
@@ -287,8 +305,9 @@ static dslash_status need_scratch(dslash_t h) {
     const size_t bytes = 3 * (size_t)h->plan.vh_local * sizeof(double2);
     for (void*& v : h->cg_vec)
         if (!v) CU(h, cudaMalloc(&v, bytes));
-    if (!h->cg_partial) CU(h, cudaMalloc(&h->cg_partial, kRedBlocks * sizeof(double)));
-    if (!h->cg_partial2) CU(h, cudaMalloc(&h->cg_partial2, kRedBlocks * sizeof(double)));
+    if (!h->cg_partial) CU(h, cudaMalloc(&h->cg_partial, kRedBlocks * sizeof(double2)));
+    if (!h->cg_partial2) CU(h, cudaMalloc(&h->cg_partial2, kRedBlocks * sizeof(double2)));
+    if (!h->cg_dd) CU(h, cudaMalloc(&h->cg_dd, (1 + kMaxRanks) * sizeof(double2)));
     if (!h->cg_bar) {
         CU(h, cudaMalloc(&h->cg_bar, sizeof(unsigned long long)));
         CU(h, cudaMemset(h->cg_bar, 0, sizeof(unsigned long long)));
@@ -298,11 +317,24 @@ static dslash_status need_scratch(dslash_t h) {
     return DSLASH_OK;
 }
 
-// the partials of one reduction -> global sum over all ranks in device scalar `slot`
+// the partials of one reduction -> global sum over all ranks in device scalar `slot`: this rank's
+// double-double sum, then (several ranks) an all-gather of every rank's and their sum in rank
+// order.  NCCL groups gather with ncclAllGather; the P2P transport (no communicator, e.g. several
+// ranks on one GPU) through the ranks' IPC-mapped control blocks (hisq_p2p_gather).
 static dslash_status reduce_to_slot(dslash_t h, cudaStream_t s, double* slot) {
-    k_finalize<<<1, kRedThreads, 0, s>>>(h->cg_partial, kRedBlocks, slot);
+    const int n = h->plan.nranks;
+    k_finalize<<<1, kRedThreads, 0, s>>>(h->cg_partial, kRedBlocks, h->cg_dd, n == 1 ? slot : nullptr);
     CU(h, cudaGetLastError());
-    if (h->nccl) NC(h, ncclAllReduce(slot, slot, 1, ncclDouble, ncclSum, h->nccl, s));
+    if (n == 1) return DSLASH_OK;
+    const double2* all = h->cg_dd + 1;
+    if (h->nccl) {
+        NC(h, ncclAllGather(h->cg_dd, h->cg_dd + 1, 2, ncclDouble, h->nccl, s));
+    } else {
+        dslash_status st = hisq_p2p_gather(h, s, h->cg_dd, &all);
+        if (st != DSLASH_OK) return st;
+    }
+    k_rank_sum<<<1, 1, 0, s>>>(all, n, slot);
+    CU(h, cudaGetLastError());
     return DSLASH_OK;
 }
 
@@ -324,8 +356,10 @@ static dslash_status check_solver_args(dslash_t h, const void* a, const void* b,
     if (h->precision == DSLASH_F32)
         return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the solver works on fp64 vectors (DSLASH_F64 or DSLASH_MIXED)");
     if (!h->loaded) return hisq_fail(h, DSLASH_ERR_STATE, "solver before load_links");
-    if (reduces && h->plan.nranks > 1 && !h->nccl)
-        return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "dot products across ranks need an NCCL communicator");
+    if (reduces && h->plan.nranks > 1 && !h->nccl && h->transport != DSLASH_TRANSPORT_P2P)
+        return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "dot products across ranks need NCCL or the P2P transport");
+    if (h->plan.nranks > kMaxRanks)
+        return hisq_fail(h, DSLASH_ERR_UNSUPPORTED, "the solver sums over at most %d ranks", kMaxRanks);
     if (!a || !b || ((uintptr_t)a & 15) || ((uintptr_t)b & 15))
         return hisq_fail(h, DSLASH_ERR_ARG, "NULL or misaligned vector");
     const uintptr_t n = 3 * (uintptr_t)h->plan.vh_local * sizeof(double2);
@@ -422,7 +456,7 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
         cudaGetLastError();
         h->cg_fused = (ok && ok32 && !getenv("HISQ_CG_UNFUSED")) ? 1 : 0;
     }
-    const bool fused = h->cg_fused == 1 && !h->nccl;
+    const bool fused = h->cg_fused == 1 && h->plan.nranks == 1;
     // HISQ_CG_PROFILE=1: host time per iteration spent enqueueing vs waiting, to stderr
     static const bool prof = getenv("HISQ_CG_PROFILE") != nullptr;
     using clk = std::chrono::steady_clock;
@@ -444,8 +478,8 @@ static dslash_status cg_core(dslash_t h, V2* x, V2* r, V2* p, V2* q, V2* t, int3
             int64_t n_v = n;
             double* pq_slot = &sc[2];
             const double* rr_c = rr_cur;
-            double* part = h->cg_partial;
-            double* part2 = h->cg_partial2;
+            double2* part = h->cg_partial;
+            double2* part2 = h->cg_partial2;
             unsigned long long* bar = h->cg_bar;
             double* rr_host = host_rr_dev + k;  // host_rr[k], written by the kernel
             void* args[] = {&x,    &r,    &p,     &q,   &m2_v,   &rr_c,    &pq_slot, &rr_new,

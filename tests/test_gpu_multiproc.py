@@ -18,6 +18,7 @@ import oracle
 pytestmark = pytest.mark.gpu
 
 SEED = 3
+CG_MASS = 0.1
 
 
 def _free_port():
@@ -32,14 +33,35 @@ def _rank_main(rank, world, port, gdims, grid, kw, parity, napply, nrhs, q):
     import torch
     import torch.distributed as dist
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
-    torch.cuda.set_device(0)
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    kw = dict(kw)
+    mode = kw.pop("_mode", "apply")              # "apply", "cg" or "cg_mixed"
+    distinct = kw.pop("_distinct", False)        # one GPU per rank (needs >= world GPUs)
+    transport = kw.pop("transport", "p2p")
+    dev = rank if distinct else 0
+    torch.cuda.set_device(dev)
+    if transport == "nccl":
+        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", dev))
+    else:
+        dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         from paper_conf_sc_dufekgaad024_b200 import Dslash
-        D = Dslash(gdims, grid, rank=rank, world_size=world, transport="p2p", **kw)
+        D = Dslash(gdims, grid, rank=rank, world_size=world, transport=transport, **kw)
         o, e = D.origin, D.local_dims
         fat, lng = fieldgen.workload_links(gdims, origin=o, extent=e)
         D.load_links(fat, lng)
+        if mode != "apply":
+            b = torch.from_numpy(fieldgen.vector_cb(gdims, SEED, parity, origin=o, extent=e)).cuda()
+            x = D.empty_vector()
+            if mode == "cg":
+                ok, it, res = D.cg(x, b, parity, CG_MASS, rel_tol=1e-10, max_iter=2000)
+                info = (ok, it, res)
+            else:
+                ok, it, outer, res = D.cg_mixed(x, b, parity, CG_MASS, rel_tol=1e-10, inner_tol=1e-3, max_iter=4000)
+                info = (ok, it, outer, res)
+            torch.cuda.synchronize()
+            q.put((rank, tuple(o), tuple(e), x.cpu().numpy(), info))
+            D.close()
+            return
         if nrhs == 1:
             src = torch.from_numpy(fieldgen.vector_cb(gdims, SEED, 1 - parity, origin=o, extent=e)).cuda()
             out = D.empty_vector()
@@ -52,10 +74,10 @@ def _rank_main(rank, world, port, gdims, grid, kw, parity, napply, nrhs, q):
             for _ in range(napply):
                 D.apply_multi(out, src, parity)
         torch.cuda.synchronize()
-        q.put((rank, tuple(o), tuple(e), out.cpu().numpy()))
+        q.put((rank, tuple(o), tuple(e), out.cpu().numpy(), None))
         D.close()
     except Exception as exc:  # pragma: no cover - reported to the parent
-        q.put((rank, None, None, repr(exc)))
+        q.put((rank, None, None, repr(exc), None))
     finally:
         dist.destroy_process_group()
 
@@ -63,14 +85,14 @@ def _rank_main(rank, world, port, gdims, grid, kw, parity, napply, nrhs, q):
 def _gather(results, gdims, nrhs):
     lx, ly, lz, lt = gdims
     full = np.zeros((nrhs, 3, lt, lz, ly, lx // 2), np.complex128)
-    for rank, o, e, out in results:
+    for rank, o, e, out, _ in results:
         assert o is not None, out
         v = out.reshape(nrhs, 3, e[3], e[2], e[1], e[0] // 2)
         full[:, :, o[3]:o[3] + e[3], o[2]:o[2] + e[2]] = v
     return full.reshape(nrhs, 3, -1)
 
 
-def _run(world, gdims, grid, kw=None, parity=0, napply=3, nrhs=1):
+def _run(world, gdims, grid, kw=None, parity=0, napply=3, nrhs=1, infos=None):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -79,9 +101,11 @@ def _run(world, gdims, grid, kw=None, parity=0, napply=3, nrhs=1):
              for r in range(world)]
     for p in procs:
         p.start()
-    res = [q.get(timeout=300) for _ in procs]
+    res = [q.get(timeout=600) for _ in procs]
     for p in procs:
         p.join(timeout=120)
+    if infos is not None:
+        infos.extend(r[4] for r in sorted(res, key=lambda r: r[0]))
     return _gather(res, gdims, nrhs)
 
 
@@ -147,3 +171,109 @@ def test_multirank_p2p_overlap_dirs(gdims, grid):
         fat, lng = fieldgen.workload_links(gdims)
         o = oracle.full_to_cb(oracle.dslash(fat, lng, fieldgen.vector(gdims, SEED), 1), 1)
         assert oracle.normwise_error(got[0], o) <= (1e-12 if tol == 1e-14 else 1e-5)
+
+
+
+def _single_cg(gdims, parity, mixed=False, kw=None):
+    import torch
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    fat, lng = fieldgen.workload_links(gdims)
+    with Dslash(gdims, **(kw or {})) as D:
+        D.load_links(fat, lng)
+        b = torch.from_numpy(fieldgen.vector_cb(gdims, SEED, parity)).cuda()
+        x = D.empty_vector()
+        if mixed:
+            info = D.cg_mixed(x, b, parity, CG_MASS, rel_tol=1e-10, inner_tol=1e-3, max_iter=4000)
+        else:
+            info = D.cg(x, b, parity, CG_MASS, rel_tol=1e-10, max_iter=2000)
+        torch.cuda.synchronize()
+        return x.cpu().numpy()[None], info
+
+
+@pytest.mark.parametrize("gdims,grid", [((8, 8, 8, 16), (1, 1, 1, 2)), ((8, 8, 16, 8), (1, 1, 2, 1)),
+                                        ((8, 8, 8, 8), (1, 1, 2, 2)), ((8, 8, 8, 24), (1, 1, 1, 3))])
+@pytest.mark.parametrize("mixed", [False, True])
+def test_multirank_p2p_cg_bitwise(gdims, grid, mixed):
+    """§8(f)-3 across ranks without NCCL (several ranks on one GPU): the dot products' per-rank
+    double-double sums meet through the ranks' IPC-mapped control blocks and every rank adds them
+    in rank order (hisq_p2p_gather).  The solve is decomposition-independent: the gathered x,
+    the iteration count and the true residual equal the 1-rank solve's BITWISE (plain CG and
+    mixed-precision CG), and x solves the system like the oracle CG's."""
+    world = grid[2] * grid[3]
+    parity = 0
+    infos = []
+    got = _run(world, gdims, grid, {"_mode": "cg_mixed" if mixed else "cg"}, parity, infos=infos)
+    ref, ref_info = _single_cg(gdims, parity, mixed)
+    assert all(i[0] for i in infos), infos
+    assert all(i == infos[0] for i in infos), infos                  # every rank: same counts and residual
+    assert tuple(infos[0]) == tuple(ref_info), (infos[0], ref_info)
+    assert np.array_equal(got, ref)
+    from oracle import cg as ocg
+    fat, lng = fieldgen.workload_links(gdims)
+    b_full = oracle.cb_to_full(fieldgen.vector_cb(gdims, SEED, parity), gdims, parity)
+    x_ref, _ = ocg.cg(fat, lng, b_full, parity, CG_MASS, rel_tol=1e-10, max_iter=2000)
+    assert oracle.normwise_error(got[0], oracle.full_to_cb(x_ref, parity)) <= 1e-8
+
+
+def test_multirank_p2p_cg_push():
+    """CG with the producer push across 2 ranks (push in every exchange, P2P reductions)."""
+    gdims, grid = (8, 8, 8, 16), (1, 1, 1, 2)
+    infos = []
+    got = _run(2, gdims, grid, {"_mode": "cg", "push": True}, 1, infos=infos)
+    ref, ref_info = _single_cg(gdims, 1)
+    assert tuple(infos[0]) == tuple(ref_info)
+    assert np.array_equal(got, ref)
+
+
+# ---------------------------------------------------------------------------- distinct GPUs
+# The same data paths across DISTINCT devices (NVLink peers on a B200 node): NCCL send/recv
+# between two GPUs, P2P copy-engine puts into another GPU's IPC-mapped ghosts, and the producer
+# push storing into a peer GPU's memory from the kernel epilogue.  Collected always, run when at
+# least two GPUs are visible (the driver's one-GPU boxes skip them).
+
+def _ngpu():
+    import torch
+    return torch.cuda.device_count()
+
+
+@pytest.mark.parametrize("transport,extra", [("nccl", {}), ("p2p", {}), ("p2p", {"push": True}),
+                                             ("nccl", {"overlap": "dirs"}), ("nccl", {"precision": "mixed"})])
+@pytest.mark.parametrize("gdims,grid", [((8, 8, 8, 16), (1, 1, 1, 2)), ((8, 8, 16, 8), (1, 1, 2, 1)),
+                                        ((16, 16, 16, 16), (1, 1, 2, 2))])
+def test_distinct_gpus_apply(transport, extra, gdims, grid):
+    world = grid[2] * grid[3]
+    if _ngpu() < world:
+        pytest.skip(f"needs {world} GPUs, {_ngpu()} visible")
+    kw = {"_distinct": True, "transport": transport, **extra}
+    parity = 1
+    got = _run(world, gdims, grid, kw, parity)
+    single_kw = {k: v for k, v in extra.items() if k not in ("push", "overlap")}
+    ref = _single(gdims, single_kw, parity)
+    prec = extra.get("precision", "f64")
+    if extra.get("overlap") == "dirs":
+        assert oracle.normwise_error(got[0], ref[0]) <= (1e-14 if prec == "f64" else 1e-6)
+    else:
+        assert np.array_equal(got, ref)
+    fat, lng = fieldgen.workload_links(gdims)
+    o = oracle.full_to_cb(oracle.dslash(fat, lng, fieldgen.vector(gdims, SEED), parity), parity)
+    assert oracle.normwise_error(got[0], o) <= (1e-12 if prec == "f64" else 1e-5)
+
+
+@pytest.mark.parametrize("transport,extra", [("nccl", {}), ("p2p", {}), ("p2p", {"push": True})])
+def test_distinct_gpus_cg(transport, extra):
+    gdims, grid = (8, 8, 8, 16), (1, 1, 1, 2)
+    if _ngpu() < 2:
+        pytest.skip(f"needs 2 GPUs, {_ngpu()} visible")
+    infos = []
+    got = _run(2, gdims, grid, {"_mode": "cg", "_distinct": True, "transport": transport, **extra}, 0, infos=infos)
+    ref, ref_info = _single_cg(gdims, 0)
+    assert tuple(infos[0]) == tuple(ref_info)
+    assert np.array_equal(got, ref)
+
+
+def test_distinct_gpus_multi_rhs_nccl():
+    gdims, grid = (8, 8, 8, 16), (1, 1, 1, 2)
+    if _ngpu() < 2:
+        pytest.skip(f"needs 2 GPUs, {_ngpu()} visible")
+    got = _run(2, gdims, grid, {"_distinct": True, "transport": "nccl"}, 0, napply=2, nrhs=3)
+    assert np.array_equal(got, _single(gdims, {}, 0, nrhs=3))

@@ -596,3 +596,32 @@ def test_nccl_self_option_errors(torch_cuda):
         D.load_links(fat, lng)
         with pytest.raises(DslashError):           # after load_links
             _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_SELF_NCCL, 0)
+
+
+@pytest.mark.parametrize("mask", [0x8, 0x4, 0xC])
+def test_load_links_halo_caller_slabs(torch_cuda, mask):
+    """dslash_load_links_halo: the caller hands over the 3 link slices below the origin (here,
+    with neighbour = self, the lattice's own top slices, host memory); the internal links equal
+    those of the library's own exchange bitwise."""
+    import ctypes
+    from paper_conf_sc_dufekgaad024_b200 import Dslash, _abi
+    dims = (8, 10, 12, 14)
+    fat = fieldgen.links(dims, 91, "gauss")
+    lng = fieldgen.links(dims, 92, "gauss")
+    with Dslash(dims, force_halo=mask) as D:
+        D.load_links(fat, lng)
+        want = [D.get_links(q) for q in (0, 1)]
+    keep = []
+    sf, sl = [0] * 4, [0] * 4
+    for d, axis in ((3, 0), (2, 1)):
+        if not (mask >> d) & 1:
+            continue
+        for k, arr in enumerate((fat, lng)):
+            top = np.ascontiguousarray(np.take(arr, range(arr.shape[axis] - 3, arr.shape[axis]), axis=axis))
+            keep.append(top)
+            (sf if k == 0 else sl)[d] = top.ctypes.data
+    with Dslash(dims, force_halo=mask) as D:
+        _abi.dslash_load_links_halo(D.h, fat.ctypes.data, lng.ctypes.data, sf, sl, 0, 0)
+        got = [D.get_links(q) for q in (0, 1)]
+    for q in (0, 1):
+        assert np.array_equal(got[q], want[q])
