@@ -237,6 +237,15 @@ DSLASH_API int64_t dslash_ipc_blob_size(void);
 DSLASH_API dslash_status dslash_get_ipc_blob(dslash_t h, void* blob);
 DSLASH_API dslash_status dslash_open_ipc_blobs(dslash_t h, const void* blobs);
 
+/* Device selection for callers without their own CUDA runtime (e.g. plain C): the library
+ * links its own copy of the CUDA runtime, so these act on the library's current device of the
+ * calling thread, the device dslash_create binds a handle to.  dslash_set_device wraps
+ * cudaSetDevice (DSLASH_ERR_ARG for an index out of range, DSLASH_ERR_CUDA otherwise);
+ * dslash_device_count returns the number of visible devices (0 when none or on error).  Call
+ * them before any other CUDA use in a forked child process. */
+DSLASH_API dslash_status dslash_set_device(int32_t device);
+DSLASH_API int32_t dslash_device_count(void);
+
 /* Write a fresh ncclUniqueId (128 bytes) to id_out.  Call on rank 0 only. */
 DSLASH_API dslash_status dslash_get_unique_id(void* id_out);
 

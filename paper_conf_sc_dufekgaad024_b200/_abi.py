@@ -84,6 +84,8 @@ _SIGS = {
     "dslash_create": ([_i4, _i4, ctypes.c_int32, ctypes.c_int32, _vp, ctypes.c_int32, ctypes.c_int32,
                        ctypes.POINTER(_h)], ctypes.c_int),
     "dslash_get_unique_id": ([_vp], ctypes.c_int),
+    "dslash_set_device": ([ctypes.c_int32], ctypes.c_int),
+    "dslash_device_count": ([], ctypes.c_int32),
     "dslash_ipc_blob_size": ([], ctypes.c_int64),
     "dslash_get_ipc_blob": ([_h, _vp], ctypes.c_int),
     "dslash_open_ipc_blobs": ([_h, _vp], ctypes.c_int),
@@ -146,6 +148,14 @@ def dslash_plan(global_dims, proc_grid=(1, 1, 1, 1), rank=0, nranks=1, force_hal
     p = dslash_plan_t()
     check(lib.dslash_plan(i4(global_dims), i4(proc_grid), rank, nranks, force_halo_mask, ctypes.byref(p)))
     return p
+
+
+def dslash_set_device(device: int) -> None:
+    check(lib.dslash_set_device(int(device)))
+
+
+def dslash_device_count() -> int:
+    return int(lib.dslash_device_count())
 
 
 def dslash_get_unique_id() -> bytes:

@@ -56,17 +56,19 @@ def build(force: bool = False, verbose: bool = False) -> str:
     link = ["nvcc", *ARCH, "-shared", "-o", LIB, *objs, "-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
             "-Xlinker", "-rpath=" + os.path.join(nccl, "lib")]
     subprocess.check_call(link)
-    build_c_demo()
+    build_c_demo("c_api_demo")
+    build_c_demo("c_p2p_demo")
     return LIB
 
 
-def build_c_demo() -> str:
-    """examples/c_api_demo: the library used from plain C (the boundary is a C ABI)."""
-    src = os.path.join(ROOT, "examples", "c_api_demo.c")
-    exe = os.path.join(ROOT, "examples", "c_api_demo")
+def build_c_demo(name: str = "c_api_demo") -> str:
+    """examples/<name>: the library used from plain C (the boundary is a C ABI).  c_api_demo: one
+    rank; c_p2p_demo: a forked multi-rank P2P partition (no Python, no MPI)."""
+    src = os.path.join(ROOT, "examples", name + ".c")
+    exe = os.path.join(ROOT, "examples", name)
     if os.path.exists(src):
-        subprocess.check_call(["gcc", "-std=c99", "-O2", src, "-I", os.path.join(ROOT, "include"), "-L", HERE,
-                               "-lhisq_dslash", "-Wl,-rpath," + HERE, "-lm", "-o", exe])
+        subprocess.check_call(["gcc", "-std=gnu99", "-O2", src, "-I", os.path.join(ROOT, "include"), "-L", HERE,
+                               "-lhisq_dslash", "-Wl,-rpath," + HERE, "-lpthread", "-lm", "-o", exe])
     return exe
 
 

@@ -139,6 +139,23 @@ extern "C" dslash_status dslash_plan(const int32_t G[4], const int32_t P[4], int
 }
 
 // ============================================================================ handle
+extern "C" int32_t dslash_device_count(void) {
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    return n;
+}
+
+extern "C" dslash_status dslash_set_device(int32_t device) {
+    const int n = dslash_device_count();
+    if (device < 0 || device >= n) return fail(nullptr, DSLASH_ERR_ARG, "device %d not in [0, %d)", device, n);
+    cudaError_t e = cudaSetDevice(device);
+    if (e != cudaSuccess) return fail(nullptr, DSLASH_ERR_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(e));
+    return DSLASH_OK;
+}
+
 extern "C" dslash_status dslash_get_unique_id(void* id_out) {
     if (!id_out) return fail(nullptr, DSLASH_ERR_ARG, "NULL id_out");
     ncclUniqueId id;
