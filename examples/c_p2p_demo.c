@@ -176,6 +176,7 @@ static int check_single(shared_hdr* hdr, const double complex* out_e, const doub
     printf("c_p2p_demo: %d ranks, global %dx%dx%dx%d t-partitioned over P2P, link halo in load_links: "
            "gathered chi %s the 1-rank chi bitwise; anti-Hermiticity rel.diff=%.2e\n",
            nranks, G[0], G[1], G[2], G[3], equal ? "EQUALS" : "DIFFERS FROM", rel);
+    fflush(stdout);  /* the child leaves with _exit, which does not flush stdio */
     CHECK(dslash_destroy(h));
     free(fat);
     free(lng);
