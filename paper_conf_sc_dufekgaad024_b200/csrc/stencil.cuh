@@ -364,11 +364,12 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
     // whole warps (not the staged kernel): each quarter-warp (8 lanes) takes 8 consecutive sites of
     // ONE group, so a 16-byte load of a quarter-warp touches one 128-byte line (one L1 wavefront)
     // instead of two; the warp still covers the same 16 sites
-    constexpr bool kQuarterRuns = LANES == 1 && RHSL == 2 && !STAGED;
+    constexpr bool kQuarterRuns = LANES == 1 && (RHSL == 2 || RHSL == 4) && !STAGED;
     const int rl = (RHSL == 1)    ? 0
-                   : kQuarterRuns ? (int)((gid >> 3) & 1)
+                   : kQuarterRuns ? (int)((gid >> 3) % RHSL)
                                   : (int)((gid / LANES) % RHSL);
-    const int64_t site = kQuarterRuns ? ((gid >> 5) << 4) + (((gid >> 4) & 1) << 3) + (gid & 7) : gid / (LANES * RHSL);
+    const int64_t site = kQuarterRuns ? (gid >> 5) * (32 / RHSL) + ((gid >> 3) / RHSL) % (4 / RHSL) * 8 + (gid & 7)
+                                      : gid / (LANES * RHSL);
     const bool valid = site < site_end;
     if (LANES == 1 && !valid) return;
     V2 acc[NRHS][3];
