@@ -1428,9 +1428,7 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
     const int bs = h->block ? h->block : kDefaultBlock;
     const int minb = h->min_blocks ? h->min_blocks : kDefaultMinBlocks;
     // right-hand sides are register-blocked per thread; 8 of them use 2 thread groups of 4
-    static const int n8v = getenv("HISQ_N8_VARIANT") ? atoi(getenv("HISQ_N8_VARIANT")) : 0;
-    const int rhsl8 = lanes != 1 ? 2 : (n8v == 2 || n8v == 3) ? 4 : n8v == 4 ? 1 : 2;
-    const int64_t threads = sites * lanes * (nrhs == 8 ? rhsl8 : 1);
+    const int64_t threads = sites * lanes * (nrhs == 8 ? 2 : 1);
     const unsigned grid = (unsigned)((threads + bs - 1) / bs);
     dslash_s::TimedLaunch* tl = nullptr;
     dslash_status st = timing_begin(h, kind, s, &tl);

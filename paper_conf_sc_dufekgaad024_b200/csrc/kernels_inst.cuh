@@ -6,8 +6,6 @@
 // 12% occupancy).
 #pragma once
 
-#include <cstdlib>
-
 #include "dispatch.h"
 #include "stencil.cuh"
 
@@ -18,19 +16,7 @@ StencilFn pick_minb(int minb, int nrhs) {
     switch (nrhs) {
         case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 2>;
         case 4: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4>;
-        case 8: {
-            // HISQ_N8_VARIANT (measurement aid): 0 = 2 groups x 4 (MINB 2), 1 = 2 x 4 (MINB 1),
-            // 2 = 4 x 2 (MINB 2), 3 = 4 x 2 (MINB 1), 4 = 1 x 8 (MINB 1)
-            static const int v = getenv("HISQ_N8_VARIANT") ? atoi(getenv("HISQ_N8_VARIANT")) : 0;
-            if (LANES == 1) switch (v) {
-                case 1: return dslash_kernel<LR, VR, LANES, GHOST, 1, RECON, 4, 2>;
-                case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 2, 4>;
-                case 3: return dslash_kernel<LR, VR, LANES, GHOST, 1, RECON, 2, 4>;
-                case 4: return dslash_kernel<LR, VR, LANES, GHOST, 1, RECON, 8, 1>;
-                default: break;
-            }
-            return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2>;  // 2 thread groups x 4 RHS each
-        }
+        case 8: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2>;  // 2 thread groups x 4 RHS each
         default: break;
     }
     switch (minb) {
