@@ -96,6 +96,8 @@ def parse(argv=None):
                     help="halo transport for N > 1: NCCL send/recv, or copy-engine puts into IPC-mapped ghosts")
     ap.add_argument("--no-pdl", action="store_true",
                     help="ordinary launches instead of programmatic dependent launch (DSLASH_OPT_PDL)")
+    ap.add_argument("--halo-dryrun", action="store_true",
+                    help="timing aid: the exchange keeps its stream structure but moves no bytes (results WRONG)")
     ap.add_argument("--breakdown-steps", type=int, default=200,
                     help="steps of the separate per-kernel-event pass after the timed region (0: none)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -466,6 +468,8 @@ def main():
                transport=args.transport if world > 1 or args.force_halo else "nccl",
                self_nccl=bool(args.self_nccl and world == 1 and args.force_halo and args.transport == "nccl"),
                stage=args.stage)
+    if args.halo_dryrun:
+        _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_HALO_DRYRUN, 1)
     origin, extent = D.origin, D.local_dims
     fat, lng = fieldgen.workload_links(gdims, origin=origin, extent=extent)
     D.load_links(fat, lng)
@@ -661,6 +665,7 @@ def main():
                            "kernel": args.kernel, "stage": bool(args.stage), "block": args.block or None,
                            "precision": args.precision, "long_link_recon": args.recon, "nrhs": nrhs,
                            "overlap": "none" if args.no_overlap else args.overlap, "pdl": not args.no_pdl,
+                           "halo_dryrun_results_invalid": True if args.halo_dryrun else None,
                            "per_kernel_events_in_timed_region": bool(args.flush_l2),
                            "transport": args.transport if world > 1 else None,
                            "colocated_ranks_on_one_gpu": bool(args.colocate) or None,
