@@ -6,6 +6,7 @@
 // itself runs in the kernels of stencil.cuh / links.cuh.
 #include <nccl.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -988,6 +989,44 @@ dslash_status hisq_p2p_gather(dslash_t h, cudaStream_t s, const double2* mine, c
 // ============================================================================ halo exchange
 static bool any_halo(const dslash_plan_t& p) { return p.halo[2] || p.halo[3]; }
 
+// Face copy within this GPU (self-neighbour ghosts, the z-face pack for NCCL): `height` rows of
+// `width` bytes, 16-byte words when every pitch and pointer allows, else 8-byte words.  An SM
+// kernel on the (high-priority) communication stream instead of cudaMemcpy2DAsync: measured on
+// B200 the 2-D device-to-device copy of 2 x 2.36 MB took ~37 us beside a bandwidth-bound
+// stencil kernel and cost it ~6.7 us; the kernel moves the same bytes at HBM speed.
+template <typename W>
+__global__ void __launch_bounds__(256) face_copy_kernel(char* __restrict__ dst, size_t dpitch,
+                                                        const char* __restrict__ src, size_t spitch,
+                                                        int64_t words_per_row, int64_t rows) {
+    const int64_t n = words_per_row * rows;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = i / words_per_row, w = i - r * words_per_row;
+        reinterpret_cast<W*>(dst + r * dpitch)[w] = __ldcs(reinterpret_cast<const W*>(src + r * spitch) + w);
+    }
+}
+
+static int num_sms(dslash_t h);
+
+static dslash_status copy_faces(dslash_t h, void* dst, size_t dpitch, const void* src, size_t spitch, size_t width,
+                                size_t height, cudaStream_t st, bool local) {
+    if (!width || !height) return DSLASH_OK;
+    if (!local) {
+        CU(h, cudaMemcpy2DAsync(dst, dpitch, src, spitch, width, height, cudaMemcpyDeviceToDevice, st));
+        return DSLASH_OK;
+    }
+    const bool w16 = ((dpitch | spitch | width | (uintptr_t)dst | (uintptr_t)src) & 15) == 0;
+    const size_t ws = w16 ? 16 : 8;
+    const int64_t words = (int64_t)(width / ws), total = words * (int64_t)height;
+    const int64_t cap = (int64_t)num_sms(h) * 2;
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((total + 255) / 256, cap));
+    if (w16)
+        face_copy_kernel<int4><<<grid, 256, 0, st>>>((char*)dst, dpitch, (const char*)src, spitch, words, (int64_t)height);
+    else
+        face_copy_kernel<int2><<<grid, 256, 0, st>>>((char*)dst, dpitch, (const char*)src, spitch, words, (int64_t)height);
+    CU(h, cudaGetLastError());
+    return DSLASH_OK;
+}
+
 // an interval of class `kind` whose start is recorded on stream s now (DSLASH_OPT_TIMING; *out =
 // nullptr when timing is off); the caller records (*out)->b at its end
 static dslash_status timing_begin(dslash_t h, int kind, cudaStream_t s, dslash_s::TimedLaunch** out);
@@ -1084,21 +1123,26 @@ static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaSt
             for (int side = 0; side < 2; ++side)
                 if (wt(h->comm, (unsigned long long)(uintptr_t)(h->flags + 8 + 2 * d + side), e - 1, 0) != 0)
                     return fail(h, DSLASH_ERR_CUDA, "cuStreamWaitValue32 (free) failed");
+    // faces to another rank: copy engines (no SM; NVLink between devices); to myself: a copy kernel
     if (p.halo[3]) {
         const size_t tslab = 3 * lxh * L1 * L2;
         const size_t b = bank_off(h, 3, e);
-        CU(h, cudaMemcpy2DAsync(h->peer_ghost[3][0] + b, tslab * es, src, vh * es, tslab * es, rows,
-                                cudaMemcpyDeviceToDevice, h->comm));
-        CU(h, cudaMemcpy2DAsync(h->peer_ghost[3][1] + b, tslab * es, src + (vh - tslab) * es, vh * es, tslab * es, rows,
-                                cudaMemcpyDeviceToDevice, h->comm));
+        st = copy_faces(h, h->peer_ghost[3][0] + b, tslab * es, src, vh * es, tslab * es, rows, h->comm,
+                        p.nbr_rank[3][0] == p.rank);
+        if (st == DSLASH_OK)
+            st = copy_faces(h, h->peer_ghost[3][1] + b, tslab * es, src + (vh - tslab) * es, vh * es, tslab * es, rows,
+                            h->comm, p.nbr_rank[3][1] == p.rank);
+        if (st != DSLASH_OK) return st;
     }
     if (p.halo[2]) {
         const size_t zrow = lxh * L1;
         const size_t b = bank_off(h, 2, e);
-        CU(h, cudaMemcpy2DAsync(h->peer_ghost[2][0] + b, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
-                                cudaMemcpyDeviceToDevice, h->comm));
-        CU(h, cudaMemcpy2DAsync(h->peer_ghost[2][1] + b, 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es,
-                                3 * zrow * es, rows * L3, cudaMemcpyDeviceToDevice, h->comm));
+        st = copy_faces(h, h->peer_ghost[2][0] + b, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
+                        h->comm, p.nbr_rank[2][0] == p.rank);
+        if (st == DSLASH_OK)
+            st = copy_faces(h, h->peer_ghost[2][1] + b, 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es,
+                            3 * zrow * es, rows * L3, h->comm, p.nbr_rank[2][1] == p.rank);
+        if (st != DSLASH_OK) return st;
     }
     for (int d = 3; d >= 2; --d)
         if (p.halo[d])
@@ -1186,10 +1230,10 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
     if (p.halo[3]) {
         if (!exch_remote(h, 3)) {
             // minus ghost <- my top slices, plus ghost <- my bottom slices (periodic self-halo)
-            CU(h, cudaMemcpy2DAsync(h->ghost[3][0], tslab * es, src + (vh - tslab) * es, vh * es, tslab * es, rows,
-                                    cudaMemcpyDeviceToDevice, h->comm));
-            CU(h, cudaMemcpy2DAsync(h->ghost[3][1], tslab * es, src, vh * es, tslab * es, rows,
-                                    cudaMemcpyDeviceToDevice, h->comm));
+            dslash_status st = copy_faces(h, h->ghost[3][0], tslab * es, src + (vh - tslab) * es, vh * es, tslab * es,
+                                          rows, h->comm, true);
+            if (st == DSLASH_OK) st = copy_faces(h, h->ghost[3][1], tslab * es, src, vh * es, tslab * es, rows, h->comm, true);
+            if (st != DSLASH_OK) return st;
         } else {
             nccl_work = true;
         }
@@ -1200,10 +1244,12 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
         const bool self = !exch_remote(h, 2);
         char* to_minus = self ? h->ghost[2][1] : h->zsend[0];  // my bottom slices
         char* to_plus = self ? h->ghost[2][0] : h->zsend[1];   // my top slices
-        CU(h, cudaMemcpy2DAsync(to_minus, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
-                                cudaMemcpyDeviceToDevice, h->comm));
-        CU(h, cudaMemcpy2DAsync(to_plus, 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es, 3 * zrow * es,
-                                rows * L3, cudaMemcpyDeviceToDevice, h->comm));
+        dslash_status st = copy_faces(h, to_minus, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
+                                      h->comm, true);
+        if (st == DSLASH_OK)
+            st = copy_faces(h, to_plus, 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es, 3 * zrow * es,
+                            rows * L3, h->comm, true);
+        if (st != DSLASH_OK) return st;
         if (!self) nccl_work = true;
     }
     if (nccl_work) {
@@ -1582,13 +1628,18 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         }
         st = launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
         if (st != DSLASH_OK) return st;
-        if ((st = dslash_halo_wait(h, (dslash_stream_t)h->bstream)) != DSLASH_OK) return st;
-        if (push_out && (st = push_wait_free(h, h->bstream)) != DSLASH_OK) return st;
-        st = launch_rhs(h, Kp, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, h->bstream, nrhs);
+        // HISQ_BND_SAME_STREAM=1 (measurement aid): the boundary kernel on the caller's stream
+        static const bool same = getenv("HISQ_BND_SAME_STREAM") != nullptr;
+        cudaStream_t bs = same ? s : h->bstream;
+        if ((st = dslash_halo_wait(h, (dslash_stream_t)bs)) != DSLASH_OK) return st;
+        if (push_out && (st = push_wait_free(h, bs)) != DSLASH_OK) return st;
+        st = launch_rhs(h, Kp, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, bs, nrhs);
         if (st != DSLASH_OK) return st;
-        if (push_out && (st = push_signal(h, h->bstream, out, nrhs)) != DSLASH_OK) return st;
-        CU(h, cudaEventRecord(h->ev_bdone, h->bstream));
-        CU(h, cudaStreamWaitEvent(s, h->ev_bdone, 0));
+        if (push_out && (st = push_signal(h, bs, out, nrhs)) != DSLASH_OK) return st;
+        if (!same) {
+            CU(h, cudaEventRecord(h->ev_bdone, h->bstream));
+            CU(h, cudaStreamWaitEvent(s, h->ev_bdone, 0));
+        }
         if (span != (size_t)-1) CU(h, cudaEventRecord(h->tpool[span].b, s));
         return DSLASH_OK;
     }
