@@ -1628,18 +1628,13 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
         }
         st = launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
         if (st != DSLASH_OK) return st;
-        // HISQ_BND_SAME_STREAM=1 (measurement aid): the boundary kernel on the caller's stream
-        static const bool same = getenv("HISQ_BND_SAME_STREAM") != nullptr;
-        cudaStream_t bs = same ? s : h->bstream;
-        if ((st = dslash_halo_wait(h, (dslash_stream_t)bs)) != DSLASH_OK) return st;
-        if (push_out && (st = push_wait_free(h, bs)) != DSLASH_OK) return st;
-        st = launch_rhs(h, Kp, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, bs, nrhs);
+        if ((st = dslash_halo_wait(h, (dslash_stream_t)h->bstream)) != DSLASH_OK) return st;
+        if (push_out && (st = push_wait_free(h, h->bstream)) != DSLASH_OK) return st;
+        st = launch_rhs(h, Kp, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, h->bstream, nrhs);
         if (st != DSLASH_OK) return st;
-        if (push_out && (st = push_signal(h, bs, out, nrhs)) != DSLASH_OK) return st;
-        if (!same) {
-            CU(h, cudaEventRecord(h->ev_bdone, h->bstream));
-            CU(h, cudaStreamWaitEvent(s, h->ev_bdone, 0));
-        }
+        if (push_out && (st = push_signal(h, h->bstream, out, nrhs)) != DSLASH_OK) return st;
+        CU(h, cudaEventRecord(h->ev_bdone, h->bstream));
+        CU(h, cudaStreamWaitEvent(s, h->ev_bdone, 0));
         if (span != (size_t)-1) CU(h, cudaEventRecord(h->tpool[span].b, s));
         return DSLASH_OK;
     }

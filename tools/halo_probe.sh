@@ -5,8 +5,6 @@ run() { timeout 300 $B "$@" 2>/dev/null | python -c "
 import json,sys; d=json.loads(sys.stdin.readline()); b=(d['roofline'].get('breakdown') or {})
 print('%-45s %8.2f us/step  span %s  int %s  bnd %s  exch %s' % (' '.join(sys.argv[1:]), d['ms_per_step']*1e3, b.get('span_us'), b.get('interior_us'), b.get('boundary_us'), b.get('exchange_us')))" "$@"; }
 for i in 1 2; do
-HISQ_BND_SAME_STREAM=1 run --force-halo 8
-HISQ_BND_SAME_STREAM=1 run --force-halo 12
 run
 run --no-pdl
 run --force-halo 8
