@@ -6,8 +6,6 @@
 // 12% occupancy).
 #pragma once
 
-#include <cstdlib>
-
 #include "dispatch.h"
 #include "stencil.cuh"
 
@@ -18,15 +16,7 @@ StencilFn pick_minb(int minb, int nrhs) {
     switch (nrhs) {
         case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 2>;
         case 4: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4>;
-        case 8: {
-            // HISQ_N8_LB (measurement aid): register budget of the 8-RHS kernel via launch bounds
-            // 1 = (128 threads, 3 blocks): <= 168 regs; 2 = (64, 5): <= 200; 3 = (96, 4): <= 168
-            static const int v = getenv("HISQ_N8_LB") ? atoi(getenv("HISQ_N8_LB")) : 0;
-            if (v == 1) return dslash_kernel<LR, VR, LANES, GHOST, 3, RECON, 4, 2, 128>;
-            if (v == 2) return dslash_kernel<LR, VR, LANES, GHOST, 5, RECON, 4, 2, 64>;
-            if (v == 3) return dslash_kernel<LR, VR, LANES, GHOST, 4, RECON, 4, 2, 96>;
-            return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2>;  // 2 thread groups x 4 RHS each
-        }
+        case 8: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2>;  // 2 thread groups x 4 RHS each
         default: break;
     }
     switch (minb) {

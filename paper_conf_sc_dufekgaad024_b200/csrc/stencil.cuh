@@ -668,9 +668,8 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
     }
 }
 
-template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1, int RHSL = 1,
-          int MAXT = 256>
-__global__ void __launch_bounds__(MAXT, MINB) dslash_kernel(const StencilParams P) {
+template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1, int RHSL = 1>
+__global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P) {
     // every block has started: the next PDL-launched apply may begin filling freed SMs
     asm volatile("griddepcontrol.launch_dependents;");
     dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
