@@ -370,14 +370,6 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                                   : (int)((gid / LANES) % RHSL);
     const int64_t site = kQuarterRuns ? (gid >> 5) * (32 / RHSL) + ((gid >> 3) / RHSL) % (4 / RHSL) * 8 + (gid & 7)
                                       : gid / (LANES * RHSL);
-    // Split links (fp64 full matrices, 2 thread groups of a site in quarter-warp runs: lanes l and
-    // l ^ 8 hold the same site): each of the two threads loads alternate entries of every matrix
-    // (e = 2k + rl) and they swap them with a pair shuffle, so a thread keeps half a matrix in
-    // registers and a hop's 5 + 3 NRHS loads fit in flight under the 128-register budget
-    // (profiles/r02/mrhs/).  Entries are applied in row-major order e = 3i + j, each to every
-    // right-hand side, so each accumulator acc[r][i] still receives j = 0, 1, 2 in order, hop after
-    // hop: the bits equal those of the single-RHS apply.
-    constexpr bool kSplitLinks = kQuarterRuns && RHSL == 2 && RECON == 18 && sizeof(LR) == 8;
     const bool valid = site < site_end;
     if (LANES == 1 && !valid) return;
     V2 acc[NRHS][3];
@@ -407,11 +399,8 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
         // (not in the ghost pass, whose first hop is never a ghost hop for LANES 1 / 2)
         if (sizeof(LR) != 4 && !(GHOST && P.halo_pass == kPassGhost)) {
             const L2* lp0 = links + link_index<LANES, RECON>((STAGED ? K - 1 : 0) * LANES + lane, 0, 0, P.vh, s.cb);
-            // (split links: no prefetch; 20 more live registers across the first direction spill)
-            if constexpr (!kSplitLinks) {
 #pragma unroll
-                for (int e = 0; e < 9; ++e) U0[e] = to_cplx<V2>(widen(ld_stream(lp0 + (int64_t)e * 4 * P.vh, pol_stream)));
-            }
+            for (int e = 0; e < 9; ++e) U0[e] = to_cplx<V2>(widen(ld_stream(lp0 + (int64_t)e * 4 * P.vh, pol_stream)));
         }
         if constexpr (!STAGED) asm volatile("griddepcontrol.wait;\n\tmov.b64 %0, %1;" : "=l"(in) : "l"(P.in) : "memory");
         const uint32_t plane_b = STAGED ? (uint32_t)(T.rows * P.lxh * sizeof(V2)) : 0u;  // bytes per staged plane
@@ -512,51 +501,6 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                                 matvec_acc<true>(acc[r], Ub, v);
                             } else {
                                 matvec_acc<false>(acc[r], Ua, v);
-                            }
-                        }
-                    }
-                }
-            } else if constexpr (kSplitLinks) {
-                const unsigned pair = (1u << (threadIdx.x & 31)) | (1u << ((threadIdx.x & 31) ^ 8));
-                // not unrolled: one hop's loads at a time (unrolled, the compiler hoists later hops'
-                // loads and spills ~2 KB per thread)
-#pragma unroll 1
-                for (int l = 0; l < 4; ++l) {
-                    const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
-                    const SrcRef<V2> src = source<V2, GHOST>(P, in, mu, h, s, rl * NRHS);
-                    if (GHOST && P.halo_pass == kPassGhost && !src.ghost) continue;  // both lanes of the pair alike
-                    const bool zap = GHOST && P.halo_pass == kPassLocal && src.ghost;
-                    const L2* lp = links + link_index<LANES, RECON>(mu, l, 0, P.vh, s.cb);
-                    V2 own[5];  // entries 2k + rl of the matrix
-#pragma unroll
-                    for (int k = 0; k < 4; ++k)
-                        own[k] = to_cplx<V2>(widen(ld_stream(lp + (int64_t)(2 * k + rl) * 4 * P.vh, pol_stream)));
-                    own[4].x = own[4].y = VR(0);   // entry 8 (rl = 0); entry 9 does not exist (rl = 1)
-                    if (rl == 0) own[4] = to_cplx<V2>(widen(ld_stream(lp + (int64_t)8 * 4 * P.vh, pol_stream)));
-                    V2 v[NRHS][3];
-#pragma unroll
-                    for (int r = 0; r < NRHS; ++r)
-#pragma unroll
-                        for (int c = 0; c < 3; ++c) {
-                            v[r][c] = ld_reuse(src.p + (int64_t)r * 3 * src.stride + c * src.stride, pol_keep);
-                            if (GHOST) zero_if(v[r][c], zap);
-                        }
-#pragma unroll
-                    for (int k = 0; k < 5; ++k) {
-                        V2 other;
-                        other.x = __shfl_xor_sync(pair, own[k].x, 8);
-                        other.y = __shfl_xor_sync(pair, own[k].y, 8);
-#pragma unroll
-                        for (int q = 0; q < 2; ++q) {
-                            const int e = 2 * k + q;
-                            if (e >= 9) continue;
-                            const V2 u = (q == rl) ? own[k] : other;
-#pragma unroll
-                            for (int r = 0; r < NRHS; ++r) {
-                                if (l & 1)
-                                    cmsub(acc[r][e / 3], u, v[r][e % 3]);
-                                else
-                                    cmadd(acc[r][e / 3], u, v[r][e % 3]);
                             }
                         }
                     }
@@ -727,14 +671,6 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1, int RHSL = 1>
 __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P) {
     // every block has started: the next PDL-launched apply may begin filling freed SMs
-    asm volatile("griddepcontrol.launch_dependents;");
-    dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
-                                                         P.box_start[P.nbox]);
-}
-
-// the same kernel under an exact register cap (__maxnreg__; measurement aid for the 8-RHS kernel)
-template <typename LR, typename VR, int LANES, bool GHOST, int MAXREG, int RECON, int NRHS = 1, int RHSL = 1>
-__global__ void __maxnreg__(MAXREG) dslash_kernel_r(const StencilParams P) {
     asm volatile("griddepcontrol.launch_dependents;");
     dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
                                                          P.box_start[P.nbox]);
