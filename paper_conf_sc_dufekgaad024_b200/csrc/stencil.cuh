@@ -91,28 +91,46 @@ template <typename V2>
 __device__ __forceinline__ V2 cconj(V2 a) {
     return V2{a.x, -a.y};
 }
-// fp32 reconstruction (recon-9 is rebuilt in the precision its parameters are stored in) takes the
-// hardware approximations: MUFU sin/cos of pi*a for |a| <= 1 (abs. error ~4e-7) and rsqrt; fp64
-// keeps the libdevice routines
+// fp32 reconstruction (recon-9 is rebuilt in the precision its parameters are stored in).  FAST:
+// the hardware approximations, MUFU sin/cos of pi*a for |a| <= 1 (abs. error ~4e-7) and rsqrt;
+// otherwise the accurate fp32 routines (sincospif, sqrtf).  The rebuild divides by
+// n = |a2|^2 + |a3|^2, so its absolute error is amplified by 1/n on links near the
+// parameterisation's singular set: at 32^4 the MUFU rebuild made mixed recon-9 71x (f32 7x) less
+// accurate than recon-18, the accurate one ~1x (profiles/r02/recon9_accuracy/).  fp64 keeps the
+// libdevice routines.
+template <bool FAST>
 __device__ __forceinline__ void sincospi_r(double a, double* s, double* c) { sincospi(a, s, c); }
-__device__ __forceinline__ void sincospi_r(float a, float* s, float* c) { __sincosf(a * 3.14159265358979f, s, c); }
+template <bool FAST>
+__device__ __forceinline__ void sincospi_r(float a, float* s, float* c) {
+    if (FAST)
+        __sincosf(a * 3.14159265358979f, s, c);
+    else
+        sincospif(a, s, c);
+}
+template <bool FAST>
 __device__ __forceinline__ double sqrt0_r(double x) { return sqrt(fmax(x, 0.0)); }
-__device__ __forceinline__ float sqrt0_r(float x) { return x > 0.f ? x * rsqrtf(x) : 0.f; }
+template <bool FAST>
+__device__ __forceinline__ float sqrt0_r(float x) { return FAST ? (x > 0.f ? x * rsqrtf(x) : 0.f) : sqrtf(fmaxf(x, 0.f)); }
 __device__ __forceinline__ double rcp_r(double x) { return 1.0 / x; }
 __device__ __forceinline__ float rcp_r(float x) { return __frcp_rn(x); }
 
+// HISQ_RECON9_FAST (compile-time, default 0): the hardware approximations in the fp32 rebuild
+#ifndef HISQ_RECON9_FAST
+#define HISQ_RECON9_FAST 0
+#endif
+
 // SCALE = false leaves U = W and only returns z = s e^{i pi psi} (the stencil multiplies the
 // 3-vector W v by z instead of the 9 entries of W)
-template <bool SCALE = true, typename V2, typename R>
+template <bool SCALE = true, bool FAST = false, typename V2, typename R>
 __device__ __forceinline__ V2 reconstruct_9(V2 U[9], R s, R psi) {
     const V2 a2 = U[1], a3 = U[2], b1 = U[3];
     const R n = a2.x * a2.x + a2.y * a2.y + a3.x * a3.x + a3.y * a3.y;
-    const R a1m = sqrt0_r(R(1) - n);
-    const R c1m = sqrt0_r(n - (b1.x * b1.x + b1.y * b1.y));
+    const R a1m = sqrt0_r<FAST>(R(1) - n);
+    const R c1m = sqrt0_r<FAST>(n - (b1.x * b1.x + b1.y * b1.y));
     R sa, ca, sc, cc, sp, cp;
-    sincospi_r(U[0].x, &sa, &ca);  // angles are stored in units of pi: no large-argument reduction
-    sincospi_r(U[0].y, &sc, &cc);
-    sincospi_r(psi, &sp, &cp);
+    sincospi_r<FAST>(U[0].x, &sa, &ca);  // angles are stored in units of pi: no large-argument reduction
+    sincospi_r<FAST>(U[0].y, &sc, &cc);
+    sincospi_r<FAST>(psi, &sp, &cp);
     const V2 a1{a1m * ca, a1m * sa}, c1{c1m * cc, c1m * sc};
     const R inv = rcp_r(n);
     const V2 a1b1 = cmul(cconj(a1), b1), a1c1 = cmul(cconj(a1), c1);
@@ -449,16 +467,16 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     V2 za, zb;  // recon-9: Nf = za Wa, Nb = zb Wb (the psi pair is entry 4: (psi_f, 0, psi_b, 0))
                     if constexpr (RECON == 9) {
                         if (j == 1) {
-                            // rebuilt in fp32, the precision the parameters are stored in (mixed
-                            // widens the result: an fp64 rebuild of fp32 data adds no accuracy)
+                            // rebuilt in fp32, the precision the parameters are stored in, with
+                            // the accurate fp32 routines (mixed widens the result)
                             float2 fa[9], fb[9];
 #pragma unroll
                             for (int e = 0; e < 4; ++e) {
                                 fa[e] = make_float2(L9w[e].x, L9w[e].y);
                                 fb[e] = make_float2(L9w[e].z, L9w[e].w);
                             }
-                            const float2 zfa = reconstruct_9<false>(fa, (float)P.long_scale, L9w[4].x);
-                            const float2 zfb = reconstruct_9<false>(fb, (float)P.long_scale, L9w[4].z);
+                            const float2 zfa = reconstruct_9<false, HISQ_RECON9_FAST>(fa, (float)P.long_scale, L9w[4].x);
+                            const float2 zfb = reconstruct_9<false, HISQ_RECON9_FAST>(fb, (float)P.long_scale, L9w[4].z);
 #pragma unroll
                             for (int e = 0; e < 9; ++e) {
                                 Ua[e] = to_cplx<V2>(widen(fa[e]));
