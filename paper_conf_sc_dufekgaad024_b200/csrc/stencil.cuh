@@ -91,13 +91,14 @@ template <typename V2>
 __device__ __forceinline__ V2 cconj(V2 a) {
     return V2{a.x, -a.y};
 }
-// fp32 reconstruction (recon-9 is rebuilt in the precision its parameters are stored in).  FAST:
-// the hardware approximations, MUFU sin/cos of pi*a for |a| <= 1 (abs. error ~4e-7) and rsqrt;
-// otherwise the accurate fp32 routines (sincospif, sqrtf).  The rebuild divides by
-// n = |a2|^2 + |a3|^2, so its absolute error is amplified by 1/n on links near the
-// parameterisation's singular set: at 32^4 the MUFU rebuild made mixed recon-9 71x (f32 7x) less
-// accurate than recon-18, the accurate one ~1x (profiles/r02/recon9_accuracy/).  fp64 keeps the
-// libdevice routines.
+// fp32 reconstruction (recon-9 is rebuilt in the precision its parameters are stored in).  FAST
+// (the default): the hardware approximations, MUFU sin/cos of pi*a for |a| <= 1 (abs. error ~4e-7)
+// and rsqrt; otherwise the accurate fp32 routines (sincospif, sqrtf).  Measured at 32^4
+// (profiles/r02/recon9_accuracy/): both give the same normwise error, 2.0e-6 for f32 and mixed
+// recon-9 (recon-18: 2.9e-7 / 2.8e-8), because the error comes from rounding the STORED parameters
+// to fp32 and the parameterisation's conditioning (|c1| = sqrt(n - |b1|^2) cancels, and b2..c3
+// divide by n = |a2|^2 + |a3|^2), not from the rebuild arithmetic; the accurate routines only cost
+// time (mixed 83.0 -> 91.9 us).  fp64 keeps the libdevice routines.
 template <bool FAST>
 __device__ __forceinline__ void sincospi_r(double a, double* s, double* c) { sincospi(a, s, c); }
 template <bool FAST>
@@ -114,9 +115,9 @@ __device__ __forceinline__ float sqrt0_r(float x) { return FAST ? (x > 0.f ? x *
 __device__ __forceinline__ double rcp_r(double x) { return 1.0 / x; }
 __device__ __forceinline__ float rcp_r(float x) { return __frcp_rn(x); }
 
-// HISQ_RECON9_FAST (compile-time, default 0): the hardware approximations in the fp32 rebuild
+// HISQ_RECON9_FAST (compile-time, default 1): the hardware approximations in the fp32 rebuild
 #ifndef HISQ_RECON9_FAST
-#define HISQ_RECON9_FAST 0
+#define HISQ_RECON9_FAST 1
 #endif
 
 // SCALE = false leaves U = W and only returns z = s e^{i pi psi} (the stencil multiplies the
@@ -467,8 +468,9 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     V2 za, zb;  // recon-9: Nf = za Wa, Nb = zb Wb (the psi pair is entry 4: (psi_f, 0, psi_b, 0))
                     if constexpr (RECON == 9) {
                         if (j == 1) {
-                            // rebuilt in fp32, the precision the parameters are stored in, with
-                            // the accurate fp32 routines (mixed widens the result)
+                            // rebuilt in fp32, the precision the parameters are stored in (mixed
+                            // widens the result; its accuracy is set by the fp32 parameters, see
+                            // sincospi_r)
                             float2 fa[9], fb[9];
 #pragma unroll
                             for (int e = 0; e < 4; ++e) {
