@@ -580,7 +580,7 @@ def main():
                      "launches_per_step": launches_per_step}
     achieved = algo_bytes_site * dom_sites / (kern_ms * 1e-3) / 1e9
     variant = (args.kernel + ("-stage" if args.stage else "") + ("" if args.precision == "f64" else f"-{args.precision}")
-               + ("" if args.recon == 18 else f"-r{args.recon}"))
+               + ("" if args.recon == 18 else f"-r{args.recon}") + (f"-n{nrhs}" if nrhs > 1 else ""))
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4), "traffic": ncu_traffic(variant, extent), "kernel": kname,
             "bytes_per_launch": algo_bytes_site * dom_sites, "bytes_per_site": algo_bytes_site,

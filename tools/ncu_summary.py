@@ -49,6 +49,7 @@ def main():
     ap.add_argument("--out", default=os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
                                                   "profiles", "ncu_summary.json"))
     ap.add_argument("--note", default="")
+    ap.add_argument("--bytes-per-site", type=int, default=2400, help="algorithmic bytes per target site")
     a = ap.parse_args()
     rs = rows(a.report)
     launches = [r for r in rs if "dslash" in r["kernel"]]
@@ -58,7 +59,7 @@ def main():
     entry = {"variant": a.variant, "local_dims": local, "report": os.path.basename(a.report),
              "kernel": launches[0]["kernel"], "launches": len(launches),
              "dram_bytes_per_launch": int(sum(dram) / len(dram)),
-             "algorithmic_bytes_per_launch": 2400 * vh,
+             "algorithmic_bytes_per_launch": a.bytes_per_site * vh,
              "duration_us": [round(r["gpu__time_duration.sum"] * 1e6, 2) for r in launches],
              "metrics": launches[-1], "note": a.note}
     try:
