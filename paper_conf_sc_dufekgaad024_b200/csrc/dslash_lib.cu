@@ -994,14 +994,33 @@ static bool any_halo(const dslash_plan_t& p) { return p.halo[2] || p.halo[3]; }
 // kernel on the (high-priority) communication stream instead of cudaMemcpy2DAsync: measured on
 // B200 the 2-D device-to-device copy of 2 x 2.36 MB took ~37 us beside a bandwidth-bound
 // stencil kernel and cost it ~6.7 us; the kernel moves the same bytes at HBM speed.
+// (4 words per thread per pass, loads first: enough bytes in flight to run at HBM speed when the
+// exchange is exposed, e.g. a partition with no interior site)
 template <typename W>
 __global__ void __launch_bounds__(256) face_copy_kernel(char* __restrict__ dst, size_t dpitch,
                                                         const char* __restrict__ src, size_t spitch,
                                                         int64_t words_per_row, int64_t rows) {
+    constexpr int U = 4;
     const int64_t n = words_per_row * rows;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t r = i / words_per_row, w = i - r * words_per_row;
-        reinterpret_cast<W*>(dst + r * dpitch)[w] = __ldcs(reinterpret_cast<const W*>(src + r * spitch) + w);
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i0 < n; i0 += U * stride) {
+        W v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t i = i0 + u * stride;
+            if (i < n) {
+                const int64_t r = i / words_per_row, w = i - r * words_per_row;
+                v[u] = __ldcs(reinterpret_cast<const W*>(src + r * spitch) + w);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t i = i0 + u * stride;
+            if (i < n) {
+                const int64_t r = i / words_per_row, w = i - r * words_per_row;
+                reinterpret_cast<W*>(dst + r * dpitch)[w] = v[u];
+            }
+        }
     }
 }
 
@@ -1017,8 +1036,8 @@ static dslash_status copy_faces(dslash_t h, void* dst, size_t dpitch, const void
     const bool w16 = ((dpitch | spitch | width | (uintptr_t)dst | (uintptr_t)src) & 15) == 0;
     const size_t ws = w16 ? 16 : 8;
     const int64_t words = (int64_t)(width / ws), total = words * (int64_t)height;
-    const int64_t cap = (int64_t)num_sms(h) * 2;
-    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((total + 255) / 256, cap));
+    const int64_t cap = (int64_t)num_sms(h) * 8;
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((total + 4 * 256 - 1) / (4 * 256), cap));
     if (w16)
         face_copy_kernel<int4><<<grid, 256, 0, st>>>((char*)dst, dpitch, (const char*)src, spitch, words, (int64_t)height);
     else
