@@ -989,19 +989,28 @@ dslash_status hisq_p2p_gather(dslash_t h, cudaStream_t s, const double2* mine, c
 // ============================================================================ halo exchange
 static bool any_halo(const dslash_plan_t& p) { return p.halo[2] || p.halo[3]; }
 
-// Face copy within this GPU (self-neighbour ghosts, the z-face pack for NCCL): `height` rows of
-// `width` bytes, 16-byte words when every pitch and pointer allows, else 8-byte words.  An SM
-// kernel on the (high-priority) communication stream instead of cudaMemcpy2DAsync: measured on
-// B200 the 2-D device-to-device copy of 2 x 2.36 MB took ~37 us beside a bandwidth-bound
-// stencil kernel and cost it ~6.7 us; the kernel moves the same bytes at HBM speed.
-// (4 words per thread per pass, loads first: enough bytes in flight to run at HBM speed when the
-// exchange is exposed, e.g. a partition with no interior site)
+// Face copies within this GPU (self-neighbour ghosts, the z-face pack for NCCL): up to 4 segments
+// of `height` rows of `width` bytes, all in ONE kernel on the (high-priority) communication stream
+// instead of cudaMemcpy2DAsync: measured on B200 the 2-D device-to-device copies of 2 x 2.36 MB
+// took ~37 us beside a bandwidth-bound stencil kernel and cost it ~6.7 us per apply.  16-byte
+// words when every pitch and pointer allows, else 8-byte words; 4 words per thread in flight.
+// Copies to another rank's memory stay on the copy engines (cudaMemcpy2DAsync, NVLink).
+struct CopySeg {
+    char* dst;
+    const char* src;
+    size_t dpitch, spitch;
+    int64_t words, rows;  // words per row, rows
+};
+struct CopySet {
+    CopySeg seg[4];
+    int n;
+};
+
 template <typename W>
-__global__ void __launch_bounds__(256) face_copy_kernel(char* __restrict__ dst, size_t dpitch,
-                                                        const char* __restrict__ src, size_t spitch,
-                                                        int64_t words_per_row, int64_t rows) {
+__global__ void __launch_bounds__(256) face_copy_kernel(const CopySet C) {
     constexpr int U = 4;
-    const int64_t n = words_per_row * rows;
+    const CopySeg& S = C.seg[blockIdx.y];
+    const int64_t n = S.words * S.rows;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t i0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i0 < n; i0 += U * stride) {
         W v[U];
@@ -1009,16 +1018,16 @@ __global__ void __launch_bounds__(256) face_copy_kernel(char* __restrict__ dst, 
         for (int u = 0; u < U; ++u) {
             const int64_t i = i0 + u * stride;
             if (i < n) {
-                const int64_t r = i / words_per_row, w = i - r * words_per_row;
-                v[u] = __ldcs(reinterpret_cast<const W*>(src + r * spitch) + w);
+                const int64_t r = i / S.words, w = i - r * S.words;
+                v[u] = __ldcs(reinterpret_cast<const W*>(S.src + r * S.spitch) + w);
             }
         }
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             const int64_t i = i0 + u * stride;
             if (i < n) {
-                const int64_t r = i / words_per_row, w = i - r * words_per_row;
-                reinterpret_cast<W*>(dst + r * dpitch)[w] = v[u];
+                const int64_t r = i / S.words, w = i - r * S.words;
+                reinterpret_cast<W*>(S.dst + r * S.dpitch)[w] = v[u];
             }
         }
     }
@@ -1026,25 +1035,50 @@ __global__ void __launch_bounds__(256) face_copy_kernel(char* __restrict__ dst, 
 
 static int num_sms(dslash_t h);
 
-static dslash_status copy_faces(dslash_t h, void* dst, size_t dpitch, const void* src, size_t spitch, size_t width,
-                                size_t height, cudaStream_t st, bool local) {
-    if (!width || !height) return DSLASH_OK;
-    if (!local) {
-        CU(h, cudaMemcpy2DAsync(dst, dpitch, src, spitch, width, height, cudaMemcpyDeviceToDevice, st));
+struct FaceCopies {
+    struct Raw {
+        void* dst;
+        const void* src;
+        size_t dpitch, spitch, width, height;
+    } raw[4];
+    int n = 0;
+    // a local segment is batched; a copy into another rank's memory goes to the copy engines now
+    dslash_status add(dslash_t h, void* dst, size_t dpitch, const void* src, size_t spitch, size_t width,
+                      size_t height, cudaStream_t st, bool local) {
+        if (!width || !height) return DSLASH_OK;
+        if (!local) {
+            CU(h, cudaMemcpy2DAsync(dst, dpitch, src, spitch, width, height, cudaMemcpyDeviceToDevice, st));
+            return DSLASH_OK;
+        }
+        raw[n++] = {dst, src, dpitch, spitch, width, height};
         return DSLASH_OK;
     }
-    const bool w16 = ((dpitch | spitch | width | (uintptr_t)dst | (uintptr_t)src) & 15) == 0;
-    const size_t ws = w16 ? 16 : 8;
-    const int64_t words = (int64_t)(width / ws), total = words * (int64_t)height;
-    const int64_t cap = (int64_t)num_sms(h) * 8;
-    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((total + 4 * 256 - 1) / (4 * 256), cap));
-    if (w16)
-        face_copy_kernel<int4><<<grid, 256, 0, st>>>((char*)dst, dpitch, (const char*)src, spitch, words, (int64_t)height);
-    else
-        face_copy_kernel<int2><<<grid, 256, 0, st>>>((char*)dst, dpitch, (const char*)src, spitch, words, (int64_t)height);
-    CU(h, cudaGetLastError());
-    return DSLASH_OK;
-}
+    dslash_status flush(dslash_t h, cudaStream_t st) {
+        if (!n) return DSLASH_OK;
+        uintptr_t bits = 0;
+        for (int k = 0; k < n; ++k)
+            bits |= raw[k].dpitch | raw[k].spitch | raw[k].width | (uintptr_t)raw[k].dst | (uintptr_t)raw[k].src;
+        const bool w16 = (bits & 15) == 0;
+        const size_t ws = w16 ? 16 : 8;
+        CopySet C{};
+        C.n = n;
+        int64_t most = 0;
+        for (int k = 0; k < n; ++k) {
+            C.seg[k] = {(char*)raw[k].dst, (const char*)raw[k].src, raw[k].dpitch, raw[k].spitch,
+                        (int64_t)(raw[k].width / ws), (int64_t)raw[k].height};
+            most = std::max<int64_t>(most, C.seg[k].words * C.seg[k].rows);
+        }
+        const int64_t cap = (int64_t)num_sms(h) * 8 / n;
+        const dim3 grid((unsigned)std::max<int64_t>(1, std::min<int64_t>((most + 4 * 256 - 1) / (4 * 256), cap)), n);
+        if (w16)
+            face_copy_kernel<int4><<<grid, 256, 0, st>>>(C);
+        else
+            face_copy_kernel<int2><<<grid, 256, 0, st>>>(C);
+        CU(h, cudaGetLastError());
+        n = 0;
+        return DSLASH_OK;
+    }
+};
 
 // an interval of class `kind` whose start is recorded on stream s now (DSLASH_OPT_TIMING; *out =
 // nullptr when timing is off); the caller records (*out)->b at its end
@@ -1142,27 +1176,29 @@ static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaSt
             for (int side = 0; side < 2; ++side)
                 if (wt(h->comm, (unsigned long long)(uintptr_t)(h->flags + 8 + 2 * d + side), e - 1, 0) != 0)
                     return fail(h, DSLASH_ERR_CUDA, "cuStreamWaitValue32 (free) failed");
-    // faces to another rank: copy engines (no SM; NVLink between devices); to myself: a copy kernel
+    // faces to another rank: copy engines (no SM; NVLink between devices); to myself: one copy kernel
+    FaceCopies fc;
     if (p.halo[3]) {
         const size_t tslab = 3 * lxh * L1 * L2;
         const size_t b = bank_off(h, 3, e);
-        st = copy_faces(h, h->peer_ghost[3][0] + b, tslab * es, src, vh * es, tslab * es, rows, h->comm,
-                        p.nbr_rank[3][0] == p.rank);
+        st = fc.add(h, h->peer_ghost[3][0] + b, tslab * es, src, vh * es, tslab * es, rows, h->comm,
+                    p.nbr_rank[3][0] == p.rank);
         if (st == DSLASH_OK)
-            st = copy_faces(h, h->peer_ghost[3][1] + b, tslab * es, src + (vh - tslab) * es, vh * es, tslab * es, rows,
-                            h->comm, p.nbr_rank[3][1] == p.rank);
+            st = fc.add(h, h->peer_ghost[3][1] + b, tslab * es, src + (vh - tslab) * es, vh * es, tslab * es, rows,
+                        h->comm, p.nbr_rank[3][1] == p.rank);
         if (st != DSLASH_OK) return st;
     }
     if (p.halo[2]) {
         const size_t zrow = lxh * L1;
         const size_t b = bank_off(h, 2, e);
-        st = copy_faces(h, h->peer_ghost[2][0] + b, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
-                        h->comm, p.nbr_rank[2][0] == p.rank);
+        st = fc.add(h, h->peer_ghost[2][0] + b, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
+                    h->comm, p.nbr_rank[2][0] == p.rank);
         if (st == DSLASH_OK)
-            st = copy_faces(h, h->peer_ghost[2][1] + b, 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es,
-                            3 * zrow * es, rows * L3, h->comm, p.nbr_rank[2][1] == p.rank);
+            st = fc.add(h, h->peer_ghost[2][1] + b, 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es,
+                        3 * zrow * es, rows * L3, h->comm, p.nbr_rank[2][1] == p.rank);
         if (st != DSLASH_OK) return st;
     }
+    if ((st = fc.flush(h, h->comm)) != DSLASH_OK) return st;
     for (int d = 3; d >= 2; --d)
         if (p.halo[d])
             for (int side = 0; side < 2; ++side)
@@ -1246,12 +1282,13 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
     }
     bool nccl_work = false;
     const size_t tslab = 3 * lxh * L1 * L2;  // sites in 3 t-slices of one parity
+    FaceCopies fc;                           // copies within this GPU: one kernel (flushed below)
     if (p.halo[3]) {
         if (!exch_remote(h, 3)) {
             // minus ghost <- my top slices, plus ghost <- my bottom slices (periodic self-halo)
-            dslash_status st = copy_faces(h, h->ghost[3][0], tslab * es, src + (vh - tslab) * es, vh * es, tslab * es,
-                                          rows, h->comm, true);
-            if (st == DSLASH_OK) st = copy_faces(h, h->ghost[3][1], tslab * es, src, vh * es, tslab * es, rows, h->comm, true);
+            dslash_status st = fc.add(h, h->ghost[3][0], tslab * es, src + (vh - tslab) * es, vh * es, tslab * es,
+                                      rows, h->comm, true);
+            if (st == DSLASH_OK) st = fc.add(h, h->ghost[3][1], tslab * es, src, vh * es, tslab * es, rows, h->comm, true);
             if (st != DSLASH_OK) return st;
         } else {
             nccl_work = true;
@@ -1263,13 +1300,17 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
         const bool self = !exch_remote(h, 2);
         char* to_minus = self ? h->ghost[2][1] : h->zsend[0];  // my bottom slices
         char* to_plus = self ? h->ghost[2][0] : h->zsend[1];   // my top slices
-        dslash_status st = copy_faces(h, to_minus, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
-                                      h->comm, true);
+        dslash_status st = fc.add(h, to_minus, 3 * zrow * es, src, L2 * zrow * es, 3 * zrow * es, rows * L3,
+                                  h->comm, true);
         if (st == DSLASH_OK)
-            st = copy_faces(h, to_plus, 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es, 3 * zrow * es,
-                            rows * L3, h->comm, true);
+            st = fc.add(h, to_plus, 3 * zrow * es, src + (L2 - 3) * zrow * es, L2 * zrow * es, 3 * zrow * es,
+                        rows * L3, h->comm, true);
         if (st != DSLASH_OK) return st;
         if (!self) nccl_work = true;
+    }
+    {
+        dslash_status st = fc.flush(h, h->comm);  // the z pack precedes the sends on the comm stream
+        if (st != DSLASH_OK) return st;
     }
     if (nccl_work) {
         if (!h->nccl) return fail(h, DSLASH_ERR_STATE, "halo to another rank without an NCCL communicator");
