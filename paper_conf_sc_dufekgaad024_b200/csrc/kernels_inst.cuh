@@ -6,8 +6,6 @@
 // 12% occupancy).
 #pragma once
 
-#include <cstdlib>
-
 #include "dispatch.h"
 #include "stencil.cuh"
 
@@ -18,15 +16,7 @@ StencilFn pick_minb(int minb, int nrhs) {
     switch (nrhs) {
         case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 2>;
         case 4: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4>;
-        case 8: {
-            // HISQ_N8_MAXREG (measurement aid): register cap of the 8-RHS kernel
-            static const int v = getenv("HISQ_N8_MAXREG") ? atoi(getenv("HISQ_N8_MAXREG")) : 0;
-            if (LANES == 1 && v == 120) return dslash_kernel_r<LR, VR, LANES, GHOST, 120, RECON, 4, 2>;
-            if (LANES == 1 && v == 112) return dslash_kernel_r<LR, VR, LANES, GHOST, 112, RECON, 4, 2>;
-            if (LANES == 1 && v == 104) return dslash_kernel_r<LR, VR, LANES, GHOST, 104, RECON, 4, 2>;
-            if (LANES == 1 && v == 96) return dslash_kernel_r<LR, VR, LANES, GHOST, 96, RECON, 4, 2>;
-            return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2>;  // 2 thread groups x 4 RHS each
-        }
+        case 8: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2>;  // 2 thread groups x 4 RHS each
         default: break;
     }
     switch (minb) {

@@ -696,14 +696,6 @@ __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P
                                                          P.box_start[P.nbox]);
 }
 
-// the same kernel under an exact register cap (__maxnreg__; measurement aid for the 8-RHS kernel)
-template <typename LR, typename VR, int LANES, bool GHOST, int MAXREG, int RECON, int NRHS = 1, int RHSL = 1>
-__global__ void __maxnreg__(MAXREG) dslash_kernel_r(const StencilParams P) {
-    asm volatile("griddepcontrol.launch_dependents;");
-    dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
-                                                         P.box_start[P.nbox]);
-}
-
 // The neighbour-staged variant (DSLASH_OPT_STAGE): one tile of P.stage_ty full x-rows per block
 // (blockDim = lxh * stage_ty * LANES * RHSL threads), the tile's source rows y0-3 .. y0+TY+2 in
 // dynamic shared memory (NRHS * RHSL * 3 * (TY + 6) * lxh complex).  Boxes span full x and y, so
