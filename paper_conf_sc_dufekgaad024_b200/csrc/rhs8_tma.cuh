@@ -37,6 +37,13 @@ __host__ __device__ constexpr size_t rhs8_smem_bytes() {
     return (size_t)kRhs8Warps * kRhs8Stages * kRhs8StageBytes + (size_t)kRhs8Warps * kRhs8Stages * 8;
 }
 
+// ld_reuse that keeps its place among the other volatile asm of the kernel
+__device__ __forceinline__ double2 ld_reuse_ordered(const double2* p, uint64_t pol) {
+    double2 r;
+    asm volatile("ld.global.nc.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(r.x), "=d"(r.y) : "l"(p), "l"(pol));
+    return r;
+}
+
 __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, int c0, int c1, int c2, uint64_t* bar,
                                             uint64_t pol) {
     asm volatile(
@@ -48,6 +55,7 @@ __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, i
 
 // P: the full-lattice box (enumeration order = cb order), vh a multiple of kRhs8Sites; in/out hold
 // 8 vectors [8][3][vh].
+template <int UNROLL>
 __global__ void __launch_bounds__(32 * kRhs8Warps, 2)
     dslash_rhs8_tma_kernel(const __grid_constant__ CUtensorMap tmap, const StencilParams P) {
     using V2 = double2;
@@ -89,8 +97,11 @@ __global__ void __launch_bounds__(32 * kRhs8Warps, 2)
         for (int r = 0; r < NRHS; ++r)
 #pragma unroll
             for (int c = 0; c < 3; ++c) acc[r][c].x = acc[r][c].y = 0.0;
-        // hops not unrolled: unrolled, the compiler hoists every hop's 12 neighbour loads and spills
-#pragma unroll 1
+        // unrolled by direction (the 4 hops of a direction: l known at compile time, mu at run
+        // time); the neighbour loads are volatile asm (ld_reuse_ordered), so the compiler cannot
+        // hoist later hops' loads above this hop's shared-memory reads (fully unrolled and hoisted,
+        // the kernel spilled 3.5 KB)
+#pragma unroll UNROLL
         for (int j = 0; j < 16; ++j) {
             const int mu = j >> 2, l = j & 3;
             const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
@@ -99,7 +110,8 @@ __global__ void __launch_bounds__(32 * kRhs8Warps, 2)
 #pragma unroll
             for (int r = 0; r < NRHS; ++r)
 #pragma unroll
-                for (int c = 0; c < 3; ++c) v[r][c] = ld_reuse(src.p + (int64_t)r * 3 * src.stride + c * src.stride, pol_keep);
+                for (int c = 0; c < 3; ++c)
+                    v[r][c] = ld_reuse_ordered(src.p + (int64_t)r * 3 * src.stride + c * src.stride, pol_keep);
             mbar_wait(&full[j & 3], (j >> 2) & 1);
             const V2* st = reinterpret_cast<const V2*>(ring + (j & 3) * kRhs8StageBytes);
             // entry by entry from shared memory (4 registers, not a 36-register matrix), each applied
