@@ -33,7 +33,8 @@ StencilFn pick_f64_r9_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_f32_r9_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_mixed_r9_stage(bool ghost, int lanes, int nrhs);
 
-constexpr int kRhs8Sites = 16;  // sites per warp tile of the TMA-fed 8-RHS kernel
+// sites per warp tile of the TMA-fed 8-RHS kernel (the tensor map's box width)
+int rhs8_tile_sites();
 
 // the TMA-fed 8-RHS kernel (rhs8_tma.cuh; fp64, recon 18, SITE layout, full-lattice box): a
 // persistent grid of up to 2 CTAs per SM, programmatic dependent launch when pdl

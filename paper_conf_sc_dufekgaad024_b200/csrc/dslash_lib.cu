@@ -1557,7 +1557,7 @@ static EncodeTiledFn encode_tiled_fn() {
 static bool rhs8_tma_serves(dslash_t h, const StencilParams& K, bool ghost, int nrhs) {
     const dslash_plan_t& p = h->plan;
     if (!h->rhs8_tma || nrhs != 8 || ghost || h->kernel != DSLASH_KERNEL_SITE || h->precision != DSLASH_F64 ||
-        h->recon != 18 || h->stage || K.nbox != 1 || K.vh % kRhs8Sites || !encode_tiled_fn())
+        h->recon != 18 || h->stage || K.nbox != 1 || K.vh % rhs8_tile_sites() || !encode_tiled_fn())
         return false;
     for (int d = 0; d < 4; ++d)
         if (K.box[0].lo[d] != 0 || K.box[0].n[d] != p.local_dims[d]) return false;
@@ -1570,7 +1570,7 @@ static dslash_status rhs8_tma_launch(dslash_t h, const StencilParams& K, cudaStr
     if (h->rhs8_map_links[parity] != K.links) {
         const cuuint64_t dims[3] = {(cuuint64_t)(2 * K.vh), 4, 36};
         const cuuint64_t strides[2] = {(cuuint64_t)(K.vh * 16), (cuuint64_t)(4 * K.vh * 16)};
-        const cuuint32_t box[3] = {2 * kRhs8Sites, 1, 9};
+        const cuuint32_t box[3] = {(cuuint32_t)(2 * rhs8_tile_sites()), 1, 9};
         const cuuint32_t estr[3] = {1, 1, 1};
         if (enc(&h->rhs8_map[parity], CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<void*>(K.links), dims, strides,
                 box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,

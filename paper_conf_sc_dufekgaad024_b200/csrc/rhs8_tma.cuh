@@ -29,13 +29,19 @@
 
 namespace hisq {
 
-constexpr int kRhs8Stages = 4;                      // ring depth per warp (a hop every 4 ahead)
-constexpr uint32_t kRhs8StageBytes = 9 * kRhs8Sites * 16;  // one matrix of the tile
-constexpr int kRhs8Warps = 8;                       // warps per CTA (256 threads, 2 CTAs per SM)
+constexpr int kRhs8Stages = 4;  // ring depth per warp (a hop every 4 ahead)
 
-__host__ __device__ constexpr size_t rhs8_smem_bytes() {
-    return (size_t)kRhs8Warps * kRhs8Stages * kRhs8StageBytes + (size_t)kRhs8Warps * kRhs8Stages * 8;
-}
+// NRHS right-hand sides per thread, RHSL = 8 / NRHS thread groups per site (quarter-warp runs of
+// 8 sites), TS = 32 / RHSL sites per warp tile; WARPS per CTA, MINB CTAs per SM
+template <int NRHS>
+struct Rhs8Cfg {
+    static constexpr int RHSL = 8 / NRHS;
+    static constexpr int TS = 32 / RHSL;
+    static constexpr uint32_t kStage = 9 * TS * 16;  // one matrix of the tile
+    static constexpr int WARPS = NRHS == 4 ? 8 : 8;
+    static constexpr int MINB = NRHS == 4 ? 2 : 3;
+    static constexpr size_t smem() { return (size_t)WARPS * kRhs8Stages * (kStage + 8); }
+};
 
 // ld_reuse that keeps its place among the other volatile asm of the kernel
 __device__ __forceinline__ double2 ld_reuse_ordered(const double2* p, uint64_t pol) {
@@ -53,22 +59,23 @@ __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, i
         : "memory");
 }
 
-// P: the full-lattice box (enumeration order = cb order), vh a multiple of kRhs8Sites; in/out hold
+// P: the full-lattice box (enumeration order = cb order), vh a multiple of the tile; in/out hold
 // 8 vectors [8][3][vh].
-template <int UNROLL>
-__global__ void __launch_bounds__(32 * kRhs8Warps, 2)
+template <int UNROLL, int NRHS>
+__global__ void __launch_bounds__(32 * Rhs8Cfg<NRHS>::WARPS, Rhs8Cfg<NRHS>::MINB)
     dslash_rhs8_tma_kernel(const __grid_constant__ CUtensorMap tmap, const StencilParams P) {
     using V2 = double2;
-    constexpr int NRHS = 4;
+    using C = Rhs8Cfg<NRHS>;
+    constexpr int TS = C::TS;
+    constexpr uint32_t kStageB = C::kStage;
     asm volatile("griddepcontrol.launch_dependents;");
     extern __shared__ __align__(128) unsigned char smem[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    unsigned char* ring = smem + (size_t)warp * kRhs8Stages * kRhs8StageBytes;
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + (size_t)kRhs8Warps * kRhs8Stages * kRhs8StageBytes) +
-                     warp * kRhs8Stages;
-    const int64_t ntiles = P.vh / kRhs8Sites;
-    const int64_t nw = (int64_t)gridDim.x * kRhs8Warps;
-    int64_t tile = (int64_t)blockIdx.x * kRhs8Warps + warp;
+    unsigned char* ring = smem + (size_t)warp * kRhs8Stages * kStageB;
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + (size_t)C::WARPS * kRhs8Stages * kStageB) + warp * kRhs8Stages;
+    const int64_t ntiles = P.vh / TS;
+    const int64_t nw = (int64_t)gridDim.x * C::WARPS;
+    int64_t tile = (int64_t)blockIdx.x * C::WARPS + warp;
     const uint64_t pol_first = policy_evict_first();
     const uint64_t pol_keep = policy_evict_last();
     if (lane == 0) {
@@ -79,19 +86,18 @@ __global__ void __launch_bounds__(32 * kRhs8Warps, 2)
     // hop j = 4 mu + l of a tile lives in stage j & 3 with phase (j >> 2) & 1 (4 uses per tile)
     auto issue = [&](int64_t t, int j) {  // lane 0
         uint64_t* bar = &full[j & 3];
-        mbar_arrive_expect_tx(bar, kRhs8StageBytes);
-        tma_load_3d(ring + (j & 3) * kRhs8StageBytes, &tmap, (int)(2 * t * kRhs8Sites), j >> 2, 9 * (j & 3), bar,
-                    pol_first);
+        mbar_arrive_expect_tx(bar, kStageB);
+        tma_load_3d(ring + (j & 3) * kStageB, &tmap, (int)(2 * t * TS), j >> 2, 9 * (j & 3), bar, pol_first);
     };
     // links are read-only: the first tile's first 4 matrices are requested before the PDL wait
     if (lane == 0 && tile < ntiles)
         for (int j = 0; j < kRhs8Stages; ++j) issue(tile, j);
     const void* in;
     asm volatile("griddepcontrol.wait;\n\tmov.b64 %0, %1;" : "=l"(in) : "l"(P.in) : "memory");
-    const int rl = (lane >> 3) & 1;
-    const int sl = ((lane >> 4) << 3) + (lane & 7);
+    const int rl = (lane >> 3) % C::RHSL;                       // right-hand-side group
+    const int sl = ((lane >> 3) / C::RHSL) * 8 + (lane & 7);    // site in the tile
     for (; tile < ntiles; tile += nw) {
-        const Site s = decode_site(P, tile * kRhs8Sites + sl);
+        const Site s = decode_site(P, tile * TS + sl);
         V2 acc[NRHS][3];
 #pragma unroll
         for (int r = 0; r < NRHS; ++r)
@@ -113,13 +119,13 @@ __global__ void __launch_bounds__(32 * kRhs8Warps, 2)
                 for (int c = 0; c < 3; ++c)
                     v[r][c] = ld_reuse_ordered(src.p + (int64_t)r * 3 * src.stride + c * src.stride, pol_keep);
             mbar_wait(&full[j & 3], (j >> 2) & 1);
-            const V2* st = reinterpret_cast<const V2*>(ring + (j & 3) * kRhs8StageBytes);
+            const V2* st = reinterpret_cast<const V2*>(ring + (j & 3) * kStageB);
             // entry by entry from shared memory (4 registers, not a 36-register matrix), each applied
             // to the 4 right-hand sides; acc[r][i] receives columns j = 0, 1, 2 in order, as in
             // matvec_acc
 #pragma unroll
             for (int e = 0; e < 9; ++e) {
-                const V2 u = lds(st + e * kRhs8Sites + sl);
+                const V2 u = lds(st + e * TS + sl);
 #pragma unroll
                 for (int r = 0; r < NRHS; ++r) {
                     if (l & 1)
