@@ -96,8 +96,6 @@ def parse(argv=None):
                     help="halo transport for N > 1: NCCL send/recv, or copy-engine puts into IPC-mapped ghosts")
     ap.add_argument("--no-pdl", action="store_true",
                     help="ordinary launches instead of programmatic dependent launch (DSLASH_OPT_PDL)")
-    ap.add_argument("--no-rhs8-tma", action="store_true",
-                    help="8 RHS: the register-blocked kernel instead of the TMA-fed one (DSLASH_OPT_RHS8_TMA 0)")
     ap.add_argument("--halo-dryrun", action="store_true",
                     help="timing aid: the exchange keeps its stream structure but moves no bytes (results WRONG)")
     ap.add_argument("--breakdown-steps", type=int, default=200,
@@ -472,8 +470,6 @@ def main():
                stage=args.stage)
     if args.halo_dryrun:
         _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_HALO_DRYRUN, 1)
-    if args.no_rhs8_tma:
-        _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_RHS8_TMA, 0)
     origin, extent = D.origin, D.local_dims
     fat, lng = fieldgen.workload_links(gdims, origin=origin, extent=extent)
     D.load_links(fat, lng)

@@ -133,12 +133,6 @@ enum {
                                    from the stencil kernel's epilogue (peer memory over NVLink), so
                                    the next apply, whose source that output is, moves no bytes.
                                    0 (default): off                                                 */
-    DSLASH_OPT_RHS8_TMA = 15,   /* 1 (default): 8-right-hand-side applies of an fp64 SITE-kernel handle
-                                   with full long links and no halo run the TMA-fed kernel: each warp
-                                   streams its 16-site tile's link matrices into a 4-deep ring of
-                                   shared-memory stages with cp.async.bulk.tensor (mbarrier
-                                   completion) and gathers only the neighbours itself; bitwise the
-                                   register kernel's results.  0: the register kernel; any time   */
     DSLASH_OPT_MIN_BLOCKS = 5   /* register budget of the stencil kernel, as the minimum number of
                                    resident 256-thread blocks per SM: 2 (<= 128 registers), 3 (<= 80),
                                    4 (<= 64); 0 = default; any time                                    */

@@ -26,7 +26,7 @@ DSLASH_KERNEL_SITE, DSLASH_KERNEL_DIR4, DSLASH_KERNEL_DIR2 = 0, 1, 2
 DSLASH_OPT_KERNEL, DSLASH_OPT_BLOCK, DSLASH_OPT_FORCE_HALO, DSLASH_OPT_OVERLAP, DSLASH_OPT_TIMING, \
     DSLASH_OPT_MIN_BLOCKS, DSLASH_OPT_LONG_RECON = range(7)
 DSLASH_OPT_TRANSPORT, DSLASH_OPT_PDL, DSLASH_OPT_SELF_NCCL, DSLASH_OPT_STAGE = range(8, 12)
-DSLASH_OPT_HALO_DRYRUN, DSLASH_OPT_PUSH, DSLASH_OPT_RHS8_TMA = 13, 14, 15
+DSLASH_OPT_HALO_DRYRUN, DSLASH_OPT_PUSH = 13, 14
 DSLASH_TRANSPORT_NCCL, DSLASH_TRANSPORT_P2P = 0, 1
 DSLASH_OVERLAP_NONE, DSLASH_OVERLAP_SITES, DSLASH_OVERLAP_DIRS = 0, 1, 2
 OVERLAPS = {"none": DSLASH_OVERLAP_NONE, "sites": DSLASH_OVERLAP_SITES, "dirs": DSLASH_OVERLAP_DIRS}

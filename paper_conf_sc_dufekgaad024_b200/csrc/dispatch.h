@@ -1,8 +1,6 @@
 // dispatch.h -- kernel selection across the per-precision translation units (kernels_*.cu).
 #pragma once
 
-#include <cuda.h>
-
 #include "common.cuh"
 #include "stencil.cuh"
 
@@ -32,12 +30,5 @@ StencilFn pick_mixed_r12_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_f64_r9_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_f32_r9_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_mixed_r9_stage(bool ghost, int lanes, int nrhs);
-
-// sites per warp tile of the TMA-fed 8-RHS kernel (the tensor map's box width)
-int rhs8_tile_sites();
-
-// the TMA-fed 8-RHS kernel (rhs8_tma.cuh; fp64, recon 18, SITE layout, full-lattice box): a
-// persistent grid of up to 2 CTAs per SM, programmatic dependent launch when pdl
-cudaError_t launch_rhs8_tma(const CUtensorMap& map, const StencilParams& P, int nsm, bool pdl, cudaStream_t s);
 
 }  // namespace hisq

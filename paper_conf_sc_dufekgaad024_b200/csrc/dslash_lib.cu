@@ -393,9 +393,6 @@ extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t valu
             h->pushed_src = nullptr;
             return alloc_halo(h, kP2PMaxRhs);
         }
-        case DSLASH_OPT_RHS8_TMA:
-            h->rhs8_tma = value != 0;
-            return DSLASH_OK;
         case DSLASH_OPT_MIN_BLOCKS:
             if (value != 0 && (value < 2 || value > 4))
                 return fail(h, DSLASH_ERR_ARG, "min_blocks %lld must be 0, 2, 3 or 4", (long long)value);
@@ -1530,68 +1527,9 @@ static int num_sms(dslash_t h) {
     return n;
 }
 
-// cuTensorMapEncodeTiled through the runtime's driver entry point (no link-time libcuda)
-typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
-                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
-                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-static EncodeTiledFn encode_tiled_fn() {
-    static EncodeTiledFn fn = nullptr;
-    static bool tried = false;
-    if (!tried) {
-        tried = true;
-        void* p = nullptr;
-        cudaDriverEntryPointQueryResult q;
-        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
-            q == cudaDriverEntryPointSuccess)
-            fn = (EncodeTiledFn)p;
-        else
-            cudaGetLastError();
-    }
-    return fn;
-}
-
-// The TMA-fed 8-RHS kernel (rhs8_tma.cuh) serves 8 right-hand sides of an fp64 SITE-layout handle
-// with full long links over the full-lattice box (no halo); everything else takes the register
-// kernels.  Its tensor map views the parity's links as doubles [entry 36][mu 4][2 vh]; one box is
-// one matrix (9 entries) of 16 consecutive sites.
-static bool rhs8_tma_serves(dslash_t h, const StencilParams& K, bool ghost, int nrhs) {
-    const dslash_plan_t& p = h->plan;
-    if (!h->rhs8_tma || nrhs != 8 || ghost || h->kernel != DSLASH_KERNEL_SITE || h->precision != DSLASH_F64 ||
-        h->recon != 18 || h->stage || K.nbox != 1 || K.vh % rhs8_tile_sites() || !encode_tiled_fn())
-        return false;
-    for (int d = 0; d < 4; ++d)
-        if (K.box[0].lo[d] != 0 || K.box[0].n[d] != p.local_dims[d]) return false;
-    return true;
-}
-
-static dslash_status rhs8_tma_launch(dslash_t h, const StencilParams& K, cudaStream_t s) {
-    const int parity = K.links == h->links[0] ? 0 : 1;
-    EncodeTiledFn enc = encode_tiled_fn();
-    if (h->rhs8_map_links[parity] != K.links) {
-        const cuuint64_t dims[3] = {(cuuint64_t)(2 * K.vh), 4, 36};
-        const cuuint64_t strides[2] = {(cuuint64_t)(K.vh * 16), (cuuint64_t)(4 * K.vh * 16)};
-        const cuuint32_t box[3] = {(cuuint32_t)(2 * rhs8_tile_sites()), 1, 9};
-        const cuuint32_t estr[3] = {1, 1, 1};
-        if (enc(&h->rhs8_map[parity], CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<void*>(K.links), dims, strides,
-                box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
-            return fail(h, DSLASH_ERR_CUDA, "cuTensorMapEncodeTiled failed for the 8-RHS link map");
-        h->rhs8_map_links[parity] = K.links;
-    }
-    CU(h, launch_rhs8_tma(h->rhs8_map[parity], K, num_sms(h), h->pdl != 0, s));
-    return DSLASH_OK;
-}
-
 static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int kind, cudaStream_t s, int nrhs) {
     const int64_t sites = K.box_start[K.nbox];
     if (sites == 0) return DSLASH_OK;
-    if (rhs8_tma_serves(h, K, ghost, nrhs)) {  // the TMA-fed 8-RHS kernel
-        dslash_s::TimedLaunch* tl = nullptr;
-        dslash_status st = timing_begin(h, kind, s, &tl);
-        if (st == DSLASH_OK) st = rhs8_tma_launch(h, K, s);
-        if (st == DSLASH_OK && tl) CU(h, cudaEventRecord(tl->b, s));
-        return st;
-    }
     const int lanes = lanes_of(h->kernel);
     if (h->stage) return launch_stage(h, K, ghost, kind, s, nrhs, lanes);
     const int bs = h->block ? h->block : nrhs == 8 ? kDefaultBlockRhs8 : kDefaultBlock;

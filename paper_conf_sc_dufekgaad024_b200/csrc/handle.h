@@ -101,11 +101,6 @@ struct dslash_s {
     char* peer_lslab[4] = {};           // my plus neighbour's lslab[d]
     unsigned int link_epoch = 0;
     unsigned int red_epoch = 0;         // cross-rank reductions so far
-    // TMA-fed 8-RHS kernel (rhs8_tma.cuh): the tensor map of each parity's links, rebuilt when the
-    // link array it describes changes; rhs8_tma = DSLASH_OPT_RHS8_TMA
-    CUtensorMap rhs8_map[2] = {};
-    const void* rhs8_map_links[2] = {nullptr, nullptr};
-    int rhs8_tma = 1;
     char* peer_ghost[4][2] = {};        // [d][0]: minus nbr's plus ghost; [d][1]: plus nbr's minus ghost
     unsigned int* peer_ready[4][2] = {};  // the ready flag of that ghost
     unsigned int* peer_free[4][2] = {};   // [d][0]: minus nbr's free_from[d][1]; [d][1]: plus nbr's free_from[d][0]

@@ -638,34 +638,3 @@ def test_c_p2p_demo_runs(torch_cuda, args):
     r = subprocess.run([exe, *args], capture_output=True, text=True, timeout=300)
     assert r.returncode == 0, r.stdout + r.stderr
     assert "EQUALS" in r.stdout
-
-
-@pytest.mark.parametrize("dims", [(8, 10, 12, 14), (16, 16, 16, 16), (32, 32, 32, 32), (6, 8, 10, 12)])
-def test_rhs8_tma_kernel_bitwise(torch_cuda, dims):
-    """The TMA-fed 8-RHS kernel (DSLASH_OPT_RHS8_TMA, on by default for fp64 SITE handles without a
-    halo) gives the register kernel's bits for every right-hand side, and the oracle's values.
-    (6, 8, 10, 12): Vh = 2880 is a multiple of the 16-site tile; a lattice whose Vh is not takes
-    the register kernel.)"""
-    import torch
-    from paper_conf_sc_dufekgaad024_b200 import Dslash, _abi
-    fat, lng = fieldgen.workload_links(dims)
-    parity = 0
-    src = torch.stack([torch.from_numpy(fieldgen.vector_cb(dims, 110 + r, 1)) for r in range(8)]).cuda()
-    outs = []
-    with Dslash(dims, kernel="site", parity_mask=parity) as D:
-        D.load_links(fat, lng)
-        for tma in (1, 0, 1):
-            _abi.dslash_set_option(D.h, _abi.DSLASH_OPT_RHS8_TMA, tma)
-            out = torch.empty_like(src)
-            D.apply_multi(out, src, parity)
-            torch.cuda.synchronize()
-            outs.append(out.cpu())
-        single = D(src[5].contiguous(), parity).cpu()
-    assert torch.equal(outs[0], outs[1]) and torch.equal(outs[0], outs[2])
-    assert torch.equal(outs[0][5], single)
-    lex = oracle.lex_sites_of_parity(dims, parity)
-    pick = np.unique(np.concatenate([[0, lex.size - 1], np.random.default_rng(8).choice(lex.size, min(2048, lex.size),
-                                                                                       replace=False)]))
-    for r in (0, 7):
-        ref = oracle.dslash_sites(fat, lng, fieldgen.vector(dims, 110 + r), lex[pick])
-        assert oracle.normwise_error(outs[0][r].numpy()[:, pick].T, ref) <= TOL
