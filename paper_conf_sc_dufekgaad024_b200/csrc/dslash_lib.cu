@@ -1404,8 +1404,9 @@ static StencilFn pick_kernel(int precision, int recon, int lanes, int minb, int 
 
 // defaults chosen by measurement on B200 (tools/sweep.py; profiles/README.md): at 32^4 and 48^4
 // every mapping is best at <= 128 registers (min 2 blocks of 256), LANES 1/2 at 64-128 threads
-// (8 right-hand sides: 256-thread blocks, 382-389 vs 390-400 us at 64; profiles/r02/mrhs/)
-static constexpr int kDefaultBlock = 64, kDefaultBlockRhs8 = 256, kDefaultMinBlocks = 2;
+// (4 / 8 right-hand sides: 128 / 256-thread blocks, 229.0 vs 231.7 us and 382-389 vs 390-400 us at
+// 64; profiles/r02/mrhs/, profiles/r02/misc/)
+static constexpr int kDefaultBlock = 64, kDefaultBlockRhs4 = 128, kDefaultBlockRhs8 = 256, kDefaultMinBlocks = 2;
 
 static StencilFn pick_stage_kernel(int precision, int recon, bool ghost, int lanes, int nrhs) {
     const bool r12 = recon == 12;
@@ -1532,7 +1533,10 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
     if (sites == 0) return DSLASH_OK;
     const int lanes = lanes_of(h->kernel);
     if (h->stage) return launch_stage(h, K, ghost, kind, s, nrhs, lanes);
-    const int bs = h->block ? h->block : nrhs == 8 ? kDefaultBlockRhs8 : kDefaultBlock;
+    const int bs = h->block                ? h->block
+                   : nrhs == 8 ? kDefaultBlockRhs8
+                   : nrhs == 4 ? kDefaultBlockRhs4
+                               : kDefaultBlock;
     const int minb = h->min_blocks ? h->min_blocks : kDefaultMinBlocks;
     // right-hand sides are register-blocked per thread; 8 of them use 2 thread groups of 4
     const int64_t threads = sites * lanes * (nrhs == 8 ? 2 : 1);
