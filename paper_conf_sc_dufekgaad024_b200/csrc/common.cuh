@@ -51,6 +51,20 @@ __device__ __forceinline__ double2 ld_reuse(const double2* p, uint64_t pol) {
     return r;
 }
 
+// a reused vector that THIS SM will not read again (the z / t hops: their other consumers run on
+// other SMs): L2 evict_last like ld_reuse, but no L1 line, so it does not evict the x / y rows
+// the block's own threads reuse
+__device__ __forceinline__ double2 ld_reuse_na(const double2* p, uint64_t pol) {
+    double2 r;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(r.x), "=d"(r.y) : "l"(p), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ float2 ld_reuse_na(const float2* p, uint64_t pol) {
+    float2 r;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f32 {%0, %1}, [%2], %3;" : "=f"(r.x), "=f"(r.y) : "l"(p), "l"(pol));
+    return r;
+}
+
 __device__ __forceinline__ void st_stream(double2* p, double2 v) {
     asm volatile("st.global.cs.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
 }

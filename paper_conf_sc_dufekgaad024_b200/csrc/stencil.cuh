@@ -323,8 +323,9 @@ __device__ __forceinline__ float2 lds_at(uint32_t a, float2*) {
 
 // one neighbour colour component: from the staged tile (shared address sa + off_b) or from global
 template <typename V2>
-__device__ __forceinline__ V2 ld_src(bool staged, uint32_t sa, uint32_t off_b, const V2* p, uint64_t pol) {
-    return staged ? lds_at(sa + off_b, (V2*)nullptr) : ld_reuse(p, pol);
+__device__ __forceinline__ V2 ld_src(bool staged, uint32_t sa, uint32_t off_b, const V2* p, uint64_t pol,
+                                     bool no_l1 = false) {
+    return staged ? lds_at(sa + off_b, (V2*)nullptr) : no_l1 ? ld_reuse_na(p, pol) : ld_reuse(p, pol);
 }
 
 // v = 0 when z (a select, so acc + U * 0 leaves acc's value unchanged without a branch)
@@ -347,6 +348,12 @@ __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[
                 cmadd(acc[i], U[3 * i + j], v[j]);
         }
 }
+
+// z / t hop vectors bypass L1 (their other consumers run on other SMs; compile-time experiment)
+#ifndef HISQ_ZT_NO_L1
+#define HISQ_ZT_NO_L1 1
+#endif
+constexpr bool kZtNoL1 = HISQ_ZT_NO_L1 != 0;
 
 // ---------------------------------------------------------------- the stencil kernel
 // LANES consecutive threads per target site (1 = thread per site, the paper's 1LP mapping;
@@ -502,7 +509,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 #pragma unroll
                             for (int c = 0; c < 3; ++c) {
                                 v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride,
-                                              pol_keep);
+                                              pol_keep, kZtNoL1 && mu >= 2);
                                 if (GHOST) zero_if(v[c], zap);
                             }
                             if (RECON == 9 && j == 1) {
@@ -578,7 +585,8 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     V2 v[3];
 #pragma unroll
                     for (int c = 0; c < 3; ++c) {
-                        v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride, pol_keep);
+                        v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride, pol_keep,
+                                      kZtNoL1 && mu >= 2);
                         if (GHOST) zero_if(v[c], zap);
                     }
                     if (RECON == 9 && l >= 2) {
