@@ -10,7 +10,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libhisq_dslash.so")
+# HISQ_DSLASH_LIB: another build of the same library (A/B measurement of a compile-time variant)
+LIB_PATH = os.environ.get("HISQ_DSLASH_LIB") or os.path.join(_HERE, "libhisq_dslash.so")
 HEADER = os.path.join(os.path.dirname(_HERE), "include", "hisq_dslash.h")
 
 DSLASH_OK, DSLASH_ERR_ARG, DSLASH_ERR_STATE, DSLASH_ERR_CUDA, DSLASH_ERR_NCCL, DSLASH_ERR_OOM, \

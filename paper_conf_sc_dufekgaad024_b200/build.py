@@ -25,19 +25,24 @@ def sources():
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    """Compile every csrc/*.cu to an object in parallel (sm_100a, -lineinfo) and link the .so."""
-    if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= max(os.path.getmtime(s) for s in sources()):
-        return LIB
+def build(force: bool = False, verbose: bool = False, defines=(), out: str = None) -> str:
+    """Compile every csrc/*.cu to an object in parallel (sm_100a, -lineinfo) and link the .so.
+
+    defines / out (measurement aid for A/B runs): extra -D flags and another output path; such a
+    variant builds in its own object directory and is loaded with HISQ_DSLASH_LIB=<out>."""
+    lib = out or LIB
+    if not force and os.path.exists(lib) and os.path.getmtime(lib) >= max(os.path.getmtime(s) for s in sources()):
+        return lib
     from concurrent.futures import ThreadPoolExecutor
 
     nccl = nccl_dir()
-    objdir = os.path.join(HERE, "build")
+    objdir = os.path.join(HERE, "build") if out is None else out + ".objs"
     os.makedirs(objdir, exist_ok=True)
     common = ["nvcc", *ARCH, "-lineinfo", "-O3", "-std=c++17", "-Xcompiler", "-fPIC,-fvisibility=hidden",
               "-I", os.path.join(nccl, "include"), "-I", os.path.join(ROOT, "include")]
     if verbose:
         common.append("-Xptxas=-v")
+    common += ["-D" + d for d in defines]
     cus = sorted(glob.glob(os.path.join(HERE, "csrc", "*.cu")))
     objs = [os.path.join(objdir, os.path.basename(c)[:-3] + ".o") for c in cus]
 
@@ -53,9 +58,11 @@ def build(force: bool = False, verbose: bool = False) -> str:
     for src, r in zip(cus, results):
         if r.returncode != 0:
             raise RuntimeError(f"nvcc failed on {src}:\n{r.stderr}")
-    link = ["nvcc", *ARCH, "-shared", "-o", LIB, *objs, "-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
+    link = ["nvcc", *ARCH, "-shared", "-o", lib, *objs, "-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
             "-Xlinker", "-rpath=" + os.path.join(nccl, "lib")]
     subprocess.check_call(link)
+    if out is not None:
+        return lib
     build_c_demo("c_api_demo")
     build_c_demo("c_p2p_demo")
     return LIB
