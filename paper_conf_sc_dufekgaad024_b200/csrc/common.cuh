@@ -65,21 +65,6 @@ __device__ __forceinline__ float2 ld_reuse_na(const float2* p, uint64_t pol) {
     return r;
 }
 
-// volatile twins of ld_stream / ld_reuse: they keep their program order relative to each other, so
-// the compiler cannot sink a hop's loads below the previous hop's arithmetic (HISQ_ORDERED_LOADS)
-__device__ __forceinline__ double2 ld_stream_o(const double2* p, uint64_t pol) {
-    double2 r;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;"
-                 : "=d"(r.x), "=d"(r.y)
-                 : "l"(p), "l"(pol));
-    return r;
-}
-__device__ __forceinline__ double2 ld_reuse_o(const double2* p, uint64_t pol) {
-    double2 r;
-    asm volatile("ld.global.nc.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(r.x), "=d"(r.y) : "l"(p), "l"(pol));
-    return r;
-}
-
 __device__ __forceinline__ void st_stream(double2* p, double2 v) {
     asm volatile("st.global.cs.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
 }

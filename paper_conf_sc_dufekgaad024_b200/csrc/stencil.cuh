@@ -354,11 +354,6 @@ __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[
 #define HISQ_ZT_NO_L1 1
 #endif
 constexpr bool kZtNoL1 = HISQ_ZT_NO_L1 != 0;
-// multi-RHS fp64: volatile (program-ordered) link and neighbour loads (compile-time experiment)
-#ifndef HISQ_ORDERED_LOADS
-#define HISQ_ORDERED_LOADS 0
-#endif
-constexpr bool kOrdered = HISQ_ORDERED_LOADS != 0;
 
 // ---------------------------------------------------------------- the stencil kernel
 // LANES consecutive threads per target site (1 = thread per site, the paper's 1LP mapping;
@@ -577,9 +572,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                 } else {
 #pragma unroll
                     for (int e = 0; e < elems_of<RECON>(l); ++e)
-                        U[e] = to_cplx<V2>(widen(kOrdered && NRHS > 1 && sizeof(LR) == 8
-                                                     ? ld_stream_o(reinterpret_cast<const double2*>(lp + (int64_t)e * 4 * P.vh), pol_stream)
-                                                     : ld_stream(lp + (int64_t)e * 4 * P.vh, pol_stream)));
+                        U[e] = to_cplx<V2>(widen(ld_stream(lp + (int64_t)e * 4 * P.vh, pol_stream)));
                 }
                 if (elems_of<RECON>(l) == 6) reconstruct_row2(U, (VR)P.long_inv_scale);
                 V2 z9;  // recon-9: N = z9 W
@@ -592,11 +585,8 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                     V2 v[3];
 #pragma unroll
                     for (int c = 0; c < 3; ++c) {
-                        if (kOrdered && NRHS > 1 && sizeof(VR) == 8 && !stg)
-                            v[c] = to_cplx<V2>(ld_reuse_o(reinterpret_cast<const double2*>(src.p + roff + c * src.stride), pol_keep));
-                        else
-                            v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride, pol_keep,
-                                          kZtNoL1 && mu >= 2);
+                        v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride, pol_keep,
+                                      kZtNoL1 && mu >= 2);
                         if (GHOST) zero_if(v[c], zap);
                     }
                     if (RECON == 9 && l >= 2) {
