@@ -85,6 +85,8 @@ class Dslash:
             # send/recv to this rank (the P = 2 message pattern on one GPU)
             assert world_size == 1 and transport == "nccl", "self_nccl is a one-rank NCCL-transport option"
             uid = _abi.dslash_get_unique_id()
+        # the library links its own CUDA runtime: bind the handle to torch's current device explicitly
+        _abi.dslash_set_device(torch.cuda.current_device())
         self.h = _abi.dslash_create(self.global_dims, self.proc_grid, parity_mask, _abi.PRECISIONS[precision], uid,
                                     world_size, rank)
         try:

@@ -304,6 +304,7 @@ extern "C" dslash_status dslash_create(const int32_t G[4], const int32_t P[4], i
 }
 
 extern "C" dslash_status dslash_set_option(dslash_t h, int32_t key, int64_t value) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     switch (key) {
         case DSLASH_OPT_KERNEL:
@@ -422,6 +423,7 @@ static dslash_status p2p_prepare(dslash_t h);
 // as fat / lng); where absent for a halo direction with another rank as neighbour, NCCL fetches them
 static dslash_status load_links_impl(dslash_t h, const void* fat, const void* lng, const void* const* slab_fat_in,
                                      const void* const* slab_lng_in, int32_t on_device, dslash_stream_t stream) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!fat || !lng) return fail(h, DSLASH_ERR_ARG, "NULL link pointer");
     cudaStream_t s = (cudaStream_t)stream;
@@ -778,6 +780,7 @@ dslash_status hisq_convert_links_sloppy(dslash_t h, int parity) {
 }
 
 extern "C" dslash_status dslash_get_links(dslash_t h, int32_t parity, void* out_host) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!out_host || (parity & ~1)) return fail(h, DSLASH_ERR_ARG, "NULL output or bad parity");
     if (!h->loaded || !h->links[parity]) return fail(h, DSLASH_ERR_STATE, "links of parity %d not loaded", parity);
@@ -863,6 +866,7 @@ static constexpr int32_t kIpcMagic = 0x48495352;  // "HISR" (layout 2: control b
 extern "C" int64_t dslash_ipc_blob_size(void) { return (int64_t)sizeof(IpcBlob); }
 
 extern "C" dslash_status dslash_get_ipc_blob(dslash_t h, void* blob) {
+    DeviceGuard device_guard(h);
     if (!h || !blob) return fail(h, DSLASH_ERR_ARG, "NULL argument");
     if (h->transport != DSLASH_TRANSPORT_P2P) return fail(h, DSLASH_ERR_STATE, "set DSLASH_TRANSPORT_P2P first");
     dslash_status st = alloc_lslab(h);
@@ -901,6 +905,7 @@ static dslash_status ipc_open(dslash_t h, void** p, cudaIpcMemHandle_t handle) {
 // Every rank's control block (reduction slots, flags); the neighbours' ghosts and the plus
 // neighbours' link-slab buffers.
 extern "C" dslash_status dslash_open_ipc_blobs(dslash_t h, const void* blobs) {
+    DeviceGuard device_guard(h);
     if (!h || !blobs) return fail(h, DSLASH_ERR_ARG, "NULL argument");
     if (h->transport != DSLASH_TRANSPORT_P2P) return fail(h, DSLASH_ERR_STATE, "set DSLASH_TRANSPORT_P2P first");
     if (h->p2p_ready) return fail(h, DSLASH_ERR_STATE, "IPC blobs already opened");
@@ -1346,6 +1351,7 @@ static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaS
 }
 
 extern "C" dslash_status dslash_halo_start(dslash_t h, const void* in, int32_t src_parity, dslash_stream_t stream) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!in || ((uintptr_t)in & 15)) return fail(h, DSLASH_ERR_ARG, "in is NULL or not 16-byte aligned");
     if (src_parity & ~1) return fail(h, DSLASH_ERR_ARG, "src_parity %d not in {0,1}", src_parity);
@@ -1356,6 +1362,7 @@ extern "C" dslash_status dslash_halo_start(dslash_t h, const void* in, int32_t s
 // `stream` waits until this rank's ghosts hold the current epoch's faces and its own sends are
 // done (P2P: my ready flags, raised by the neighbours; NCCL / self copies: the comm event).
 extern "C" dslash_status dslash_halo_wait(dslash_t h, dslash_stream_t stream) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!h->halo_pending) return DSLASH_OK;
     if (h->transport == DSLASH_TRANSPORT_P2P) {
@@ -1601,6 +1608,7 @@ dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, 
 
 static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs,
                                 dslash_stream_t stream, bool push_out) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (parity & ~1) return fail(h, DSLASH_ERR_ARG, "parity %d not in {0,1}", parity);
     if (nrhs < 1) return fail(h, DSLASH_ERR_ARG, "nrhs %d < 1", nrhs);
@@ -1736,6 +1744,7 @@ extern "C" dslash_status dslash_apply_multi(dslash_t h, int32_t nrhs, void* out,
 
 extern "C" dslash_status dslash_apply_host(dslash_t h, void* out_host, const void* in_host, int32_t parity,
                                            dslash_stream_t stream) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!out_host || !in_host) return fail(h, DSLASH_ERR_ARG, "NULL host buffer");
     const size_t bytes = 3 * (size_t)h->plan.vh_local * vec_elem(h);
@@ -1752,6 +1761,7 @@ extern "C" dslash_status dslash_apply_host(dslash_t h, void* out_host, const voi
 extern "C" dslash_status dslash_apply_host_batch(dslash_t h, int32_t n, void* const* out_host,
                                                  const void* const* in_host, int32_t parity,
                                                  dslash_stream_t stream) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (n < 0 || (n > 0 && (!out_host || !in_host))) return fail(h, DSLASH_ERR_ARG, "bad batch arguments");
     if (!h->loaded) return fail(h, DSLASH_ERR_STATE, "apply before load_links");
@@ -1804,6 +1814,7 @@ extern "C" dslash_status dslash_apply_host_batch(dslash_t h, int32_t n, void* co
 
 // ============================================================================ misc
 extern "C" dslash_status dslash_sync(dslash_t h) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     CU(h, cudaStreamSynchronize(h->comm));
     CU(h, cudaDeviceSynchronize());
@@ -1817,6 +1828,7 @@ extern "C" dslash_status dslash_sync(dslash_t h) {
 }
 
 extern "C" dslash_status dslash_kernel_timing(dslash_t h, int32_t which, double* total_ms, int64_t* launches) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!total_ms || !launches) return fail(h, DSLASH_ERR_ARG, "NULL output");
     double tot = 0.0;
@@ -1841,6 +1853,7 @@ extern "C" dslash_status dslash_kernel_timing(dslash_t h, int32_t which, double*
 
 extern "C" dslash_status dslash_timeline(dslash_t h, int64_t max_entries, int32_t* kinds, double* start_ms,
                                          double* end_ms, int64_t* n) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (!n || (max_entries > 0 && (!kinds || !start_ms || !end_ms))) return fail(h, DSLASH_ERR_ARG, "NULL output");
     *n = (int64_t)h->tused;
@@ -1858,6 +1871,7 @@ extern "C" dslash_status dslash_timeline(dslash_t h, int64_t max_entries, int32_
 }
 
 extern "C" dslash_status dslash_kernel_timing_reset(dslash_t h) {
+    DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (h->tused) CU(h, cudaEventSynchronize(h->tpool[h->tused - 1].b));
     h->tused = 0;
@@ -1873,6 +1887,7 @@ extern "C" dslash_status dslash_get_plan(dslash_t h, dslash_plan_t* plan) {
 extern "C" int64_t dslash_local_half_volume(dslash_t h) { return h ? h->plan.vh_local : -1; }
 
 extern "C" dslash_status dslash_destroy(dslash_t h) {
+    DeviceGuard device_guard(h);
     if (!h) return DSLASH_OK;
     if (h->comm) cudaStreamSynchronize(h->comm);
     cudaDeviceSynchronize();

@@ -119,6 +119,20 @@ struct dslash_s {
     std::string msg;
 };
 
+// Every entry point that touches the GPU runs on the handle's device (several handles on several
+// devices in one process) and restores the caller's current device on return.
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(const dslash_s* h) {
+        int cur = 0;
+        if (h && cudaGetDevice(&cur) == cudaSuccess && cur != h->device && cudaSetDevice(h->device) == cudaSuccess)
+            prev = cur;
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
 // Record a failure on the handle (first error wins) or, with h == NULL, in the thread's last
 // error; returns st.
 dslash_status hisq_fail(dslash_t h, dslash_status st, const char* fmt, ...);

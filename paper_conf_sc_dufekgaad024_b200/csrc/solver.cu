@@ -385,6 +385,7 @@ static dslash_status normal_apply(dslash_t h, V2* q, const V2* p, int32_t parity
 
 extern "C" dslash_status dslash_normal_apply(dslash_t h, void* out, const void* in, int32_t parity, double mass,
                                              dslash_stream_t stream) {
+    DeviceGuard device_guard(h);
     dslash_status st = check_solver_args(h, out, in, parity, false);  // no dot product
     if (st != DSLASH_OK) return st;
     if ((st = need_scratch(h)) != DSLASH_OK) return st;
@@ -556,6 +557,7 @@ static dslash_status true_residual(dslash_t h, double2* r, const double2* x, con
 extern "C" dslash_status dslash_cg(dslash_t h, void* x_out, const void* b_in, int32_t parity, double mass,
                                    double rel_tol, int32_t max_iter, int32_t* iters, double* rel_resid,
                                    dslash_stream_t stream) {
+    DeviceGuard device_guard(h);
     dslash_status st = check_solver_args(h, x_out, b_in, parity);
     if (st != DSLASH_OK) return st;
     if (!(rel_tol > 0.0) || max_iter < 1) return hisq_fail(h, DSLASH_ERR_ARG, "rel_tol must be > 0 and max_iter >= 1");
@@ -640,6 +642,7 @@ struct SloppyScope {
 extern "C" dslash_status dslash_cg_mixed(dslash_t h, void* x_out, const void* b_in, int32_t parity, double mass,
                                          double rel_tol, double inner_tol, int32_t max_iter, int32_t* iters,
                                          int32_t* outer_iters, double* rel_resid, dslash_stream_t stream) {
+    DeviceGuard device_guard(h);
     dslash_status st = check_solver_args(h, x_out, b_in, parity);
     if (st != DSLASH_OK) return st;
     if (h->precision != DSLASH_F64)
