@@ -277,3 +277,38 @@ def test_distinct_gpus_multi_rhs_nccl():
         pytest.skip(f"needs 2 GPUs, {_ngpu()} visible")
     got = _run(2, gdims, grid, {"_distinct": True, "transport": "nccl"}, 0, napply=2, nrhs=3)
     assert np.array_equal(got, _single(gdims, {}, 0, nrhs=3))
+
+
+def test_two_handles_two_devices_one_process():
+    """Two handles in one process on different GPUs, used interleaved while torch's current device
+    is the other one: every entry point runs on its handle's device (DeviceGuard) and leaves the
+    caller's current device as it was."""
+    import torch
+    if _ngpu() < 2:
+        pytest.skip(f"needs 2 GPUs, {_ngpu()} visible")
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 8, 8, 16)
+    fat, lng = fieldgen.workload_links(dims)
+    handles = []
+    for dev in (0, 1):
+        torch.cuda.set_device(dev)
+        D = Dslash(dims)
+        D.load_links(fat, lng)
+        handles.append(D)
+    src = [torch.from_numpy(fieldgen.vector_cb(dims, SEED, 1)).to(f"cuda:{d}") for d in (0, 1)]
+    outs = []
+    for it in range(3):
+        for d, D in enumerate(handles):
+            torch.cuda.set_device(1 - d)                         # the OTHER device is current
+            with torch.cuda.device(d):
+                o = torch.empty_like(src[d])
+                D.apply(o, src[d], 0, torch.cuda.current_stream(d))
+            assert torch.cuda.current_device() == 1 - d
+            outs.append(o)
+    torch.cuda.synchronize(0)
+    torch.cuda.synchronize(1)
+    ref = outs[0].cpu()
+    for o in outs:
+        assert torch.equal(o.cpu(), ref)
+    for D in handles:
+        D.close()
