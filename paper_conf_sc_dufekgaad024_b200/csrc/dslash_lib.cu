@@ -1024,7 +1024,7 @@ __global__ void __launch_bounds__(256) face_copy_kernel(const CopySet C) {
             const int64_t i = i0 + u * stride;
             if (i < n) {
                 const int64_t r = i / S.words, w = i - r * S.words;
-                v[u] = __ldcs(reinterpret_cast<const W*>(S.src + r * S.spitch) + w);
+                v[u] = __ldg(reinterpret_cast<const W*>(S.src + r * S.spitch) + w);  // default L2 policy: the stencil reads these lines too
             }
         }
 #pragma unroll
