@@ -1540,10 +1540,14 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
     if (sites == 0) return DSLASH_OK;
     const int lanes = lanes_of(h->kernel);
     if (h->stage) return launch_stage(h, K, ghost, kind, s, nrhs, lanes);
-    const int bs = h->block                ? h->block
-                   : nrhs == 8 ? kDefaultBlockRhs8
-                   : nrhs == 4 ? kDefaultBlockRhs4
-                               : kDefaultBlock;
+    // recon-9 on the site kernel (its default): 256 / 128 / 64 threads for fp64 / mixed / fp32
+    // (profiles/r02/recon9_blocks/: 150.6 vs 152.7 us, 86.9 vs 88.0 us, 75.9 vs 77.3 us)
+    const int r9_block = h->precision == DSLASH_F64 ? 256 : h->precision == DSLASH_MIXED ? 128 : 64;
+    const int bs = h->block                        ? h->block
+                   : nrhs == 8                     ? kDefaultBlockRhs8
+                   : nrhs == 4                     ? kDefaultBlockRhs4
+                   : (h->recon == 9 && lanes == 1) ? r9_block
+                                                   : kDefaultBlock;
     const int minb = h->min_blocks ? h->min_blocks : kDefaultMinBlocks;
     // right-hand sides are register-blocked per thread; 8 of them use 2 thread groups of 4
     const int64_t threads = sites * lanes * (nrhs == 8 ? 2 : 1);
