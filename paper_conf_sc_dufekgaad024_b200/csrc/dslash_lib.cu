@@ -1047,6 +1047,7 @@ struct FaceCopies {
         size_t dpitch, spitch, width, height;
     } raw[4];
     int n = 0;
+    cudaStream_t stream_of_pending = nullptr;
     // a local segment is batched; a copy into another rank's memory goes to the copy engines now
     dslash_status add(dslash_t h, void* dst, size_t dpitch, const void* src, size_t spitch, size_t width,
                       size_t height, cudaStream_t st, bool local) {
@@ -1055,6 +1056,11 @@ struct FaceCopies {
             CU(h, cudaMemcpy2DAsync(dst, dpitch, src, spitch, width, height, cudaMemcpyDeviceToDevice, st));
             return DSLASH_OK;
         }
+        if (n == 4) {  // (an exchange has at most 4 local segments; flush rather than overflow)
+            dslash_status st = flush(h, stream_of_pending);
+            if (st != DSLASH_OK) return st;
+        }
+        stream_of_pending = st;
         raw[n++] = {dst, src, dpitch, spitch, width, height};
         return DSLASH_OK;
     }
