@@ -1057,8 +1057,8 @@ struct FaceCopies {
             return DSLASH_OK;
         }
         if (n == 4) {  // (an exchange has at most 4 local segments; flush rather than overflow)
-            dslash_status st = flush(h, stream_of_pending);
-            if (st != DSLASH_OK) return st;
+            const dslash_status fs = flush(h, stream_of_pending);
+            if (fs != DSLASH_OK) return fs;
         }
         stream_of_pending = st;
         raw[n++] = {dst, src, dpitch, spitch, width, height};
