@@ -357,16 +357,6 @@ __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[
 #define HISQ_ZT_NO_L1 1
 #endif
 constexpr bool kZtNoL1 = HISQ_ZT_NO_L1 != 0;
-// 8 right-hand sides (fp64, full links, interior): links copied to shared memory by cp.async a hop
-// ahead (compile-time switch, measured A/B)
-#ifndef HISQ_RHS8_ASYNC
-#define HISQ_RHS8_ASYNC 1
-#endif
-constexpr bool kRhs8Async = HISQ_RHS8_ASYNC != 0;
-#ifndef HISQ_RHS8_UNROLL
-#define HISQ_RHS8_UNROLL 4
-#endif
-constexpr int kRhs8Unroll = HISQ_RHS8_UNROLL;
 
 // ---------------------------------------------------------------- the stencil kernel
 // LANES consecutive threads per target site (1 = thread per site, the paper's 1LP mapping;
@@ -404,8 +394,6 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
     // ONE group, so a 16-byte load of a quarter-warp touches one 128-byte line (one L1 wavefront)
     // instead of two; the warp still covers the same 16 sites
     constexpr bool kQuarterRuns = LANES == 1 && (RHSL == 2 || RHSL == 4) && !STAGED;
-    constexpr bool kAsyncLinks = kRhs8Async && kQuarterRuns && RHSL == 2 && NRHS == 4 && RECON == 18 &&
-                                 sizeof(LR) == 8 && sizeof(VR) == 8 && !GHOST;
     const int rl = (RHSL == 1)    ? 0
                    : kQuarterRuns ? (int)((gid >> 3) % RHSL)
                                   : (int)((gid / LANES) % RHSL);
@@ -436,61 +424,6 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
             asm volatile("griddepcontrol.wait;\n\tmov.b64 %0, %1;" : "=l"(in) : "l"(P.in) : "memory");
             if (threadIdx.x == 0) stage_tile_issue(P, in, T, NRHS * RHSL, pol_keep);
         }
-        if constexpr (kAsyncLinks) {
-            // 8 right-hand sides, fp64 full links (HISQ_RHS8_ASYNC): the link matrices of hop j + 2
-            // are copied global -> shared memory by the threads themselves (cp.async, no registers)
-            // while hop j computes, so the DRAM latency of the link stream leaves the warps'
-            // critical path and a matrix never occupies 36 registers; the two threads of a site
-            // (lanes l and l ^ 8) each copy alternate entries of one shared copy per site.  Entries
-            // are applied in row-major order to every right-hand side: acc[r][i] receives j = 0, 1,
-            // 2 in order, hop after hop, as in matvec_acc, so the bits are the register kernel's.
-            __shared__ double2 lk[2][9][128];
-            const int ls = (int)(site - (int64_t)blockIdx.x * (blockDim.x >> 1));
-            const unsigned pair = (1u << (threadIdx.x & 31)) | (1u << ((threadIdx.x & 31) ^ 8));
-            const double2* dl = reinterpret_cast<const double2*>(links);
-            auto issue = [&](int j) {
-                const double2* lp = dl + link_index<1>(j >> 2, j & 3, 0, P.vh, s.cb);
-#pragma unroll
-                for (int e = 0; e < 9; ++e)
-                    if ((e & 1) == rl) cp_async16(&lk[j & 1][e][ls], lp + (int64_t)e * 4 * P.vh, pol_stream);
-                cp_async_commit();
-            };
-            issue(0);
-            issue(1);
-            const void* in;
-            asm volatile("griddepcontrol.wait;\n\tmov.b64 %0, %1;" : "=l"(in) : "l"(P.in) : "memory");
-#pragma unroll(kRhs8Unroll)
-            for (int j = 0; j < 16; ++j) {
-                const int mu = j >> 2, l = j & 3;
-                const int h = (l == 0) ? 1 : (l == 1) ? -1 : (l == 2) ? 3 : -3;
-                const SrcRef<V2> src = source<V2, false>(P, in, mu, h, s, rl * NRHS);
-                V2 v[NRHS][3];
-#pragma unroll
-                for (int r = 0; r < NRHS; ++r)
-#pragma unroll
-                    for (int c = 0; c < 3; ++c)
-                        v[r][c] = ld_src(false, 0u, 0u, src.p + (int64_t)r * 3 * src.stride + c * src.stride, pol_keep,
-                                         kZtNoL1 && mu >= 2);
-                cp_async_wait_1();   // hop j's copies (this thread's) have landed
-                __syncwarp(pair);    // ... and the partner's
-#pragma unroll
-                for (int e = 0; e < 9; ++e) {
-                    const V2 u = to_cplx<V2>(lds(&lk[j & 1][e][ls]));
-#pragma unroll
-                    for (int r = 0; r < NRHS; ++r) {
-                        if (l & 1)
-                            cmsub(acc[r][e / 3], u, v[r][e % 3]);
-                        else
-                            cmadd(acc[r][e / 3], u, v[r][e % 3]);
-                    }
-                }
-                __syncwarp(pair);    // both have read stage j & 1: refill it with hop j + 2
-                if (j + 2 < 16)
-                    issue(j + 2);
-                else
-                    cp_async_commit();  // (empty group: keeps wait_group 1 exact)
-            }
-        } else {
         V2 U0[9];
         // (not in the ghost pass, whose first hop is never a ghost hop for LANES 1 / 2)
         if (sizeof(LR) != 4 && !(GHOST && P.halo_pass == kPassGhost)) {
@@ -680,7 +613,6 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
             }
             }  // unpaired links
         }
-        }  // kAsyncLinks
     }
     if (LANES > 1) {
         // butterfly over the lanes of a site: every lane ends with the same bits
