@@ -159,3 +159,52 @@ def test_32_nccl_self_halo(torch_cuda, links32, psi_full):
     parity = 0
     for ss, got in _run_chain(torch_cuda, links32, psi_full, parity, force_halo=0xC, self_nccl=True):
         _check(got, fat, lng, psi_full(ss[0]), parity, "f64", ("nccl", ss))
+
+
+# ---------------------------------------------------------------------------- 48^4 and its per-GPU volumes
+DIMS48 = (48, 48, 48, 48)
+
+
+@pytest.fixture(scope="module")
+def links48():
+    return fieldgen.workload_links(DIMS48)
+
+
+def _check48(torch, fat, lng, dims, parity, precision, what, nsample=2048, **kw):
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    with Dslash(dims, parity_mask=parity, precision=precision, **kw) as D:
+        D.load_links(fat, lng)
+        src = torch.from_numpy(fieldgen.vector_cb(dims, 401, 1 - parity)).to(D.dtype).cuda()
+        out = D.empty_vector()
+        for _ in range(2):                              # back to back, PDL
+            D.apply(out, src, parity)
+        torch.cuda.synchronize()
+        got = out.cpu().numpy()
+    lex = oracle.lex_sites_of_parity(dims, parity)
+    pick = np.unique(np.concatenate([[0, 1, lex.size - 2, lex.size - 1],
+                                     np.random.default_rng(48).choice(lex.size, nsample, replace=False)]))
+    ref = oracle.dslash_sites(fat, lng, fieldgen.vector(dims, 401), lex[pick])
+    err = oracle.normwise_error(got[:, pick].T.astype(np.complex128), ref)
+    assert err <= TOL[precision], (what, err)
+    if precision != "f64":
+        assert err > 1e-12, (what, err)
+
+
+@pytest.mark.parametrize("precision,recon", [("f32", 18), ("mixed", 18), ("f64", 12), ("f64", 9), ("f32", 12)])
+def test_48_precisions_and_recon(torch_cuda, links48, precision, recon):
+    """The strong-scaling lattice (BASELINE.json configs[3]) on one GPU, reduced precision and
+    long-link compression, sampled against the oracle."""
+    fat, lng = links48
+    _check48(torch_cuda, fat, lng, DIMS48, 1, precision, (precision, recon), recon=recon,
+             kernel="site" if recon == 9 else "dir2")
+
+
+@pytest.mark.parametrize("dims,mask,overlap", [((48, 48, 48, 6), 0x8, "sites"), ((48, 48, 48, 6), 0x8, "dirs"),
+                                               ((48, 48, 24, 12), 0xC, "sites"), ((48, 48, 48, 12), 0x8, "sites")])
+@pytest.mark.parametrize("precision", ["f64", "mixed"])
+def test_48_per_gpu_volumes_self_halo(torch_cuda, dims, mask, overlap, precision):
+    """The per-GPU volumes of 48^4 on 8 GPUs (t8: 48^3 x 6, no interior site; z2 x t4: 48^2 x 24 x
+    12, choose_grid's pick) and on 4 (48^3 x 12), through the self-halo in the bench's launch
+    configuration, sampled against the oracle of that (periodic) lattice."""
+    fat, lng = fieldgen.workload_links(dims)
+    _check48(torch_cuda, fat, lng, dims, 0, precision, (dims, mask, overlap), force_halo=mask, overlap=overlap)
