@@ -97,7 +97,7 @@ enum {
                                    precisions (dslash_cg_mixed's fp32 copies are rebuilt in full);
                                    load_links
                                    verifies that every long link
-                                   is rebuilt within 1e-12 s, which also rejects links near the
+                                   is rebuilt within 1e-11 s, which also rejects links near the
                                    parameterisation's singular set |a2|^2 + |a3|^2 -> 0 (e.g.
                                    multiples of the identity): DSLASH_ERR_ARG.
                                    Before load_links                                                  */
