@@ -164,16 +164,19 @@ def test_full_size_32_halo_path(torch_cuda, mask):
     assert torch.equal(outs[0], outs[1]) and torch.equal(outs[0], outs[2])
 
 
-def test_large_lattice_64x64x64x32(torch_cuda):
+@pytest.mark.parametrize("recon", [18, 9])
+def test_large_lattice_64x64x64x32(torch_cuda, recon):
     """A large local volume (Vh = 4.2M, 9.7 GB of links per parity): 64-bit indexing and grid
-    sizes; 2048 sampled sites vs the oracle (first/last sites included)."""
+    sizes; 2048 sampled sites vs the oracle (first/last sites included).  recon-9 too: its load
+    check must accept the 33 M long links of a random lattice (the rebuild's worst-link error grows
+    with the lattice, DESIGN.md §12 f-2b)."""
     import torch
     from paper_conf_sc_dufekgaad024_b200 import Dslash, _abi
     dims = (64, 64, 64, 32)
     fat, lng = fieldgen.workload_links(dims)
     psi = fieldgen.vector(dims, fieldgen.SEED_PSI)
     parity = 0
-    with Dslash(dims, parity_mask=_abi.DSLASH_EVEN) as D:
+    with Dslash(dims, parity_mask=_abi.DSLASH_EVEN, recon=recon, kernel="site" if recon == 9 else "dir2") as D:
         D.load_links(fat, lng)
         out = D(torch.from_numpy(fieldgen.vector_cb(dims, fieldgen.SEED_PSI, 1)).cuda(), parity)
         torch.cuda.synchronize()
