@@ -215,6 +215,27 @@ def test_multirank_p2p_cg_bitwise(gdims, grid, mixed):
     assert oracle.normwise_error(got[0], oracle.full_to_cb(x_ref, parity)) <= 1e-8
 
 
+@pytest.mark.parametrize("kw", [{"recon": 9, "kernel": "site"}, {"recon": 12}, {"overlap": "dirs"}])
+@pytest.mark.parametrize("mixed", [False, True])
+def test_multirank_p2p_cg_variants(kw, mixed):
+    """CG and mixed CG over 2 colocated ranks with compressed long links or the split-by-direction
+    overlap: the same iterates as the 1-rank solve (recon-9 / recon-12 bitwise; the split by
+    direction sums boundary sites in another order, so its solve is compared with the oracle)."""
+    gdims, grid = (8, 8, 8, 16), (1, 1, 1, 2)
+    infos = []
+    got = _run(2, gdims, grid, {"_mode": "cg_mixed" if mixed else "cg", **kw}, 0, infos=infos)
+    assert all(i[0] for i in infos), infos
+    if kw.get("overlap") != "dirs":
+        ref, ref_info = _single_cg(gdims, 0, mixed, kw)
+        assert tuple(infos[0]) == tuple(ref_info), (infos[0], ref_info)
+        assert np.array_equal(got, ref)
+    from oracle import cg as ocg
+    fat, lng = fieldgen.workload_links(gdims)
+    b_full = oracle.cb_to_full(fieldgen.vector_cb(gdims, SEED, 0), gdims, 0)
+    x_ref, _ = ocg.cg(fat, lng, b_full, 0, CG_MASS, rel_tol=1e-10, max_iter=2000)
+    assert oracle.normwise_error(got[0], oracle.full_to_cb(x_ref, 0)) <= 1e-8
+
+
 def test_multirank_p2p_cg_push():
     """CG with the producer push across 2 ranks (push in every exchange, P2P reductions)."""
     gdims, grid = (8, 8, 8, 16), (1, 1, 1, 2)
