@@ -8,22 +8,6 @@
 
 #include "dispatch.h"
 #include "stencil.cuh"
-#include "stencil_mrhs.cuh"
-
-// HISQ_MRHS_PIPE (compile-time, measurement aid): 8 right-hand sides through the explicitly
-// pipelined kernel (stencil_mrhs.cuh) with MINB / link distance LD / vector distance VD
-#ifndef HISQ_MRHS_PIPE
-#define HISQ_MRHS_PIPE 0
-#endif
-#ifndef HISQ_MRHS_MINB
-#define HISQ_MRHS_MINB 1
-#endif
-#ifndef HISQ_MRHS_LD
-#define HISQ_MRHS_LD 1
-#endif
-#ifndef HISQ_MRHS_VD
-#define HISQ_MRHS_VD 1
-#endif
 
 namespace hisq {
 
@@ -32,10 +16,7 @@ StencilFn pick_minb(int minb, int nrhs) {
     switch (nrhs) {
         case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 2>;
         case 4: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4>;
-        case 8:
-            if constexpr (HISQ_MRHS_PIPE && !GHOST && LANES == 1 && sizeof(LR) == 8 && RECON != 9)
-                return dslash_mrhs_kernel<LR, VR, RECON, 4, 2, HISQ_MRHS_MINB, HISQ_MRHS_LD, HISQ_MRHS_VD>;
-            return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2>;  // 2 thread groups x 4 RHS each
+        case 8: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2>;  // 2 thread groups x 4 RHS each
         default: break;
     }
     switch (minb) {

@@ -193,39 +193,6 @@ __device__ __forceinline__ Site decode_site(const StencilParams& P, int64_t gid)
     return s;
 }
 
-#ifndef HISQ_TILE8
-#define HISQ_TILE8 0
-#endif
-#ifndef HISQ_TILE8_TY
-#define HISQ_TILE8_TY 4
-#endif
-// site -> (x, y, z, t) for the tiled 8-RHS order: within a tile xh fastest, then TY rows, then
-// z0 / z0 + 2, then t0 / t0 + 2; tiles by y, then z pairs (z0 = 4 (p / 2) + p % 2), then t pairs
-template <int TY>
-__device__ __forceinline__ Site decode_site_tiled(const StencilParams& P, int64_t gid) {
-    const Box& B = P.box[0];
-    uint32_t r = (uint32_t)gid;
-    const uint32_t lxh = (uint32_t)(B.n[0] >> 1);
-    Site s;
-    s.xh = (int)(r % lxh) + (B.lo[0] >> 1);
-    r /= lxh;
-    const int yl = (int)(r % TY);
-    r /= TY;
-    const int zs = (int)(r & 1), ts = (int)((r >> 1) & 1);
-    r >>= 2;
-    const uint32_t nyt = (uint32_t)B.n[1] / TY, nzp = (uint32_t)B.n[2] / 2;
-    const int yt = (int)(r % nyt);
-    r /= nyt;
-    const int zp = (int)(r % nzp);
-    const int tp = (int)(r / nzp);
-    s.y = yt * TY + yl + B.lo[1];
-    s.z = (zp >> 1) * 4 + (zp & 1) + 2 * zs + B.lo[2];
-    s.t = (tp >> 1) * 4 + (tp & 1) + 2 * ts + B.lo[3];
-    s.x = 2 * s.xh + ((P.parity + s.y + s.z + s.t) & 1);
-    s.cb = s.xh + (int64_t)P.lxh * (s.y + (int64_t)P.L[1] * (s.z + (int64_t)P.L[2] * s.t));
-    return s;
-}
-
 template <typename V2>
 struct SrcRef {
     const V2* p;  // colour component c at p[c * stride]
@@ -391,28 +358,6 @@ __device__ __forceinline__ void matvec_acc(V2 acc[3], const V2 U[9], const V2 v[
 #endif
 constexpr bool kZtNoL1 = HISQ_ZT_NO_L1 != 0;
 
-// Software prefetch a few hops ahead (compile-time measurement aid): HISQ_PF_DIST hops ahead,
-// links / vectors into L2 (1) or L1 (2) or not at all (0), for launches of >= HISQ_PF_MINRHS RHS.
-#ifndef HISQ_PF_DIST
-#define HISQ_PF_DIST 0
-#endif
-#ifndef HISQ_PF_LINK
-#define HISQ_PF_LINK 1
-#endif
-#ifndef HISQ_PF_VEC
-#define HISQ_PF_VEC 1
-#endif
-#ifndef HISQ_PF_MINRHS
-#define HISQ_PF_MINRHS 8
-#endif
-template <int LEVEL>
-__device__ __forceinline__ void prefetch_line(const void* p) {
-    if (LEVEL == 2)
-        asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
-    else if (LEVEL == 1)
-        asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
-}
-
 // ---------------------------------------------------------------- the stencil kernel
 // LANES consecutive threads per target site (1 = thread per site, the paper's 1LP mapping;
 // 4 = one lane per direction, the paper's 3LP-1 site x direction split with a shuffle
@@ -456,11 +401,6 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                                       : gid / (LANES * RHSL);
     const bool valid = site < site_end;
     if (LANES == 1 && !valid) return;
-    // HISQ_TILE8 (measurement aid): 8-RHS interior sites enumerated in tiles of TY rows x 2 z x 2 t
-    // planes (stride 2), so the z / t hop sources of a tile's planes overlap in L1
-    constexpr bool kTile8 = HISQ_TILE8 && kQuarterRuns && RHSL == 2 && !GHOST && !STAGED;
-    const bool tiled = kTile8 && P.nbox == 1 && (P.box[0].n[1] % HISQ_TILE8_TY) == 0 && (P.box[0].n[2] % 4) == 0 &&
-                       (P.box[0].n[3] % 4) == 0;
     V2 acc[NRHS][3];
 #pragma unroll
     for (int r = 0; r < NRHS; ++r)
@@ -470,7 +410,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
     if (valid) {
         const uint64_t pol_stream = policy_evict_first();
         const uint64_t pol_keep = policy_evict_last();
-        s = tiled ? decode_site_tiled<HISQ_TILE8_TY>(P, site) : decode_site(P, site);
+        s = decode_site(P, site);
         const L2* links = static_cast<const L2*>(P.links);
         // Programmatic dependent launch (DSLASH_OPT_PDL): the links are read-only, so the first
         // matrix (unpaired layouts) is fetched before waiting for the previous grid; psi (and the
@@ -616,29 +556,6 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                                     pol_stream)));
                     }
                 }
-#if HISQ_PF_DIST > 0
-                if constexpr (LANES == 1 && !STAGED && !GHOST && NRHS * RHSL >= HISQ_PF_MINRHS) {
-                    // software prefetch of hop q + D (no destination registers): lane j of each
-                    // 8-site run touches lines j, j + 8, ... of the hop's link entries (group 0
-                    // only: the groups share links) and the group's (rhs, colour) planes
-                    const int q2 = kk * 4 + l + HISQ_PF_DIST;
-                    if (q2 < 4 * K) {
-                        const int mu2 = q2 / 4, l2 = q2 % 4;
-                        const int h2 = (l2 == 0) ? 1 : (l2 == 1) ? -1 : (l2 == 2) ? 3 : -3;
-                        const SrcRef<V2> s2 = source<V2, GHOST>(P, in, mu2, h2, s, rl * NRHS);
-                        const L2* lp2 = links + link_index<LANES, RECON>(mu2, l2, 0, P.vh, s.cb);
-                        const int nl = (HISQ_PF_LINK && rl == 0 && !(RECON == 9 && l2 >= 2)) ? elems_of<RECON>(l2) : 0;
-                        const int nv = HISQ_PF_VEC ? NRHS * 3 : 0;
-                        const int j = (int)(gid & 7);
-#pragma unroll
-                        for (int it0 = 0; it0 < elems_of<RECON>(0) + NRHS * 3; it0 += 8) {
-                            const int it = it0 + j;
-                            if (it < nl) prefetch_line<HISQ_PF_LINK>(lp2 + (int64_t)it * 4 * P.vh);
-                            else if (it < nl + nv) prefetch_line<HISQ_PF_VEC>(s2.p + (int64_t)(it - nl) * s2.stride);
-                        }
-                    }
-                }
-#endif
                 const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0, false} : source<V2, GHOST>(P, in, mu, h, s, rl * NRHS);
                 const uint32_t sa = stg ? staged_addr<V2>(P, T, sbase, mu, h, s, rl * NRHS) : 0u;
                 // split-by-direction passes: the ghost pass takes only the ghost hops (the link of
@@ -672,7 +589,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 #pragma unroll
                     for (int c = 0; c < 3; ++c) {
                         v[c] = ld_src(stg, sa, (uint32_t)(r * 3 + c) * plane_b, src.p + roff + c * src.stride, pol_keep,
-                                      kZtNoL1 && mu >= 2 && !tiled);
+                                      kZtNoL1 && mu >= 2);
                         if (GHOST) zero_if(v[c], zap);
                     }
                     if (RECON == 9 && l >= 2) {
@@ -782,13 +699,8 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
     }
 }
 
-#ifndef HISQ_TILE8_BLOCK
-#define HISQ_TILE8_BLOCK 256
-#endif
 template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1, int RHSL = 1>
-__global__ void __launch_bounds__((HISQ_TILE8 && NRHS * RHSL == 8 && !GHOST) ? HISQ_TILE8_BLOCK : 256,
-                                  (HISQ_TILE8 && NRHS * RHSL == 8 && !GHOST) ? 256 * MINB / HISQ_TILE8_BLOCK : MINB)
-    dslash_kernel(const StencilParams P) {
+__global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P) {
     // every block has started: the next PDL-launched apply may begin filling freed SMs
     asm volatile("griddepcontrol.launch_dependents;");
     dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
