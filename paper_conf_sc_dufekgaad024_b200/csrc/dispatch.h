@@ -31,8 +31,4 @@ StencilFn pick_f64_r9_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_f32_r9_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_mixed_r9_stage(bool ghost, int lanes, int nrhs);
 
-// the 8-RHS kernel with TMA-fed links (stencil_mrhs.cuh): nullptr unless fp64 links and vectors
-StencilFn pick_f64_r18_rhs8_tma(int variant, size_t* smem);
-StencilFn pick_f64_r12_rhs8_tma(int variant, size_t* smem);
-
 }  // namespace hisq

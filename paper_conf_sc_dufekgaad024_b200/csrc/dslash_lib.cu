@@ -1546,47 +1546,11 @@ static int num_sms(dslash_t h) {
     return n;
 }
 
-// 8 right-hand sides with the link stream on the TMA engine (stencil_mrhs.cuh): fp64, interior,
-// one box of full x, y and z extents (16 consecutive target sites per warp), the site mapping.
-// HISQ_RHS8_TMA=<variant> selects it (measurement stage; -1 / unset: off)
-static int rhs8_tma_variant() {
-    static const int v = getenv("HISQ_RHS8_TMA") ? atoi(getenv("HISQ_RHS8_TMA")) : -1;
-    return v;
-}
-
-static bool rhs8_tma_ok(dslash_t h, const StencilParams& K, bool ghost, int lanes, int nrhs, int64_t sites) {
-    return nrhs == 8 && !ghost && lanes == 1 && !h->block && h->precision == DSLASH_F64 && h->recon != 9 &&
-           rhs8_tma_variant() >= 0 && K.nbox == 1 && K.box[0].n[0] == K.L[0] && K.box[0].n[1] == K.L[1] &&
-           K.box[0].n[2] == K.L[2] && sites % 16 == 0;
-}
-
-static dslash_status launch_rhs8_tma(dslash_t h, const StencilParams& K, int kind, cudaStream_t s, int64_t sites) {
-    size_t smem = 0;
-    StencilFn fn = h->recon == 12 ? pick_f64_r12_rhs8_tma(rhs8_tma_variant(), &smem)
-                                  : pick_f64_r18_rhs8_tma(rhs8_tma_variant(), &smem);
-    if (!fn) return fail(h, DSLASH_ERR_UNSUPPORTED, "no TMA-link kernel for this configuration");
-    static std::vector<StencilFn> smem_set;  // opt-in above 48 KB, once per kernel
-    bool done = false;
-    for (StencilFn f : smem_set) done = done || f == fn;
-    if (!done) {
-        CU(h, cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        smem_set.push_back(fn);
-    }
-    const unsigned grid = (unsigned)((sites * 2 + 255) / 256);
-    dslash_s::TimedLaunch* tl = nullptr;
-    dslash_status st = timing_begin(h, kind, s, &tl);
-    if (st != DSLASH_OK) return st;
-    CU(h, launch_pdl(h->pdl, fn, K, grid, 256, smem, s));
-    if (tl) CU(h, cudaEventRecord(tl->b, s));
-    return DSLASH_OK;
-}
-
 static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int kind, cudaStream_t s, int nrhs) {
     const int64_t sites = K.box_start[K.nbox];
     if (sites == 0) return DSLASH_OK;
     const int lanes = lanes_of(h->kernel);
     if (h->stage) return launch_stage(h, K, ghost, kind, s, nrhs, lanes);
-    if (rhs8_tma_ok(h, K, ghost, lanes, nrhs, sites)) return launch_rhs8_tma(h, K, kind, s, sites);
     // recon-9 on the site kernel (its default): 256 / 128 / 64 threads for fp64 / mixed / fp32
     // (profiles/r02/recon9_blocks/: 150.6 vs 152.7 us, 86.9 vs 88.0 us, 75.9 vs 77.3 us)
     const int r9_block = h->precision == DSLASH_F64 ? 256 : h->precision == DSLASH_MIXED ? 128 : 64;

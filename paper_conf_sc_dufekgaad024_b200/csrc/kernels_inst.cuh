@@ -8,7 +8,6 @@
 
 #include "dispatch.h"
 #include "stencil.cuh"
-#include "stencil_mrhs.cuh"
 
 namespace hisq {
 
@@ -59,23 +58,6 @@ StencilFn pick_stage(bool ghost, int lanes, int nrhs) {
     return ghost ? pick_stage_n<LR, VR, 2, true, RECON>(nrhs) : pick_stage_n<LR, VR, 2, false, RECON>(nrhs);
 }
 
-// the 8-RHS kernel with the link stream on the TMA engine (stencil_mrhs.cuh): fp64 links and
-// vectors, recon 18 / 12; variant = (stages, distance) 0: (4, 2), 1: (4, 3), 2: (3, 2), 3: (6, 4)
-template <typename LR, typename VR, int RECON>
-StencilFn pick_rhs8_tma(int variant, size_t* smem) {
-    if constexpr (sizeof(LR) == 8 && sizeof(VR) == 8 && RECON != 9) {
-        switch (variant) {
-            case 1: *smem = rhs8_tma_smem<4>(); return dslash_rhs8_tma_kernel<RECON, 4, 3>;
-            case 2: *smem = rhs8_tma_smem<3>(); return dslash_rhs8_tma_kernel<RECON, 3, 2>;
-            case 3: *smem = rhs8_tma_smem<6>(); return dslash_rhs8_tma_kernel<RECON, 6, 4>;
-            default: *smem = rhs8_tma_smem<4>(); return dslash_rhs8_tma_kernel<RECON, 4, 2>;
-        }
-    }
-    (void)variant;
-    *smem = 0;
-    return nullptr;
-}
-
 }  // namespace hisq
 
 #define HISQ_DEFINE_PICK(NAME, LR, VR, RECON)                                                                  \
@@ -84,5 +66,4 @@ StencilFn pick_rhs8_tma(int variant, size_t* smem) {
         return pick_any<LR, VR, RECON>(ghost, lanes, minb, nrhs);                                             \
     }                                                                                                         \
     StencilFn NAME##_stage(bool ghost, int lanes, int nrhs) { return pick_stage<LR, VR, RECON>(ghost, lanes, nrhs); } \
-    StencilFn NAME##_rhs8_tma(int variant, size_t* smem) { return pick_rhs8_tma<LR, VR, RECON>(variant, smem); }       \
     }
