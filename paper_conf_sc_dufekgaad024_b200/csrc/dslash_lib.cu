@@ -274,12 +274,12 @@ extern "C" dslash_status dslash_create(const int32_t G[4], const int32_t P[4], i
         fail(h, DSLASH_ERR_CUDA, "cudaGetDevice: %s", cudaGetErrorString(e));
         return bail(DSLASH_ERR_CUDA);
     }
-    // the exchange and the boundary kernel get the greatest stream priority: their blocks are
-    // dispatched ahead of the interior kernel's pending blocks once their inputs are ready
+    // the exchange and the boundary kernel (queued behind it on the same stream) get the greatest
+    // stream priority: their blocks are dispatched ahead of the interior kernel's pending blocks
+    // once their inputs are ready
     int prio_lo = 0, prio_hi = 0;
     cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
     if ((e = cudaStreamCreateWithPriority(&h->comm, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
-        (e = cudaStreamCreateWithPriority(&h->bstream, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
         (e = cudaEventCreateWithFlags(&h->ev_bdone, cudaEventDisableTiming)) != cudaSuccess ||
         (e = cudaEventCreateWithFlags(&h->ev_start, cudaEventDisableTiming)) != cudaSuccess ||
         (e = cudaEventCreateWithFlags(&h->ev_halo, cudaEventDisableTiming)) != cudaSuccess) {
@@ -1697,8 +1697,8 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
     // one launch on the caller's stream after it, no boundary stream and join (measured equal,
     // 153.7 vs 153.8 us per apply at 48^3 x 6 with a t self-halo)
     if (h->overlap == DSLASH_OVERLAP_SITES && p.interior_sites > 0) {
-        // interior on the caller's stream; boundary on the handle's boundary stream as soon as the
-        // halo lands, so it fills the SMs the interior kernel's tail leaves idle; then the caller's
+        // interior on the caller's stream; boundary on the exchange stream as soon as the halo
+        // lands, so it fills the SMs the interior kernel's tail leaves idle; then the caller's
         // stream joins (the two kernels write disjoint sites of out)
         // span of the two overlapping kernels (DSLASH_TIMING_SPAN): interior start -> join
         // (an index, not a pointer: the launches below may grow tpool)
@@ -1714,14 +1714,19 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
             h->tpool[span].kind = DSLASH_TIMING_SPAN;
             CU(h, cudaEventRecord(h->tpool[span].a, s));
         }
+        // the boundary kernel is queued on the exchange's own (high-priority) stream right behind
+        // the exchange: no cross-stream wait between the faces and the kernel that reads them
+        // (round 3, profiles/r03/halo/: t 185.2 -> 182.9 us, t + z 186.7 -> 185.0 us per apply
+        // against 178.9 us without a halo, vs a separate boundary stream)
+        cudaStream_t bs = h->comm;
         st = launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
         if (st != DSLASH_OK) return st;
-        if ((st = dslash_halo_wait(h, (dslash_stream_t)h->bstream)) != DSLASH_OK) return st;
-        if (push_out && (st = push_wait_free(h, h->bstream)) != DSLASH_OK) return st;
-        st = launch_rhs(h, Kp, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, h->bstream, nrhs);
+        if ((st = dslash_halo_wait(h, (dslash_stream_t)bs)) != DSLASH_OK) return st;
+        if (push_out && (st = push_wait_free(h, bs)) != DSLASH_OK) return st;
+        st = launch_rhs(h, Kp, p.boundary, p.n_boundary, true, DSLASH_TIMING_BOUNDARY, bs, nrhs);
         if (st != DSLASH_OK) return st;
-        if (push_out && (st = push_signal(h, h->bstream, out, nrhs)) != DSLASH_OK) return st;
-        CU(h, cudaEventRecord(h->ev_bdone, h->bstream));
+        if (push_out && (st = push_signal(h, bs, out, nrhs)) != DSLASH_OK) return st;
+        CU(h, cudaEventRecord(h->ev_bdone, bs));
         CU(h, cudaStreamWaitEvent(s, h->ev_bdone, 0));
         if (span != (size_t)-1) CU(h, cudaEventRecord(h->tpool[span].b, s));
         return DSLASH_OK;
@@ -1947,7 +1952,6 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
     if (h->ev_start) cudaEventDestroy(h->ev_start);
     if (h->ev_halo) cudaEventDestroy(h->ev_halo);
     if (h->comm) cudaStreamDestroy(h->comm);
-    if (h->bstream) cudaStreamDestroy(h->bstream);
     if (h->ev_bdone) cudaEventDestroy(h->ev_bdone);
     delete h;
     return DSLASH_OK;

@@ -50,7 +50,6 @@ struct dslash_s {
     cudaEvent_t ev_in_ready[kSlots] = {}, ev_in_free[kSlots] = {}, ev_out_ready[kSlots] = {},
                 ev_out_free[kSlots] = {}, ev_batch = nullptr;
     cudaStream_t comm = nullptr;
-    cudaStream_t bstream = nullptr;  // boundary kernels (overlap the interior kernel's tail)
     cudaEvent_t ev_start = nullptr, ev_halo = nullptr, ev_bdone = nullptr;
     bool halo_pending = false;
     ncclComm_t nccl = nullptr;
