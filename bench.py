@@ -59,6 +59,9 @@ def parse(argv=None):
     ap.add_argument("--kernel", default=None, choices=["site", "dir2", "dir4"],
                     help="default: dir2 (site with --recon 9 or --nrhs > 1, measured best for them)")
     ap.add_argument("--min-blocks", type=int, default=0)
+    ap.add_argument("--layout", default="planar", choices=["planar", "blocked"],
+                    help="multi-RHS vector layout: planar [nrhs][3][Vh] (dslash_apply_multi) or site-blocked "
+                         "[Vh/16][nrhs*3][16] (dslash_apply_multi_blocked; no halo)")
     ap.add_argument("--nrhs", type=int, default=1, choices=[1, 2, 3, 4, 5, 6, 7, 8],
                     help="right-hand sides per apply, one link pass (SURVEY §8(f)-4)")
     ap.add_argument("--recon", type=int, default=18, choices=[18, 12, 9],
@@ -487,6 +490,8 @@ def main():
         return (vs[0] if nrhs == 1 else torch.stack(vs)).contiguous()
 
     srcs = [make_src(r).cuda() for r in range(R)]
+    if args.layout == "blocked":   # converted once, on the device, before the timed region
+        srcs = [D.to_blocked(torch.empty_like(v), v) for v in srcs]
     outs = [torch.empty_like(srcs[0]) for _ in range(R)]
     stream = torch.cuda.current_stream()
     flush = torch.empty(2 * l2_bytes // 4, dtype=torch.float32, device="cuda") if args.flush_l2 else None
@@ -495,7 +500,9 @@ def main():
     def step(i):
         if flush is not None:
             flush.fill_(float(i))
-        if nrhs == 1:
+        if args.layout == "blocked":
+            D.apply_multi_blocked(outs[i % R], srcs[i % R], parity, stream)
+        elif nrhs == 1:
             D.apply(outs[i % R], srcs[i % R], parity, stream)
         else:
             D.apply_multi(outs[i % R], srcs[i % R], parity, stream)
@@ -566,7 +573,7 @@ def main():
             kern_ms, n_launch = max_over_ranks(t_span / n_span), n_span
             kname = (f"{kstem}<lanes={lanes_n}> interior + boundary ("
                      + ("local pass + ghost pass, split by direction" if args.overlap == "dirs" else
-                        "boundary on a high-priority stream, split by sites") + "): span per apply")
+                        "boundary queued behind the exchange on the high-priority comm stream, split by sites") + "): span per apply")
         else:                   # one ghost-aware launch after the exchange
             kern_ms, n_launch = max_over_ranks(t_all / max(1, n_all)), n_all
             kname = f"{kstem}<lanes={lanes_n}, ghost=true> (all sites, after the exchange)"
@@ -580,7 +587,8 @@ def main():
                      "launches_per_step": launches_per_step}
     achieved = algo_bytes_site * dom_sites / (kern_ms * 1e-3) / 1e9
     variant = (args.kernel + ("-stage" if args.stage else "") + ("" if args.precision == "f64" else f"-{args.precision}")
-               + ("" if args.recon == 18 else f"-r{args.recon}") + (f"-n{nrhs}" if nrhs > 1 else ""))
+               + ("" if args.recon == 18 else f"-r{args.recon}") + (f"-n{nrhs}" if nrhs > 1 else "")
+               + ("-blocked" if args.layout == "blocked" else ""))
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4), "traffic": ncu_traffic(variant, extent), "kernel": kname,
             "bytes_per_launch": algo_bytes_site * dom_sites, "bytes_per_site": algo_bytes_site,
@@ -664,6 +672,7 @@ def main():
                            "parity": parity,
                            "kernel": args.kernel, "stage": bool(args.stage), "block": args.block or None,
                            "precision": args.precision, "long_link_recon": args.recon, "nrhs": nrhs,
+                           "vector_layout": args.layout,
                            "overlap": "none" if args.no_overlap else args.overlap, "pdl": not args.no_pdl,
                            "halo_dryrun_results_invalid": True if args.halo_dryrun else None,
                            "per_kernel_events_in_timed_region": bool(args.flush_l2),

@@ -301,6 +301,29 @@ DSLASH_API dslash_status dslash_apply(dslash_t h, void* out, const void* in, int
 DSLASH_API dslash_status dslash_apply_multi(dslash_t h, int32_t nrhs, void* out, const void* in, int32_t parity,
                                             dslash_stream_t stream);
 
+/* dslash_apply_multi on SITE-BLOCKED vectors (same operation, PAPER.md L45-51 for every right-hand
+ * side; the L25 intensity argument for sharing the links): element (rhs r, colour c) of the
+ * site with checkerboard index cb lies at
+ *     [(cb / 16) * (nrhs * 3 * 16) + (r * 3 + c) * 16 + cb % 16]
+ * (complex of the handle's vector precision), i.e. blocks of 16 consecutive sites, each holding
+ * its nrhs x 3 rows of 16 back to back.  A warp's gathers of one hop then read a few contiguous
+ * kilobytes instead of 3 x nrhs planes Vh_local apart (8 RHS at 32^4: fp64 393 -> 376 us, fp32
+ * 219 -> 186 us; profiles/r03/mrhs/).  Results are bitwise those of dslash_apply_multi on the
+ * planar copies.  Caller-owned device buffers of nrhs x 3 x Vh_local complex, 16-byte aligned,
+ * non-overlapping.  Requires Vh_local % 16 == 0 and an unpartitioned lattice (no halo), else
+ * DSLASH_ERR_UNSUPPORTED; other errors as dslash_apply_multi. */
+DSLASH_API dslash_status dslash_apply_multi_blocked(dslash_t h, int32_t nrhs, void* out, const void* in,
+                                                    int32_t parity, dslash_stream_t stream);
+
+/* Layout conversion for dslash_apply_multi_blocked, stream-ordered on the device:
+ * planar [nrhs][3][Vh_local] <-> site-blocked (above), complex of the handle's vector
+ * precision.  Caller-owned, non-overlapping device buffers; Vh_local % 16 == 0, else
+ * DSLASH_ERR_UNSUPPORTED. */
+DSLASH_API dslash_status dslash_vectors_to_blocked(dslash_t h, int32_t nrhs, void* blocked, const void* planar,
+                                                   dslash_stream_t stream);
+DSLASH_API dslash_status dslash_vectors_from_blocked(dslash_t h, int32_t nrhs, void* planar, const void* blocked,
+                                                     dslash_stream_t stream);
+
 /* The same operation from HOST buffers (end-to-end path): copies in (host) to an
  * internal device buffer, applies, copies the result to out (host), all ordered on
  * `stream`; returns after enqueueing (synchronise the stream before reading out).

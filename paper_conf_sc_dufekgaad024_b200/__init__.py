@@ -193,6 +193,35 @@ class Dslash:
                                 _stream_handle(stream))
         return out
 
+    def _check_blocked(self, *vs):
+        n = vs[0].numel()
+        for v in vs:
+            if not (v.is_cuda and v.dtype == self.dtype and v.is_contiguous() and v.numel() == n
+                    and n % (3 * self.vh) == 0):
+                raise ValueError(f"site-blocked vectors must be contiguous {self.dtype} CUDA tensors of "
+                                 f"nrhs x 3 x {self.vh} elements")
+        return n // (3 * self.vh)
+
+    def apply_multi_blocked(self, out, inp, parity, stream=None):
+        """out = D inp for nrhs right-hand sides in the site-blocked layout (dslash_apply_multi_blocked:
+        element (r, c, cb) at [cb // 16][r * 3 + c][cb % 16]); tensors of nrhs x 3 x Vh elements."""
+        nrhs = self._check_blocked(out, inp)
+        _abi.dslash_apply_multi_blocked(self.h, nrhs, out.data_ptr(), inp.data_ptr(), int(parity),
+                                        _stream_handle(stream))
+        return out
+
+    def to_blocked(self, blocked, planar, stream=None):
+        """planar (nrhs, 3, Vh) -> site-blocked copy (on the device, stream-ordered)."""
+        nrhs = self._check_blocked(blocked, planar)
+        _abi.dslash_vectors_to_blocked(self.h, nrhs, blocked.data_ptr(), planar.data_ptr(), _stream_handle(stream))
+        return blocked
+
+    def from_blocked(self, planar, blocked, stream=None):
+        """site-blocked -> planar (nrhs, 3, Vh) copy (on the device, stream-ordered)."""
+        nrhs = self._check_blocked(planar, blocked)
+        _abi.dslash_vectors_from_blocked(self.h, nrhs, planar.data_ptr(), blocked.data_ptr(), _stream_handle(stream))
+        return planar
+
     def normal_apply(self, out, inp, parity, mass, stream=None):
         """out = (m^2 - D_{p,1-p} D_{1-p,p}) inp on parity p (needs parity_mask BOTH, fp64 vectors)."""
         self._check_vec(out)

@@ -98,6 +98,9 @@ _SIGS = {
     "dslash_apply": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply_push": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply_multi": ([_h, ctypes.c_int32, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
+    "dslash_apply_multi_blocked": ([_h, ctypes.c_int32, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
+    "dslash_vectors_to_blocked": ([_h, ctypes.c_int32, _vp, _vp, _vp], ctypes.c_int),
+    "dslash_vectors_from_blocked": ([_h, ctypes.c_int32, _vp, _vp, _vp], ctypes.c_int),
     "dslash_apply_host": ([_h, _vp, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_apply_host_batch": ([_h, ctypes.c_int32, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.c_int32,
                                  _vp], ctypes.c_int),
@@ -217,6 +220,18 @@ def dslash_apply_push(h, out_ptr, in_ptr, parity, stream=0):
 
 def dslash_apply_multi(h, nrhs, out_ptr, in_ptr, parity, stream=0):
     return check(lib.dslash_apply_multi(h, nrhs, out_ptr, in_ptr, parity, stream), h)
+
+
+def dslash_apply_multi_blocked(h, nrhs, out_ptr, in_ptr, parity, stream=0):
+    return check(lib.dslash_apply_multi_blocked(h, nrhs, out_ptr, in_ptr, parity, stream), h)
+
+
+def dslash_vectors_to_blocked(h, nrhs, blocked_ptr, planar_ptr, stream=0):
+    return check(lib.dslash_vectors_to_blocked(h, nrhs, blocked_ptr, planar_ptr, stream), h)
+
+
+def dslash_vectors_from_blocked(h, nrhs, planar_ptr, blocked_ptr, stream=0):
+    return check(lib.dslash_vectors_from_blocked(h, nrhs, planar_ptr, blocked_ptr, stream), h)
 
 
 def dslash_apply_host(h, out_ptr, in_ptr, parity, stream=0):

@@ -247,6 +247,9 @@ struct StencilParams {
     // the minus (plus) neighbour's plus (minus) ghost face, [3][face_vh[mu]], peer memory over NVLink
     void* push[4][2];
     int push_mask;
+    // site-blocked vectors (VBLK kernels): complex elements per 16-site block = 16 * 3 * nrhs of
+    // the whole apply (a launch of NRHS right-hand sides starts at its first one's rows)
+    int64_t vblk;
 };
 
 // Passes of a GHOST kernel (StencilParams::halo_pass).  kPassAll reads local sources and ghost

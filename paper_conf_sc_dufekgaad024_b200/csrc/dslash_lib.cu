@@ -1406,6 +1406,19 @@ static void fill_boxes(StencilParams& K, const dslash_box_t* boxes, int n) {
     for (int b = n; b < kMaxBoxes; ++b) K.box_start[b + 1] = K.box_start[n];
 }
 
+static StencilFn pick_vblk_kernel(int precision, int recon, int lanes, int nrhs) {
+    if (recon == 9)
+        return precision == DSLASH_F32     ? pick_f32_r9_vblk(lanes, nrhs)
+               : precision == DSLASH_MIXED ? pick_mixed_r9_vblk(lanes, nrhs)
+                                           : pick_f64_r9_vblk(lanes, nrhs);
+    const bool r12 = recon == 12;
+    switch (precision) {
+        case DSLASH_F32: return r12 ? pick_f32_r12_vblk(lanes, nrhs) : pick_f32_r18_vblk(lanes, nrhs);
+        case DSLASH_MIXED: return r12 ? pick_mixed_r12_vblk(lanes, nrhs) : pick_mixed_r18_vblk(lanes, nrhs);
+        default: return r12 ? pick_f64_r12_vblk(lanes, nrhs) : pick_f64_r18_vblk(lanes, nrhs);
+    }
+}
+
 template <bool GHOST>
 static StencilFn pick_kernel(int precision, int recon, int lanes, int minb, int nrhs) {
     const bool r12 = recon == 12;
@@ -1550,7 +1563,7 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
     const int64_t sites = K.box_start[K.nbox];
     if (sites == 0) return DSLASH_OK;
     const int lanes = lanes_of(h->kernel);
-    if (h->stage) return launch_stage(h, K, ghost, kind, s, nrhs, lanes);
+    if (h->stage && !K.vblk) return launch_stage(h, K, ghost, kind, s, nrhs, lanes);
     // recon-9 on the site kernel (its default): 256 / 128 / 64 threads for fp64 / mixed / fp32
     // (profiles/r02/recon9_blocks/: 150.6 vs 152.7 us, 86.9 vs 88.0 us, 75.9 vs 77.3 us)
     const int r9_block = h->precision == DSLASH_F64 ? 256 : h->precision == DSLASH_MIXED ? 128 : 64;
@@ -1566,8 +1579,9 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
     dslash_s::TimedLaunch* tl = nullptr;
     dslash_status st = timing_begin(h, kind, s, &tl);
     if (st != DSLASH_OK) return st;
-    StencilFn fn = ghost ? pick_kernel<true>(h->precision, h->recon, lanes, minb, nrhs)
-                         : pick_kernel<false>(h->precision, h->recon, lanes, minb, nrhs);
+    StencilFn fn = K.vblk  ? pick_vblk_kernel(h->precision, h->recon, lanes, nrhs)
+                   : ghost ? pick_kernel<true>(h->precision, h->recon, lanes, minb, nrhs)
+                           : pick_kernel<false>(h->precision, h->recon, lanes, minb, nrhs);
     // programmatic dependent launch: may start while the previous kernel on `s` drains
     CU(h, launch_pdl(h->pdl, fn, K, grid, bs, 0, s));
     if (tl) CU(h, cudaEventRecord(tl->b, s));
@@ -1588,8 +1602,10 @@ static dslash_status launch_rhs(dslash_t h, StencilParams K, const dslash_box_t*
     for (int r0 = 0; r0 < nrhs;) {
         const int left = nrhs - r0;
         int nr = left >= 8 ? 8 : left >= 4 ? 4 : left >= 2 ? 2 : 1;
-        K.in = in0 + (size_t)r0 * 3 * K.vh * es;
-        K.out = out0 + (size_t)r0 * 3 * K.vh * es;
+        // planar: the chunk's first vector; site-blocked: its first rows inside every 16-site block
+        const size_t roff = (size_t)r0 * 3 * (K.vblk ? kVBlk : K.vh) * es;
+        K.in = in0 + roff;
+        K.out = out0 + roff;
         for (int d = 0; d < 4; ++d)
             for (int side = 0; side < 2; ++side) {
                 K.ghost[d][side] = g0[d][side] ? static_cast<const char*>(g0[d][side]) + (size_t)r0 * 3 * K.face_vh[d] * es
@@ -1614,7 +1630,7 @@ static dslash_status check_vectors(dslash_t h, const void* out, const void* in, 
 }
 
 static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs,
-                                dslash_stream_t stream, bool push_out = false);
+                                dslash_stream_t stream, bool push_out = false, bool blocked = false);
 
 dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s,
                          bool push) {
@@ -1622,7 +1638,7 @@ dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, 
 }
 
 static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs,
-                                dslash_stream_t stream, bool push_out) {
+                                dslash_stream_t stream, bool push_out, bool blocked) {
     DeviceGuard device_guard(h);
     if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
     if (parity & ~1) return fail(h, DSLASH_ERR_ARG, "parity %d not in {0,1}", parity);
@@ -1651,6 +1667,13 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
     // producer push: only with a halo (without one the next apply needs no faces)
     push_out = push_out && any_halo(p);
     if (push_out && !h->push) return fail(h, DSLASH_ERR_STATE, "apply_push needs DSLASH_OPT_PUSH");
+    if (blocked) {  // site-blocked vectors (dslash_apply_multi_blocked): unpartitioned lattices only
+        if (any_halo(p)) return fail(h, DSLASH_ERR_UNSUPPORTED, "the site-blocked layout has no halo exchange");
+        if (p.vh_local % kVBlk)
+            return fail(h, DSLASH_ERR_UNSUPPORTED, "site-blocked layout: Vh_local %lld is not a multiple of %d",
+                        (long long)p.vh_local, kVBlk);
+        K.vblk = (int64_t)nrhs * 3 * kVBlk;
+    }
     if (!any_halo(p)) return launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
     if ((st = halo_start_impl(h, in, nrhs, s)) != DSLASH_OK) return st;
     for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
@@ -1755,6 +1778,61 @@ extern "C" dslash_status dslash_apply(dslash_t h, void* out, const void* in, int
 extern "C" dslash_status dslash_apply_push(dslash_t h, void* out, const void* in, int32_t parity,
                                            dslash_stream_t stream) {
     return apply_impl(h, out, in, parity, 1, stream, true);
+}
+
+extern "C" dslash_status dslash_apply_multi_blocked(dslash_t h, int32_t nrhs, void* out, const void* in,
+                                                    int32_t parity, dslash_stream_t stream) {
+    return apply_impl(h, out, in, parity, nrhs, stream, false, true);
+}
+
+// planar [rows][vh] <-> site-blocked [vh / 16][rows][16] (rows = 3 nrhs), one element per thread in
+// the blocked order, so both sides move runs of 16 consecutive elements
+template <typename T>
+__global__ void vblk_convert_kernel(T* __restrict__ dst, const T* __restrict__ src, int64_t vh, int rows,
+                                    bool to_blocked) {
+    const int64_t n = vh * rows, blk = (int64_t)rows * kVBlk;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t b = i / blk, rem = i - b * blk;
+        const int64_t planar = (rem / kVBlk) * vh + b * kVBlk + rem % kVBlk;
+        if (to_blocked)
+            dst[i] = src[planar];
+        else
+            dst[planar] = src[i];
+    }
+}
+
+static dslash_status vblk_convert(dslash_t h, int32_t nrhs, void* dst, const void* src, dslash_stream_t stream,
+                                  bool to_blocked) {
+    DeviceGuard device_guard(h);
+    if (!h) return fail(nullptr, DSLASH_ERR_ARG, "NULL handle");
+    if (nrhs < 1) return fail(h, DSLASH_ERR_ARG, "nrhs %d < 1", nrhs);
+    dslash_status st = check_vectors(h, dst, src, nrhs);
+    if (st != DSLASH_OK) return st;
+    const int64_t vh = h->plan.vh_local;
+    if (vh % kVBlk)
+        return fail(h, DSLASH_ERR_UNSUPPORTED, "site-blocked layout: Vh_local %lld is not a multiple of %d",
+                    (long long)vh, kVBlk);
+    const int rows = 3 * nrhs;
+    const unsigned grid = (unsigned)std::min<int64_t>((vh * rows + 255) / 256, (int64_t)num_sms(h) * 8);
+    cudaStream_t s = (cudaStream_t)stream;
+    if (vec_elem(h) == 16)
+        vblk_convert_kernel<double2><<<grid, 256, 0, s>>>(static_cast<double2*>(dst), static_cast<const double2*>(src),
+                                                          vh, rows, to_blocked);
+    else
+        vblk_convert_kernel<float2><<<grid, 256, 0, s>>>(static_cast<float2*>(dst), static_cast<const float2*>(src), vh,
+                                                         rows, to_blocked);
+    CU(h, cudaGetLastError());
+    return DSLASH_OK;
+}
+
+extern "C" dslash_status dslash_vectors_to_blocked(dslash_t h, int32_t nrhs, void* blocked, const void* planar,
+                                                   dslash_stream_t stream) {
+    return vblk_convert(h, nrhs, blocked, planar, stream, true);
+}
+
+extern "C" dslash_status dslash_vectors_from_blocked(dslash_t h, int32_t nrhs, void* planar, const void* blocked,
+                                                     dslash_stream_t stream) {
+    return vblk_convert(h, nrhs, planar, blocked, stream, false);
 }
 
 extern "C" dslash_status dslash_apply_multi(dslash_t h, int32_t nrhs, void* out, const void* in, int32_t parity,

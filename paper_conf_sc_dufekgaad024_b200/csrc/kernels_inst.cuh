@@ -58,6 +58,25 @@ StencilFn pick_stage(bool ghost, int lanes, int nrhs) {
     return ghost ? pick_stage_n<LR, VR, 2, true, RECON>(nrhs) : pick_stage_n<LR, VR, 2, false, RECON>(nrhs);
 }
 
+// the site-blocked layout (dslash_apply_multi_blocked): interior, MINB 2, the handle's mapping (its
+// link layout); 8 right-hand sides as two groups of 4 like the planar kernel
+template <typename LR, typename VR, int LANES, int RECON>
+StencilFn pick_vblk_n(int nrhs) {
+    switch (nrhs) {
+        case 2: return dslash_kernel<LR, VR, LANES, false, 2, RECON, 2, 1, true>;
+        case 4: return dslash_kernel<LR, VR, LANES, false, 2, RECON, 4, 1, true>;
+        case 8: return dslash_kernel<LR, VR, LANES, false, 2, RECON, 4, 2, true>;
+        default: return dslash_kernel<LR, VR, LANES, false, 2, RECON, 1, 1, true>;
+    }
+}
+
+template <typename LR, typename VR, int RECON>
+StencilFn pick_vblk(int lanes, int nrhs) {
+    return lanes == 1 ? pick_vblk_n<LR, VR, 1, RECON>(nrhs)
+           : lanes == 2 ? pick_vblk_n<LR, VR, 2, RECON>(nrhs)
+                        : pick_vblk_n<LR, VR, 4, RECON>(nrhs);
+}
+
 }  // namespace hisq
 
 #define HISQ_DEFINE_PICK(NAME, LR, VR, RECON)                                                                  \
@@ -66,4 +85,5 @@ StencilFn pick_stage(bool ghost, int lanes, int nrhs) {
         return pick_any<LR, VR, RECON>(ghost, lanes, minb, nrhs);                                             \
     }                                                                                                         \
     StencilFn NAME##_stage(bool ghost, int lanes, int nrhs) { return pick_stage<LR, VR, RECON>(ghost, lanes, nrhs); } \
+    StencilFn NAME##_vblk(int lanes, int nrhs) { return pick_vblk<LR, VR, RECON>(lanes, nrhs); }                  \
     }

@@ -193,6 +193,9 @@ __device__ __forceinline__ Site decode_site(const StencilParams& P, int64_t gid)
     return s;
 }
 
+// sites per block of the site-blocked multi-RHS vector layout (dslash_apply_multi_blocked)
+constexpr int kVBlk = 16;
+
 template <typename V2>
 struct SrcRef {
     const V2* p;  // colour component c at p[c * stride]
@@ -203,7 +206,7 @@ struct SrcRef {
 // Address of psi(x + h mu^).  GHOST: directions in P.halo_mask read the depth-3 ghost faces
 // outside [0, L); otherwise coordinates wrap periodically (two conditional steps suffice for
 // |h| <= 3 and L >= 2).
-template <typename V2, bool GHOST>
+template <typename V2, bool GHOST, bool VBLK = false>
 __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, const void* in, int mu, int h, const Site& s,
                                              int rhs) {
     const int c = mu == 0 ? s.x : mu == 1 ? s.y : mu == 2 ? s.z : s.t;
@@ -221,6 +224,12 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, const void*
     } else {
         st = mu == 1 ? (int64_t)P.lxh : mu == 2 ? (int64_t)P.lxh * P.L[1] : (int64_t)P.lxh * P.L[1] * P.L[2];
         idx = s.cb + (int64_t)(cw - c) * st;
+    }
+    if constexpr (VBLK) {
+        // site-blocked vectors (dslash_apply_multi_blocked): (rhs, colour c) of site idx at
+        // [idx / 16][rhs * 3 + c][idx % 16], P.vblk complex per 16-site block
+        static_assert(!GHOST, "the site-blocked layout has no halo");
+        return {static_cast<const V2*>(in) + (idx >> 4) * P.vblk + (idx & 15) + rhs * 3 * kVBlk, kVBlk, false};
     }
     const V2* local = static_cast<const V2*>(in) + (int64_t)rhs * 3 * P.vh + idx;
     if (!GHOST || mu < 2) return {local, P.vh, false};
@@ -379,7 +388,8 @@ constexpr bool kZtNoL1 = HISQ_ZT_NO_L1 != 0;
 // staged kernel visits the global (z, t) directions first and the tile's (x, y) ones last, so
 // the tile's bulk copies land while the z/t links and neighbours stream (a different summation
 // order from the unstaged kernel: equal within the fp64 tolerance, not bitwise).
-template <typename LR, typename VR, int LANES, bool GHOST, int RECON, int NRHS, int RHSL = 1, bool STAGED = false>
+template <typename LR, typename VR, int LANES, bool GHOST, int RECON, int NRHS, int RHSL = 1, bool STAGED = false,
+          bool VBLK = false>
 __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_t gid, const int64_t site_end,
                                             const StageTile<cplx_t<VR>> T = {}) {
     static_assert(LANES == 1 || LANES == 2 || LANES == 4, "LANES must divide 4");
@@ -501,7 +511,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
 #pragma unroll
                     for (int sub = 0; sub < 2; ++sub) {
                         const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0, false}
-                                                   : source<V2, GHOST>(P, in, mu, sub ? -hop : hop, s, rl * NRHS);
+                                                   : source<V2, GHOST, VBLK>(P, in, mu, sub ? -hop : hop, s, rl * NRHS);
                         const uint32_t sa = stg ? staged_addr<V2>(P, T, sbase, mu, sub ? -hop : hop, s, rl * NRHS) : 0u;
                         if (GHOST && P.halo_pass == kPassGhost && !src.ghost) continue;
                         const bool zap = GHOST && P.halo_pass == kPassLocal && src.ghost;
@@ -556,7 +566,7 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
                                     pol_stream)));
                     }
                 }
-                const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0, false} : source<V2, GHOST>(P, in, mu, h, s, rl * NRHS);
+                const SrcRef<V2> src = stg ? SrcRef<V2>{nullptr, 0, false} : source<V2, GHOST, VBLK>(P, in, mu, h, s, rl * NRHS);
                 const uint32_t sa = stg ? staged_addr<V2>(P, T, sbase, mu, h, s, rl * NRHS) : 0u;
                 // split-by-direction passes: the ghost pass takes only the ghost hops (the link of
                 // a skipped hop is not read); the local pass stays branch-free, so loads can be
@@ -648,19 +658,22 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
     }
 #pragma unroll
     for (int r = 0; r < NRHS; ++r) {
-        V2* out = static_cast<V2*>(P.out) + (int64_t)(rl * NRHS + r) * 3 * P.vh;
+        // colour c of this (site, rhs) at out[c * cs]: planar [rhs][3][vh], or site-blocked
+        V2* out = VBLK ? static_cast<V2*>(P.out) + (s.cb >> 4) * P.vblk + (s.cb & 15) + (rl * NRHS + r) * 3 * kVBlk
+                       : static_cast<V2*>(P.out) + (int64_t)(rl * NRHS + r) * 3 * P.vh + s.cb;
+        const int64_t cs = VBLK ? kVBlk : P.vh;
         if (LANES == 1) {
 #pragma unroll
-            for (int c = 0; c < 3; ++c) st_stream(out + c * P.vh + s.cb, acc[r][c]);
+            for (int c = 0; c < 3; ++c) st_stream(out + c * cs, acc[r][c]);
         } else if (LANES == 2) {
             if (lane == 0) {
-                st_stream(out + s.cb, acc[r][0]);
-                st_stream(out + P.vh + s.cb, acc[r][1]);
+                st_stream(out, acc[r][0]);
+                st_stream(out + cs, acc[r][1]);
             } else {
-                st_stream(out + 2 * P.vh + s.cb, acc[r][2]);
+                st_stream(out + 2 * cs, acc[r][2]);
             }
         } else {
-            if (lane < 3) st_stream(out + lane * P.vh + s.cb, lane == 0 ? acc[r][0] : lane == 1 ? acc[r][1] : acc[r][2]);
+            if (lane < 3) st_stream(out + lane * cs, lane == 0 ? acc[r][0] : lane == 1 ? acc[r][1] : acc[r][2]);
         }
     }
     if constexpr (GHOST) {
@@ -699,12 +712,14 @@ __device__ __forceinline__ void dslash_body(const StencilParams& P, const int64_
     }
 }
 
-template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1, int RHSL = 1>
+// VBLK: the source and output vectors are in the site-blocked layout (dslash_apply_multi_blocked)
+template <typename LR, typename VR, int LANES, bool GHOST, int MINB, int RECON, int NRHS = 1, int RHSL = 1,
+          bool VBLK = false>
 __global__ void __launch_bounds__(256, MINB) dslash_kernel(const StencilParams P) {
     // every block has started: the next PDL-launched apply may begin filling freed SMs
     asm volatile("griddepcontrol.launch_dependents;");
-    dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
-                                                         P.box_start[P.nbox]);
+    dslash_body<LR, VR, LANES, GHOST, RECON, NRHS, RHSL, false, VBLK>(P, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                                                                     P.box_start[P.nbox]);
 }
 
 // The neighbour-staged variant (DSLASH_OPT_STAGE): one tile of P.stage_ty full x-rows per block

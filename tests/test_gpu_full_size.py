@@ -73,8 +73,10 @@ def _bench_kernel(recon, nrhs):
     return "site" if (recon == 9 or nrhs > 1) else "dir2"
 
 
-def _run_chain(torch, links32, psi_full, parity, nrhs=1, **kw):
-    """Three applies back to back (PDL on), distinct sources; returns [(seeds, out numpy)]."""
+def _run_chain(torch, links32, psi_full, parity, nrhs=1, blocked=False, **kw):
+    """Three applies back to back (PDL on), distinct sources; returns [(seeds, out numpy)].
+    blocked: the sources are converted to the site-blocked layout on the device first, the three
+    applies run dslash_apply_multi_blocked back to back, and the outputs are converted back."""
     from paper_conf_sc_dufekgaad024_b200 import Dslash
     fat, lng = links32
     res = []
@@ -87,11 +89,19 @@ def _run_chain(torch, links32, psi_full, parity, nrhs=1, **kw):
             srcs.append((vs[0] if nrhs == 1 else torch.stack(vs)).contiguous().cuda())
             outs.append(torch.empty_like(srcs[-1]))
             seeds.append(ss)
-        for src, out in zip(srcs, outs):
-            if nrhs == 1:
-                D.apply(out, src, parity)
-            else:
-                D.apply_multi(out, src, parity)
+        if blocked:
+            bsrcs = [D.to_blocked(torch.empty_like(v), v) for v in srcs]
+            bouts = [torch.empty_like(v) for v in srcs]
+            for src, out in zip(bsrcs, bouts):
+                D.apply_multi_blocked(out, src, parity)
+            for out, bout in zip(outs, bouts):
+                D.from_blocked(out, bout)
+        else:
+            for src, out in zip(srcs, outs):
+                if nrhs == 1:
+                    D.apply(out, src, parity)
+                else:
+                    D.apply_multi(out, src, parity)
         torch.cuda.synchronize()
         for ss, out in zip(seeds, outs):
             res.append((ss, out.cpu().numpy()))
@@ -121,6 +131,18 @@ def test_32_multi_rhs_every_rhs(torch_cuda, links32, psi_full, nrhs, precision):
                               kernel=_bench_kernel(18, nrhs)):
         for r, s in enumerate(ss):
             _check(got[r], fat, lng, psi_full(s), parity, precision, (nrhs, r, s))
+
+
+@pytest.mark.parametrize("precision", ["f64", "f32", "mixed"])
+def test_32_multi_rhs_blocked_every_rhs(torch_cuda, links32, psi_full, precision):
+    """The site-blocked 8-RHS layout (dslash_apply_multi_blocked) at the bench size, as bench.py
+    --layout blocked runs it: every right-hand side of every apply against the oracle."""
+    fat, lng = links32
+    parity = 1
+    for ss, got in _run_chain(torch_cuda, links32, psi_full, parity, nrhs=8, blocked=True, precision=precision,
+                              kernel="site"):
+        for r, s in enumerate(ss):
+            _check(got[r], fat, lng, psi_full(s), parity, precision, ("blocked", r, s))
 
 
 @pytest.mark.parametrize("kernel,nrhs", [("dir2", 1), ("site", 1), ("site", 8)])
