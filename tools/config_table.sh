@@ -20,6 +20,10 @@ run --nrhs 2
 run --nrhs 4
 run --nrhs 8
 run --precision f32 --nrhs 8
+run --nrhs 8 --layout blocked
+run --precision f32 --nrhs 8 --layout blocked
+run --precision mixed --nrhs 8 --layout blocked
+run --precision f32 --nrhs 4 --layout blocked
 run --stage
 run --local 48,48,48,48
 run --local 48,48,48,48 --precision f32

@@ -1,0 +1,18 @@
+#!/bin/bash
+# End-of-round evidence on one GPU box (from the repo root): bash tools/gpu_final.sh <name>
+n=${1:-r03_final}
+bash tools/gpu_run.sh $n \
+  "timeout 2400 python -m pytest tests -m gpu -q --timeout 900" \
+  "timeout 300 python -c 'import __graft_entry__ as g; g.smoke()'" \
+  "timeout 300 python bench.py --steps 20 --warmup 5" \
+  "timeout 300 python bench.py --no-cpu-baseline" \
+  "timeout 600 python bench.py --impl reference --steps 20 --warmup 5" \
+  "bash tools/gpu_ncu.sh gpurun_out/$n/ncu_headline" \
+  "bash tools/gpu_ncu.sh gpurun_out/$n/ncu_n8 --nrhs 8" \
+  "bash tools/gpu_ncu.sh gpurun_out/$n/ncu_n8_blocked --nrhs 8 --layout blocked" \
+  "bash tools/gpu_ncu.sh gpurun_out/$n/ncu_n8_f32_blocked --nrhs 8 --layout blocked --precision f32" \
+  "bash tools/gpu_sanitize.sh gpurun_out/$n/sanitize" \
+  "bash tools/config_table.sh" \
+  "bash tools/halo_probe.sh" \
+  "timeout 300 python bench.py --nrhs 8 --layout blocked --precision f32 --no-cpu-baseline" \
+  "timeout 300 python bench.py --nrhs 8 --no-cpu-baseline"

@@ -57,4 +57,16 @@ for kw in cases:
         assert err <= tol, (kw, err)
         assert torch.equal(mo[0], mo[1])
         n += 1
+# round 3: the site-blocked multi-RHS layout (conversion kernels + the VBLK stencil), 8 RHS
+for kw in (dict(kernel="site"), dict(kernel="dir2"), dict(precision="f32", kernel="site"),
+           dict(precision="mixed", kernel="site", recon=12), dict(recon=9, kernel="site")):
+    with Dslash(dims, **kw) as D:
+        D.load_links(fat, lng)
+        multi = torch.stack([src[1] * (k + 1) for k in range(8)]).to(D.dtype).contiguous()
+        planar = D.apply_multi(torch.empty_like(multi), multi, 0)
+        bout = D.apply_multi_blocked(torch.empty_like(multi), D.to_blocked(torch.empty_like(multi), multi), 0)
+        back = D.from_blocked(torch.empty_like(multi), bout)
+        torch.cuda.synchronize()
+        assert torch.equal(back, planar), kw
+        n += 1
 print(f"sanitize_run: {n} configurations OK")
