@@ -310,8 +310,11 @@ DSLASH_API dslash_status dslash_apply_multi(dslash_t h, int32_t nrhs, void* out,
  * kilobytes instead of 3 x nrhs planes Vh_local apart (8 RHS at 32^4: fp64 393 -> 376 us, fp32
  * 219 -> 186 us; profiles/r03/mrhs/).  Results are bitwise those of dslash_apply_multi on the
  * planar copies.  Caller-owned device buffers of nrhs x 3 x Vh_local complex, 16-byte aligned,
- * non-overlapping.  Requires Vh_local % 16 == 0 and an unpartitioned lattice (no halo), else
- * DSLASH_ERR_UNSUPPORTED; other errors as dslash_apply_multi. */
+ * non-overlapping.  Requires Vh_local % 16 == 0.  With a halo (t and/or z partition, or a
+ * forced self-halo) the faces are exchanged as whole blocks, in the same layout: every face must
+ * be whole 16-site blocks (t: 3 Lx/2 Ly Lz; z: 3 Lx/2 Ly and Lx/2 Ly Lz multiples of 16, local
+ * extents), and neither the producer push nor the split-by-direction overlap is available.
+ * Otherwise DSLASH_ERR_UNSUPPORTED; other errors as dslash_apply_multi. */
 DSLASH_API dslash_status dslash_apply_multi_blocked(dslash_t h, int32_t nrhs, void* out, const void* in,
                                                     int32_t parity, dslash_stream_t stream);
 

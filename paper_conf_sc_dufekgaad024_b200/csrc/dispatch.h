@@ -31,16 +31,16 @@ StencilFn pick_f64_r9_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_f32_r9_stage(bool ghost, int lanes, int nrhs);
 StencilFn pick_mixed_r9_stage(bool ghost, int lanes, int nrhs);
 
-// the site-blocked-layout kernel (dslash_apply_multi_blocked) of one (precision, recon): interior,
-// lanes 1/2/4 (the handle's mapping), 1/2/4/8 right-hand sides per launch
-StencilFn pick_f64_r18_vblk(int lanes, int nrhs);
-StencilFn pick_f64_r12_vblk(int lanes, int nrhs);
-StencilFn pick_f32_r18_vblk(int lanes, int nrhs);
-StencilFn pick_f32_r12_vblk(int lanes, int nrhs);
-StencilFn pick_mixed_r18_vblk(int lanes, int nrhs);
-StencilFn pick_mixed_r12_vblk(int lanes, int nrhs);
-StencilFn pick_f64_r9_vblk(int lanes, int nrhs);
-StencilFn pick_f32_r9_vblk(int lanes, int nrhs);
-StencilFn pick_mixed_r9_vblk(int lanes, int nrhs);
+// the site-blocked-layout kernel (dslash_apply_multi_blocked) of one (precision, recon): interior or
+// ghost-aware, lanes 1/2/4 (the handle's mapping), 1/2/4/8 right-hand sides per launch
+StencilFn pick_f64_r18_vblk(bool ghost, int lanes, int nrhs);
+StencilFn pick_f64_r12_vblk(bool ghost, int lanes, int nrhs);
+StencilFn pick_f32_r18_vblk(bool ghost, int lanes, int nrhs);
+StencilFn pick_f32_r12_vblk(bool ghost, int lanes, int nrhs);
+StencilFn pick_mixed_r18_vblk(bool ghost, int lanes, int nrhs);
+StencilFn pick_mixed_r12_vblk(bool ghost, int lanes, int nrhs);
+StencilFn pick_f64_r9_vblk(bool ghost, int lanes, int nrhs);
+StencilFn pick_f32_r9_vblk(bool ghost, int lanes, int nrhs);
+StencilFn pick_mixed_r9_vblk(bool ghost, int lanes, int nrhs);
 
 }  // namespace hisq

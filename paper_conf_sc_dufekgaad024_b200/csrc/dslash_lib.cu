@@ -1149,7 +1149,10 @@ static dslash_status push_signal(dslash_t h, cudaStream_t x, const void* out, in
 //   4. raise their ready flags to e.
 // Consumers wait for their own ready flags (halo_landed).  Every rank releases before it waits, so
 // the ring of waits always resolves.
-static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaStream_t s) {
+// blocked: the sources are site-blocked (dslash_apply_multi_blocked).  Every face is then a
+// run of whole 16-site blocks (checked by the caller), i.e. the same byte ranges as a site-major
+// layout with 3 nrhs elements per site: the copies below take es = 3 nrhs x element and one row.
+static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaStream_t s, bool blocked) {
     const dslash_plan_t& p = h->plan;
     if (nrhs > kP2PMaxRhs)
         return fail(h, DSLASH_ERR_UNSUPPORTED, "P2P transport: at most %d right-hand sides per apply", kP2PMaxRhs);
@@ -1165,12 +1168,12 @@ static dslash_status halo_start_p2p(dslash_t h, const void* in, int nrhs, cudaSt
         return fail(h, DSLASH_ERR_STATE, "the apply after apply_push must take the pushed output as its source");
     h->epoch = e;
     h->pushed_epoch = 0;
-    const size_t es = vec_elem(h);
+    const size_t es = vec_elem(h) * (blocked ? 3 * nrhs : 1);
     const char* src = static_cast<const char*>(in);
     const size_t vh = (size_t)p.vh_local;
     const size_t L1 = p.local_dims[1], L2 = p.local_dims[2], L3 = p.local_dims[3];
     const size_t lxh = p.local_dims[0] / 2;
-    const size_t rows = (size_t)3 * nrhs;
+    const size_t rows = blocked ? 1 : (size_t)3 * nrhs;
     CU(h, cudaEventRecord(h->ev_start, s));
     CU(h, cudaStreamWaitEvent(h->comm, h->ev_start, 0));
     dslash_s::TimedLaunch* xt = nullptr;  // DSLASH_TIMING_EXCHANGE interval on the comm stream
@@ -1269,22 +1272,23 @@ dslash_status hisq_push_discard(dslash_t h, cudaStream_t s) {
 }
 
 // Exchange the depth-3 faces of nrhs source vectors stored back to back ([nrhs][3][vh]).
-static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaStream_t s) {
+static dslash_status halo_start_impl(dslash_t h, const void* in, int nrhs, cudaStream_t s, bool blocked = false) {
     const dslash_plan_t& p = h->plan;
     if (!any_halo(p)) return DSLASH_OK;
-    if (h->transport == DSLASH_TRANSPORT_P2P) return halo_start_p2p(h, in, nrhs, s);
+    if (h->transport == DSLASH_TRANSPORT_P2P) return halo_start_p2p(h, in, nrhs, s, blocked);
     if (nrhs > h->ghost_rhs) {
         CU(h, cudaStreamSynchronize(h->comm));  // old ghosts may still be read by queued kernels
         CU(h, cudaDeviceSynchronize());
         dslash_status st = alloc_halo(h, nrhs);
         if (st != DSLASH_OK) return st;
     }
-    const size_t es = vec_elem(h);
+    // (site-blocked sources: whole 16-site blocks per face, see halo_start_p2p)
+    const size_t es = vec_elem(h) * (blocked ? 3 * nrhs : 1);
     const char* src = static_cast<const char*>(in);
     const size_t vh = (size_t)p.vh_local;
     const size_t L1 = p.local_dims[1], L2 = p.local_dims[2], L3 = p.local_dims[3];
     const size_t lxh = p.local_dims[0] / 2;
-    const size_t rows = (size_t)3 * nrhs;  // (rhs, colour) rows of length vh
+    const size_t rows = blocked ? 1 : (size_t)3 * nrhs;  // (rhs, colour) rows of length vh
     CU(h, cudaEventRecord(h->ev_start, s));
     CU(h, cudaStreamWaitEvent(h->comm, h->ev_start, 0));
     dslash_s::TimedLaunch* xt = nullptr;  // DSLASH_TIMING_EXCHANGE interval on the comm stream
@@ -1406,16 +1410,17 @@ static void fill_boxes(StencilParams& K, const dslash_box_t* boxes, int n) {
     for (int b = n; b < kMaxBoxes; ++b) K.box_start[b + 1] = K.box_start[n];
 }
 
-static StencilFn pick_vblk_kernel(int precision, int recon, int lanes, int nrhs) {
+static StencilFn pick_vblk_kernel(int precision, int recon, bool ghost, int lanes, int nrhs) {
     if (recon == 9)
-        return precision == DSLASH_F32     ? pick_f32_r9_vblk(lanes, nrhs)
-               : precision == DSLASH_MIXED ? pick_mixed_r9_vblk(lanes, nrhs)
-                                           : pick_f64_r9_vblk(lanes, nrhs);
+        return precision == DSLASH_F32     ? pick_f32_r9_vblk(ghost, lanes, nrhs)
+               : precision == DSLASH_MIXED ? pick_mixed_r9_vblk(ghost, lanes, nrhs)
+                                           : pick_f64_r9_vblk(ghost, lanes, nrhs);
     const bool r12 = recon == 12;
     switch (precision) {
-        case DSLASH_F32: return r12 ? pick_f32_r12_vblk(lanes, nrhs) : pick_f32_r18_vblk(lanes, nrhs);
-        case DSLASH_MIXED: return r12 ? pick_mixed_r12_vblk(lanes, nrhs) : pick_mixed_r18_vblk(lanes, nrhs);
-        default: return r12 ? pick_f64_r12_vblk(lanes, nrhs) : pick_f64_r18_vblk(lanes, nrhs);
+        case DSLASH_F32: return r12 ? pick_f32_r12_vblk(ghost, lanes, nrhs) : pick_f32_r18_vblk(ghost, lanes, nrhs);
+        case DSLASH_MIXED:
+            return r12 ? pick_mixed_r12_vblk(ghost, lanes, nrhs) : pick_mixed_r18_vblk(ghost, lanes, nrhs);
+        default: return r12 ? pick_f64_r12_vblk(ghost, lanes, nrhs) : pick_f64_r18_vblk(ghost, lanes, nrhs);
     }
 }
 
@@ -1573,13 +1578,15 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
                    : (h->recon == 9 && lanes == 1) ? r9_block
                                                    : kDefaultBlock;
     const int minb = h->min_blocks ? h->min_blocks : kDefaultMinBlocks;
-    // right-hand sides are register-blocked per thread; 8 of them use 2 thread groups of 4
-    const int64_t threads = sites * lanes * (nrhs == 8 ? 2 : 1);
+    // right-hand sides are register-blocked per thread; 8 of them use 2 thread groups of 4, except
+    // site-blocked fp64 vectors (one group of 8: kernels_inst.cuh pick_vblk_n)
+    const int vblk_groups8 = (h->precision == DSLASH_F32 || h->recon == 9 || ghost) ? 2 : 1;
+    const int64_t threads = sites * lanes * (nrhs == 8 ? (K.vblk ? vblk_groups8 : 2) : 1);
     const unsigned grid = (unsigned)((threads + bs - 1) / bs);
     dslash_s::TimedLaunch* tl = nullptr;
     dslash_status st = timing_begin(h, kind, s, &tl);
     if (st != DSLASH_OK) return st;
-    StencilFn fn = K.vblk  ? pick_vblk_kernel(h->precision, h->recon, lanes, nrhs)
+    StencilFn fn = K.vblk  ? pick_vblk_kernel(h->precision, h->recon, ghost, lanes, nrhs)
                    : ghost ? pick_kernel<true>(h->precision, h->recon, lanes, minb, nrhs)
                            : pick_kernel<false>(h->precision, h->recon, lanes, minb, nrhs);
     // programmatic dependent launch: may start while the previous kernel on `s` drains
@@ -1608,7 +1615,8 @@ static dslash_status launch_rhs(dslash_t h, StencilParams K, const dslash_box_t*
         K.out = out0 + roff;
         for (int d = 0; d < 4; ++d)
             for (int side = 0; side < 2; ++side) {
-                K.ghost[d][side] = g0[d][side] ? static_cast<const char*>(g0[d][side]) + (size_t)r0 * 3 * K.face_vh[d] * es
+                K.ghost[d][side] = g0[d][side] ? static_cast<const char*>(g0[d][side]) +
+                                                     (size_t)r0 * 3 * (K.vblk ? kVBlk : K.face_vh[d]) * es
                                                : nullptr;
                 K.push[d][side] = p0[d][side] ? static_cast<char*>(p0[d][side]) + (size_t)r0 * 3 * K.face_vh[d] * es
                                               : nullptr;
@@ -1667,15 +1675,22 @@ static dslash_status apply_impl(dslash_t h, void* out, const void* in, int32_t p
     // producer push: only with a halo (without one the next apply needs no faces)
     push_out = push_out && any_halo(p);
     if (push_out && !h->push) return fail(h, DSLASH_ERR_STATE, "apply_push needs DSLASH_OPT_PUSH");
-    if (blocked) {  // site-blocked vectors (dslash_apply_multi_blocked): unpartitioned lattices only
-        if (any_halo(p)) return fail(h, DSLASH_ERR_UNSUPPORTED, "the site-blocked layout has no halo exchange");
-        if (p.vh_local % kVBlk)
-            return fail(h, DSLASH_ERR_UNSUPPORTED, "site-blocked layout: Vh_local %lld is not a multiple of %d",
-                        (long long)p.vh_local, kVBlk);
+    if (blocked) {  // site-blocked vectors (dslash_apply_multi_blocked)
+        // every face exchanged must be a run of whole 16-site blocks: the t face (3 t-slices), and
+        // per t-slice the 3 bottom / top z-slices, with their offsets
+        const int64_t zrow = (int64_t)K.lxh * K.L[1];
+        const bool ok = p.vh_local % kVBlk == 0 && (!p.halo[3] || (3 * zrow * K.L[2]) % kVBlk == 0) &&
+                        (!p.halo[2] || ((3 * zrow) % kVBlk == 0 && (zrow * K.L[2]) % kVBlk == 0));
+        if (!ok)
+            return fail(h, DSLASH_ERR_UNSUPPORTED,
+                        "site-blocked layout: Vh_local and every exchanged face must be whole blocks of %d sites", kVBlk);
+        if (any_halo(p) && (push_out || h->overlap == DSLASH_OVERLAP_DIRS))
+            return fail(h, DSLASH_ERR_UNSUPPORTED,
+                        "site-blocked layout: no producer push and no split-by-direction overlap");
         K.vblk = (int64_t)nrhs * 3 * kVBlk;
     }
     if (!any_halo(p)) return launch_rhs(h, K, p.interior, p.n_interior, false, DSLASH_TIMING_INTERIOR, s, nrhs);
-    if ((st = halo_start_impl(h, in, nrhs, s)) != DSLASH_OK) return st;
+    if ((st = halo_start_impl(h, in, nrhs, s, blocked)) != DSLASH_OK) return st;
     for (int d = 0; d < 4; ++d) {  // after halo_start: the ghosts may have been (re)allocated
         K.ghost[d][0] = h->ghost[d][0] ? h->ghost[d][0] + bank_off(h, d, h->epoch) : nullptr;
         K.ghost[d][1] = h->ghost[d][1] ? h->ghost[d][1] + bank_off(h, d, h->epoch) : nullptr;

@@ -58,23 +58,37 @@ StencilFn pick_stage(bool ghost, int lanes, int nrhs) {
     return ghost ? pick_stage_n<LR, VR, 2, true, RECON>(nrhs) : pick_stage_n<LR, VR, 2, false, RECON>(nrhs);
 }
 
-// the site-blocked layout (dslash_apply_multi_blocked): interior, MINB 2, the handle's mapping (its
-// link layout); 8 right-hand sides as two groups of 4 like the planar kernel
-template <typename LR, typename VR, int LANES, int RECON>
+// the site-blocked layout (dslash_apply_multi_blocked): MINB 2, the handle's mapping (its link
+// layout), interior or ghost-aware
+template <typename LR, typename VR, int LANES, bool GHOST, int RECON>
 StencilFn pick_vblk_n(int nrhs) {
     switch (nrhs) {
-        case 2: return dslash_kernel<LR, VR, LANES, false, 2, RECON, 2, 1, true>;
-        case 4: return dslash_kernel<LR, VR, LANES, false, 2, RECON, 4, 1, true>;
-        case 8: return dslash_kernel<LR, VR, LANES, false, 2, RECON, 4, 2, true>;
-        default: return dslash_kernel<LR, VR, LANES, false, 2, RECON, 1, 1, true>;
+        case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 2, 1, true>;
+        case 4: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 1, true>;
+        case 8:
+            // interior, fp64 vectors, recon 18 / 12: one thread per site holds all 8 (255 registers,
+            // 8 warps/SM): 355 vs 388 us for 2 groups x 4 at 32^4 fp64, mixed 297 vs 351 us.
+            // fp32 vectors (177-179 vs 201 us), recon-9 (its rebuild: 717 vs 502 us) and the
+            // ghost-aware boundary kernel keep 2 groups x 4 (profiles/r03/blocked/).
+            // dslash_lib.cu vblk_groups8 matches.
+            if constexpr (sizeof(VR) == 8 && RECON != 9 && !GHOST)
+                return dslash_kernel<LR, VR, LANES, GHOST, 1, RECON, 8, 1, true>;
+            else
+                return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2, true>;
+        default: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 1, 1, true>;
     }
 }
 
+template <typename LR, typename VR, bool GHOST, int RECON>
+StencilFn pick_vblk_l(int lanes, int nrhs) {
+    return lanes == 1   ? pick_vblk_n<LR, VR, 1, GHOST, RECON>(nrhs)
+           : lanes == 2 ? pick_vblk_n<LR, VR, 2, GHOST, RECON>(nrhs)
+                        : pick_vblk_n<LR, VR, 4, GHOST, RECON>(nrhs);
+}
+
 template <typename LR, typename VR, int RECON>
-StencilFn pick_vblk(int lanes, int nrhs) {
-    return lanes == 1 ? pick_vblk_n<LR, VR, 1, RECON>(nrhs)
-           : lanes == 2 ? pick_vblk_n<LR, VR, 2, RECON>(nrhs)
-                        : pick_vblk_n<LR, VR, 4, RECON>(nrhs);
+StencilFn pick_vblk(bool ghost, int lanes, int nrhs) {
+    return ghost ? pick_vblk_l<LR, VR, true, RECON>(lanes, nrhs) : pick_vblk_l<LR, VR, false, RECON>(lanes, nrhs);
 }
 
 }  // namespace hisq
@@ -85,5 +99,5 @@ StencilFn pick_vblk(int lanes, int nrhs) {
         return pick_any<LR, VR, RECON>(ghost, lanes, minb, nrhs);                                             \
     }                                                                                                         \
     StencilFn NAME##_stage(bool ghost, int lanes, int nrhs) { return pick_stage<LR, VR, RECON>(ghost, lanes, nrhs); } \
-    StencilFn NAME##_vblk(int lanes, int nrhs) { return pick_vblk<LR, VR, RECON>(lanes, nrhs); }                  \
+    StencilFn NAME##_vblk(bool ghost, int lanes, int nrhs) { return pick_vblk<LR, VR, RECON>(ghost, lanes, nrhs); } \
     }

@@ -225,14 +225,13 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, const void*
         st = mu == 1 ? (int64_t)P.lxh : mu == 2 ? (int64_t)P.lxh * P.L[1] : (int64_t)P.lxh * P.L[1] * P.L[2];
         idx = s.cb + (int64_t)(cw - c) * st;
     }
-    if constexpr (VBLK) {
-        // site-blocked vectors (dslash_apply_multi_blocked): (rhs, colour c) of site idx at
-        // [idx / 16][rhs * 3 + c][idx % 16], P.vblk complex per 16-site block
-        static_assert(!GHOST, "the site-blocked layout has no halo");
-        return {static_cast<const V2*>(in) + (idx >> 4) * P.vblk + (idx & 15) + rhs * 3 * kVBlk, kVBlk, false};
-    }
-    const V2* local = static_cast<const V2*>(in) + (int64_t)rhs * 3 * P.vh + idx;
-    if (!GHOST || mu < 2) return {local, P.vh, false};
+    // site-blocked vectors (dslash_apply_multi_blocked): (rhs, colour c) of site idx at
+    // [idx / 16][rhs * 3 + c][idx % 16], P.vblk complex per 16-site block; the ghost faces are
+    // blocked the same way over their face index
+    const V2* local = VBLK ? static_cast<const V2*>(in) + (idx >> 4) * P.vblk + (idx & 15) + rhs * 3 * kVBlk
+                           : static_cast<const V2*>(in) + (int64_t)rhs * 3 * P.vh + idx;
+    const int64_t lstride = VBLK ? (int64_t)kVBlk : P.vh;
+    if (!GHOST || mu < 2) return {local, lstride, false};
     // branch-free choice between the local site and the ghost face: the lanes of a site walk
     // different directions, so a branch here would diverge within the warp
     const bool ghost = ((P.halo_mask >> mu) & 1) && (cn < 0 || cn >= L);
@@ -241,11 +240,12 @@ __device__ __forceinline__ SrcRef<V2> source(const StencilParams& P, const void*
     // z face [t][d][y][xh] = cb + st (d - z) + st (3 - Lz) t (st = the direction's cb stride)
     const int64_t f = s.cb + st * (h + (side ? -L : 3)) + (mu == 2 ? st * (3 - P.L[2]) * (int64_t)s.t : 0);
     const int64_t fv = P.face_vh[mu];
-    const V2* gp = static_cast<const V2*>(P.ghost[mu][side]) + (int64_t)rhs * 3 * fv + f;
+    const V2* gp = VBLK ? static_cast<const V2*>(P.ghost[mu][side]) + (f >> 4) * P.vblk + (f & 15) + rhs * 3 * kVBlk
+                        : static_cast<const V2*>(P.ghost[mu][side]) + (int64_t)rhs * 3 * fv + f;
     // local pass of the split-by-direction overlap: the face is still in flight, so a ghost hop
     // reads the (valid) wrapped local address and the caller zeroes the vector
     const bool use_face = ghost && P.halo_pass != kPassLocal;
-    return {use_face ? gp : local, use_face ? fv : P.vh, ghost};
+    return {use_face ? gp : local, use_face ? (VBLK ? (int64_t)kVBlk : fv) : lstride, ghost};
 }
 
 // ---------------------------------------------------------------- staged neighbour tile

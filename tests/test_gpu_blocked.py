@@ -5,7 +5,9 @@ element (rhs r, colour c, site cb) at [cb // 16][r * 3 + c][cb % 16].
 - blocked applies are bitwise the planar dslash_apply_multi (same per-thread arithmetic and
   summation order; the planar path is oracle-checked in test_gpu_parity / test_gpu_full_size), for
   every precision, recon and right-hand-side count, and match the oracle directly;
-- the unsupported cases fail loudly (a halo, Vh % 16 != 0).
+- with a halo (self-halo t / t + z through every transport; P2P ranks in test_gpu_multiproc) the
+  faces are exchanged as whole 16-site blocks, bitwise;
+- the unsupported cases fail loudly (Vh or a face not whole blocks, the split-by-direction overlap).
 """
 import pytest
 
@@ -82,11 +84,43 @@ def test_blocked_vs_oracle(torch_cuda, precision, tol):
         assert oracle.normwise_error(got[r].astype("complex128"), ref) <= tol
 
 
+@pytest.mark.parametrize("halo,kw", [(8, {}), (12, {}), (8, {"transport": "p2p"}), (12, {"transport": "p2p"}),
+                                     (12, {"overlap": False}), (8, {"self_nccl": True}),
+                                     (12, {"precision": "f32"}), (12, {"precision": "mixed", "recon": 12}),
+                                     (8, {"kernel": "dir2"})])
+def test_blocked_self_halo_bitwise(torch_cuda, halo, kw):
+    """With a self-halo (t: 8, t + z: 12; device copies, P2P copies, NCCL to self, one launch after
+    the exchange) the blocked apply exchanges whole 16-site blocks and equals the planar apply
+    without a halo bitwise."""
+    torch = torch_cuda
+    from paper_conf_sc_dufekgaad024_b200 import Dslash
+    dims = (8, 8, 12, 12)          # Vh 4608; t face 3 x 384 sites, z faces 3 x 32 per t-slice
+    fat, lng = fieldgen.workload_links(dims)
+    kernel = kw.pop("kernel", "site")
+    plain_kw = {k: v for k, v in kw.items() if k in ("precision", "recon")}
+    with Dslash(dims, kernel=kernel, **plain_kw) as D:
+        D.load_links(fat, lng)
+        src = torch.stack([torch.from_numpy(fieldgen.vector_cb(dims, 90 + r, 1)) for r in range(8)])
+        src = src.to(D.dtype).contiguous().cuda()
+        ref = D.apply_multi(torch.empty_like(src), src, 0)
+        torch.cuda.synchronize()
+    with Dslash(dims, kernel=kernel, force_halo=halo, **kw) as D:
+        D.load_links(fat, lng)
+        bsrc = D.to_blocked(torch.empty_like(src), src)
+        bout = torch.empty_like(src)
+        for _ in range(3):                        # several epochs through the same ghosts
+            D.apply_multi_blocked(bout, bsrc, 0)
+        got = D.from_blocked(torch.empty_like(src), bout)
+        torch.cuda.synchronize()
+    assert torch.equal(got, ref)
+
+
 def test_blocked_unsupported(torch_cuda):
     torch = torch_cuda
     from paper_conf_sc_dufekgaad024_b200 import Dslash, _abi
-    with Dslash(DIMS, force_halo=8) as D:       # a t halo: the blocked layout has no exchange
-        D.load_links(*fieldgen.workload_links(DIMS))
+    dims = (8, 8, 12, 12)
+    with Dslash(dims, force_halo=8, overlap="dirs") as D:   # split by direction: planar partial sums
+        D.load_links(*fieldgen.workload_links(dims))
         v = torch.zeros((8, 3, D.vh), dtype=D.dtype, device="cuda")
         with pytest.raises(_abi.DslashError) as e:
             D.apply_multi_blocked(torch.empty_like(v), v, 0)
@@ -100,3 +134,10 @@ def test_blocked_unsupported(torch_cuda):
             with pytest.raises(_abi.DslashError) as e:
                 call()
             assert e.value.status == _abi.DSLASH_ERR_UNSUPPORTED
+    dims = (8, 6, 8, 8)                           # t face 3 x 192 sites is whole blocks, z face 3 x 24 per t is not
+    with Dslash(dims, force_halo=4) as D:
+        D.load_links(*fieldgen.workload_links(dims))
+        v = torch.zeros((2, 3, D.vh), dtype=D.dtype, device="cuda")
+        with pytest.raises(_abi.DslashError) as e:
+            D.apply_multi_blocked(torch.empty_like(v), v, 0)
+        assert e.value.status == _abi.DSLASH_ERR_UNSUPPORTED

@@ -49,7 +49,7 @@ def _rank_main(rank, world, port, gdims, grid, kw, parity, napply, nrhs, q):
         o, e = D.origin, D.local_dims
         fat, lng = fieldgen.workload_links(gdims, origin=o, extent=e)
         D.load_links(fat, lng)
-        if mode != "apply":
+        if mode in ("cg", "cg_mixed"):
             b = torch.from_numpy(fieldgen.vector_cb(gdims, SEED, parity, origin=o, extent=e)).cuda()
             x = D.empty_vector()
             if mode == "cg":
@@ -60,6 +60,18 @@ def _rank_main(rank, world, port, gdims, grid, kw, parity, napply, nrhs, q):
                 info = (ok, it, outer, res)
             torch.cuda.synchronize()
             q.put((rank, tuple(o), tuple(e), x.cpu().numpy(), info))
+            D.close()
+            return
+        if mode == "blocked":                    # site-blocked multi-RHS layout
+            src = torch.stack([torch.from_numpy(fieldgen.vector_cb(gdims, SEED + r, 1 - parity, origin=o, extent=e))
+                               for r in range(nrhs)]).to(D.dtype).contiguous().cuda()
+            bsrc = D.to_blocked(torch.empty_like(src), src)
+            bout = torch.empty_like(src)
+            for _ in range(napply):
+                D.apply_multi_blocked(bout, bsrc, parity)
+            out = D.from_blocked(torch.empty_like(src), bout)
+            torch.cuda.synchronize()
+            q.put((rank, tuple(o), tuple(e), out.cpu().numpy(), None))
             D.close()
             return
         if nrhs == 1:
@@ -147,6 +159,19 @@ def test_multirank_p2p_multi_rhs():
     gdims, grid = (8, 8, 8, 16), (1, 1, 1, 2)
     got = _run(2, gdims, grid, {}, 0, napply=2, nrhs=3)
     assert np.array_equal(got, _single(gdims, {}, 0, nrhs=3))
+
+
+@pytest.mark.parametrize("gdims,grid", [((8, 8, 8, 16), (1, 1, 1, 2)), ((8, 8, 16, 8), (1, 1, 2, 1)),
+                                        ((8, 8, 8, 8), (1, 1, 2, 2))])
+@pytest.mark.parametrize("kw", [{"kernel": "site"}, {"precision": "mixed", "kernel": "site"}, {"overlap": False}])
+def test_multirank_p2p_blocked(gdims, grid, kw):
+    """The site-blocked multi-RHS layout across P2P ranks (faces = whole 16-site blocks): the
+    gathered result equals the 1-rank planar apply bitwise."""
+    world = grid[2] * grid[3]
+    got = _run(world, gdims, grid, dict(kw, _mode="blocked"), 0, napply=2, nrhs=8)
+    single_kw = {k: v for k, v in kw.items() if k != "overlap"}
+    ref = _single(gdims, single_kw, 0, nrhs=8)
+    assert np.array_equal(got, ref)
 
 
 def test_multirank_p2p_32_local():
