@@ -395,6 +395,21 @@ DSLASH_API dslash_status dslash_cg_mixed(dslash_t h, void* x, const void* b, int
                                          double rel_tol, double inner_tol, int32_t max_iter, int32_t* iters,
                                          int32_t* outer_iters, double* rel_resid, dslash_stream_t stream);
 
+/* CG for nrhs <= 8 independent systems A_p x_r = b_r (A_p as dslash_cg) that share every pass over
+ * the links (SURVEY.md §8(f)-3 on the §8(f)-4 multi-RHS stencil): each
+ * iteration applies the stencil twice to all nrhs directions at once
+ * (dslash_apply_multi_blocked), then every system advances on its own scalars
+ * (Hestenes-Stiefel, double-double dot products).  A system whose residual met rel_tol is frozen
+ * while the others continue.  x, b: device buffers of nrhs x 3 x Vh_local fp64 complex in the
+ * SITE-BLOCKED layout (dslash_apply_multi_blocked; dslash_vectors_to_blocked converts).
+ * iters[r]: the iteration at which system r converged (max_iter if it did not); rel_resid[r]: its
+ * true |b_r - A x_r| / |b_r| (each array nrhs long, or NULL).  Requires a DSLASH_F64 or
+ * DSLASH_MIXED handle with parity_mask DSLASH_BOTH, one rank, nonzero mass, the blocked layout's
+ * conditions; synchronous; DSLASH_ERR_NOT_CONVERGED (not sticky) if a system did not converge. */
+DSLASH_API dslash_status dslash_cg_multi_blocked(dslash_t h, int32_t nrhs, void* x, const void* b, int32_t parity,
+                                                 double mass, double rel_tol, int32_t max_iter, int32_t* iters,
+                                                 double* rel_resid, dslash_stream_t stream);
+
 /* Halo exchange only: start sending the depth-3 faces of `in` (source parity
  * src_parity) after the work already queued on `stream`; dslash_halo_wait makes
  * `stream` wait for the ghost zones.  No-op when no direction has a halo.  Exposed

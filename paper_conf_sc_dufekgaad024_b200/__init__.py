@@ -238,6 +238,14 @@ class Dslash:
                                      int(max_iter), _stream_handle(stream))
         return st == _abi.DSLASH_OK, it, res
 
+    def cg_multi_blocked(self, x, b, parity, mass, rel_tol=1e-10, max_iter=1000, stream=None):
+        """CG for nrhs <= 8 systems sharing every link pass (dslash_cg_multi_blocked); x, b: site-blocked
+        fp64 tensors of nrhs x 3 x Vh elements.  Returns (all converged, [iterations], [true rel. residual])."""
+        nrhs = self._check_blocked(x, b)
+        st, its, res = _abi.dslash_cg_multi_blocked(self.h, nrhs, x.data_ptr(), b.data_ptr(), int(parity), float(mass),
+                                                    float(rel_tol), int(max_iter), _stream_handle(stream))
+        return st == _abi.DSLASH_OK, its, res
+
     def cg_mixed(self, x, b, parity, mass, rel_tol=1e-10, inner_tol=1e-4, max_iter=5000, stream=None):
         """Mixed-precision CG (fp32 inner solves, fp64 defect correction) for the same system as
         cg(); returns (converged, inner iterations, outer corrections, true rel. residual)."""

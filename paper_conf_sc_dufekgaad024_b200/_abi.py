@@ -110,6 +110,9 @@ _SIGS = {
     "dslash_cg_mixed": ([_h, _vp, _vp, ctypes.c_int32, ctypes.c_double, ctypes.c_double, ctypes.c_double,
                          ctypes.c_int32, ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_int32),
                          ctypes.POINTER(ctypes.c_double), _vp], ctypes.c_int),
+    "dslash_cg_multi_blocked": ([_h, ctypes.c_int32, _vp, _vp, ctypes.c_int32, ctypes.c_double, ctypes.c_double,
+                                 ctypes.c_int32, ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_double), _vp],
+                                ctypes.c_int),
     "dslash_halo_start": ([_h, _vp, ctypes.c_int32, _vp], ctypes.c_int),
     "dslash_halo_wait": ([_h, _vp], ctypes.c_int),
     "dslash_sync": ([_h], ctypes.c_int),
@@ -260,6 +263,16 @@ def dslash_cg(h, x_ptr, b_ptr, parity, mass, rel_tol, max_iter, stream=0):
     if st not in (DSLASH_OK, DSLASH_ERR_NOT_CONVERGED):
         check(st, h)
     return st, it.value, res.value
+
+
+def dslash_cg_multi_blocked(h, nrhs, x_ptr, b_ptr, parity, mass, rel_tol, max_iter, stream=0):
+    """Returns (status, [iterations per system], [true relative residual per system])."""
+    its = (ctypes.c_int32 * nrhs)()
+    res = (ctypes.c_double * nrhs)()
+    st = lib.dslash_cg_multi_blocked(h, nrhs, x_ptr, b_ptr, parity, mass, rel_tol, max_iter, its, res, stream)
+    if st not in (DSLASH_OK, DSLASH_ERR_NOT_CONVERGED):
+        check(st, h)
+    return st, list(its), list(res)
 
 
 def dslash_cg_mixed(h, x_ptr, b_ptr, parity, mass, rel_tol, inner_tol, max_iter, stream=0):

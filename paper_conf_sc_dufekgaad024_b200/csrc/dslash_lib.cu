@@ -1800,6 +1800,10 @@ extern "C" dslash_status dslash_apply_multi_blocked(dslash_t h, int32_t nrhs, vo
     return apply_impl(h, out, in, parity, nrhs, stream, false, true);
 }
 
+dslash_status hisq_apply_blocked(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s) {
+    return apply_impl(h, out, in, parity, nrhs, (dslash_stream_t)s, false, true);
+}
+
 // planar [rows][vh] <-> site-blocked [vh / 16][rows][16] (rows = 3 nrhs), one element per thread in
 // the blocked order, so both sides move runs of 16 consecutive elements
 template <typename T>
@@ -2026,6 +2030,9 @@ extern "C" dslash_status dslash_destroy(dslash_t h) {
         if (v) cudaFree(v);
     for (void* v : h->links32)
         if (v) cudaFree(v);
+    for (void* v : h->cgm_vec)
+        if (v) cudaFree(v);
+    if (h->cgm_small) cudaFree(h->cgm_small);
     for (void* v : h->cg_vec)
         if (v) cudaFree(v);
     if (h->cg_partial) cudaFree(h->cg_partial);

@@ -62,6 +62,11 @@ struct dslash_s {
     // conjugate-gradient scratch (solver.cu): r, p, q on the target parity, t on the other one,
     // block partial sums and the reduced scalars
     void* cg_vec[4] = {};
+    // dslash_cg_multi_blocked scratch (solver_multi.cu): r, p, q, t of cgm_bytes each, grown on demand,
+    // and its partials / scalars / convergence record
+    void* cgm_vec[4] = {};
+    size_t cgm_bytes = 0;
+    void* cgm_small = nullptr;
     // mixed-precision solver (dslash_cg_mixed): fp32 e, r, p, q, t and the fp32 links per parity
     void* cg_vec32[5] = {};
     void* links32[2] = {};
@@ -181,3 +186,5 @@ dslash_status hisq_convert_links_sloppy(dslash_t h, int parity);
 // push the faces of out into the neighbours' ghosts for the next apply (DSLASH_OPT_PUSH)
 dslash_status hisq_apply(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s,
                          bool push = false);
+// the same on site-blocked vectors (dslash_apply_multi_blocked)
+dslash_status hisq_apply_blocked(dslash_t h, void* out, const void* in, int32_t parity, int32_t nrhs, cudaStream_t s);
