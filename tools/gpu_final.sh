@@ -1,5 +1,6 @@
 #!/bin/bash
 # End-of-round evidence on one GPU box (from the repo root): bash tools/gpu_final.sh <name>
+# (compute-sanitizer is closed on this pool: tools/gpu_sanitize.sh is run separately where it is open)
 n=${1:-r03_final}
 bash tools/gpu_run.sh $n \
   "timeout 2400 python -m pytest tests -m gpu -q --timeout 900" \
@@ -11,8 +12,9 @@ bash tools/gpu_run.sh $n \
   "bash tools/gpu_ncu.sh gpurun_out/$n/ncu_n8 --nrhs 8" \
   "bash tools/gpu_ncu.sh gpurun_out/$n/ncu_n8_blocked --nrhs 8 --layout blocked" \
   "bash tools/gpu_ncu.sh gpurun_out/$n/ncu_n8_f32_blocked --nrhs 8 --layout blocked --precision f32" \
-  "bash tools/gpu_sanitize.sh gpurun_out/$n/sanitize" \
   "bash tools/config_table.sh" \
   "bash tools/halo_probe.sh" \
-  "timeout 300 python bench.py --nrhs 8 --layout blocked --precision f32 --no-cpu-baseline" \
-  "timeout 300 python bench.py --nrhs 8 --no-cpu-baseline"
+  "bash tools/strong_probe.sh" \
+  "timeout 600 python tools/bench_cg_multi.py" \
+  "timeout 300 python bench.py --nrhs 8 --layout blocked --no-cpu-baseline" \
+  "timeout 300 python bench.py --nrhs 8 --layout blocked --precision f32 --no-cpu-baseline"
