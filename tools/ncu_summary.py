@@ -1,6 +1,6 @@
 """Summarise ncu reports into profiles/ (JSON + markdown rows).
 
-python tools/ncu_summary.py <report.ncu-rep> --variant site --local 32,32,32,32 [--out profiles/ncu_summary.json]
+python tools/ncu_summary.py <report.ncu-rep | full_raw.csv> --variant site --local 32,32,32,32 [--out profiles/ncu_summary.json]
 Reads `ncu -i ... --page raw --csv`, keeps the metrics the roofline uses, and merges one entry
 per (variant, local_dims) into the JSON file bench.py reads for `roofline.traffic`.
 """
@@ -22,7 +22,12 @@ SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
 
 
 def rows(rep):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True, check=True).stdout
+    if rep.endswith(".csv"):  # an exported `--page raw --csv` (gpu_ncu.sh full_raw.csv)
+        with open(rep) as f:
+            out = f.read()
+    else:
+        out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True,
+                             check=True).stdout
     r = list(csv.reader(io.StringIO(out)))
     hdr, units = r[0], r[1]
     res = []
