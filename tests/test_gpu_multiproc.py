@@ -325,6 +325,18 @@ def test_distinct_gpus_multi_rhs_nccl():
     assert np.array_equal(got, _single(gdims, {}, 0, nrhs=3))
 
 
+@pytest.mark.parametrize("transport", ["nccl", "p2p"])
+@pytest.mark.parametrize("gdims,grid", [((8, 8, 8, 16), (1, 1, 1, 2)), ((8, 8, 16, 8), (1, 1, 2, 1))])
+def test_distinct_gpus_blocked(transport, gdims, grid):
+    """The site-blocked 8-RHS layout across two GPUs (faces as whole 16-site blocks over NCCL or
+    NVLink peer copies): bitwise the 1-rank planar apply."""
+    if _ngpu() < 2:
+        pytest.skip(f"needs 2 GPUs, {_ngpu()} visible")
+    got = _run(2, gdims, grid, {"_distinct": True, "transport": transport, "kernel": "site", "_mode": "blocked"}, 0,
+               napply=2, nrhs=8)
+    assert np.array_equal(got, _single(gdims, {"kernel": "site"}, 0, nrhs=8))
+
+
 def test_two_handles_two_devices_one_process():
     """Two handles in one process on different GPUs, used interleaved while torch's current device
     is the other one: every entry point runs on its handle's device (DeviceGuard) and leaves the
