@@ -1579,8 +1579,8 @@ static dslash_status launch(dslash_t h, const StencilParams& K, bool ghost, int 
                                                    : kDefaultBlock;
     const int minb = h->min_blocks ? h->min_blocks : kDefaultMinBlocks;
     // right-hand sides are register-blocked per thread; 8 of them use 2 thread groups of 4, except
-    // site-blocked fp64 vectors (one group of 8: kernels_inst.cuh pick_vblk_n)
-    const int vblk_groups8 = (h->precision == DSLASH_F32 || h->recon == 9 || ghost) ? 2 : 1;
+    // interior site-blocked launches without recon-9 (one group of 8: kernels_inst.cuh pick_vblk_n)
+    const int vblk_groups8 = (h->recon == 9 || ghost) ? 2 : 1;
     const int64_t threads = sites * lanes * (nrhs == 8 ? (K.vblk ? vblk_groups8 : 2) : 1);
     const unsigned grid = (unsigned)((threads + bs - 1) / bs);
     dslash_s::TimedLaunch* tl = nullptr;

@@ -66,13 +66,14 @@ StencilFn pick_vblk_n(int nrhs) {
         case 2: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 2, 1, true>;
         case 4: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 1, true>;
         case 8:
-            // interior, fp64 vectors, recon 18 / 12: one thread per site holds all 8 (255 registers,
-            // 8 warps/SM): 355 vs 388 us for 2 groups x 4 at 32^4 fp64, mixed 297 vs 351 us.
-            // fp32 vectors (177-179 vs 201 us), recon-9 (its rebuild: 717 vs 502 us) and the
-            // ghost-aware boundary kernel keep 2 groups x 4 (profiles/r03/blocked/).
-            // dslash_lib.cu vblk_groups8 matches.
-            if constexpr (sizeof(VR) == 8 && RECON != 9 && !GHOST)
-                return dslash_kernel<LR, VR, LANES, GHOST, 1, RECON, 8, 1, true>;
+            // interior, recon 18 / 12: one thread per site holds all 8 right-hand sides; fp64 vectors
+            // (f64, mixed) at 255 registers and 8 warps/SM: 355 vs 388 us for 2 groups x 4 at 32^4
+            // fp64, mixed 297 vs 351 us; fp32 vectors at 128 registers and 16 warps/SM: 167 vs
+            // 178 us (recon-12 161 vs 181 us).  Recon-9 (its rebuild needs the registers: 717 vs
+            // 502 us) and the ghost-aware boundary kernel keep 2 groups x 4
+            // (profiles/r03/blocked/).  dslash_lib.cu vblk_groups8 matches.
+            if constexpr (RECON != 9 && !GHOST)
+                return dslash_kernel<LR, VR, LANES, GHOST, sizeof(VR) == 8 ? 1 : 2, RECON, 8, 1, true>;
             else
                 return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 4, 2, true>;
         default: return dslash_kernel<LR, VR, LANES, GHOST, 2, RECON, 1, 1, true>;
