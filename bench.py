@@ -57,7 +57,7 @@ def parse(argv=None):
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--kernel", default=None, choices=["site", "dir2", "dir4"],
-                    help="default: dir2 (site with --recon 9 or --nrhs > 1, measured best for them)")
+                    help="default: dir2 (site with --recon 9, --nrhs > 1 or --precision mixed, measured best for them)")
     ap.add_argument("--min-blocks", type=int, default=0)
     ap.add_argument("--layout", default="planar", choices=["planar", "blocked"],
                     help="multi-RHS vector layout: planar [nrhs][3][Vh] (dslash_apply_multi) or site-blocked "
@@ -115,7 +115,10 @@ def parse(argv=None):
                          "of a per-rank number and rank 0 prints one JSON line (no CUDA)")
     args = ap.parse_args(argv)
     if args.kernel is None:
-        args.kernel = "site" if (args.recon == 9 or args.nrhs > 1) else "dir2"
+        # measured per configuration (profiles/r03/recon_mapping_ab.txt, mapping_mixed_ab.txt): site for
+        # recon-9, multi-RHS and mixed precision (mixed 96.2 vs 99.9 us, mixed recon-12 83.4 vs 88.6),
+        # dir2 otherwise (fp64 / fp32: +1%)
+        args.kernel = "site" if (args.recon == 9 or args.nrhs > 1 or args.precision == "mixed") else "dir2"
     return args
 
 

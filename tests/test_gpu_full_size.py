@@ -68,9 +68,9 @@ def _check(got_cb, fat, lng, psi, parity, precision, what):
     return err
 
 
-def _bench_kernel(recon, nrhs):
-    # bench.py's default mapping: site for recon-9 and multi-RHS, dir2 otherwise
-    return "site" if (recon == 9 or nrhs > 1) else "dir2"
+def _bench_kernel(recon, nrhs, precision="f64"):
+    # bench.py's default mapping: site for recon-9, multi-RHS and mixed precision, dir2 otherwise
+    return "site" if (recon == 9 or nrhs > 1 or precision == "mixed") else "dir2"
 
 
 def _run_chain(torch, links32, psi_full, parity, nrhs=1, blocked=False, **kw):
@@ -115,7 +115,7 @@ def test_32_precisions_and_recon(torch_cuda, links32, psi_full, precision, recon
     """fp32 / mixed (§8(f)-1), recon-12 and recon-9 in every precision (§8(f)-2)."""
     fat, lng = links32
     parity = 0
-    kernel = _bench_kernel(recon, 1)
+    kernel = _bench_kernel(recon, 1, precision)
     for ss, got in _run_chain(torch_cuda, links32, psi_full, parity, precision=precision, recon=recon,
                               kernel=kernel):
         _check(got, fat, lng, psi_full(ss[0]), parity, precision, (precision, recon, ss))
