@@ -307,9 +307,9 @@ DSLASH_API dslash_status dslash_apply_multi(dslash_t h, int32_t nrhs, void* out,
  *     [(cb / 16) * (nrhs * 3 * 16) + (r * 3 + c) * 16 + cb % 16]
  * (complex of the handle's vector precision), i.e. blocks of 16 consecutive sites, each holding
  * its nrhs x 3 rows of 16 back to back.  A warp's gathers of one hop then read a few contiguous
- * kilobytes instead of 3 x nrhs planes Vh_local apart (8 RHS at 32^4: fp64 393 -> 376 us, fp32
- * 219 -> 186 us; profiles/r03/mrhs/).  Results are bitwise those of dslash_apply_multi on the
- * planar copies.  Caller-owned device buffers of nrhs x 3 x Vh_local complex, 16-byte aligned,
+ * kilobytes instead of 3 x nrhs planes Vh_local apart, and one thread can hold all 8 right-hand
+ * sides (8 RHS at 32^4: fp64 391 -> 355 us, fp32 219 -> 166 us; profiles/r03/blocked/).  Results
+ * are bitwise those of dslash_apply_multi on the planar copies.  Caller-owned device buffers of nrhs x 3 x Vh_local complex, 16-byte aligned,
  * non-overlapping.  Requires Vh_local % 16 == 0.  With a halo (t and/or z partition, or a
  * forced self-halo) the faces are exchanged as whole blocks, in the same layout: every face must
  * be whole 16-site blocks (t: 3 Lx/2 Ly Lz; z: 3 Lx/2 Ly and Lx/2 Ly Lz multiples of 16, local
